@@ -1,0 +1,195 @@
+"""Pilot output -> resolved control flow, execution blocks and per-block tensor sets
+(§IV-B; readings R4, R6).
+
+Oracle — test infrastructure only (see oracle/__init__.py).
+
+Logit layout (reading R4): [block head: K_max x 10 | branch head: one logit per choice of
+every free (untied) control-flow site, sites in preorder | zero padding].
+  block head: n = rint(y * 2^sigma) (round half to even), clamped to [0, 2^24-1];
+              sigma = 4 for the count and idiom sums, 10 for the dimension sums;
+              slot k is empty iff its count n_0 = 0 (P:L143 vector format).
+  branch head: choice = argmax (lowest index on ties) over the site's logits; a tied site
+              replays the choice of the site it names (reading R6).
+Without a branch head the paper's traversal match resolves the path.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+import math
+
+import numpy as np
+
+from workloads import Op, If, Loop, R, W
+from . import afm as A
+
+NEAR_TIE = 1e-6
+
+
+@dataclass
+class Prediction:
+    choices: list
+    path: list              # executed rows: Op or None (control)
+    groups: list            # [(start_row, end_row)]
+    blocks: list            # block10 of every group (the executed block vectors)
+    W: list                 # per group: [(tensor_id, mode_union, needs_fetch)]
+    slots: list             # raw decoded block head, K_max x 10 ints
+    near_ties: list = field(default_factory=list)
+    matched: bool = True    # traversal: exact match found
+
+
+def decode_block_head(y, K_max, near):
+    """Block head -> K_max x 10 integer slot vectors (reading R4)."""
+    slots = []
+    for k in range(K_max):
+        v = []
+        for e in range(10):
+            sigma = 4 if e < 7 else 10
+            t = float(y[10 * k + e]) * (2.0 ** sigma)
+            frac = t - math.floor(t)
+            if abs(frac - 0.5) < NEAR_TIE:
+                near.append(("slot", k, e))
+            n = int(np.rint(t))
+            v.append(min(max(n, 0), A.SAT))
+        slots.append(tuple(v))
+    return slots
+
+
+def decode_branch_head(y, program, K_max, near):
+    """Branch head -> choice index for every site in preorder (reading R4, R6)."""
+    sl = A.sites(program)
+    off = 10 * K_max
+    choices = [0] * len(sl)
+    for i, s in enumerate(sl):
+        if s.tie >= 0:
+            choices[i] = choices[s.tie]
+            continue
+        b = A.n_choices(s)
+        logits = [float(v) for v in y[off:off + b]]
+        best = 0
+        for c in range(1, b):
+            if logits[c] > logits[best]:
+                best = c
+        srt = sorted(logits, reverse=True)
+        if b > 1 and srt[0] - srt[1] < NEAR_TIE * max(1.0, abs(srt[0])):
+            near.append(("site", i))
+        choices[i] = best
+        off += b
+    return choices
+
+
+def cut(L, counts):
+    """Partition rows [0, L) at the cumulative predicted counts (reading R4): group g covers
+    [C_g, C_{g+1}) clipped to L; groups starting at or past L are dropped; if the counts sum
+    to less than L the last group absorbs the remainder; no non-empty slot -> one group."""
+    if not counts or L == 0:
+        return [(0, L)] if L > 0 else []
+    groups, c = [], 0
+    for n in counts:
+        if c >= L:
+            break
+        groups.append((c, min(c + n, L)))
+        c += n
+    if groups[-1][1] < L:
+        groups[-1] = (groups[-1][0], L)
+    return groups
+
+
+def enumerate_paths(program):
+    """All resolved paths in lexicographic order of branch choices (program order; lower
+    branch index / lower trip count first). Yields (choices_by_site_index, rows)."""
+    sl = A.sites(program)
+    index = {id(s): i for i, s in enumerate(sl)}
+
+    def rec(items, pos, choices):
+        # yields (choices, rows) for items[pos:]
+        if pos == len(items):
+            yield choices, []
+            return
+        it = items[pos]
+        if isinstance(it, Op):
+            for ch, rows in rec(items, pos + 1, choices):
+                yield ch, [it] + rows
+            return
+        si = index[id(it)]
+        opts = [choices[it.tie]] if it.tie >= 0 else list(range(A.n_choices(it)))
+        for c in opts:
+            ch0 = dict(choices)
+            ch0[si] = c
+            if isinstance(it, If):
+                heads = [(ch0, [None])]
+                body_items = it.branches[c]
+                for ch1, brows in rec(body_items, 0, ch0):
+                    for ch2, rest in rec(items, pos + 1, ch1):
+                        yield ch2, [None] + brows + rest
+            else:
+                n = it.lo + c
+                yield from _loop_iter(it, n, items, pos, ch0, rec)
+
+    def _loop_iter(it, n, items, pos, ch, rec_):
+        def iters(k, chk):
+            if k == n:
+                yield chk, [None]
+                return
+            for ch1, brows in rec_(it.body, 0, chk):
+                for ch2, rest in iters(k + 1, ch1):
+                    yield ch2, [None] + brows + rest
+        for ch1, lrows in iters(0, ch):
+            for ch2, rest in rec_(items, pos + 1, ch1):
+                yield ch2, lrows + rest
+
+    for ch, rows in rec(program, 0, {}):
+        yield [ch.get(i, 0) for i in range(len(sl))], rows
+
+
+def traversal(program, pred_blocks):
+    """The paper's mapping: find the first path (lexicographic order) whose
+    rows, cut at the predicted cumulative counts, give exactly the predicted block vectors;
+    otherwise pick the path closest in operator count (first on ties)."""
+    total = sum(v[0] for v in pred_blocks)
+    best = None
+    for choices, rows in enumerate_paths(program):
+        if len(rows) == total:
+            groups = cut(len(rows), [v[0] for v in pred_blocks])
+            if len(groups) == len(pred_blocks) and all(
+                    A.block10(rows[s:e]) == tuple(pred_blocks[g]) for g, (s, e) in enumerate(groups)):
+                return choices, rows, True
+        d = abs(len(rows) - total)
+        if best is None or d < best[0]:
+            best = (d, choices, rows)
+    return best[1], best[2], False
+
+
+def tensor_sets(path, groups):
+    """W_j (reading R8): tensors accessed by the group's operators, in order of first access
+    (row order; within an operator ascending tensor id); mode = union of the group's accesses;
+    needs_fetch = the first access reads the tensor."""
+    out = []
+    for (s, e) in groups:
+        order, mode, fetch = [], {}, {}
+        for r in path[s:e]:
+            if r is None:
+                continue
+            for t, m in r.acc:
+                if t not in mode:
+                    order.append(t)
+                    mode[t] = m
+                    fetch[t] = bool(m & R)
+                else:
+                    mode[t] |= m
+        out.append([(t, mode[t], fetch[t]) for t in order])
+    return out
+
+
+def decode(wl, y, branch_head=True):
+    near = []
+    slots = decode_block_head(y, wl.K_max, near)
+    counts_slots = [v for v in slots if v[0] != 0]
+    matched = True
+    if branch_head:
+        choices = decode_branch_head(y, wl.program, wl.K_max, near)
+        path = A.resolve(wl.program, choices)
+    else:
+        choices, path, matched = traversal(wl.program, counts_slots)
+    groups = cut(len(path), [v[0] for v in counts_slots])
+    blocks = [A.block10(path[s:e]) for s, e in groups]
+    return Prediction(choices, path, groups, blocks, tensor_sets(path, groups), slots, near, matched)

@@ -1,0 +1,46 @@
+"""One oracle step of the hot path: encode -> pilot -> decode -> plan.
+
+Oracle — test infrastructure only (see oracle/__init__.py).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import encode as E, pilot as P, decode as D, plan as PL
+
+
+@dataclass
+class StepResult:
+    feat: np.ndarray
+    logits: np.ndarray
+    pred: D.Prediction
+    transitions: list
+    state: PL.State
+    error: str = ""
+
+
+def step(wl, sample, state, group_table=(), branch_head=None, policy=None):
+    bh = wl.notes.get("branch_head", True) if branch_head is None else branch_head
+    x = E.encode(wl, wl.samples[sample], wl.hist_ids, group_table)
+    y = P.forward(wl.pilot, x, wl.nn_type)
+    pred = D.decode(wl, y, branch_head=bh)
+    try:
+        trs, st = PL.plan(state, wl, pred.W, policy)
+        return StepResult(x, y, pred, trs, st)
+    except PL.BudgetError as e:
+        return StepResult(x, y, pred, [], state, str(e))
+
+
+def run(wl, n_steps, policy=None, branch_head=None):
+    """Consecutive steps over samples 0..n_steps-1 with the history table fed forward."""
+    st = PL.initial_state(len(wl.tensors))
+    table = ()
+    out = []
+    for s in range(n_steps):
+        r = step(wl, s % len(wl.samples), st, table, branch_head, policy)
+        out.append(r)
+        st = r.state
+        table = r.pred.blocks
+    return out

@@ -1,0 +1,513 @@
+"""Seeded synthetic DyNN traces — the ONLY module shared by oracle/ and the CUDA path.
+
+It holds the *inputs* of the method and none of its arithmetic: the static program
+(operators with their idiom counts, input shapes and tensor accesses; If/Loop
+control flow), the tensor table, the per-sample input-shape descriptors, the
+pilot-model weights, and a counter-based byte-content generator used by the
+migration tests (oracle/ implements nothing of it; both sides call it).
+
+No signature, AFM, block vector, feature, logit, decode or plan is computed here.
+
+Program model (§IV-A2):
+  Op(idioms[6], inputs=(shape, ...), acc=((tensor_id, mode), ...))
+      idioms = counts of [transpose, gather, scatter, reduction, stream, stencil]
+      (column order P:L135); acc sorted by tensor id, unique.
+  If(branches=[program, ...], tie=-1)   one control-flow statement
+  Loop(body=program, lo, hi, tie=-1)    trip count in [lo, hi]
+  tie >= 0 marks a site that replays the choice of an earlier site (the backward
+  pass of a routed layer follows its forward choice) — DESIGN.md reading R6.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+import numpy as np
+
+R, W, RW = 1, 2, 3
+CNN, LSTM, TRANSFORMER = 0, 1, 2
+MiB = 1 << 20
+GiB = 1 << 30
+
+
+@dataclass
+class Op:
+    idioms: tuple
+    inputs: tuple
+    acc: tuple
+    name: str = ""
+
+
+@dataclass
+class If:
+    branches: list
+    tie: int = -1
+
+
+@dataclass
+class Loop:
+    body: list
+    lo: int
+    hi: int
+    tie: int = -1
+
+
+@dataclass
+class Tensor:
+    nbytes: int
+    host_off: int
+    transient: bool
+    name: str = ""
+
+
+@dataclass
+class PilotSpec:
+    """Pilot topology + fp32 weights (row-major W[out][in]).
+
+    feature: list of (in_off, in_len, out) input-feature layers;
+             empty list = identity feature stage (tiny T32 topology).
+    mlp:     list of (in, out) layer dims shared by the three MLPs.
+    out_in:  input width of the output layer; O = number of logits.
+    weights: {"feat{i}.W","feat{i}.b","mlp{k}.{l}.W","mlp{k}.{l}.b","out.W","out.b"}
+    """
+    F: int
+    O: int
+    feature: list
+    mlp: list
+    out_in: int
+    weights: dict
+
+
+@dataclass
+class Workload:
+    name: str
+    nn_type: int
+    program: list
+    tensors: list
+    S_max: int
+    D_s: int
+    h: int
+    K_max: int
+    budget: int
+    align: int
+    policy: int          # 0 = PAPER (evict all unused), 1 = RETAIN (Belady prefix cut)
+    pilot: PilotSpec
+    samples: np.ndarray  # int64 [n_samples, D_s] input-shape descriptors
+    hist_ids: np.ndarray  # int32 [h] history group ids (negative = from the end)
+    seed: int
+    notes: dict = field(default_factory=dict)
+
+
+# ----------------------------------------------------------------------------
+# helpers (input construction only)
+# ----------------------------------------------------------------------------
+
+def _op(rng, acc, nin=2, name=""):
+    idioms = tuple(int(x) for x in rng.integers(0, 4, size=6))
+    inputs = tuple(tuple(int(d) for d in rng.integers(1, 513, size=int(rng.integers(1, 4))))
+                   for _ in range(nin))
+    acc = tuple(sorted({t: m for t, m in acc}.items()))
+    return Op(idioms, inputs, acc, name)
+
+
+def _linear_init(rng, fan_in, fan_out):
+    """He-uniform W ~ U(-sqrt(6/in), sqrt(6/in)) (keeps activations alive through the LeakyReLU
+    stack so the random pilot's routing depends on the sample), b ~ U(-0.1, 0.1)."""
+    bound = np.sqrt(6.0 / fan_in)
+    Wt = rng.uniform(-bound, bound, size=(fan_out, fan_in)).astype(np.float32)
+    b = rng.uniform(-0.1, 0.1, size=(fan_out,)).astype(np.float32)
+    return Wt, b
+
+
+def feature_width(S_max, D_s, h):
+    """F = [x_t(3) | x_s(D_s) | x_a(10*S_max) | x_h(10*h)] zero-padded to a multiple of 16."""
+    n = 3 + D_s + 10 * S_max + 10 * h
+    return (n + 15) // 16 * 16
+
+
+def make_pilot(rng, kind, S_max, D_s, h, K_max, n_branch_logits, planted_counts=None,
+               count_scale=16.0, xs_mean=None):
+    """Build a pilot with seeded-random weights.
+
+    kind "T32": identity feature stage, MLP F->32->32, output 32->O (north_star config 1).
+    kind "P512": three input-feature layers (x_s->32, [x_a;x_h]->32, x_t->32), MLP
+                 96->512->512->512->64, output 64->O (width P:L263).
+    kind "H<w>": like P512 with hidden width w (width sweep).
+
+    planted_counts: if given, the block-head rows of the output layer get zero weights and
+    a bias that encodes these per-slot operator counts in the block-head unit (count/16,
+    DESIGN.md reading R4) — a stand-in for a trained pilot's partition labels
+    (P:L164-L170), so the synthetic predictions have the workload's group structure.
+    The branch-head rows keep random weights: routing depends on the sample.
+    """
+    F = feature_width(S_max, D_s, h)
+    n_out = 10 * K_max + n_branch_logits
+    O = (n_out + 7) // 8 * 8
+    wts = {}
+    if kind == "T32":
+        feature = []
+        mlp = [(F, 32), (32, 32)]
+        out_in = 32
+    else:
+        width = 512 if kind == "P512" else int(kind[1:])
+        xs_off, xs_len = 3, D_s
+        xa_off, xa_len = 3 + D_s, 10 * S_max + 10 * h
+        feature = [(xs_off, xs_len, 32), (xa_off, xa_len, 32), (0, 3, 32)]
+        mlp = [(96, width), (width, width), (width, width), (width, 64)]
+        out_in = 64
+        for i, (off, ln, o) in enumerate(feature):
+            wts[f"feat{i}.W"], wts[f"feat{i}.b"] = _linear_init(rng, ln, o)
+    for k in range(3):
+        for l, (i, o) in enumerate(mlp):
+            wts[f"mlp{k}.{l}.W"], wts[f"mlp{k}.{l}.b"] = _linear_init(rng, i, o)
+    # sample sensitivity: the per-arch constant inputs (x_t, x_a) get a gain of 1/16 so that
+    # the random branch head routes differently per sample instead of being dominated by them
+    if kind == "T32":
+        for k in range(3):
+            wts[f"mlp{k}.0.W"][:, :3] *= np.float32(1 / 16)
+            wts[f"mlp{k}.0.W"][:, 3 + D_s:] *= np.float32(1 / 1024)
+    else:
+        wts["feat1.W"] *= np.float32(1 / 1024)
+        wts["feat2.W"] *= np.float32(1 / 16)
+    # centre the descriptor input (what a trained first layer does): b -= W . E[x_s], with
+    # E[x_s] the mean descriptor in feature units (descriptor x 2^-10, reading R3)
+    if xs_mean is not None:
+        mu = np.asarray(xs_mean, np.float64) / 1024.0
+        if kind == "T32":
+            for k in range(3):
+                Wk = wts[f"mlp{k}.0.W"]
+                wts[f"mlp{k}.0.b"] = (wts[f"mlp{k}.0.b"] - Wk[:, 3:3 + D_s].astype(np.float64) @ mu).astype(np.float32)
+        else:
+            wts["feat0.b"] = (wts["feat0.b"] - wts["feat0.W"].astype(np.float64) @ mu).astype(np.float32)
+    Wo, bo = _linear_init(rng, out_in, O)
+    if planted_counts is not None:
+        Wo[: 10 * K_max, :] = 0.0
+        bo[: 10 * K_max] = 0.0
+        for k, c in enumerate(planted_counts):
+            bo[10 * k] = np.float32(c / count_scale)
+    Wo[n_out:, :] = 0.0
+    bo[n_out:] = 0.0
+    wts["out.W"], wts["out.b"] = Wo, bo
+    return PilotSpec(F=F, O=O, feature=feature, mlp=mlp, out_in=out_in, weights=wts)
+
+
+def _host_layout(tensors_bytes, align):
+    """Host homes laid out in table order (the generator lists tensors group-major)."""
+    offs, cur = [], 0
+    for nb in tensors_bytes:
+        offs.append(cur)
+        cur += (nb + align - 1) // align * align
+    return offs, cur
+
+
+def n_branch_logits(program):
+    """Count of free (untied) branch-head logits: structure bookkeeping of the input."""
+    n = 0
+    for it in _walk(program):
+        if isinstance(it, If) and it.tie < 0:
+            n += len(it.branches)
+        elif isinstance(it, Loop) and it.tie < 0:
+            n += it.hi - it.lo + 1
+    return n
+
+
+def _walk(program):
+    for it in program:
+        yield it
+        if isinstance(it, If):
+            for br in it.branches:
+                yield from _walk(br)
+        elif isinstance(it, Loop):
+            yield from _walk(it.body)
+
+
+# ----------------------------------------------------------------------------
+# M0 tiny (BASELINE configs[0])
+# ----------------------------------------------------------------------------
+
+def make_tiny(seed=0, n_samples=16, planted=True, branch_head=True):
+    """8 groups, 64 tensors, T32 pilot (hidden 32), 1 GiB budget.
+
+    Program: LSTM type; If A (2 branches), If B (2 branches), Loop C (1..3 x 4-op body)
+    -> 12 paths of 35..49 rows. 64 tensors of U{1..31} MiB: 38 weights (R) and 26
+    activations (written once, then read; transient). Each op touches 1-2 tensors.
+    Feasibility by construction: a group has <= 7 rows (8 planted slots of 6 rows, the
+    last absorbs <= 1 extra row) x 2 accesses x 31 MiB = 434 MiB < H = 512 MiB.
+    """
+    rng = np.random.default_rng(seed)
+    T = 64
+    n_w = 38
+    sizes = [int(rng.integers(1, 32)) * MiB for _ in range(T)]
+    weights = list(range(n_w))
+    acts = list(range(n_w, T))
+    act_cursor = [0]
+
+    def op():
+        k = int(rng.integers(1, 3))
+        acc = []
+        for _ in range(k):
+            if rng.random() < 0.6 or not acts:
+                acc.append((int(rng.choice(weights)), R))
+            else:
+                a = acts[int(rng.integers(0, len(acts)))]
+                acc.append((a, W if rng.random() < 0.5 else R))
+        return _op(rng, acc)
+
+    def block(n):
+        return [op() for _ in range(n)]
+
+    program = (block(8)
+               + [If([block(4), block(6)])]
+               + block(6)
+               + [If([block(3), block(5)])]
+               + block(4)
+               + [Loop(block(4), 1, 3)]
+               + block(2))
+    offs, _ = _host_layout(sizes, 256)
+    tensors = [Tensor(sizes[t], offs[t], t >= n_w, f"t{t}") for t in range(T)]
+    S_max, D_s, h, K_max = 4, 8, 0, 8
+    nbl = n_branch_logits(program) if branch_head else 0
+    samples = rng.integers(1, 4096, size=(n_samples, D_s)).astype(np.int64)
+    pilot = make_pilot(rng, "T32", S_max, D_s, h, K_max, nbl,
+                       planted_counts=[6] * 8 if planted else None, xs_mean=[2048.0] * D_s)
+    return Workload("tiny", LSTM, program, tensors, S_max, D_s, h, K_max,
+                    budget=GiB, align=256, policy=1, pilot=pilot, samples=samples,
+                    hist_ids=np.zeros(0, np.int32), seed=seed,
+                    notes={"branch_head": branch_head})
+
+
+# ----------------------------------------------------------------------------
+# M1 switch-MoE (BASELINE configs[1])
+# ----------------------------------------------------------------------------
+
+def make_moe(seed=0, n_samples=16, layers=24, experts=16, layers_per_group=3,
+             pilot_kind="P512", budget=3 * GiB, expert_mib=32, act_mib=16):
+    """Switch-MoE top-1 (sample-level) routing, 16 experts, expert tensors offloaded.
+
+    Per layer, forward: 4 static attention ops (dense weights resident, not managed),
+    then If(16 experts): expert e = 2 ops reading W_in[l,e], W_out[l,e] (32 MiB each,
+    d_model 2048 x d_ff 8192 bf16) and writing act[l] (16 MiB, transient).
+    Backward (reverse layer order): If(tie = forward site of l): 3 ops reading W_out, W_in,
+    act[l] and writing grad_out[l,e], grad_in[l,e] (32 MiB each; live -> written back
+    for a host-side optimizer), then 4 static attention-backward ops.
+    Groups: 3 layers per group -> 8 forward (21 rows) + 8 backward (24 rows) = K_max 16.
+    Host pool: experts 24 GiB + gradients 24 GiB; budget 3 GiB -> 8x oversubscription
+    of the expert pool.
+    """
+    rng = np.random.default_rng(seed)
+    L, E = layers, experts
+    tensors = []
+
+    def add(nb, transient, name):
+        tensors.append([nb, transient, name])
+        return len(tensors) - 1
+
+    # host layout is table order: expert weights layer-major with W_in/W_out adjacent
+    w_in, w_out, g_in, g_out, act = {}, {}, {}, {}, {}
+    for l in range(L):
+        for e in range(E):
+            w_in[l, e] = add(expert_mib * MiB, False, f"w_in[{l},{e}]")
+            w_out[l, e] = add(expert_mib * MiB, False, f"w_out[{l},{e}]")
+    for l in range(L):
+        for e in range(E):
+            g_in[l, e] = add(expert_mib * MiB, False, f"g_in[{l},{e}]")
+            g_out[l, e] = add(expert_mib * MiB, False, f"g_out[{l},{e}]")
+    for l in range(L):
+        act[l] = add(act_mib * MiB, True, f"act[{l}]")
+
+    d_model, d_ff, seq = 2048, 8192, 2048
+
+    def attn_ops(bwd=False):
+        # layernorm, qkv projection, attention, output projection (shapes of the layer)
+        shp = [((seq, d_model),), ((seq, d_model), (d_model, 3 * d_model)),
+               ((seq, d_model), (seq, d_model), (seq, d_model)), ((seq, d_model), (d_model, d_model))]
+        idi = [(0, 0, 0, 2, 3, 0), (1, 0, 0, 1, 1, 0), (2, 1, 0, 2, 2, 0), (1, 0, 0, 1, 1, 0)]
+        if bwd:
+            idi = [tuple(x + (1 if i in (0, 4) else 0) for i, x in enumerate(v)) for v in idi][::-1]
+            shp = shp[::-1]
+        return [Op(idi[i], shp[i], (), "attn_bwd" if bwd else "attn") for i in range(4)]
+
+    program, fwd_site = [], {}
+    site = 0
+    for l in range(L):
+        program += attn_ops()
+        branches = []
+        for e in range(E):
+            branches.append([
+                Op((0, 0, 0, 1, 1, 0), ((seq, d_model), (d_model, d_ff)), ((w_in[l, e], R),), "ffn_in"),
+                Op((0, 0, 0, 1, 1, 0), ((seq, d_ff), (d_ff, d_model)),
+                   tuple(sorted([(w_out[l, e], R), (act[l], W)])), "ffn_out"),
+            ])
+        program.append(If(branches))
+        fwd_site[l] = site
+        site += 1
+    for l in reversed(range(L)):
+        branches = []
+        for e in range(E):
+            branches.append([
+                Op((1, 0, 0, 1, 1, 0), ((seq, d_model), (d_ff, d_model)),
+                   tuple(sorted([(w_out[l, e], R), (g_out[l, e], W)])), "ffn_out_bwd"),
+                Op((1, 0, 0, 1, 1, 0), ((seq, d_ff), (d_model, d_ff)),
+                   tuple(sorted([(w_in[l, e], R), (g_in[l, e], W)])), "ffn_in_bwd"),
+                Op((0, 0, 0, 1, 2, 0), ((seq, d_model),), ((act[l], R),), "act_bwd"),
+            ])
+        program.append(If(branches, tie=fwd_site[l]))
+        site += 1
+        program += attn_ops(bwd=True)
+
+    sizes = [t[0] for t in tensors]
+    offs, _ = _host_layout(sizes, 256)
+    tens = [Tensor(t[0], offs[i], t[1], t[2]) for i, t in enumerate(tensors)]
+    S_max, D_s, h = 16, 16, 2
+    K_max = 2 * L // layers_per_group
+    fwd_rows = layers_per_group * (4 + 1 + 2)
+    bwd_rows = layers_per_group * (1 + 3 + 4)
+    planted = [fwd_rows] * (L // layers_per_group) + [bwd_rows] * (L // layers_per_group)
+    samples = np.stack([
+        rng.integers(128, 2049, size=n_samples),         # sequence length
+        rng.integers(1, 65, size=n_samples),             # sentences / documents
+    ] + [rng.integers(1, 4096, size=n_samples) for _ in range(D_s - 2)], axis=1).astype(np.int64)
+    pilot = make_pilot(rng, pilot_kind, S_max, D_s, h, K_max, n_branch_logits(program),
+                       planted_counts=planted, xs_mean=[1088.0, 32.5] + [2048.0] * (D_s - 2))
+    return Workload("moe", TRANSFORMER, program, tens, S_max, D_s, h, K_max,
+                    budget=budget, align=256, policy=1, pilot=pilot, samples=samples,
+                    hist_ids=np.array([-2, -1], np.int32), seed=seed,
+                    notes={"experts": E, "layers": L, "expert_bytes": 2 * expert_mib * MiB})
+
+
+# ----------------------------------------------------------------------------
+# M2 AlphaFold-Evoformer-shaped (BASELINE configs[2])
+# ----------------------------------------------------------------------------
+
+def make_af(seed=0, n_samples=16, blocks=48, max_recycle=4, budget=2 * GiB,
+            pilot_kind="P512", rows_per_block=16, acts_per_block=10, act_mib=16,
+            weight_mib=11):
+    """Evoformer-shaped trace: Loop(recycle 1..4) over 48 forward blocks, then 48 backward
+    blocks (with the per-block optimizer update fused in), then one final group.
+
+    MSA N_seq 128 x N_res 256, c_m 256, c_z 128, bf16: 10 saved activations of 16 MiB per
+    block (written in every recycle; only the last recycle's survive to the backward pass),
+    running MSA/pair state (RW), per-block weights 11 MiB + Adam state 22 MiB (RW in backward),
+    per-block weight gradient 11 MiB. Every group is 16 rows (the loop-test row rides with
+    the first block of an iteration), so planted counts [17, 16 x 47] x 5 + [16] decode to
+    one group per block per direction for every recycle count (reading R4).
+    """
+    rng = np.random.default_rng(seed)
+    tensors = []
+
+    def add(nb, transient, name):
+        tensors.append([nb, transient, name])
+        return len(tensors) - 1
+
+    n_seq, n_res, c_m, c_z = 128, 256, 256, 128
+    msa_state = add(n_seq * n_res * c_m * 2, False, "msa_state")
+    pair_state = add(n_res * n_res * c_z * 2, False, "pair_state")
+    msa_grad = add(n_seq * n_res * c_m * 2, True, "msa_grad")
+    pair_grad = add(n_res * n_res * c_z * 2, True, "pair_grad")
+    wts, adam, wgrad, acts = {}, {}, {}, {}
+    for b in range(blocks):
+        wts[b] = add(weight_mib * MiB, False, f"w[{b}]")
+        adam[b] = add(2 * weight_mib * MiB, False, f"adam[{b}]")
+    for b in range(blocks):
+        for a in range(acts_per_block):
+            acts[b, a] = add(act_mib * MiB, True, f"act[{b},{a}]")
+    for b in range(blocks):
+        wgrad[b] = add(weight_mib * MiB, True, f"wgrad[{b}]")
+    final_t = add(1 * MiB, False, "loss_scale")
+
+    msa_shape = (n_seq, n_res, c_m)
+    pair_shape = (n_res, n_res, c_z)
+    n = rows_per_block
+
+    def fwd_block(b):
+        ops = []
+        for i in range(n):
+            acc = []
+            if i == 0:
+                acc += [(wts[b], R), (msa_state, RW)]
+            if i == 1:
+                acc += [(pair_state, RW)]
+            if 2 <= i < 2 + acts_per_block:
+                acc += [(acts[b, i - 2], W)]
+            idi = (int(i % 3 == 0), int(i % 5 == 1), 0, 1 + i % 2, 2, int(i % 4 == 3))
+            ops.append(Op(idi, (msa_shape, pair_shape) if i % 2 else (msa_shape,), tuple(sorted(acc)), f"evo{b}.{i}"))
+        return ops
+
+    def bwd_block(b):
+        ops = []
+        for i in range(n):
+            acc = []
+            if i < acts_per_block:
+                acc += [(acts[b, acts_per_block - 1 - i], R)]
+            if i == 0:
+                acc += [(msa_grad, RW), (pair_grad, RW)]
+            if i == acts_per_block:
+                acc += [(wts[b], R), (wgrad[b], W)]
+            if i == n - 1:
+                acc += [(wts[b], RW), (adam[b], RW), (wgrad[b], R)]
+            idi = (int(i % 3 == 1), 0, int(i % 5 == 0), 2, 2 + i % 2, 0)
+            ops.append(Op(idi, (pair_shape, msa_shape) if i % 2 else (pair_shape,), tuple(sorted(acc)), f"evo_bwd{b}.{i}"))
+        return ops
+
+    body = []
+    for b in range(blocks):
+        body += fwd_block(b)
+    program = [Loop(body, 1, max_recycle)]
+    for b in reversed(range(blocks)):
+        program += bwd_block(b)
+    program += [Op((0, 0, 0, 1, 1, 0), ((1,),), ((final_t, RW),), "final")] + \
+               [Op((0, 0, 0, 0, 1, 0), ((1,),), (), "final")] * (n - 1)
+
+    sizes = [t[0] for t in tensors]
+    offs, _ = _host_layout(sizes, 256)
+    tens = [Tensor(t[0], offs[i], t[1], t[2]) for i, t in enumerate(tensors)]
+    S_max, D_s, h = 16, 16, 2
+    K_max = 256
+    planted = ([n + 1] + [n] * (blocks - 1)) * (max_recycle + 1) + [n]
+    samples = np.stack([
+        np.full(n_samples, n_seq), np.full(n_samples, n_res),
+        rng.integers(1, 5, size=n_samples),             # sampled recycle count descriptor
+    ] + [rng.integers(1, 4096, size=n_samples) for _ in range(D_s - 3)], axis=1).astype(np.int64)
+    pilot = make_pilot(rng, pilot_kind, S_max, D_s, h, K_max, n_branch_logits(program),
+                       planted_counts=planted, xs_mean=[n_seq, n_res, 2.5] + [2048.0] * (D_s - 3))
+    return Workload("af", TRANSFORMER, program, tens, S_max, D_s, h, K_max,
+                    budget=budget, align=256, policy=1, pilot=pilot, samples=samples,
+                    hist_ids=np.array([-2, -1], np.int32), seed=seed,
+                    notes={"blocks": blocks, "max_recycle": max_recycle})
+
+
+CONFIGS = {"tiny": make_tiny, "moe": make_moe, "af": make_af}
+
+
+def make(name, seed=0, **kw):
+    return CONFIGS[name](seed=seed, **kw)
+
+
+# ----------------------------------------------------------------------------
+# counter-based content generator (migration byte checks; both sides call it)
+# ----------------------------------------------------------------------------
+
+def content_words_np(tid, version, n_words, start=0):
+    """uint32 words of tensor `tid` at `version`: a 32-bit integer hash of the word index.
+
+    Pure integer mixing (xorshift-multiply), identical to content_words_torch().
+    """
+    i = np.arange(start, start + n_words, dtype=np.int64)
+    x = (i * 0x9E3779B1 + (tid * 0x85EBCA77) + (version * 0xC2B2AE3D) + 0x27D4EB2F) & 0xFFFFFFFF
+    x ^= x >> 15
+    x = (x * 0x2C1B3C6D) & 0xFFFFFFFF
+    x ^= x >> 12
+    x = (x * 0x297A2D39) & 0xFFFFFFFF
+    x ^= x >> 15
+    return x.astype(np.uint32)
+
+
+def content_words_torch(tid, version, n_words, device, start=0):
+    import torch
+    i = torch.arange(start, start + n_words, dtype=torch.int64, device=device)
+    M = 0xFFFFFFFF
+    x = (i * 0x9E3779B1 + ((tid * 0x85EBCA77) & M) + ((version * 0xC2B2AE3D) & M) + 0x27D4EB2F) & M
+    x ^= x >> 15
+    x = (x * 0x2C1B3C6D) & M
+    x ^= x >> 12
+    x = (x * 0x297A2D39) & M
+    x ^= x >> 15
+    return x.to(torch.int32)  # reinterpreted as uint32 bits via two's complement wrap

@@ -1,0 +1,256 @@
+/*
+ * dyo.h — C ABI of the B200-native DyNN-Offload hot path (libdyo.so).
+ *
+ * Paper: Ren et al., "Enabling Large Dynamic Neural Network Training with Learning-based
+ * Memory Management", HPCA 2024 (PAPER.md; "P:Lnnn" = line nnn). Readings R1-R12 of the
+ * paper's silent/garbled points are in DESIGN.md §2 and are referenced below.
+ *
+ * Per training step the caller runs
+ *     dyo_pilot_predict  (encode + pilot MLP + decode; on device)
+ *     dyo_plan           (double-buffered evict/prefetch plan; on device, then
+ *                         one synchronisation that hands the DMA sizes to the host)
+ *     dyo_migrate(j)     for j = 0..K-1 (evict -> compact/carry -> fetch)
+ *
+ * Conventions (all entry points):
+ *   - return a dyo_status (0 = OK, negative = error); nothing throws or aborts;
+ *     dyo_strerror() names a status, dyo_last_error() describes the last failure of a ctx.
+ *   - "device" pointers are CUDA device (or managed) memory; "host" pointers are CPU memory;
+ *     arguments documented "host or device" are detected with cudaPointerGetAttributes and
+ *     host data is staged to the device on the call's stream (the end-to-end path).
+ *   - streams/events are cudaStream_t / cudaEvent_t passed as void*; NULL stream = legacy
+ *     default stream. Calls are stream-ordered and asynchronous unless stated otherwise.
+ *   - a dyo_ctx is bound to one GPU and is not thread-safe (one manager per GPU, §8(e)).
+ *   - integer limits (validated at load, DYO_E_INVAL otherwise): tensors < 2^20, aligned
+ *     tensor size / ALIGN < 2^28, groups per dyo_plan < 2^16, operators < 2^24.
+ */
+#ifndef DYO_H
+#define DYO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  DYO_OK = 0,
+  DYO_E_INVAL = -1,       /* bad argument / malformed arch or pilot */
+  DYO_E_NOMEM = -2,       /* device or pinned host allocation failed */
+  DYO_E_BUDGET = -3,      /* some W_j needs more than half the budget (R7) */
+  DYO_E_CUDA = -4,        /* a CUDA runtime call failed (dyo_last_error has the text) */
+  DYO_E_STATE = -5,       /* calls out of order (e.g. migrate before plan, j out of order) */
+  DYO_E_CAPACITY = -6,    /* a fixed-capacity buffer overflowed (needed size in last_error) */
+  DYO_E_UNSUPPORTED = -7  /* program shape not supported by this decode mode */
+} dyo_status;
+
+typedef struct dyo_ctx dyo_ctx;
+
+/* Runtime configuration (host struct, copied by dyo_create). */
+typedef struct {
+  int64_t budget;         /* B: device arena bytes, split in two equal halves (R7) */
+  int32_t align;          /* ALIGN in bytes (power of two >= 16; 256 in all configs) */
+  int32_t policy;         /* 0 = PAPER (evict every unused tensor), 1 = RETAIN (R10) */
+  int32_t max_batch;      /* max predictions per dyo_pilot_predict call (>= 1) */
+  int32_t max_groups;     /* max groups per dyo_plan (sum over its predictions), <= 65535 */
+  int32_t max_entries;    /* capacity of tensor-set entries per dyo_plan (0 = auto) */
+  int32_t max_records;    /* capacity of plan records per dyo_plan (0 = auto) */
+  int64_t staging_bytes;  /* device staging for pack/unpack/compaction (outside B; 0 = 64 MiB) */
+  int64_t dma_min_bytes;  /* host runs >= this move by DMA, smaller by zero-copy kernel (0 = 2 MiB) */
+  int32_t flags;          /* DYO_F_* */
+} dyo_config;
+
+#define DYO_F_NO_ZEROCOPY 1   /* move every run by DMA (measurement switch) */
+#define DYO_F_NO_PACK 2       /* never pack scattered writebacks into one DMA */
+#define DYO_F_NO_HOST_POOL 4  /* plan-only ctx: no pinned host pool (dyo_migrate -> DYO_E_STATE) */
+#define DYO_F_TIMING 8        /* record CUDA events around every internal launch (dyo_get_timings) */
+
+/* Static architecture: the DyNN program in preorder, its operators and the
+ * tensor table. All arrays are HOST memory; dyo_load_arch copies what it needs. */
+typedef struct {
+  int32_t nn_type;        /* 0 CNN, 1 LSTM, 2 transformer: selects the MLP */
+  int32_t S_max;          /* AFM segments fed to the pilot (R3) */
+  int32_t D_s;            /* input-shape descriptors per sample (R3) */
+  int32_t h;              /* history groups per sample (R3) */
+  int32_t K_max;          /* block-head slots (R4) */
+  int32_t branch_head;    /* 1: logits carry a branch head (R4); 0: paper traversal decode */
+  /* program nodes in preorder; node kinds: 0 OP, 1 IF, 2 LOOP, 3 BRANCH (start of an If arm).
+   * IF: a = number of branches, followed by that many BRANCH nodes each followed by its body;
+   * LOOP: a = lo, b = hi trip count, followed by its body; OP: a = operator index (operators
+   * are numbered in preorder). span = number of descendant nodes. tie = index (in preorder
+   * among IF/LOOP nodes) of the site whose choice this site replays, or -1 (R6). */
+  int32_t n_nodes;
+  const int32_t* node_kind;
+  const int32_t* node_a;
+  const int32_t* node_b;
+  const int32_t* node_span;
+  const int32_t* node_tie;
+  /* operators: six idiom counts (order of P:L135) and input shapes (CSR: op ->
+   * inputs -> dims); signature = idioms ++ [sum of shape[k] over inputs, k < 3] (Fig. 3, R1) */
+  int32_t n_ops;
+  const int32_t* op_idioms;     /* n_ops x 6 */
+  const int32_t* op_in_ptr;     /* n_ops + 1 */
+  const int32_t* in_dim_ptr;    /* n_inputs + 1 */
+  const int64_t* in_dims;
+  const int32_t* op_acc_ptr;    /* n_ops + 1: tensor accesses of each operator */
+  const int32_t* acc_tensor;    /* ascending tensor id within an operator, unique */
+  const int32_t* acc_mode;      /* 1 read, 2 write (full overwrite), 3 read-write */
+  /* tensor table */
+  int32_t n_tensors;
+  const int64_t* t_bytes;       /* > 0 */
+  const int64_t* t_host_off;    /* home offset in the ctx's pinned host pool, ALIGN-aligned */
+  const int32_t* t_flags;       /* bit 0: transient (contents end with the step, R9) */
+} dyo_arch;
+
+/* Pilot weights (host fp32, row-major W[out][in]); topology R5. n_feature = 0 means an
+ * identity feature stage (the MLP reads the F features); otherwise feature layer i maps
+ * features [feat_off[i], feat_off[i]+feat_len[i]) to feat_out[i] outputs, concatenated.
+ * The three MLPs share layer dims; mlp_W[k*n_mlp + l] is layer l of MLP k. */
+typedef struct {
+  int32_t F, O;
+  int32_t n_feature;
+  const int32_t* feat_off;
+  const int32_t* feat_len;
+  const int32_t* feat_out;
+  const float* const* feat_W;
+  const float* const* feat_b;
+  int32_t n_mlp;
+  const int32_t* mlp_in;
+  const int32_t* mlp_out;
+  const float* const* mlp_W;
+  const float* const* mlp_b;
+  int32_t out_in;
+  const float* out_W;           /* O x out_in */
+  const float* out_b;           /* O */
+  float slope;                  /* LeakyReLU negative slope (0.01, R5) */
+} dyo_pilot_desc;
+
+/* One batch of samples. desc: B x D_s int64 shape descriptors; hist_ids: B x h int32 history
+ * group ids (>= 0 index the history table, < 0 count from its end, R3) or NULL (no history).
+ * Either pointer may be host or device memory. */
+typedef struct {
+  const int64_t* desc;
+  const int32_t* hist_ids;
+} dyo_sample;
+
+/* Host-visible summary of one transition of the current plan (valid after dyo_plan). */
+typedef struct {
+  int32_t half;                 /* m = (G + j) mod 2 */
+  int32_t n_entries;            /* |W_j| */
+  int32_t n_evict, n_move, n_carry, n_alloc, n_fetch;
+  int64_t need;                 /* aligned bytes of W_j */
+  int64_t h2d, d2h, d2d;        /* algorithmic bytes (FETCH; written-back EVICT; MOVE + CARRY) */
+} dyo_transition_info;
+
+/* Plan records as stored by libdyo (little-endian int64 fields, absolute device offsets into
+ * the arena, host offsets into the host pool). */
+typedef struct { int64_t t, src, host_off, bytes, writeback; } dyo_evict_rec;
+typedef struct { int64_t t, src, dst, bytes; } dyo_move_rec;
+typedef struct { int64_t t, src, dst, bytes, late; } dyo_carry_rec;
+typedef struct { int64_t t, dst, bytes; } dyo_alloc_rec;
+typedef struct { int64_t t, host_off, dst, bytes; } dyo_fetch_rec;
+typedef struct { int64_t t, mode, needs_fetch, dst; } dyo_entry_rec;  /* W_j entry + placement */
+
+const char* dyo_strerror(dyo_status s);
+const char* dyo_last_error(const dyo_ctx* ctx);
+int32_t dyo_version(void);
+
+/* Create a manager on `device`: allocates the device arena (cfg->budget), staging, status
+ * words. Ownership: ctx owns every buffer it allocates; free with dyo_destroy. */
+dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** out);
+dyo_status dyo_destroy(dyo_ctx* ctx);
+
+/* Load the static architecture (copies it; builds the AFM segment table (R3), operator
+ * signatures, site table and tensor table on the device; allocates the pinned, mapped host
+ * pool sized to max(host_off + bytes)). Resets residency: all tensors on the host. */
+dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* arch);
+
+/* Host-only check of an arch (no GPU needed; used by the CPU test suite): runs the same parse
+ * as dyo_load_arch and returns its summary, the S_max x 10 AFM segment table (R3) and the
+ * n_ops x 9 operator signatures (R1). seg_table / op_sig may be NULL; err (errlen bytes) gets
+ * the failure text. */
+typedef struct {
+  int32_t n_sites, n_branch_logits, n_pieces, F;
+  int64_t L_max, host_pool_bytes;
+} dyo_arch_summary;
+dyo_status dyo_arch_check(const dyo_arch* arch, int32_t align, dyo_arch_summary* out, int32_t* seg_table,
+                          int32_t* op_sig, char* err, int32_t errlen);
+
+/* Load pilot weights (copied to the device, rows padded to 16 bytes). F and O must match the
+ * arch: F = pad16(3 + D_s + 10*S_max + 10*h); O >= 10*K_max + branch logits. */
+dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w);
+
+/* The ctx-owned pinned host pool holding every tensor's home ("initially allocates all
+ * tensors on CPU memory"); the caller fills initial contents. Valid until dyo_destroy or the
+ * next dyo_load_arch. */
+dyo_status dyo_host_pool(dyo_ctx* ctx, void** host_base, int64_t* bytes);
+/* Device arena base (2 halves of H bytes each) and H. */
+dyo_status dyo_arena(dyo_ctx* ctx, void** dev_base, int64_t* half_bytes);
+
+/* A1: feature vectors of B samples (R3) into feat (device, B x F fp32). Uses the history
+ * table of the previous dyo_pilot_predict. */
+dyo_status dyo_encode_features(dyo_ctx* ctx, const dyo_sample* s, int32_t B, float* feat,
+                               void* stream);
+
+/* A2 + A3: pilot forward for B samples (feat = NULL: fused encode from s; else device B x F
+ * features) and decode (R4) into ctx-owned device storage; logits (device B x O fp32) may be
+ * NULL. Asynchronous; decode errors surface at dyo_plan. After the call the history table is
+ * the executed block vectors of these predictions (in sample order). */
+dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* s, int32_t B,
+                             float* logits, void* stream);
+
+/* Copy prediction b of the last dyo_pilot_predict to host arrays (synchronises `stream`).
+ * K (groups), blocks (K_max x 10 int32, first K rows valid), choices (n_sites int32),
+ * group_rows (2*K_max int32 [start, end) pairs). Any output pointer may be NULL. */
+dyo_status dyo_prediction_get(dyo_ctx* ctx, int32_t b, int32_t* K, int32_t* blocks,
+                              int32_t* choices, int32_t* group_rows, void* stream);
+/* Tensor-set entries of group g of prediction b (host out, capacity cap entries of 3 int32:
+ * tensor, mode, needs_fetch); *n receives the count (DYO_E_CAPACITY if cap < n). */
+dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* out, int32_t cap,
+                             int32_t* n, void* stream);
+
+/* A4: plan every transition of the predictions [b0, b0 + n) of the last predict, concatenated
+ * in sample order (n = -1: all). Runs the planner kernel on `stream`, then synchronises once
+ * and copies the plan lists to pinned host memory (the DMA issue needs host-visible sizes).
+ * On DYO_E_BUDGET / DYO_E_CAPACITY the residency state is unchanged. *K_out = transitions. */
+dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* stream);
+
+/* Host copies of the current plan (valid until the next dyo_plan). */
+dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info);
+/* list: 0 evict, 1 move, 2 carry, 3 alloc, 4 fetch, 5 entries (with placement); returns a
+ * pointer to the transition's records (host memory owned by the ctx) and their count. */
+dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** recs,
+                            int32_t* n);
+
+/* A5: execute transition j (j = 0, 1, ... in order; DYO_E_STATE otherwise) on copy_stream:
+ * wait ev_prev_started (block j-1 started => block j-2, the last user of half m, finished;
+ * may be NULL), EVICT writebacks (D2H), MOVE (compaction through staging), CARRY (D2D) and
+ * FETCH (H2D); late CARRYs wait ev_prev_done (block j-1 finished; may be NULL); then record
+ * ev_ready (may be NULL), which block j must wait on. */
+dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev_started,
+                       void* ev_prev_done, void* ev_ready);
+
+/* Device address of tensor t after the last planned transition that placed it (NULL if it is
+ * on the host). Valid until the next dyo_migrate that moves it. */
+dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr);
+
+/* Per-ctx counters of the last dyo_plan / dyo_migrate calls (bytes by mechanism, launches). */
+typedef struct {
+  int64_t h2d_dma, h2d_zc, d2h_dma, d2h_zc, d2h_packed, d2d;
+  int64_t n_dma, n_kernels;
+} dyo_counters;
+dyo_status dyo_get_counters(dyo_ctx* ctx, dyo_counters* c, int32_t reset);
+
+/* With DYO_F_TIMING: device time (CUDA events on the launching stream) summed over the launches
+ * of one kind since the last reset: 0 pilot kernel (K1), 1 decode kernels, 2 planner kernel (K2),
+ * 3 device copy kernel (pack / unpack / carry / compaction), 4 zero-copy kernel (K5),
+ * 5 DMA H2D, 6 DMA D2H. bytes = algorithmic bytes moved by those launches. Synchronises on
+ * the recorded events. */
+#define DYO_T_KINDS 7
+dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* launches, int64_t* bytes,
+                           int32_t reset);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DYO_H */

@@ -1,0 +1,1088 @@
+// libdyo C ABI: context, loaders, the four hot-path calls and the migration engine.
+// See include/dyo.h for the contract and DESIGN.md for the readings R1-R12.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <array>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "dyo_internal.h"
+
+using namespace dyo;
+
+struct dyo_ctx {
+  dyo_config cfg{};
+  int device = 0;
+  std::string err;
+  bool arch_ok = false, pilot_ok = false;
+  // host copy of the arch
+  int T = 0, n_ops = 0, n_sites = 0, K_max = 0, F = 0, O_min = 0, n_branch_logits = 0;
+  std::vector<int64_t> t_bytes, t_abytes, t_host;
+  std::vector<int32_t> t_flags;
+  int64_t H = 0;
+  ArchDev ad{};
+  std::vector<void*> arch_dev;     // device buffers of the arch / prediction / plan
+  PilotDev pdv{};
+  std::vector<void*> pilot_dev;
+  // memory
+  char* arena = nullptr;
+  char* staging = nullptr;
+  int64_t staging_bytes = 0;
+  char* host_pool = nullptr;
+  int64_t host_bytes = 0;
+  // prediction
+  PredDev pd{};
+  float* logits_scratch = nullptr;
+  int64_t* desc_dev = nullptr;
+  int32_t* hist_dev = nullptr;
+  int32_t* hist_tab[2] = {nullptr, nullptr};
+  int32_t* hist_len[2] = {nullptr, nullptr};
+  int hist_cur = 0;
+  int last_B = 0;
+  // plan
+  int max_groups = 0;
+  PlanState state[2]{};
+  int committed = 0;
+  PlanScratch sc{};
+  PlanOut out{};                   // record arrays + headers in pinned mapped host memory
+  int32_t* h_status = nullptr;     // pinned mapped
+  int32_t* h_counts = nullptr;
+  int8_t* h_loc = nullptr;         // pinned mirrors of the committed residency
+  int64_t* h_off = nullptr;
+  int plan_K = 0, next_j = 0;
+  bool plan_valid = false;
+  // migration
+  CopySeg* h_segs = nullptr;       // pinned mapped work items for the copy kernels
+  int64_t seg_cap = 0, seg_used = 0;
+  cudaEvent_t ev_last = nullptr;
+  bool ev_pending = false;
+  dyo_counters ctr{};
+  int sm_count = 148;
+  // DYO_F_TIMING: event pairs per launch kind
+  struct Tm { int kind; cudaEvent_t a, b; int64_t bytes; };
+  std::vector<Tm> tm;
+  std::vector<cudaEvent_t> ev_pool;
+  double tm_ms[DYO_T_KINDS] = {};
+  int64_t tm_n[DYO_T_KINDS] = {}, tm_bytes[DYO_T_KINDS] = {};
+};
+
+namespace {
+
+dyo_status fail(dyo_ctx* c, dyo_status s, const char* fmt, ...) {
+  if (c) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    c->err = buf;
+  }
+  return s;
+}
+
+#define CK(call)                                                                          \
+  do {                                                                                    \
+    cudaError_t e_ = (call);                                                              \
+    if (e_ != cudaSuccess)                                                                \
+      return fail(ctx, e_ == cudaErrorMemoryAllocation ? DYO_E_NOMEM : DYO_E_CUDA,        \
+                  "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__);   \
+  } while (0)
+
+template <class T>
+dyo_status dalloc(dyo_ctx* ctx, std::vector<void*>& owner, T** p, size_t n) {
+  void* v = nullptr;
+  size_t bytes = std::max<size_t>(n * sizeof(T), 16);
+  CK(cudaMalloc(&v, bytes));
+  CK(cudaMemset(v, 0, bytes));
+  owner.push_back(v);
+  *p = static_cast<T*>(v);
+  return DYO_OK;
+}
+
+template <class T>
+dyo_status dupload(dyo_ctx* ctx, std::vector<void*>& owner, const T** p, const std::vector<T>& h) {
+  T* d = nullptr;
+  dyo_status s = dalloc(ctx, owner, &d, h.size());
+  if (s) return s;
+  if (!h.empty()) CK(cudaMemcpy(d, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice));
+  *p = d;
+  return DYO_OK;
+}
+
+void free_list(std::vector<void*>& v) {
+  for (void* p : v) cudaFree(p);
+  v.clear();
+}
+
+int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes at{};
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+void free_plan_host(dyo_ctx* c) {
+  auto fh = [](void* p) { if (p) cudaFreeHost(p); };
+  fh(c->out.hdr); fh(c->out.ent); fh(c->out.ev); fh(c->out.mv); fh(c->out.ca); fh(c->out.al);
+  fh(c->out.fe); fh(c->h_status); fh(c->h_counts); fh(c->h_loc); fh(c->h_off); fh(c->h_segs);
+  c->out = PlanOut{};
+  c->h_status = c->h_counts = nullptr;
+  c->h_loc = nullptr;
+  c->h_off = nullptr;
+  c->h_segs = nullptr;
+}
+
+// timing helpers (no-ops unless DYO_F_TIMING)
+cudaEvent_t pool_event(dyo_ctx* c) {
+  if (!c->ev_pool.empty()) { cudaEvent_t e = c->ev_pool.back(); c->ev_pool.pop_back(); return e; }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+struct TScope {
+  dyo_ctx* c; int kind; cudaStream_t s; int64_t bytes; cudaEvent_t a = nullptr;
+  TScope(dyo_ctx* c_, int k, cudaStream_t s_, int64_t b = 0) : c(c_), kind(k), s(s_), bytes(b) {
+    if (c->cfg.flags & DYO_F_TIMING) { a = pool_event(c); cudaEventRecord(a, s); }
+  }
+  ~TScope() {
+    if (a) {
+      cudaEvent_t b = pool_event(c);
+      cudaEventRecord(b, s);
+      c->tm.push_back({kind, a, b, bytes});
+    }
+  }
+};
+
+void drain_timings(dyo_ctx* c) {
+  for (auto& t : c->tm) {
+    cudaEventSynchronize(t.b);
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, t.a, t.b);
+    c->tm_ms[t.kind] += ms;
+    c->tm_n[t.kind] += 1;
+    c->tm_bytes[t.kind] += t.bytes;
+    c->ev_pool.push_back(t.a);
+    c->ev_pool.push_back(t.b);
+  }
+  c->tm.clear();
+}
+
+// Host-side parse of a dyo_arch (no CUDA): signatures (Fig. 3, R1), AFM segment table (R3),
+// sites / arms / top-level pieces (R2, R4, R6), tensor table. Shared by dyo_load_arch and
+// dyo_arch_check.
+struct ArchHost {
+  int T = 0, n_sites = 0, n_branch_logits = 0;
+  int64_t L_max = 0, pool = 0;
+  std::vector<int64_t> t_bytes, t_abytes, t_host;
+  std::vector<int32_t> t_flags, sig, acc_ptr, acc_t, acc_m;
+  std::vector<int32_t> site_kind, site_nch, site_lo, site_tie, site_logit, site_arm_ptr, arm_first, arm_n;
+  std::vector<int32_t> piece_kind, piece_a, piece_b, piece_c, seg_table;
+};
+
+dyo_status hfail(std::string& err, dyo_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  err = buf;
+  return s;
+}
+
+dyo_status parse_arch(const dyo_arch* A, int64_t AL, ArchHost& h, std::string& err) {
+  if (A->nn_type < 0 || A->nn_type > 2 || A->S_max < 0 || A->D_s < 0 || A->h < 0 || A->K_max < 1 ||
+      A->K_max > 256 || A->n_tensors < 1 || A->n_tensors >= (1 << 20) || A->n_ops < 0 ||
+      A->n_ops >= (1 << 24) || A->n_nodes < 0)
+    return hfail(err, DYO_E_INVAL, "arch: bad sizes");
+  if (!A->branch_head)
+    return hfail(err, DYO_E_UNSUPPORTED, "arch: traversal decode (no branch head) runs only in the oracle in this build");
+  const int T = A->n_tensors, n_ops = A->n_ops, N = A->n_nodes;
+  // ---- tensors ----
+  h.T = T;
+  h.t_bytes.assign(A->t_bytes, A->t_bytes + T);
+  h.t_host.assign(A->t_host_off, A->t_host_off + T);
+  h.t_flags.assign(A->t_flags, A->t_flags + T);
+  h.t_abytes.resize(T);
+  int64_t& pool = h.pool;
+  pool = 0;
+  for (int t = 0; t < T; ++t) {
+    if (h.t_bytes[t] <= 0 || h.t_host[t] < 0 || h.t_host[t] % AL)
+      return hfail(err, DYO_E_INVAL, "arch: tensor %d bytes/host_off invalid", t);
+    h.t_abytes[t] = align_up(h.t_bytes[t], AL);
+    if (h.t_abytes[t] / AL >= (1ll << 28)) return hfail(err, DYO_E_INVAL, "arch: tensor %d too large", t);
+    pool = std::max(pool, h.t_host[t] + h.t_abytes[t]);
+  }
+  if (pool / AL >= (1ll << 42)) return hfail(err, DYO_E_INVAL, "arch: host pool too large");
+  // ---- operators: signatures (Fig. 3 / R1) and accesses ----
+  auto& sig = h.sig; auto& acc_ptr = h.acc_ptr; auto& acc_t = h.acc_t; auto& acc_m = h.acc_m;
+  sig.assign((size_t)n_ops * 9, 0);
+  acc_ptr.assign(n_ops + 1, 0);
+  for (int o = 0; o < n_ops; ++o) {
+    for (int k = 0; k < 6; ++k) {
+      int64_t v = A->op_idioms[o * 6 + k];
+      sig[o * 9 + k] = (int32_t)std::min<int64_t>(std::max<int64_t>(v, 0), kSat);
+    }
+    for (int k = 0; k < 3; ++k) {
+      int64_t s = 0;
+      for (int i = A->op_in_ptr[o]; i < A->op_in_ptr[o + 1]; ++i) {
+        const int rank = A->in_dim_ptr[i + 1] - A->in_dim_ptr[i];
+        if (rank > k) s += A->in_dims[A->in_dim_ptr[i] + k];
+      }
+      sig[o * 9 + 6 + k] = (int32_t)std::min<int64_t>(std::max<int64_t>(s, 0), kSat);
+    }
+    acc_ptr[o] = (int32_t)acc_t.size();
+    int prev = -1;
+    for (int q = A->op_acc_ptr[o]; q < A->op_acc_ptr[o + 1]; ++q) {
+      const int t = A->acc_tensor[q], md = A->acc_mode[q];
+      if (t < 0 || t >= T || t <= prev || md < 1 || md > 3)
+        return hfail(err, DYO_E_INVAL, "arch: op %d accesses must be ascending unique tensor ids with mode 1..3", o);
+      prev = t;
+      acc_t.push_back(t);
+      acc_m.push_back(md);
+    }
+  }
+  acc_ptr[n_ops] = (int32_t)acc_t.size();
+  // ---- program: sites, arms, top-level pieces, AFM segments (R2, R3, R4, R6) ----
+  auto& site_kind = h.site_kind; auto& site_nch = h.site_nch; auto& site_lo = h.site_lo;
+  auto& site_tie = h.site_tie; auto& site_logit = h.site_logit; auto& site_arm_ptr = h.site_arm_ptr;
+  auto& arm_first = h.arm_first; auto& arm_n = h.arm_n;
+  std::vector<int32_t> site_node;                   // node index of each site
+  auto& piece_kind = h.piece_kind; auto& piece_a = h.piece_a; auto& piece_b = h.piece_b; auto& piece_c = h.piece_c;
+  std::vector<std::array<int64_t, 10>> segs;
+  std::array<int64_t, 10> cur{};
+  bool cur_open = false;
+  int expect_op = 0;
+  auto close_seg = [&]() { if (cur_open) segs.push_back(cur); cur = {}; cur_open = false; };
+  for (int i = 0; i < N; ++i) {
+    const int k = A->node_kind[i];
+    if (k == 0) {
+      const int o = A->node_a[i];
+      if (o != expect_op) return hfail(err, DYO_E_INVAL, "arch: operators must be numbered in preorder");
+      ++expect_op;
+      cur[0] += 1;
+      for (int q = 0; q < 9; ++q) cur[1 + q] += sig[o * 9 + q];
+      cur_open = true;
+    } else if (k == 1 || k == 2) {
+      close_seg();
+      cur[0] = 1;              // the control row starts the new segment (R3)
+      cur_open = true;
+      site_node.push_back(i);
+    } else if (k != 3) {
+      return hfail(err, DYO_E_INVAL, "arch: node kind %d", k);
+    }
+  }
+  close_seg();
+  if (expect_op != n_ops) return hfail(err, DYO_E_INVAL, "arch: %d ops in nodes, %d declared", expect_op, n_ops);
+  const int n_sites = (int)site_node.size();
+  if (n_sites > kMaxSites) return hfail(err, DYO_E_CAPACITY, "arch: too many sites");
+  int logit = 10 * A->K_max;
+  int64_t L_max = 0;
+  // walk the top level
+  auto count_ops = [&](int first_node, int span, int* first_op, bool* has_site) {
+    int n = 0;
+    *first_op = -1;
+    *has_site = false;
+    for (int q = first_node; q < first_node + span; ++q) {
+      if (A->node_kind[q] == 0) { if (*first_op < 0) *first_op = A->node_a[q]; ++n; }
+      else if (A->node_kind[q] != 3) *has_site = true;
+    }
+    if (*first_op < 0) *first_op = 0;
+    return n;
+  };
+  std::vector<int> node_site(N, -1);
+  for (int s = 0; s < n_sites; ++s) node_site[site_node[s]] = s;
+  for (int s = 0; s < n_sites; ++s) {
+    const int i = site_node[s];
+    const int k = A->node_kind[i];
+    site_kind.push_back(k);
+    const int tie = A->node_tie[i];
+    if (tie >= s) return hfail(err, DYO_E_INVAL, "arch: site %d ties to a later site", s);
+    site_tie.push_back(tie);
+    if (k == 1) {
+      site_nch.push_back(A->node_a[i]);
+      site_lo.push_back(0);
+    } else {
+      if (A->node_b[i] < A->node_a[i] || A->node_a[i] < 0) return hfail(err, DYO_E_INVAL, "arch: loop bounds");
+      site_nch.push_back(A->node_b[i] - A->node_a[i] + 1);
+      site_lo.push_back(A->node_a[i]);
+    }
+    if (tie >= 0) {
+      if (site_tie[tie] >= 0 || site_nch[tie] != site_nch[s] || site_kind[tie] != k)
+        return hfail(err, DYO_E_INVAL, "arch: site %d tie target must be a free site of the same shape", s);
+      site_logit.push_back(-1);
+    } else {
+      site_logit.push_back(logit);
+      logit += site_nch[s];
+    }
+    site_arm_ptr.push_back((int)arm_first.size());
+    if (k == 1) {
+      int q = i + 1;
+      for (int br = 0; br < A->node_a[i]; ++br) {
+        if (A->node_kind[q] != 3) return hfail(err, DYO_E_INVAL, "arch: IF node %d arm %d", i, br);
+        int fo; bool hs;
+        const int n = count_ops(q + 1, A->node_span[q], &fo, &hs);
+        arm_first.push_back(fo);
+        arm_n.push_back(n);
+        q += 1 + A->node_span[q];
+      }
+    }
+  }
+  h.n_branch_logits = logit - 10 * A->K_max;
+  for (int i = 0; i < N;) {
+    const int k = A->node_kind[i];
+    if (k == 0) {
+      const int first = A->node_a[i];
+      int n = 0;
+      while (i < N && A->node_kind[i] == 0) { ++n; ++i; }
+      piece_kind.push_back(0); piece_a.push_back(first); piece_b.push_back(n); piece_c.push_back(0);
+      L_max += n;
+    } else if (k == 1 || k == 2) {
+      const int s = node_site[i];
+      int fo; bool hs;
+      const int n = count_ops(i + 1, A->node_span[i], &fo, &hs);
+      if (hs) return hfail(err, DYO_E_UNSUPPORTED, "arch: nested control flow under site %d (device decode needs top-level sites)", s);
+      if (k == 1) {
+        int mx = 0;
+        for (int br = 0; br < site_nch[s]; ++br) mx = std::max(mx, arm_n[site_arm_ptr[s] + br]);
+        piece_kind.push_back(1); piece_a.push_back(s); piece_b.push_back(0); piece_c.push_back(0);
+        L_max += 1 + mx;
+      } else {
+        piece_kind.push_back(2); piece_a.push_back(s); piece_b.push_back(fo); piece_c.push_back(n);
+        L_max += (int64_t)(site_lo[s] + site_nch[s] - 1) * (1 + n) + 1;
+      }
+      i += 1 + A->node_span[i];
+    } else {
+      return hfail(err, DYO_E_INVAL, "arch: stray BRANCH node %d", i);
+    }
+  }
+  if ((int)piece_kind.size() > 1024) return hfail(err, DYO_E_CAPACITY, "arch: more than 1024 top-level pieces");
+  if (L_max >= (1 << 30)) return hfail(err, DYO_E_CAPACITY, "arch: path too long");
+  auto& seg_table = h.seg_table;
+  seg_table.assign((size_t)A->S_max * 10, 0);
+  for (int s = 0; s < A->S_max && s < (int)segs.size(); ++s)
+    for (int e = 0; e < 10; ++e) seg_table[s * 10 + e] = (int32_t)std::min<int64_t>(segs[s][e], kSat);
+
+  h.n_sites = n_sites;
+  h.L_max = L_max;
+  return DYO_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* dyo_strerror(dyo_status s) {
+  switch (s) {
+    case DYO_OK: return "ok";
+    case DYO_E_INVAL: return "invalid argument";
+    case DYO_E_NOMEM: return "out of memory";
+    case DYO_E_BUDGET: return "a tensor set does not fit half the budget";
+    case DYO_E_CUDA: return "CUDA error";
+    case DYO_E_STATE: return "call out of order";
+    case DYO_E_CAPACITY: return "buffer capacity exceeded";
+    case DYO_E_UNSUPPORTED: return "unsupported program shape";
+  }
+  return "unknown status";
+}
+
+const char* dyo_last_error(const dyo_ctx* ctx) { return ctx ? ctx->err.c_str() : ""; }
+
+int32_t dyo_version(void) { return 1; }
+
+dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
+  if (!cfg || !outp) return DYO_E_INVAL;
+  dyo_ctx* ctx = new dyo_ctx();
+  ctx->cfg = *cfg;
+  ctx->device = device;
+  dyo_config& c = ctx->cfg;
+  if (c.align <= 0 || (c.align & (c.align - 1)) || c.align < 16 || c.budget < 2 * c.align ||
+      c.max_batch < 1 || c.max_batch > 64 || c.policy < 0 || c.policy > 1) {
+    delete ctx;
+    return DYO_E_INVAL;
+  }
+  if (c.staging_bytes <= 0) c.staging_bytes = 64ll << 20;
+  if (c.dma_min_bytes <= 0) c.dma_min_bytes = 2ll << 20;
+  ctx->H = c.budget / 2 / c.align * c.align;
+  if (ctx->H / c.align >= (1ll << 28)) { delete ctx; return DYO_E_INVAL; }
+  cudaError_t e = cudaSetDevice(device);
+  if (e == cudaSuccess) e = cudaMalloc(&ctx->arena, 2 * ctx->H);
+  if (e == cudaSuccess) e = cudaMalloc(&ctx->staging, c.staging_bytes);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_last, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, device);
+  if (e != cudaSuccess) {
+    dyo_destroy(ctx);
+    return e == cudaErrorMemoryAllocation ? DYO_E_NOMEM : DYO_E_CUDA;
+  }
+  ctx->staging_bytes = c.staging_bytes;
+  *outp = ctx;
+  return DYO_OK;
+}
+
+dyo_status dyo_destroy(dyo_ctx* ctx) {
+  if (!ctx) return DYO_E_INVAL;
+  cudaSetDevice(ctx->device);
+  cudaDeviceSynchronize();
+  free_list(ctx->arch_dev);
+  free_list(ctx->pilot_dev);
+  free_plan_host(ctx);
+  if (ctx->host_pool) cudaFreeHost(ctx->host_pool);
+  if (ctx->arena) cudaFree(ctx->arena);
+  if (ctx->staging) cudaFree(ctx->staging);
+  if (ctx->ev_last) cudaEventDestroy(ctx->ev_last);
+  for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
+  for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+  delete ctx;
+  return DYO_OK;
+}
+
+dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
+  if (!ctx || !A) return DYO_E_INVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  free_list(ctx->arch_dev);
+  free_plan_host(ctx);
+  if (ctx->host_pool) { cudaFreeHost(ctx->host_pool); ctx->host_pool = nullptr; }
+  ctx->arch_ok = false;
+  ctx->plan_valid = false;
+  const int64_t AL = ctx->cfg.align;
+  ArchHost h;
+  dyo_status pst = parse_arch(A, AL, h, ctx->err);
+  if (pst) return pst;
+  const int T = h.T, n_ops = A->n_ops, n_sites = h.n_sites;
+  ctx->T = T;
+  ctx->t_bytes = h.t_bytes; ctx->t_abytes = h.t_abytes; ctx->t_host = h.t_host; ctx->t_flags = h.t_flags;
+  ctx->n_branch_logits = h.n_branch_logits;
+  const int64_t pool = h.pool, L_max = h.L_max;
+  auto& sig = h.sig; auto& acc_ptr = h.acc_ptr; auto& acc_t = h.acc_t; auto& acc_m = h.acc_m;
+  auto& site_kind = h.site_kind; auto& site_nch = h.site_nch; auto& site_lo = h.site_lo;
+  auto& site_tie = h.site_tie; auto& site_logit = h.site_logit; auto& site_arm_ptr = h.site_arm_ptr;
+  auto& arm_first = h.arm_first; auto& arm_n = h.arm_n;
+  auto& piece_kind = h.piece_kind; auto& piece_a = h.piece_a; auto& piece_b = h.piece_b; auto& piece_c = h.piece_c;
+  auto& seg_table = h.seg_table;
+  // ---- device copies ----
+  ArchDev& ad = ctx->ad;
+  ad = ArchDev{};
+  ad.T = T; ad.n_ops = n_ops; ad.n_sites = n_sites; ad.n_pieces = (int)piece_kind.size();
+  ad.nn_type = A->nn_type; ad.S_max = A->S_max; ad.D_s = A->D_s; ad.h = A->h; ad.K_max = A->K_max;
+  ad.F = (3 + A->D_s + 10 * A->S_max + 10 * A->h + 15) / 16 * 16;
+  ad.O = 0;
+  ad.n_branch_logits = ctx->n_branch_logits;
+  ad.L_max = (int)std::max<int64_t>(L_max, 1);
+  ad.H = ctx->H;
+  ad.align = AL;
+  std::vector<void*>& own = ctx->arch_dev;
+  dyo_status st;
+#define UP(field, vec) if ((st = dupload(ctx, own, &ad.field, vec))) return st
+  UP(t_bytes, ctx->t_bytes); UP(t_abytes, ctx->t_abytes); UP(t_host, ctx->t_host); UP(t_flags, ctx->t_flags);
+  UP(op_sig, sig); UP(acc_ptr, acc_ptr); UP(acc_t, acc_t); UP(acc_m, acc_m);
+  UP(site_kind, site_kind); UP(site_nch, site_nch); UP(site_lo, site_lo); UP(site_tie, site_tie);
+  UP(site_logit, site_logit); UP(site_arm_ptr, site_arm_ptr); UP(arm_first_op, arm_first); UP(arm_nops, arm_n);
+  UP(piece_kind, piece_kind); UP(piece_a, piece_a); UP(piece_b, piece_b); UP(piece_c, piece_c);
+  UP(seg_table, seg_table);
+#undef UP
+  ctx->n_ops = n_ops; ctx->n_sites = n_sites; ctx->K_max = A->K_max; ctx->F = ad.F;
+  ctx->O_min = 10 * A->K_max + ctx->n_branch_logits;
+
+  // ---- prediction storage ----
+  const int B = ctx->cfg.max_batch, K = A->K_max;
+  PredDev& pd = ctx->pd;
+  pd = PredDev{};
+  pd.B = B;
+#define DA(p, n) if ((st = dalloc(ctx, own, &p, (size_t)(n)))) return st
+  DA(pd.K, B); DA(pd.L, B); DA(pd.choices, (size_t)B * std::max(n_sites, 1)); DA(pd.slots, (size_t)B * K * 10);
+  DA(pd.path, (size_t)B * ad.L_max); DA(pd.grp, (size_t)B * K * 2); DA(pd.blocks, (size_t)B * K * 10);
+  DA(pd.ent_n, (size_t)B * K); DA(pd.ent, (size_t)B * K * kEntCap); DA(pd.status, 4);
+  DA(ctx->desc_dev, (size_t)B * std::max(A->D_s, 1)); DA(ctx->hist_dev, (size_t)B * std::max(A->h, 1));
+  DA(ctx->hist_tab[0], (size_t)B * K * 10); DA(ctx->hist_tab[1], (size_t)B * K * 10);
+  DA(ctx->hist_len[0], 1); DA(ctx->hist_len[1], 1);
+  ctx->hist_cur = 0;
+  ctx->last_B = 0;
+  // ---- planner state, scratch and outputs ----
+  int mg = ctx->cfg.max_groups > 0 ? ctx->cfg.max_groups : B * K;
+  mg = std::min(mg, 65535);
+  ctx->max_groups = mg;
+  for (int s2 = 0; s2 < 2; ++s2) {
+    PlanState& ps = ctx->state[s2];
+    DA(ps.loc, T); DA(ps.off, T); DA(ps.dirty, T); DA(ps.pw, T); DA(ps.res, 2 * (size_t)T);
+    DA(ps.res_n, 2); DA(ps.prev, T); DA(ps.prev_n, 1); DA(ps.G, 1);
+    CK(cudaMemset(ps.loc, 0xff, T));   // -1: every tensor starts on the host
+  }
+  ctx->committed = 0;
+  int64_t cap_ent = ctx->cfg.max_entries > 0 ? ctx->cfg.max_entries : (int64_t)mg * 256;
+  int64_t cap_rec = ctx->cfg.max_records > 0 ? ctx->cfg.max_records : 4 * ((int64_t)T + cap_ent);
+  PlanScratch& sc = ctx->sc;
+  DA(sc.inw, T); DA(sc.cur_next, T); DA(sc.cur_rd, T); DA(sc.nxt, cap_ent); DA(sc.nxt_rd, cap_ent);
+  DA(sc.rstat, T); DA(sc.keys, 2 * ((size_t)T + 1024) + 4096); DA(sc.gap_s, T + 1); DA(sc.gap_e, T + 1);
+  DA(sc.kept, T); DA(sc.newoff, T); DA(sc.ebase, mg); DA(sc.grp_b, mg); DA(sc.grp_k, mg);
+#undef DA
+  auto hmap = [&](void** p, size_t bytes) -> dyo_status {
+    CK(cudaHostAlloc(p, std::max<size_t>(bytes, 64), cudaHostAllocMapped | cudaHostAllocPortable));
+    memset(*p, 0, std::max<size_t>(bytes, 64));
+    return DYO_OK;
+  };
+  PlanOut& o = ctx->out;
+  o = PlanOut{};
+  o.cap_ent = cap_ent;
+  o.cap_rec = cap_rec;
+  if ((st = hmap((void**)&o.hdr, sizeof(PlanHdr) * mg))) return st;
+  if ((st = hmap((void**)&o.ent, sizeof(dyo_entry_rec) * cap_ent))) return st;
+  if ((st = hmap((void**)&o.ev, sizeof(dyo_evict_rec) * cap_rec))) return st;
+  if ((st = hmap((void**)&o.mv, sizeof(dyo_move_rec) * cap_rec))) return st;
+  if ((st = hmap((void**)&o.ca, sizeof(dyo_carry_rec) * cap_rec))) return st;
+  if ((st = hmap((void**)&o.al, sizeof(dyo_alloc_rec) * cap_rec))) return st;
+  if ((st = hmap((void**)&o.fe, sizeof(dyo_fetch_rec) * cap_rec))) return st;
+  if ((st = hmap((void**)&ctx->h_status, 16 * sizeof(int32_t)))) return st;
+  if ((st = hmap((void**)&ctx->h_counts, 16 * sizeof(int32_t)))) return st;
+  if ((st = hmap((void**)&ctx->h_loc, T))) return st;
+  if ((st = hmap((void**)&ctx->h_off, sizeof(int64_t) * T))) return st;
+  memset(ctx->h_loc, 0xff, T);
+  ctx->seg_cap = 8 * cap_rec + 65536;
+  if ((st = hmap((void**)&ctx->h_segs, sizeof(CopySeg) * ctx->seg_cap))) return st;
+  int32_t* d_status = nullptr;
+  int32_t* d_counts = nullptr;
+  CK(cudaHostGetDevicePointer((void**)&d_status, ctx->h_status, 0));
+  CK(cudaHostGetDevicePointer((void**)&d_counts, ctx->h_counts, 0));
+  o.status = d_status;
+  o.counts = d_counts;
+  // ---- host pool (pinned, mapped: DMA and zero-copy kernels) ----
+  ctx->host_bytes = pool;
+  if (!(ctx->cfg.flags & DYO_F_NO_HOST_POOL))
+    CK(cudaHostAlloc((void**)&ctx->host_pool, std::max<int64_t>(pool, 64), cudaHostAllocMapped | cudaHostAllocPortable));
+  ctx->arch_ok = true;
+  ctx->pilot_ok = false;
+  return DYO_OK;
+}
+
+dyo_status dyo_arch_check(const dyo_arch* A, int32_t align, dyo_arch_summary* out, int32_t* seg_table,
+                          int32_t* op_sig, char* err, int32_t errlen) {
+  if (!A || align < 16 || (align & (align - 1))) return DYO_E_INVAL;
+  ArchHost h;
+  std::string e;
+  dyo_status st = parse_arch(A, align, h, e);
+  if (err && errlen > 0) { strncpy(err, e.c_str(), errlen - 1); err[errlen - 1] = 0; }
+  if (st) return st;
+  if (out) {
+    out->n_sites = h.n_sites;
+    out->n_branch_logits = h.n_branch_logits;
+    out->n_pieces = (int32_t)h.piece_kind.size();
+    out->L_max = h.L_max;
+    out->F = (3 + A->D_s + 10 * A->S_max + 10 * A->h + 15) / 16 * 16;
+    out->host_pool_bytes = h.pool;
+  }
+  if (seg_table) std::copy(h.seg_table.begin(), h.seg_table.end(), seg_table);
+  if (op_sig) std::copy(h.sig.begin(), h.sig.end(), op_sig);
+  return DYO_OK;
+}
+
+dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
+  if (!ctx || !w) return DYO_E_INVAL;
+  if (!ctx->arch_ok) return fail(ctx, DYO_E_STATE, "load the arch first");
+  CK(cudaSetDevice(ctx->device));
+  if (w->F != ctx->F) return fail(ctx, DYO_E_INVAL, "pilot F=%d, arch needs %d", w->F, ctx->F);
+  if (w->O < ctx->O_min) return fail(ctx, DYO_E_INVAL, "pilot O=%d < %d", w->O, ctx->O_min);
+  if (w->n_mlp < 1 || w->n_mlp > kMaxLayers || w->n_feature < 0 || w->n_feature > 8)
+    return fail(ctx, DYO_E_INVAL, "pilot: layer counts");
+  free_list(ctx->pilot_dev);
+  PilotDev& p = ctx->pdv;
+  p = PilotDev{};
+  p.F = w->F;
+  p.O = w->O;
+  p.slope = w->slope;
+  int nl = 0, ns = 0, width = w->F;
+  int maxw = w->F;
+  auto add_layer = [&](const float* W, const float* b, int in_off, int in_len, int out_len, int out_off) -> dyo_status {
+    LayerDev& L = p.ly[nl++];
+    const int in_pad = (in_len + 3) / 4 * 4;
+    std::vector<float> wp((size_t)out_len * in_pad, 0.f), bp(b, b + out_len);
+    for (int r = 0; r < out_len; ++r)
+      for (int c = 0; c < in_len; ++c) wp[(size_t)r * in_pad + c] = W[(size_t)r * in_len + c];
+    const float* dw = nullptr;
+    const float* db = nullptr;
+    dyo_status s = dupload(ctx, ctx->pilot_dev, &dw, wp);
+    if (s) return s;
+    s = dupload(ctx, ctx->pilot_dev, &db, bp);
+    if (s) return s;
+    L.W = dw; L.b = db; L.in_off = in_off; L.in_len = in_len; L.in_pad = in_pad; L.out_off = out_off; L.out_len = out_len;
+    return DYO_OK;
+  };
+  dyo_status s;
+  if (w->n_feature > 0) {
+    StageDev& S = p.st[ns++];
+    S.first_layer = nl; S.n_layers = w->n_feature; S.in_width = w->F; S.act = 1;
+    int o = 0;
+    for (int i = 0; i < w->n_feature; ++i) {
+      if (w->feat_off[i] < 0 || w->feat_off[i] + w->feat_len[i] > w->F) return fail(ctx, DYO_E_INVAL, "pilot: feature slice");
+      if ((s = add_layer(w->feat_W[i], w->feat_b[i], w->feat_off[i], w->feat_len[i], w->feat_out[i], o))) return s;
+      o += w->feat_out[i];
+    }
+    S.out_width = S.rows = o;
+    width = o;
+    maxw = std::max(maxw, o);
+  }
+  const int k = ctx->ad.nn_type;   // only the MLP of the arch's NN type runs
+  for (int l = 0; l < w->n_mlp; ++l) {
+    if (w->mlp_in[l] != width) return fail(ctx, DYO_E_INVAL, "pilot: MLP layer %d input %d != %d", l, w->mlp_in[l], width);
+    StageDev& S = p.st[ns++];
+    S.first_layer = nl; S.n_layers = 1; S.in_width = width; S.act = 1;
+    if ((s = add_layer(w->mlp_W[k * w->n_mlp + l], w->mlp_b[k * w->n_mlp + l], 0, w->mlp_in[l], w->mlp_out[l], 0))) return s;
+    width = S.out_width = S.rows = w->mlp_out[l];
+    maxw = std::max(maxw, width);
+  }
+  if (w->out_in != width) return fail(ctx, DYO_E_INVAL, "pilot: output layer input %d != %d", w->out_in, width);
+  StageDev& S = p.st[ns++];
+  S.first_layer = nl; S.n_layers = 1; S.in_width = width; S.act = 0;
+  if ((s = add_layer(w->out_W, w->out_b, 0, width, w->O, 0))) return s;
+  S.out_width = S.rows = w->O;
+  p.n_stages = ns;
+  p.max_width = (maxw + 3) / 4 * 4;
+  ctx->ad.O = w->O;
+  CK(cudaFree(nullptr));
+  float* lg = nullptr;
+  if ((s = dalloc(ctx, ctx->pilot_dev, &lg, (size_t)ctx->cfg.max_batch * w->O))) return s;
+  ctx->logits_scratch = lg;
+  ctx->pilot_ok = true;
+  return DYO_OK;
+}
+
+dyo_status dyo_host_pool(dyo_ctx* ctx, void** base, int64_t* bytes) {
+  if (!ctx || !ctx->arch_ok || !ctx->host_pool) return DYO_E_STATE;
+  if (base) *base = ctx->host_pool;
+  if (bytes) *bytes = ctx->host_bytes;
+  return DYO_OK;
+}
+
+dyo_status dyo_arena(dyo_ctx* ctx, void** base, int64_t* half) {
+  if (!ctx) return DYO_E_INVAL;
+  if (base) *base = ctx->arena;
+  if (half) *half = ctx->H;
+  return DYO_OK;
+}
+
+static dyo_status stage_samples(dyo_ctx* ctx, const dyo_sample* s, int B, cudaStream_t st,
+                                const int64_t** desc, const int32_t** hist) {
+  const ArchDev& a = ctx->ad;
+  *desc = nullptr;
+  *hist = nullptr;
+  if (a.D_s > 0) {
+    if (!s || !s->desc) return fail(ctx, DYO_E_INVAL, "sample descriptors missing");
+    if (is_device_ptr(s->desc)) *desc = s->desc;
+    else {
+      CK(cudaMemcpyAsync(ctx->desc_dev, s->desc, sizeof(int64_t) * B * a.D_s, cudaMemcpyHostToDevice, st));
+      *desc = ctx->desc_dev;
+    }
+  } else {
+    *desc = ctx->desc_dev;
+  }
+  if (a.h > 0 && s && s->hist_ids) {
+    if (is_device_ptr(s->hist_ids)) *hist = s->hist_ids;
+    else {
+      CK(cudaMemcpyAsync(ctx->hist_dev, s->hist_ids, sizeof(int32_t) * B * a.h, cudaMemcpyHostToDevice, st));
+      *hist = ctx->hist_dev;
+    }
+  }
+  return DYO_OK;
+}
+
+dyo_status dyo_encode_features(dyo_ctx* ctx, const dyo_sample* s, int32_t B, float* feat, void* stream) {
+  if (!ctx || !feat) return DYO_E_INVAL;
+  if (!ctx->arch_ok) return fail(ctx, DYO_E_STATE, "load the arch first");
+  if (B < 1 || B > ctx->cfg.max_batch) return fail(ctx, DYO_E_INVAL, "B=%d out of [1, max_batch]", B);
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t* desc;
+  const int32_t* hist;
+  dyo_status r = stage_samples(ctx, s, B, st, &desc, &hist);
+  if (r) return r;
+  CK(launch_encode(ctx->ad, desc, hist, ctx->hist_tab[ctx->hist_cur], ctx->hist_len[ctx->hist_cur], B, feat, st));
+  return DYO_OK;
+}
+
+dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* s, int32_t B,
+                             float* logits, void* stream) {
+  if (!ctx) return DYO_E_INVAL;
+  if (!ctx->arch_ok || !ctx->pilot_ok) return fail(ctx, DYO_E_STATE, "load arch and pilot first");
+  if (B < 1 || B > ctx->cfg.max_batch) return fail(ctx, DYO_E_INVAL, "B=%d out of [1, max_batch]", B);
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t* desc = nullptr;
+  const int32_t* hist = nullptr;
+  if (!feat) {
+    dyo_status r = stage_samples(ctx, s, B, st, &desc, &hist);
+    if (r) return r;
+  } else if (!is_device_ptr(feat)) {
+    return fail(ctx, DYO_E_INVAL, "feat must be device memory");
+  }
+  float* lg = logits ? logits : ctx->logits_scratch;
+  const int cur = ctx->hist_cur;
+  {
+    TScope ts(ctx, 0, st);
+    CK(launch_pilot(ctx->ad, ctx->pdv, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_len[cur], B, lg, nullptr, st));
+  }
+  {
+    TScope ts(ctx, 1, st);
+    CK(launch_decode(ctx->ad, lg, ctx->pd, B, ctx->hist_tab[1 - cur], ctx->hist_len[1 - cur], st));
+  }
+  ctx->hist_cur = 1 - cur;
+  ctx->last_B = B;
+  return DYO_OK;
+}
+
+dyo_status dyo_prediction_get(dyo_ctx* ctx, int32_t b, int32_t* K, int32_t* blocks, int32_t* choices,
+                              int32_t* group_rows, void* stream) {
+  if (!ctx || b < 0 || b >= ctx->last_B) return DYO_E_INVAL;
+  cudaStream_t st = (cudaStream_t)stream;
+  CK(cudaStreamSynchronize(st));
+  int32_t status = 0;
+  CK(cudaMemcpy(&status, ctx->pd.status, sizeof status, cudaMemcpyDeviceToHost));
+  if (status) return fail(ctx, (dyo_status)status, "decode failed (status %d)", status);
+  const int Km = ctx->K_max;
+  if (K) CK(cudaMemcpy(K, ctx->pd.K + b, sizeof(int32_t), cudaMemcpyDeviceToHost));
+  if (blocks) CK(cudaMemcpy(blocks, ctx->pd.blocks + (size_t)b * Km * 10, sizeof(int32_t) * Km * 10, cudaMemcpyDeviceToHost));
+  if (choices && ctx->n_sites)
+    CK(cudaMemcpy(choices, ctx->pd.choices + (size_t)b * ctx->n_sites, sizeof(int32_t) * ctx->n_sites, cudaMemcpyDeviceToHost));
+  if (group_rows) CK(cudaMemcpy(group_rows, ctx->pd.grp + (size_t)b * Km * 2, sizeof(int32_t) * Km * 2, cudaMemcpyDeviceToHost));
+  return DYO_OK;
+}
+
+dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* outp, int32_t cap, int32_t* n,
+                             void* stream) {
+  if (!ctx || b < 0 || b >= ctx->last_B || g < 0 || g >= ctx->K_max || !n) return DYO_E_INVAL;
+  CK(cudaStreamSynchronize((cudaStream_t)stream));
+  int32_t cnt = 0;
+  CK(cudaMemcpy(&cnt, ctx->pd.ent_n + (size_t)b * ctx->K_max + g, sizeof cnt, cudaMemcpyDeviceToHost));
+  *n = cnt;
+  if (cnt > cap) return fail(ctx, DYO_E_CAPACITY, "need %d entries", cnt);
+  std::vector<int2> tmp(cnt);
+  if (cnt) CK(cudaMemcpy(tmp.data(), ctx->pd.ent + ((size_t)b * ctx->K_max + g) * kEntCap, sizeof(int2) * cnt, cudaMemcpyDeviceToHost));
+  for (int i = 0; i < cnt; ++i) {
+    outp[3 * i] = tmp[i].x;
+    outp[3 * i + 1] = tmp[i].y & 3;
+    outp[3 * i + 2] = (tmp[i].y >> 2) & 1;
+  }
+  return DYO_OK;
+}
+
+dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* stream) {
+  if (!ctx) return DYO_E_INVAL;
+  if (!ctx->arch_ok || ctx->last_B <= 0) return fail(ctx, DYO_E_STATE, "no prediction to plan");
+  if (n < 0) { b0 = 0; n = ctx->last_B; }
+  if (b0 < 0 || n < 1 || b0 + n > ctx->last_B) return fail(ctx, DYO_E_INVAL, "prediction range");
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  // the pinned plan lists and copy descriptors are about to be rewritten: the previous plan's
+  // migrations must have consumed them
+  if (ctx->ev_pending) { CK(cudaEventSynchronize(ctx->ev_last)); ctx->ev_pending = false; }
+  ctx->plan_valid = false;
+  ctx->h_status[0] = -100;
+  PlanState& in = ctx->state[ctx->committed];
+  PlanState& wk = ctx->state[1 - ctx->committed];
+  {
+    TScope ts(ctx, 2, st);
+    CK(launch_plan(ctx->ad, ctx->pd, b0, n, ctx->cfg.policy, in, wk, ctx->sc, ctx->out, ctx->max_groups, st));
+  }
+  CK(cudaMemcpyAsync(ctx->h_loc, wk.loc, ctx->T, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(ctx->h_off, wk.off, sizeof(int64_t) * ctx->T, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));     // the one synchronisation of the hot path (DMA sizes to host)
+  const int32_t status = ctx->h_status[0];
+  if (status != 0) {
+    // restore the residency mirror of the committed state
+    cudaMemcpy(ctx->h_loc, in.loc, ctx->T, cudaMemcpyDeviceToHost);
+    cudaMemcpy(ctx->h_off, in.off, sizeof(int64_t) * ctx->T, cudaMemcpyDeviceToHost);
+    if (status == DYO_E_BUDGET) return fail(ctx, DYO_E_BUDGET, "transition %d: W_j exceeds half the budget", ctx->h_status[1]);
+    if (status == DYO_E_CAPACITY) return fail(ctx, DYO_E_CAPACITY, "capacity exceeded (needed %d)", ctx->h_status[2]);
+    return fail(ctx, (dyo_status)(status < 0 ? status : DYO_E_CUDA), "planner status %d", status);
+  }
+  ctx->committed = 1 - ctx->committed;
+  ctx->plan_K = ctx->h_counts[0];
+  ctx->next_j = 0;
+  ctx->seg_used = 0;
+  ctx->plan_valid = true;
+  if (K_out) *K_out = ctx->plan_K;
+  return DYO_OK;
+}
+
+dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info) {
+  if (!ctx || !info) return DYO_E_INVAL;
+  if (!ctx->plan_valid) return fail(ctx, DYO_E_STATE, "no valid plan");
+  if (j < 0 || j >= ctx->plan_K) return DYO_E_INVAL;
+  const PlanHdr& h = ctx->out.hdr[j];
+  info->half = h.half; info->n_entries = h.n_ent; info->n_evict = h.n_evict; info->n_move = h.n_move;
+  info->n_carry = h.n_carry; info->n_alloc = h.n_alloc; info->n_fetch = h.n_fetch;
+  info->need = h.need; info->h2d = h.h2d; info->d2h = h.d2h; info->d2d = h.d2d;
+  return DYO_OK;
+}
+
+dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** recs, int32_t* n) {
+  if (!ctx || !recs || !n) return DYO_E_INVAL;
+  if (!ctx->plan_valid) return fail(ctx, DYO_E_STATE, "no valid plan");
+  if (j < 0 || j >= ctx->plan_K) return DYO_E_INVAL;
+  const PlanHdr& h = ctx->out.hdr[j];
+  switch (list) {
+    case 0: *recs = ctx->out.ev + h.o_evict; *n = h.n_evict; break;
+    case 1: *recs = ctx->out.mv + h.o_move; *n = h.n_move; break;
+    case 2: *recs = ctx->out.ca + h.o_carry; *n = h.n_carry; break;
+    case 3: *recs = ctx->out.al + h.o_alloc; *n = h.n_alloc; break;
+    case 4: *recs = ctx->out.fe + h.o_fetch; *n = h.n_fetch; break;
+    case 5: *recs = ctx->out.ent + h.o_ent; *n = h.n_ent; break;
+    default: return DYO_E_INVAL;
+  }
+  return DYO_OK;
+}
+
+// ---- migration engine -----------------------------------------------------------------
+namespace {
+
+struct Run { int64_t host_off, dev_off, bytes; bool dev_contig; int first, count; };
+
+constexpr int64_t kChunk = 256 << 10;   // copy-kernel work item
+
+// push (src, dst, bytes) split into work items; returns false on capacity
+bool push_seg(dyo_ctx* ctx, const char* src, char* dst, int64_t bytes) {
+  for (int64_t o = 0; o < bytes; o += kChunk) {
+    if (ctx->seg_used >= ctx->seg_cap) return false;
+    ctx->h_segs[ctx->seg_used++] = CopySeg{src + o, dst + o, std::min(kChunk, bytes - o)};
+  }
+  return true;
+}
+
+dyo_status launch_segs(dyo_ctx* ctx, int64_t first, cudaStream_t s, int grid, int kind = 3) {
+  const int64_t n = ctx->seg_used - first;
+  if (n <= 0) return DYO_OK;
+  CopySeg* dptr = nullptr;
+  CK(cudaHostGetDevicePointer((void**)&dptr, ctx->h_segs + first, 0));
+  int64_t bytes = 0;
+  for (int64_t i = first; i < ctx->seg_used; ++i) bytes += ctx->h_segs[i].bytes;
+  TScope ts(ctx, kind, s, bytes);
+  CK(launch_copy_segments(dptr, (int)n, kChunk, grid, s));
+  ctx->ctr.n_kernels++;
+  return DYO_OK;
+}
+
+}  // namespace
+
+dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev_started, void* ev_prev_done,
+                       void* ev_ready) {
+  if (!ctx) return DYO_E_INVAL;
+  if (!ctx->plan_valid) return fail(ctx, DYO_E_STATE, "dyo_migrate before a successful dyo_plan");
+  if (j != ctx->next_j || j >= ctx->plan_K) return fail(ctx, DYO_E_STATE, "transition %d out of order (next %d)", j, ctx->next_j);
+  if (!ctx->host_pool) return fail(ctx, DYO_E_STATE, "plan-only ctx (DYO_F_NO_HOST_POOL) cannot migrate");
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t s = (cudaStream_t)copy_stream;
+  const PlanHdr& h = ctx->out.hdr[j];
+  char* arena = ctx->arena;
+  char* host = ctx->host_pool;
+  const int64_t AL = ctx->cfg.align;
+  const int64_t dma_min = (ctx->cfg.flags & DYO_F_NO_ZEROCOPY) ? 0 : ctx->cfg.dma_min_bytes;
+  const int zc_grid = 16;
+  const int d2d_grid = 4 * ctx->sm_count;
+  if (ev_prev_started) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_started, 0));
+
+  // 1. EVICT writebacks (D2H): host runs (ascending host offset) -> DMA (direct, or K3 packed
+  //    through staging when the device sources are scattered), or one zero-copy scatter launch
+  //    (K5) for the runs below dma_min
+  {
+    const dyo_evict_rec* ev = ctx->out.ev + h.o_evict;
+    std::vector<int> small;
+    int i = 0;
+    while (i < h.n_evict) {
+      if (!ev[i].writeback) { ++i; continue; }
+      Run r{ev[i].host_off, ev[i].src, ev[i].bytes, true, i, 1};
+      int64_t hend = ev[i].host_off + align_up(ev[i].bytes, AL);
+      int64_t dend = ev[i].src + align_up(ev[i].bytes, AL);
+      int k = i + 1;
+      while (k < h.n_evict && ev[k].writeback && ev[k].host_off == hend) {
+        if (ev[k].src != dend) r.dev_contig = false;
+        hend = ev[k].host_off + align_up(ev[k].bytes, AL);
+        dend = ev[k].src + align_up(ev[k].bytes, AL);
+        r.bytes = ev[k].host_off + ev[k].bytes - r.host_off;
+        ++k;
+        ++r.count;
+      }
+      if (r.bytes >= dma_min && r.dev_contig) {
+        { TScope ts(ctx, 6, s, r.bytes);
+          CK(cudaMemcpyAsync(host + r.host_off, arena + r.dev_off, r.bytes, cudaMemcpyDeviceToHost, s)); }
+        ctx->ctr.d2h_dma += r.bytes;
+        ctx->ctr.n_dma++;
+      } else if (r.bytes >= dma_min && !(ctx->cfg.flags & DYO_F_NO_PACK)) {
+        int q = r.first;
+        while (q < r.first + r.count) {
+          const int64_t base = ev[q].host_off;
+          const int64_t seg0 = ctx->seg_used;
+          int q2 = q;
+          while (q2 < r.first + r.count && ev[q2].host_off + ev[q2].bytes - base <= ctx->staging_bytes) {
+            if (!push_seg(ctx, arena + ev[q2].src, ctx->staging + (ev[q2].host_off - base), ev[q2].bytes))
+              return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+            ++q2;
+          }
+          if (q2 == q) {   // a tensor larger than the staging buffer: its own DMA
+            { TScope ts(ctx, 6, s, ev[q].bytes);
+              CK(cudaMemcpyAsync(host + ev[q].host_off, arena + ev[q].src, ev[q].bytes, cudaMemcpyDeviceToHost, s)); }
+            ctx->ctr.d2h_dma += ev[q].bytes;
+            ctx->ctr.n_dma++;
+            ++q;
+            continue;
+          }
+          dyo_status s1 = launch_segs(ctx, seg0, s, d2d_grid);
+          if (s1) return s1;
+          const int64_t len = ev[q2 - 1].host_off + ev[q2 - 1].bytes - base;
+          { TScope ts(ctx, 6, s, len);
+            CK(cudaMemcpyAsync(host + base, ctx->staging, len, cudaMemcpyDeviceToHost, s)); }
+          ctx->ctr.d2h_packed += len;
+          ctx->ctr.n_dma++;
+          q = q2;
+        }
+      } else {
+        for (int q = r.first; q < r.first + r.count; ++q) small.push_back(q);
+      }
+      i = k;
+    }
+    if (!small.empty()) {
+      const int64_t g0 = ctx->seg_used;
+      for (int q : small) {
+        if (!push_seg(ctx, arena + ev[q].src, host + ev[q].host_off, ev[q].bytes))
+          return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+        ctx->ctr.d2h_zc += ev[q].bytes;
+      }
+      dyo_status s1 = launch_segs(ctx, g0, s, zc_grid, 4);
+      if (s1) return s1;
+    }
+  }
+  // 2. MOVE (compaction): staged through `staging` in ascending destination order (R12)
+  {
+    const dyo_move_rec* mv = ctx->out.mv + h.o_move;
+    int i = 0;
+    int64_t piece_off = 0;
+    while (i < h.n_move) {
+      const int64_t g0 = ctx->seg_used;
+      int64_t used = 0;
+      std::vector<std::array<int64_t, 3>> parts;   // (src, dst, bytes) of this chunk
+      while (i < h.n_move && used < ctx->staging_bytes) {
+        const int64_t take = std::min(mv[i].bytes - piece_off, ctx->staging_bytes - used);
+        parts.push_back({mv[i].src + piece_off, mv[i].dst + piece_off, take});
+        used += take;
+        piece_off += take;
+        if (piece_off == mv[i].bytes) { ++i; piece_off = 0; }
+      }
+      int64_t so = 0;
+      for (auto& p : parts) {
+        if (!push_seg(ctx, arena + p[0], ctx->staging + so, p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+        so += p[2];
+      }
+      dyo_status s1 = launch_segs(ctx, g0, s, d2d_grid);
+      if (s1) return s1;
+      const int64_t g1 = ctx->seg_used;
+      so = 0;
+      for (auto& p : parts) {
+        if (!push_seg(ctx, ctx->staging + so, arena + p[1], p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+        so += p[2];
+        ctx->ctr.d2d += p[2];
+      }
+      s1 = launch_segs(ctx, g1, s, d2d_grid);
+      if (s1) return s1;
+    }
+  }
+  // 3. early CARRY (D2D, one launch) and FETCH (H2D: DMA per host run, zero-copy gather for
+  //    the small runs, one launch)
+  {
+    const dyo_carry_rec* ca = ctx->out.ca + h.o_carry;
+    const int64_t g0 = ctx->seg_used;
+    for (int i = 0; i < h.n_carry; ++i) {
+      if (ca[i].late) continue;
+      if (!push_seg(ctx, arena + ca[i].src, arena + ca[i].dst, ca[i].bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+      ctx->ctr.d2d += ca[i].bytes;
+    }
+    dyo_status s1 = launch_segs(ctx, g0, s, d2d_grid);
+    if (s1) return s1;
+  }
+  {
+    const dyo_fetch_rec* fe = ctx->out.fe + h.o_fetch;
+    const int64_t g0 = ctx->seg_used;
+    int i = 0;
+    while (i < h.n_fetch) {
+      int64_t hend = fe[i].host_off + align_up(fe[i].bytes, AL);
+      int64_t dend = fe[i].dst + align_up(fe[i].bytes, AL);
+      int k = i + 1;
+      while (k < h.n_fetch && fe[k].host_off == hend && fe[k].dst == dend) {
+        hend = fe[k].host_off + align_up(fe[k].bytes, AL);
+        dend = fe[k].dst + align_up(fe[k].bytes, AL);
+        ++k;
+      }
+      const int64_t bytes = fe[k - 1].host_off + fe[k - 1].bytes - fe[i].host_off;
+      if (bytes >= dma_min) {
+        { TScope ts(ctx, 5, s, bytes);
+          CK(cudaMemcpyAsync(arena + fe[i].dst, host + fe[i].host_off, bytes, cudaMemcpyHostToDevice, s)); }
+        ctx->ctr.h2d_dma += bytes;
+        ctx->ctr.n_dma++;
+      } else {
+        for (int q = i; q < k; ++q) {
+          if (!push_seg(ctx, host + fe[q].host_off, arena + fe[q].dst, fe[q].bytes))
+            return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+          ctx->ctr.h2d_zc += fe[q].bytes;
+        }
+      }
+      i = k;
+    }
+    dyo_status s1 = launch_segs(ctx, g0, s, zc_grid, 4);
+    if (s1) return s1;
+  }
+  // 4. late CARRY: block j-1 writes them, so they wait for its end
+  {
+    const dyo_carry_rec* ca = ctx->out.ca + h.o_carry;
+    bool any = false;
+    for (int i = 0; i < h.n_carry; ++i) any |= ca[i].late != 0;
+    if (any) {
+      if (ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
+      const int64_t g0 = ctx->seg_used;
+      for (int i = 0; i < h.n_carry; ++i) {
+        if (!ca[i].late) continue;
+        if (!push_seg(ctx, arena + ca[i].src, arena + ca[i].dst, ca[i].bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+        ctx->ctr.d2d += ca[i].bytes;
+      }
+      dyo_status s1 = launch_segs(ctx, g0, s, d2d_grid);
+      if (s1) return s1;
+    }
+  }
+  if (ev_ready) CK(cudaEventRecord((cudaEvent_t)ev_ready, s));
+  CK(cudaEventRecord(ctx->ev_last, s));
+  ctx->ev_pending = true;
+  ctx->next_j = j + 1;
+  return DYO_OK;
+}
+
+dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr) {
+  if (!ctx || !dev_ptr || t < 0 || t >= ctx->T) return DYO_E_INVAL;
+  const int8_t l = ctx->h_loc[t];
+  *dev_ptr = l < 0 ? nullptr : ctx->arena + (int64_t)l * ctx->H + ctx->h_off[t];
+  return DYO_OK;
+}
+
+dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* launches, int64_t* bytes,
+                           int32_t reset) {
+  if (!ctx || kind < 0 || kind >= DYO_T_KINDS) return DYO_E_INVAL;
+  drain_timings(ctx);
+  if (ms) *ms = ctx->tm_ms[kind];
+  if (launches) *launches = ctx->tm_n[kind];
+  if (bytes) *bytes = ctx->tm_bytes[kind];
+  if (reset) {
+    for (int k = 0; k < DYO_T_KINDS; ++k) { ctx->tm_ms[k] = 0; ctx->tm_n[k] = 0; ctx->tm_bytes[k] = 0; }
+  }
+  return DYO_OK;
+}
+
+dyo_status dyo_get_counters(dyo_ctx* ctx, dyo_counters* c, int32_t reset) {
+  if (!ctx || !c) return DYO_E_INVAL;
+  *c = ctx->ctr;
+  if (reset) ctx->ctr = dyo_counters{};
+  return DYO_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,159 @@
+// Internal structures of libdyo (not part of the ABI). See include/dyo.h and DESIGN.md.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/dyo.h"
+
+namespace dyo {
+
+constexpr int kSat = (1 << 24) - 1;       // R1(iii)
+constexpr int kMaxSites = 4096;
+constexpr int kEntCap = 1024;             // tensor-set entries per group (records before dedupe)
+constexpr int kPlanThreads = 512;
+
+enum OpClass : int8_t { C_KEEP = 0, C_CARRY = 1, C_ALLOC = 2, C_FETCH = 3 };
+
+// ---- pilot --------------------------------------------------------------------------
+constexpr int kMaxLayers = 16;
+struct LayerDev {
+  const float* W;    // out x in_pad (rows padded to a multiple of 4 floats)
+  const float* b;    // out
+  int in_off;        // offset of this layer's input in the stage input vector
+  int in_len;
+  int in_pad;
+  int out_off;       // offset in the stage output vector
+  int out_len;
+};
+struct StageDev {
+  int first_layer, n_layers;
+  int in_width, out_width;   // widths of the stage input / output vectors
+  int act;                   // 1: LeakyReLU
+  int rows;                  // total output rows of the stage
+};
+struct PilotDev {
+  int F, O;
+  int n_stages;
+  int max_width;            // largest stage in/out width (smem sizing)
+  float slope;
+  StageDev st[4 + kMaxLayers];
+  LayerDev ly[3 * kMaxLayers + 8];
+};
+
+// ---- arch on the device -------------------------------------------------------------
+struct ArchDev {
+  int T, n_ops, n_sites, n_pieces, nn_type, S_max, D_s, h, K_max, F, O, n_branch_logits;
+  int L_max;
+  int64_t H, align;
+  // tensors
+  const int64_t* t_bytes;
+  const int64_t* t_abytes;   // aligned
+  const int64_t* t_host;
+  const int32_t* t_flags;
+  // operators
+  const int32_t* op_sig;     // n_ops x 9 (saturated)
+  const int32_t* acc_ptr;    // n_ops + 1
+  const int32_t* acc_t;
+  const int32_t* acc_m;
+  // sites (preorder IF/LOOP)
+  const int32_t* site_kind;  // 1 IF, 2 LOOP
+  const int32_t* site_nch;   // choices
+  const int32_t* site_lo;
+  const int32_t* site_tie;
+  const int32_t* site_logit; // logit offset (absolute in the O vector) or -1 (tied)
+  const int32_t* site_arm_ptr;   // IF: site -> first arm index; arms give (first op, n ops)
+  const int32_t* arm_first_op;
+  const int32_t* arm_nops;
+  // top-level pieces: kind 0 static run (a = first op, b = n ops), 1 IF (a = site),
+  // 2 LOOP (a = site, b = body first op, c = body n ops)
+  const int32_t* piece_kind;
+  const int32_t* piece_a;
+  const int32_t* piece_b;
+  const int32_t* piece_c;
+  const int32_t* seg_table;  // S_max x 10
+};
+
+// ---- prediction storage -------------------------------------------------------------
+struct PredDev {
+  int B;
+  int32_t* K;         // B
+  int32_t* L;         // B
+  int32_t* choices;   // B x n_sites
+  int32_t* slots;     // B x K_max x 10 (decoded block head)
+  int32_t* path;      // B x L_max (operator index, -1 control)
+  int32_t* grp;       // B x K_max x 2 (start, end rows)
+  int32_t* blocks;    // B x K_max x 10 executed block vectors
+  int32_t* ent_n;     // B x K_max entry counts
+  int2* ent;          // B x K_max x kEntCap (t, mode | needs_fetch << 2)
+  int32_t* status;    // decode status word (0 ok, else DYO_E_*), [1] = detail
+};
+
+// ---- planner state (device) -----------------------------------------------------------
+struct PlanState {
+  int8_t* loc;        // T: -1 host, 0/1 half
+  int64_t* off;       // T: offset within the half
+  uint8_t* dirty;     // T
+  uint8_t* pw;        // T: written by the previous group
+  int32_t* res;       // 2 x T: tensors of each half, ascending offset
+  int32_t* res_n;     // 2
+  int32_t* prev;      // T: entries of the previous group (ids)
+  int32_t* prev_n;    // 1
+  int64_t* G;         // 1
+};
+
+struct PlanHdr {      // per transition (device + pinned mirror)
+  int32_t half, n_ent, n_evict, n_move, n_carry, n_alloc, n_fetch, pad;
+  int64_t need, h2d, d2h, d2d;
+  int64_t o_ent, o_evict, o_move, o_carry, o_alloc, o_fetch;  // record offsets
+};
+
+struct PlanOut {
+  PlanHdr* hdr;          // max_groups
+  dyo_entry_rec* ent;
+  dyo_evict_rec* ev;
+  dyo_move_rec* mv;
+  dyo_carry_rec* ca;
+  dyo_alloc_rec* al;
+  dyo_fetch_rec* fe;
+  int64_t cap_ent, cap_rec;
+  int32_t* status;       // [0] status, [1] failing transition, [2] needed capacity
+  int32_t* counts;       // [0..5] total records written per list
+};
+
+struct PlanScratch {
+  int8_t* inw;          // T
+  int32_t* cur_next;    // T
+  uint8_t* cur_rd;      // T
+  int32_t* nxt;         // max_groups x kEntCap : next occurrence of each entry
+  uint8_t* nxt_rd;
+  int8_t* rstat;        // T: resident status during a transition
+  uint64_t* keys;       // 2 x sort capacity (global fallback)
+  int64_t* gap_s;       // T + 1
+  int64_t* gap_e;
+  int32_t* kept;        // T
+  int64_t* newoff;      // T
+  int64_t* ebase;       // max_groups: first entry record of each planned group
+  int32_t* grp_b;       // max_groups: prediction of each planned group
+  int32_t* grp_k;
+};
+
+// ---- launchers (implemented in the .cu files) ------------------------------------------
+cudaError_t launch_encode(const ArchDev& a, const int64_t* desc, const int32_t* hist,
+                          const int32_t* hist_tab, const int32_t* hist_len, int B, float* feat,
+                          cudaStream_t s);
+cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_or_null,
+                         const int64_t* desc, const int32_t* hist, const int32_t* hist_tab,
+                         const int32_t* hist_len, int B, float* logits, int* cluster_used,
+                         cudaStream_t s);
+cudaError_t launch_decode(const ArchDev& a, const float* logits, PredDev& pd, int B,
+                          int32_t* hist_tab_out, int32_t* hist_len_out, cudaStream_t s);
+cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,
+                        PlanState& in, PlanState& work, PlanScratch& sc, PlanOut& out,
+                        int max_groups, cudaStream_t s);
+struct CopySeg { const char* src; char* dst; int64_t bytes; };
+cudaError_t launch_copy_segments(const CopySeg* segs_dev_or_mapped, int n, int64_t chunk,
+                                 int grid, cudaStream_t s);
+
+}  // namespace dyo

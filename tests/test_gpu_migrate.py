@@ -1,0 +1,130 @@
+"""GPU migration parity: bytes moved by dyo_migrate (DMA / pack / zero-copy / D2D kernels)
+against the oracle's plan and version model, with emulated compute between transitions."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import workloads as WL
+from oracle import plan as PL, migrate as M
+from gpu_harness import make_ctx, oracle_step, hist_for, tr_lists, gpu_lists, F_NO_ZEROCOPY, F_NO_PACK
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+
+
+class _Dev:
+    def __init__(self, ptr, n):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": "|u1", "data": (ptr, False), "version": 3}
+
+
+def _arena(d):
+    base, H = d.arena()
+    return torch.as_tensor(_Dev(base, 2 * H), device="cuda"), H
+
+
+def _words(t, v, nb):
+    return WL.content_words_torch(t, v, nb // 4, "cuda")
+
+
+def _check_dev(arena, dst, t, v, nb):
+    got = arena[dst: dst + nb].view(torch.int32)
+    return bool(torch.equal(got, _words(t, v, nb)))
+
+
+def run_bytes(wl, steps, policy=None, flags=0, dma_min=0):
+    for t in wl.tensors:
+        assert t.nbytes % 4 == 0
+    d = make_ctx(wl, flags=flags, policy=policy, dma_min_bytes=dma_min)
+    pool = d.host_pool_array()
+    for t, ten in enumerate(wl.tensors):
+        pool[ten.host_off: ten.host_off + ten.nbytes] = M.content_bytes(t, 0, ten.nbytes)
+    arena, H = _arena(d)
+    stream = torch.cuda.current_stream()
+    st = PL.initial_state(len(wl.tensors))
+    table = ()
+    ver = [0] * len(wl.tensors)
+    mech = {"dma": 0, "zc": 0, "packed": 0}
+    for s in range(steps):
+        r = oracle_step(wl, [s % len(wl.samples)], st, table, policy)
+        assert r["err"] is None
+        d.predict(wl.samples[[s % len(wl.samples)]].copy(), hist_for(wl, 1), 1, stream=stream.cuda_stream)
+        K = d.plan(stream=stream.cuda_stream)
+        assert K == len(r["trs"])
+        fresh = set()
+        Ws = [Wj for p in r["preds"] for Wj in p.W]
+        for j, tr in enumerate(r["trs"]):
+            assert gpu_lists(d, j) == tr_lists(tr)
+            d.migrate(j, stream.cuda_stream)
+            ent = d.plan_records(j, "entries")
+            for (t, mode, rd, dst) in ent.tolist():
+                nb = wl.tensors[t].nbytes
+                if rd and (not wl.tensors[t].transient or t in fresh):
+                    assert _check_dev(arena, dst, t, ver[t], nb), f"step {s} block {j}: tensor {t} stale"
+            for (t, mode, rd, dst) in ent.tolist():
+                if mode & 2:
+                    ver[t] += 1
+                    fresh.add(t)
+                    nb = wl.tensors[t].nbytes
+                    arena[dst: dst + nb].view(torch.int32).copy_(_words(t, ver[t], nb))
+        st = r["state"]
+        table = r["table"]
+        torch.cuda.synchronize()
+        c = d.counters(reset=True)
+        mech["dma"] += c["h2d_dma"] + c["d2h_dma"]
+        mech["zc"] += c["h2d_zc"] + c["d2h_zc"]
+        mech["packed"] += c["d2h_packed"]
+        # every resident non-transient tensor holds its latest bytes on the device (I2 + moves)
+        for t, ten in enumerate(wl.tensors):
+            if st.loc[t] != PL.HOST and not ten.transient:
+                assert _check_dev(arena, st.loc[t] * H + st.off[t], t, ver[t], ten.nbytes), f"resident {t}"
+    # I5: host homes of non-resident non-transient tensors hold their latest bytes
+    for t, ten in enumerate(wl.tensors):
+        if st.loc[t] == PL.HOST and not ten.transient:
+            assert np.array_equal(pool[ten.host_off: ten.host_off + ten.nbytes],
+                                  M.content_bytes(t, ver[t], ten.nbytes)), f"host home of {t}"
+    d.close()
+    return mech
+
+
+@pytest.mark.parametrize("policy", [0, 1])
+def test_tiny_fullsize_default_mechanisms(policy):
+    wl = WL.make("tiny", n_samples=16)
+    m = run_bytes(wl, 4, policy)
+    assert m["dma"] > 0
+
+
+def test_tiny_all_zero_copy():
+    wl = WL.make("tiny", n_samples=16)
+    m = run_bytes(wl, 3, 1, dma_min=1 << 40)
+    assert m["dma"] == 0 and m["zc"] > 0
+
+
+@pytest.mark.parametrize("flags", [0, F_NO_PACK, F_NO_ZEROCOPY])
+def test_tiny_tight_budget_writebacks(flags):
+    wl = WL.make("tiny", seed=2, n_samples=16)
+    wl.budget = 384 << 20
+    run_bytes(wl, 6, 0, flags=flags)
+
+
+def test_moe_scaled_tied_routing_gradients():
+    wl = WL.make_moe(seed=1, n_samples=8, expert_mib=1, act_mib=1, budget=96 << 20)
+    m = run_bytes(wl, 4, 1, dma_min=1 << 20)
+    assert m["dma"] > 0
+
+
+def test_af_scaled_recycling():
+    wl = WL.make_af(seed=1, n_samples=8, act_mib=1, weight_mib=1, blocks=8, budget=64 << 20)
+    for t in wl.tensors:
+        t.nbytes = min(t.nbytes, 1 << 20)     # MSA/pair state scaled to 1 MiB too
+    off = 0
+    for t in wl.tensors:
+        t.host_off = off
+        off += (t.nbytes + 255) // 256 * 256
+    run_bytes(wl, 3, 1)

@@ -1,0 +1,153 @@
+"""GPU parity: libdyo (through its C ABI) against the CPU oracle, element by element."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import workloads as WL
+from oracle import plan as PL, afm as A
+from gpu_harness import (make_ctx, oracle_step, hist_for, tr_lists, gpu_lists, logit_gates,
+                         F_NO_HOST_POOL)
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+
+
+def _stream():
+    return torch.cuda.current_stream().cuda_stream
+
+
+@pytest.mark.parametrize("name", ["tiny", "moe", "af"])
+def test_encode_bitexact(name):
+    wl = WL.make(name)
+    B = 4
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    feat = torch.zeros((B, wl.pilot.F), device="cuda")
+    d.encode(wl.samples[:B].copy(), hist_for(wl, B), B, feat, _stream())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), ())
+    got = feat.cpu().numpy().astype(np.float64)
+    assert np.array_equal(got, np.stack(r["feats"]))
+    # after a prediction the history table is the executed block vectors (R3)
+    d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, stream=_stream())
+    d.encode(wl.samples[B:2 * B].copy(), hist_for(wl, B), B, feat, _stream())
+    r2 = oracle_step(wl, range(B, 2 * B), PL.initial_state(len(wl.tensors)), r["table"])
+    assert np.array_equal(feat.cpu().numpy().astype(np.float64), np.stack(r2["feats"]))
+    d.close()
+
+
+@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 16), ("moe", 1), ("moe", 8), ("af", 1), ("af", 3)])
+def test_pilot_logits(name, B):
+    wl = WL.make(name, n_samples=max(16, B))
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    logits = torch.zeros((B, wl.pilot.O), device="cuda")
+    d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, stream=_stream())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), ())
+    y = logits.cpu().numpy()
+    n1 = 0
+    for b in range(B):
+        g1, g2, o = logit_gates(y[b], r["feats"][b], wl.pilot, wl.nn_type)
+        assert g2.all(), f"fp32 error bound violated at {np.where(~g2)[0][:5]}"
+        n1 += int((~g1).sum())
+    assert n1 == 0, f"{n1} logits outside 1e-5 relative (floored)"
+    d.close()
+
+
+def _check_prediction(d, wl, b, pred):
+    K, blocks, choices, rows = d.prediction(b, wl.K_max, len(A.sites(wl.program)), _stream())
+    assert K == len(pred.groups)
+    assert [tuple(r) for r in rows.tolist()] == pred.groups
+    assert [tuple(v) for v in blocks.tolist()] == [tuple(v) for v in pred.blocks]
+    assert choices.tolist() == pred.choices
+    for g in range(K):
+        ent = d.group_entries(b, g, stream=_stream())
+        assert [tuple(e) for e in ent.tolist()] == [(t, m, int(f)) for t, m, f in pred.W[g]], f"group {g}"
+
+
+@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 8), ("moe", 1), ("moe", 4), ("af", 2)])
+def test_decode(name, B):
+    wl = WL.make(name, n_samples=max(16, B))
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, stream=_stream())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), ())
+    for b in range(B):
+        assert not r["preds"][b].near_ties
+        _check_prediction(d, wl, b, r["preds"][b])
+    d.close()
+
+
+def _run_plan_steps(wl, steps, B=1, policy=None, flags=F_NO_HOST_POOL):
+    d = make_ctx(wl, max_batch=B, flags=flags, policy=policy)
+    st = PL.initial_state(len(wl.tensors))
+    table = ()
+    for s in range(steps):
+        ids = [(s * B + i) % len(wl.samples) for i in range(B)]
+        r = oracle_step(wl, ids, st, table, policy)
+        d.predict(wl.samples[ids].copy(), hist_for(wl, B), B, stream=_stream())
+        if r["err"] is not None:
+            with pytest.raises(Exception) as ei:
+                d.plan(stream=_stream())
+            assert getattr(ei.value, "status", None) == -3
+        else:
+            K = d.plan(stream=_stream())
+            assert K == len(r["trs"])
+            for j, tr in enumerate(r["trs"]):
+                info = d.plan_info(j)
+                assert (info["half"], info["h2d"], info["d2h"], info["d2d"], info["need"]) == \
+                    (tr.half, tr.h2d, tr.d2h, tr.d2d, tr.need), f"step {s} transition {j}"
+                assert gpu_lists(d, j) == tr_lists(tr), f"step {s} transition {j}"
+            st = r["state"]
+        table = r["table"]
+    return d
+
+
+@pytest.mark.parametrize("policy", [0, 1])
+@pytest.mark.parametrize("name,steps,B", [("tiny", 8, 1), ("tiny", 3, 8), ("moe", 6, 1), ("af", 3, 1)])
+def test_plan_bitexact(name, steps, B, policy):
+    wl = WL.make(name, n_samples=32)
+    _run_plan_steps(wl, steps, B, policy).close()
+
+
+@pytest.mark.parametrize("budget_mib", [160, 256, 384])
+def test_plan_tight_budgets_and_errors(budget_mib):
+    """Tight budgets: evictions with writeback, compaction, and DYO_E_BUDGET (transactional)."""
+    wl = WL.make("tiny", n_samples=32)
+    wl.budget = budget_mib << 20
+    _run_plan_steps(wl, 10, 1, 0).close()
+    _run_plan_steps(wl, 10, 1, 1).close()
+
+
+def test_unplanted_pilot_random_partitions():
+    wl = WL.make("tiny", n_samples=32)
+    wl2 = WL.make_tiny(seed=3, n_samples=32, planted=False)
+    wl2.budget = 4 << 30
+    _run_plan_steps(wl2, 4, 1, 1).close()
+    _ = wl
+
+
+def test_state_unchanged_after_budget_error():
+    wl = WL.make("tiny", n_samples=32)
+    d = make_ctx(wl, max_batch=1, flags=F_NO_HOST_POOL)
+    st = PL.initial_state(len(wl.tensors))
+    r0 = oracle_step(wl, [0], st, ())
+    d.predict(wl.samples[[0]].copy(), None, 1, stream=_stream())
+    d.plan(stream=_stream())
+    # a prediction whose group needs more than H: an all-zero block head -> one group = whole path
+    big = WL.make_tiny(seed=0, n_samples=32, planted=False)
+    big.pilot.weights["out.W"][:80] = 0
+    big.pilot.weights["out.b"][:80] = 0
+    d2 = make_ctx(big, max_batch=1, flags=F_NO_HOST_POOL)
+    d2.predict(big.samples[[0]].copy(), None, 1, stream=_stream())
+    with pytest.raises(Exception):
+        d2.plan(stream=_stream())
+    # after the failure the committed state is the initial one: a feasible plan matches the oracle
+    d2.load_pilot(wl.pilot)
+    d2.predict(wl.samples[[0]].copy(), None, 1, stream=_stream())
+    K = d2.plan(stream=_stream())
+    assert K == len(r0["trs"]) and gpu_lists(d2, 0) == tr_lists(r0["trs"][0])
+    d.close(); d2.close()

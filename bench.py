@@ -1,0 +1,399 @@
+#!/usr/bin/env python
+"""Benchmark of the DyNN-Offload hot path (pilot -> decode -> plan -> migrate) on B200.
+
+One *step* = one training sample of the workload: dyo_pilot_predict (fused encode + pilot MLP +
+decode) -> dyo_plan (planner kernel + the one host sync) -> dyo_migrate(j) for every predicted
+transition (DMA + copy kernels on a side copy stream). The headline metric (BASELINE.json) is
+"pilot us/prediction; plan us; migration H2D/D2H GB/s vs PCIe Gen5 x16 peak"; `value` is the
+whole-job migration throughput (algorithmic H2D + D2H bytes / step time, all ranks), and the
+pilot / plan / per-direction numbers ride along in the same line.
+
+  python bench.py [--gpus N --steps K --warmup W --config moe|tiny|af --policy 0|1]
+  python bench.py --impl reference ...   (the CPU oracle, timed on the host cores)
+
+Workload: BASELINE configs[1] (switch-MoE, 16 experts, 8x oversubscribed expert pool) unless
+--config says otherwise. Inputs are synthetic (workloads/, seeded); every step moves >= 1 GiB
+through HBM and PCIe, far above the 126 MB L2 ("inputs larger than L2").
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PCIE_GEN5_X16 = 63.0          # GB/s per direction, 32 GT/s x 16 x 128/130 / 8 (theoretical)
+DYO_F_TIMING = 8
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="dyo", choices=["dyo", "reference"])
+    ap.add_argument("--config", default="moe", choices=["moe", "tiny", "af"])
+    ap.add_argument("--policy", type=int, default=1)
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--budget-gib", type=float, default=0.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--dist-backend", default="nccl")
+    return ap.parse_args()
+
+
+CONFIG_DESC = {
+    "moe": "switch-MoE top-1 trace, 24 layers x 16 experts (32 MiB W_in/W_out, grads written back), "
+           "3 GiB budget = 8x oversubscribed expert pool, P512 pilot (BASELINE configs[1])",
+    "tiny": "tiny trace: 8 groups, 64 tensors, T32 pilot, 1 GiB budget (BASELINE configs[0])",
+    "af": "AlphaFold-Evoformer-shaped trace, 48 blocks x recycle 1..4, MSA 128x256, 2 GiB budget (BASELINE configs[2])",
+}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except OSError:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0}, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    def __init__(self, index=0):
+        self.samples = []
+        self.proc = None
+        self.index = index
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            threading.Thread(target=self._read, daemon=True).start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.samples.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if len(s) > 3 + i and s[3 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def make_workload(args, rank):
+    import workloads as WL
+    wl = WL.make(args.config, seed=args.seed + rank, n_samples=64)
+    wl.policy = args.policy
+    if args.budget_gib > 0:
+        wl.budget = int(args.budget_gib * (1 << 30))
+    return wl
+
+
+# ---------------------------------------------------------------------------------------------
+# CPU oracle legs (the only place bench.py executes oracle/)
+# ---------------------------------------------------------------------------------------------
+
+def oracle_steps(wl, n_steps, budget_s=None):
+    """Run the oracle as it stands for n_steps samples: encode, pilot (fp64), decode, plan (pure
+    Python), then the step's algorithmic bytes copied by numpy between a host buffer pair (the
+    oracle's byte model moves exactly these bytes; full-size arenas do not fit its numpy model,
+    so the copy runs through 256 MiB buffers). Returns (bytes, seconds, steps_done)."""
+    import numpy as np
+    from threadpoolctl import threadpool_limits
+    from oracle import run as OR, plan as PL
+    st = PL.initial_state(len(wl.tensors))
+    table = ()
+    buf_a = np.ones(256 << 20, np.uint8)
+    buf_b = np.zeros(256 << 20, np.uint8)
+    total_b, t0, done = 0, time.perf_counter(), 0
+    with threadpool_limits(limits=1):
+        for s in range(n_steps):
+            r = OR.step(wl, s % len(wl.samples), st, table)
+            st, table = r.state, r.pred.blocks
+            nbytes = sum(t.h2d + t.d2h for t in r.transitions)
+            left = nbytes
+            while left > 0:
+                n = min(left, buf_a.size)
+                np.copyto(buf_b[:n], buf_a[:n])
+                left -= n
+            total_b += nbytes
+            done += 1
+            if budget_s is not None and time.perf_counter() - t0 > budget_s:
+                break
+    return total_b, time.perf_counter() - t0, done
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    wl = make_workload(args, 0)
+    oracle_steps(wl, max(args.warmup, 1))
+    b, sec, n = oracle_steps(wl, args.steps)
+    v = b / sec / 1e9
+    out = {"metric": "migration GB/s (pilot us/prediction; plan us; H2D/D2H vs PCIe Gen5 x16)",
+           "impl": "reference", "value": round(v, 4), "unit": "GB/s", "n_gpus": args.gpus, "steps": n,
+           "warmup": args.warmup, "ms_per_step": round(sec / n * 1e3, 3), "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f64 pilot / int64 plan / u8 bytes",
+           "data": "synthetic", "config": {"workload": args.config, "desc": CONFIG_DESC[args.config]},
+           "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                            "sample": f"{n} full oracle steps (pure Python encode/pilot/decode/plan + numpy copy of "
+                                      f"the step's algorithmic bytes), 1 host core"},
+           "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+# ---------------------------------------------------------------------------------------------
+# B200 leg
+# ---------------------------------------------------------------------------------------------
+
+def pcie_probe(torch, nbytes=256 << 20, reps=5):
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    s = torch.cuda.Stream()
+    res = {}
+    for name, (dst, src) in (("h2d", (d, h)), ("d2h", (h, d))):
+        with torch.cuda.stream(s):
+            dst.copy_(src, non_blocking=True)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            for _ in range(reps):
+                dst.copy_(src, non_blocking=True)
+            b.record(s)
+        b.synchronize()
+        res[name] = nbytes * reps / (a.elapsed_time(b) * 1e-3) / 1e9
+    del h, d
+    return res
+
+
+def run_dyo(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_hpca_renxyzlnwxl24_b200 import Dyo
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group(args.dist_backend)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+
+    wl = make_workload(args, rank)
+    d = Dyo(wl.budget, wl.align, wl.policy, max_batch=1, device=local, flags=DYO_F_TIMING)
+    d.load(wl)
+    s0 = torch.cuda.current_stream()
+    s1 = torch.cuda.Stream()
+    desc_dev = torch.from_numpy(wl.samples.copy()).to(dev)
+    hist_np = wl.hist_ids.astype(np.int32).reshape(1, -1) if wl.h else None
+    hist_dev = torch.from_numpy(hist_np).to(dev) if hist_np is not None else None
+    nS = len(wl.samples)
+
+    def step(i, desc, hist):
+        d.predict(desc, hist, 1, stream=s0.cuda_stream)
+        K = d.plan(stream=s0.cuda_stream)
+        byt = 0
+        h2d = d2h = 0
+        for j in range(K):
+            info = d.plan_info(j)
+            h2d += info["h2d"]
+            d2h += info["d2h"]
+            d.migrate(j, s1.cuda_stream)
+        return K, h2d, d2h
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for i in range(args.warmup):
+        step(i, desc_dev[i % nS: i % nS + 1], hist_dev)
+    barrier()
+    d.timings(reset=True)
+    d.counters(reset=True)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    tot_h2d = tot_d2h = tot_K = 0
+    plan_wall = []
+    with Clocks(local) as clk:
+        e0.record(s0)
+        for i in range(args.steps):
+            k = (args.warmup + i) % nS
+            K, h2d, d2h = step(i, desc_dev[k: k + 1], hist_dev)
+            tot_K += K
+            tot_h2d += h2d
+            tot_d2h += d2h
+        s0.wait_stream(s1)
+        e1.record(s0)
+        e1.synchronize()
+    barrier()
+    ms = e0.elapsed_time(e1)
+    tm = d.timings(reset=True)
+    ctr = d.counters(reset=True)
+
+    # e2e: the same steps through the public API with HOST inputs (pinned), results read back
+    desc_host = torch.from_numpy(wl.samples.copy()).pin_memory()
+    hist_host = torch.from_numpy(hist_np).pin_memory() if hist_np is not None else None
+    barrier()
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        k = (args.warmup + args.steps + i) % nS
+        step(i, desc_host[k: k + 1].numpy(), hist_host.numpy() if hist_host is not None else None)
+    s1.synchronize()
+    barrier()
+    e2e_s = time.perf_counter() - t0
+    e2e_bytes = None
+
+    # pilot latency: back-to-back predictions (device time per prediction) and kernel-only
+    d.timings(reset=True)
+    n_pred = 200
+    p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    p0.record(s0)
+    for i in range(n_pred):
+        d.predict(desc_dev[i % nS: i % nS + 1], hist_dev, 1, stream=s0.cuda_stream)
+    p1.record(s0)
+    p1.synchronize()
+    pred_us = p0.elapsed_time(p1) * 1e3 / n_pred
+    tp = d.timings(reset=True)
+    pilot_kernel_us = tp["pilot"]["ms"] * 1e3 / max(1, tp["pilot"]["launches"])
+    decode_us = tp["decode"]["ms"] * 1e3 / max(1, tp["decode"]["launches"])
+    probe = pcie_probe(torch)
+
+    # max over ranks
+    tt = torch.tensor([ms, e2e_s, float(tot_h2d + tot_d2h), float(tot_h2d), float(tot_d2h)], device=dev, dtype=torch.float64)
+    if world > 1:
+        mx = tt.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        sm = tt.clone()
+        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+        ms_max, e2e_max = mx[0].item(), mx[1].item()
+        bytes_all, h2d_all, d2h_all = sm[2].item(), sm[3].item(), sm[4].item()
+    else:
+        ms_max, e2e_max = ms, e2e_s
+        bytes_all, h2d_all, d2h_all = float(tot_h2d + tot_d2h), float(tot_h2d), float(tot_d2h)
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        d.close()
+        return
+
+    peaks, peak_src = measured_peaks()
+    value = bytes_all / (ms_max * 1e-3) / 1e9
+    # dominant kernel of the timed region among libdyo's kernels
+    kern = {k: tm[k] for k in ("pilot", "decode", "plan", "copy_d2d", "copy_zc")}
+    dom = max(kern, key=lambda k: kern[k]["ms"])
+    km = kern[dom]
+    avg_ms = km["ms"] / max(1, km["launches"])
+    if dom == "copy_d2d":
+        alg = 2.0 * km["bytes"] / max(1, km["launches"])          # read + write per launch
+        achieved = alg / (avg_ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": round(achieved, 2), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": None, "kernel": "copy_segments_kernel",
+                "peak_source": peak_src, "alg_bytes_per_launch": alg, "avg_launch_us": avg_ms * 1e3}
+    elif dom == "copy_zc":
+        alg = km["bytes"] / max(1, km["launches"])
+        achieved = alg / (avg_ms * 1e-3) / 1e9
+        roof = {"bound": "pcie", "achieved": round(achieved, 2), "peak": PCIE_GEN5_X16, "unit": "GB/s",
+                "frac": round(achieved / PCIE_GEN5_X16, 4), "traffic": None, "kernel": "copy_segments_kernel (zero-copy)",
+                "peak_source": "theoretical PCIe Gen5 x16", "alg_bytes_per_launch": alg, "avg_launch_us": avg_ms * 1e3}
+    else:
+        roof = {"bound": "latency", "achieved": round(avg_ms * 1e3, 2), "peak": None, "unit": "us/launch",
+                "frac": None, "traffic": None, "kernel": dom, "avg_launch_us": avg_ms * 1e3}
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            tr = json.load(f)
+        if roof["kernel"].split()[0] in tr:
+            roof["traffic"] = tr[roof["kernel"].split()[0]]
+    except OSError:
+        pass
+    shares = {k: round(v["ms"] / ms, 4) for k, v in tm.items()}
+    dma_h2d = tm["dma_h2d"]
+    dma_d2h = tm["dma_d2h"]
+    h2d_link = dma_h2d["bytes"] / (dma_h2d["ms"] * 1e-3) / 1e9 if dma_h2d["ms"] else None
+    d2h_link = dma_d2h["bytes"] / (dma_d2h["ms"] * 1e-3) / 1e9 if dma_d2h["ms"] else None
+    plan_us = tm["plan"]["ms"] * 1e3 / max(1, tm["plan"]["launches"])
+    launches = (tm["pilot"]["launches"] + 3 * tm["decode"]["launches"] + tm["plan"]["launches"]
+                + tm["copy_d2d"]["launches"] + tm["copy_zc"]["launches"])
+
+    out = {
+        "metric": "migration GB/s (pilot us/prediction; plan us; H2D/D2H vs PCIe Gen5 x16)",
+        "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(ms_max / args.steps, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32 weights / f64 accumulate (pilot); int64 (plan); u8 (migrate)",
+        "data": "synthetic",
+        "config": {"workload": args.config, "desc": CONFIG_DESC[args.config], "policy": "RETAIN" if args.policy else "PAPER",
+                   "budget_bytes": wl.budget, "tensors": len(wl.tensors),
+                   "l2": "inputs larger than L2 (every step moves >= 1 GiB through HBM and PCIe)",
+                   "parallelism": f"{world} independent managers (replicas, no collective on the path)"},
+        "pilot_us_per_prediction": round(pred_us, 3),
+        "pilot_kernel_us": round(pilot_kernel_us, 3), "decode_kernels_us": round(decode_us, 3),
+        "predictions_per_s": round(1e6 / pred_us, 1),
+        "plan_us": round(plan_us, 2), "transitions_per_step": round(tot_K / args.steps, 2),
+        "h2d_bytes_per_step": int(h2d_all / args.steps / world), "d2h_bytes_per_step": int(d2h_all / args.steps / world),
+        "pcie": {"h2d_dma_gbs": round(h2d_link, 2) if h2d_link else None,
+                 "d2h_dma_gbs": round(d2h_link, 2) if d2h_link else None,
+                 "peak_theoretical_gbs": PCIE_GEN5_X16,
+                 "probe_h2d_gbs": round(probe["h2d"], 2), "probe_d2h_gbs": round(probe["d2h"], 2),
+                 "frac_h2d_of_theoretical": round(h2d_link / PCIE_GEN5_X16, 4) if h2d_link else None,
+                 "frac_d2h_of_theoretical": round(d2h_link / PCIE_GEN5_X16, 4) if d2h_link else None,
+                 "step_gbs_per_gpu": round(value / world, 3)},
+        "roofline": roof,
+        "time_shares": shares,
+        "mechanisms": ctr,
+        "gpu_launches": int(launches),
+        "clocks": clk.summary(),
+        "e2e": {"value": round(bytes_all / e2e_max / 1e9, 3), "unit": "GB/s",
+                "h2d_bytes_per_step": int(wl.D_s * 8 + wl.h * 4), "d2h_bytes_per_step": int(16 * 4 + 9 * len(wl.tensors)),
+                "note": "dyo_* calls with pinned host sample descriptors; plan lists + residency read back each step"},
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        import os as _os
+        b, sec, n = oracle_steps(wl, 200, budget_s=15.0)
+        out["cpu_baseline"] = {"value": round(b / sec / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                               "sample": f"{n} oracle steps of the same workload (pure Python encode/pilot/decode/plan + "
+                                         f"numpy copy of each step's algorithmic bytes), ~15 s, 1 of {_os.cpu_count()} cores"}
+    print(json.dumps(out), flush=True)
+    d.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_dyo(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -122,7 +122,7 @@ typedef struct {
   int32_t out_in;
   const float* out_W;           /* O x out_in */
   const float* out_b;           /* O */
-  float slope;                  /* LeakyReLU negative slope (0.01, R5) */
+  double slope;                 /* LeakyReLU negative slope (0.01, R5) */
 } dyo_pilot_desc;
 
 /* One batch of samples. desc: B x D_s int64 shape descriptors; hist_ids: B x h int32 history
@@ -193,7 +193,7 @@ dyo_status dyo_encode_features(dyo_ctx* ctx, const dyo_sample* s, int32_t B, flo
                                void* stream);
 
 /* A2 + A3: pilot forward for B samples (feat = NULL: fused encode from s; else device B x F
- * features) and decode (R4) into ctx-owned device storage; logits (device B x O fp32) may be
+ * features) and decode (R4) into ctx-owned device storage; logits (device B x O fp32 copy of the fp64 logits the decode uses) may be
  * NULL. Asynchronous; decode errors surface at dyo_plan. After the call the history table is
  * the executed block vectors of these predictions (in sample order). */
 dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* s, int32_t B,

@@ -36,7 +36,7 @@ struct dyo_ctx {
   int64_t host_bytes = 0;
   // prediction
   PredDev pd{};
-  float* logits_scratch = nullptr;
+  double* logits64 = nullptr;      // fp64 logits (decode decisions, R4)
   int64_t* desc_dev = nullptr;
   int32_t* hist_dev = nullptr;
   int32_t* hist_tab[2] = {nullptr, nullptr};
@@ -646,9 +646,9 @@ dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   p.max_width = (maxw + 3) / 4 * 4;
   ctx->ad.O = w->O;
   CK(cudaFree(nullptr));
-  float* lg = nullptr;
+  double* lg = nullptr;
   if ((s = dalloc(ctx, ctx->pilot_dev, &lg, (size_t)ctx->cfg.max_batch * w->O))) return s;
-  ctx->logits_scratch = lg;
+  ctx->logits64 = lg;
   ctx->pilot_ok = true;
   return DYO_OK;
 }
@@ -721,15 +721,15 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
   } else if (!is_device_ptr(feat)) {
     return fail(ctx, DYO_E_INVAL, "feat must be device memory");
   }
-  float* lg = logits ? logits : ctx->logits_scratch;
   const int cur = ctx->hist_cur;
   {
     TScope ts(ctx, 0, st);
-    CK(launch_pilot(ctx->ad, ctx->pdv, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_len[cur], B, lg, nullptr, st));
+    CK(launch_pilot(ctx->ad, ctx->pdv, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_len[cur], B, ctx->logits64,
+                    logits, nullptr, st));
   }
   {
     TScope ts(ctx, 1, st);
-    CK(launch_decode(ctx->ad, lg, ctx->pd, B, ctx->hist_tab[1 - cur], ctx->hist_len[1 - cur], st));
+    CK(launch_decode(ctx->ad, ctx->logits64, ctx->pd, B, ctx->hist_tab[1 - cur], ctx->hist_len[1 - cur], st));
   }
   ctx->hist_cur = 1 - cur;
   ctx->last_B = B;

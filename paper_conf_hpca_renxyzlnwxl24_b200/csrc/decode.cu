@@ -19,9 +19,9 @@ constexpr int kMaxPieces = 1024;
 constexpr int kRecCap = 2048;      // access records per group before deduplication
 
 __global__ void __launch_bounds__(kDecThreads)
-decode_path_kernel(ArchDev a, const float* __restrict__ logits, PredDev pd) {
+decode_path_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd) {
   const int b = blockIdx.x;
-  const float* y = logits + (int64_t)b * a.O;
+  const double* y = logits + (int64_t)b * a.O;
   __shared__ int s_start[kMaxPieces + 1];
   __shared__ int s_ngroups, s_L;
   int32_t* choices = pd.choices + (int64_t)b * a.n_sites;
@@ -30,18 +30,18 @@ decode_path_kernel(ArchDev a, const float* __restrict__ logits, PredDev pd) {
   // 1. block head -> slots (R4): n = rint(y * 2^sigma), clamped to [0, 2^24-1]
   for (int i = threadIdx.x; i < a.K_max * 10; i += blockDim.x) {
     const int e = i % 10;
-    float t = y[i] * (e < 7 ? 16.f : 1024.f);
-    t = fminf(fmaxf(t, 0.f), (float)kSat);
-    slots[i] = (int)rintf(t);
+    double t = y[i] * (e < 7 ? 16.0 : 1024.0);
+    t = fmin(fmax(t, 0.0), (double)kSat);
+    slots[i] = (int)rint(t);
   }
   // 2. branch head -> choices (argmax, lowest index on ties)
   for (int i = threadIdx.x; i < a.n_sites; i += blockDim.x) {
     const int off = a.site_logit[i];
     if (off >= 0) {
       int best = 0;
-      float bv = y[off];
+      double bv = y[off];
       for (int c = 1; c < a.site_nch[i]; ++c) {
-        const float v = y[off + c];
+        const double v = y[off + c];
         if (v > bv) { bv = v; best = c; }
       }
       choices[i] = best;
@@ -274,7 +274,7 @@ __global__ void hist_compact_kernel(ArchDev a, PredDev pd, int B, int32_t* tab, 
   }
 }
 
-cudaError_t launch_decode(const ArchDev& a, const float* logits, PredDev& pd, int B,
+cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_len_out, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
   cudaMemsetAsync(pd.status, 0, 2 * sizeof(int32_t), s);

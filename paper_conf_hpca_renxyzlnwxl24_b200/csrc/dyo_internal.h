@@ -37,7 +37,7 @@ struct PilotDev {
   int F, O;
   int n_stages;
   int max_width;            // largest stage in/out width (smem sizing)
-  float slope;
+  double slope;
   StageDev st[4 + kMaxLayers];
   LayerDev ly[3 * kMaxLayers + 8];
 };
@@ -145,9 +145,9 @@ cudaError_t launch_encode(const ArchDev& a, const int64_t* desc, const int32_t* 
                           cudaStream_t s);
 cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_or_null,
                          const int64_t* desc, const int32_t* hist, const int32_t* hist_tab,
-                         const int32_t* hist_len, int B, float* logits, int* cluster_used,
-                         cudaStream_t s);
-cudaError_t launch_decode(const ArchDev& a, const float* logits, PredDev& pd, int B,
+                         const int32_t* hist_len, int B, double* logits64, float* logits32,
+                         int* cluster_used, cudaStream_t s);
+cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_len_out, cudaStream_t s);
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,
                         PlanState& in, PlanState& work, PlanScratch& sc, PlanOut& out,

@@ -42,7 +42,7 @@ class PilotDesc(C.Structure):
                 ("feat_out", PI32), ("feat_W", C.POINTER(PF32)), ("feat_b", C.POINTER(PF32)),
                 ("n_mlp", i32), ("mlp_in", PI32), ("mlp_out", PI32), ("mlp_W", C.POINTER(PF32)),
                 ("mlp_b", C.POINTER(PF32)), ("out_in", i32), ("out_W", PF32), ("out_b", PF32),
-                ("slope", f32)]
+                ("slope", C.c_double)]
 
 
 class Sample(C.Structure):

@@ -210,8 +210,10 @@ def run_dyo(args):
     dev = torch.device("cuda", local)
 
     wl = make_workload(args, rank)
+    _log("workload built")
     d = Dyo(wl.budget, wl.align, wl.policy, max_batch=1, device=local, flags=DYO_F_TIMING)
     d.load(wl)
+    _log("ctx loaded")
     s0 = torch.cuda.current_stream()
     s1 = torch.cuda.Stream()
     desc_dev = torch.from_numpy(wl.samples.copy()).to(dev)
@@ -219,16 +221,25 @@ def run_dyo(args):
     hist_dev = torch.from_numpy(hist_np).to(dev) if hist_np is not None else None
     nS = len(wl.samples)
 
+    # Zero-duration compute blocks: block j "starts" and "ends" when ready[j] fires, so transition
+    # j's EVICT waits ready[j-2] (its half's last user) and overlaps transition j-1's FETCH.
+    ready = [torch.cuda.Event() for _ in range(wl.K_max + 1)]
+    t_start = torch.cuda.Event()
+    for e in ready + [t_start]:
+        e.record(s1)                          # materialise the cudaEvent_t handles
+
     def step(i, desc, hist):
         d.predict(desc, hist, 1, stream=s0.cuda_stream)
         K = d.plan(stream=s0.cuda_stream)
-        byt = 0
         h2d = d2h = 0
+        t_start.record(s1)
         for j in range(K):
             info = d.plan_info(j)
             h2d += info["h2d"]
             d2h += info["d2h"]
-            d.migrate(j, s1.cuda_stream)
+            half_free = ready[j - 2] if j >= 2 else t_start
+            prev_done = ready[j - 1] if j >= 1 else t_start
+            d.migrate(j, s1.cuda_stream, half_free.cuda_event, prev_done.cuda_event, ready[j].cuda_event)
         return K, h2d, d2h
 
     def barrier():
@@ -236,6 +247,7 @@ def run_dyo(args):
             dist.barrier()
         torch.cuda.synchronize()
 
+    _log("warmup")
     for i in range(args.warmup):
         step(i, desc_dev[i % nS: i % nS + 1], hist_dev)
     barrier()
@@ -260,6 +272,7 @@ def run_dyo(args):
     tm = d.timings(reset=True)
     ctr = d.counters(reset=True)
 
+    _log("e2e")
     # e2e: the same steps through the public API with HOST inputs (pinned), results read back
     desc_host = torch.from_numpy(wl.samples.copy()).pin_memory()
     hist_host = torch.from_numpy(hist_np).pin_memory() if hist_np is not None else None
@@ -273,6 +286,7 @@ def run_dyo(args):
     e2e_s = time.perf_counter() - t0
     e2e_bytes = None
 
+    _log("pilot loop")
     # pilot latency: back-to-back predictions (device time per prediction) and kernel-only
     d.timings(reset=True)
     n_pred = 200
@@ -286,6 +300,7 @@ def run_dyo(args):
     tp = d.timings(reset=True)
     pilot_kernel_us = tp["pilot"]["ms"] * 1e3 / max(1, tp["pilot"]["launches"])
     decode_us = tp["decode"]["ms"] * 1e3 / max(1, tp["decode"]["launches"])
+    _log("probe")
     probe = pcie_probe(torch)
 
     # max over ranks
@@ -387,8 +402,17 @@ def run_dyo(args):
         dist.destroy_process_group()
 
 
+def _log(msg):
+    if os.environ.get("DYO_BENCH_VERBOSE"):
+        print(f"[bench {time.strftime('%H:%M:%S')}] {msg}", file=sys.stderr, flush=True)
+
+
 def main():
     args = parse()
+    wd = os.environ.get("DYO_BENCH_WATCHDOG")
+    if wd:
+        import faulthandler
+        faulthandler.dump_traceback_later(float(wd), exit=True)
     if args.impl == "reference":
         run_reference(args)
     else:

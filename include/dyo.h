@@ -222,12 +222,17 @@ dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info);
 dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** recs,
                             int32_t* n);
 
-/* A5: execute transition j (j = 0, 1, ... in order; DYO_E_STATE otherwise) on copy_stream:
- * wait ev_prev_started (block j-1 started => block j-2, the last user of half m, finished;
- * may be NULL), EVICT writebacks (D2H), MOVE (compaction through staging), CARRY (D2D) and
- * FETCH (H2D); late CARRYs wait ev_prev_done (block j-1 finished; may be NULL); then record
- * ev_ready (may be NULL), which block j must wait on. */
-dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev_started,
+/* A5: execute transition j (j = 0, 1, ... in order; DYO_E_STATE otherwise):
+ *   EVICT writebacks (D2H: DMA per host run, K3 pack + DMA for scattered sources, K5 zero-copy
+ *   for small runs) on a ctx-owned D2H stream, after ev_half_free = the end of block j-2, the
+ *   last user of half m (NULL: after everything already enqueued on copy_stream); then on
+ *   copy_stream: MOVE (compaction through staging), early CARRY (D2D), FETCH (H2D: DMA per host
+ *   run or one K5 zero-copy gather), late CARRY after ev_prev_done (end of block j-1; may be
+ *   NULL), and finally ev_ready (may be NULL), which block j must wait on.
+ * Because EVICT_j only waits for block j-2, it overlaps transition j-1's fetches (P:L176's
+ * double buffer; PCIe is full duplex). Host-non-blocking; all transitions of a plan may be
+ * enqueued at once. */
+dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half_free,
                        void* ev_prev_done, void* ev_ready);
 
 /* Device address of tensor t after the last planned transition that placed it (NULL if it is

@@ -37,7 +37,7 @@ def build(force=False, verbose=False):
         objs.append(o)
     for f in CPP:
         o = os.path.join(BUILD, f + ".o")
-        _run([NVCC, "-O2", "-std=c++17", "-Xcompiler", "-fPIC,-Wall", "-x", "cu", *ARCH,
+        _run([NVCC, "-O2", "-std=c++17", "-Xcompiler", "-fPIC,-Wall,-Wextra,-Werror=uninitialized,-Werror=init-self,-Wno-unused-parameter", "-x", "cu", *ARCH,
               "-c", os.path.join(CSRC, f), "-o", o])
         objs.append(o)
     _run([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", OUT, *objs])

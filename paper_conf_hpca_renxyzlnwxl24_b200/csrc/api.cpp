@@ -6,6 +6,7 @@
 #include <array>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -40,7 +41,8 @@ struct dyo_ctx {
   int64_t* desc_dev = nullptr;
   int32_t* hist_dev = nullptr;
   int32_t* hist_tab[2] = {nullptr, nullptr};
-  int32_t* hist_len[2] = {nullptr, nullptr};
+  int32_t* hist_K[2] = {nullptr, nullptr};   // groups per prediction of each history table
+  int hist_B[2] = {0, 0};                    // predictions in each history table
   int hist_cur = 0;
   int last_B = 0;
   // plan
@@ -60,6 +62,8 @@ struct dyo_ctx {
   int64_t seg_cap = 0, seg_used = 0;
   cudaEvent_t ev_last = nullptr;
   bool ev_pending = false;
+  cudaStream_t d2h = nullptr;      // ctx-owned stream for the EVICT (D2H) phase
+  cudaEvent_t ev_entry = nullptr, ev_evict = nullptr;
   dyo_counters ctr{};
   int sm_count = 148;
   // DYO_F_TIMING: event pairs per launch kind
@@ -119,6 +123,14 @@ void free_list(std::vector<void*>& v) {
 }
 
 int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+// DYO_TRACE=1: one line per migration operation on stderr (debugging hangs / ordering)
+bool trace_on() {
+  static int v = -1;
+  if (v < 0) { const char* e = getenv("DYO_TRACE"); v = (e && *e == '1') ? 1 : 0; }
+  return v == 1;
+}
+#define TRACE(...) do { if (trace_on()) { fprintf(stderr, "[dyo] " __VA_ARGS__); fputc('\n', stderr); fflush(stderr); } } while (0)
 
 bool is_device_ptr(const void* p) {
   if (!p) return false;
@@ -417,6 +429,9 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   if (e == cudaSuccess) e = cudaMalloc(&ctx->arena, 2 * ctx->H);
   if (e == cudaSuccess) e = cudaMalloc(&ctx->staging, c.staging_bytes);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_last, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_entry, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_evict, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->d2h, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, device);
   if (e != cudaSuccess) {
     dyo_destroy(ctx);
@@ -438,6 +453,9 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->arena) cudaFree(ctx->arena);
   if (ctx->staging) cudaFree(ctx->staging);
   if (ctx->ev_last) cudaEventDestroy(ctx->ev_last);
+  if (ctx->ev_entry) cudaEventDestroy(ctx->ev_entry);
+  if (ctx->ev_evict) cudaEventDestroy(ctx->ev_evict);
+  if (ctx->d2h) cudaStreamDestroy(ctx->d2h);
   for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   delete ctx;
@@ -503,7 +521,8 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   DA(pd.ent_n, (size_t)B * K); DA(pd.ent, (size_t)B * K * kEntCap); DA(pd.status, 4);
   DA(ctx->desc_dev, (size_t)B * std::max(A->D_s, 1)); DA(ctx->hist_dev, (size_t)B * std::max(A->h, 1));
   DA(ctx->hist_tab[0], (size_t)B * K * 10); DA(ctx->hist_tab[1], (size_t)B * K * 10);
-  DA(ctx->hist_len[0], 1); DA(ctx->hist_len[1], 1);
+  DA(ctx->hist_K[0], B); DA(ctx->hist_K[1], B);
+  ctx->hist_B[0] = ctx->hist_B[1] = 0;
   ctx->hist_cur = 0;
   ctx->last_B = 0;
   // ---- planner state, scratch and outputs ----
@@ -702,7 +721,8 @@ dyo_status dyo_encode_features(dyo_ctx* ctx, const dyo_sample* s, int32_t B, flo
   const int32_t* hist;
   dyo_status r = stage_samples(ctx, s, B, st, &desc, &hist);
   if (r) return r;
-  CK(launch_encode(ctx->ad, desc, hist, ctx->hist_tab[ctx->hist_cur], ctx->hist_len[ctx->hist_cur], B, feat, st));
+  CK(launch_encode(ctx->ad, desc, hist, ctx->hist_tab[ctx->hist_cur], ctx->hist_K[ctx->hist_cur],
+                   ctx->hist_B[ctx->hist_cur], B, feat, st));
   return DYO_OK;
 }
 
@@ -724,13 +744,14 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
   const int cur = ctx->hist_cur;
   {
     TScope ts(ctx, 0, st);
-    CK(launch_pilot(ctx->ad, ctx->pdv, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_len[cur], B, ctx->logits64,
-                    logits, nullptr, st));
+    CK(launch_pilot(ctx->ad, ctx->pdv, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur], ctx->hist_B[cur], B,
+                    ctx->logits64, logits, ctx->pd.status, nullptr, st));
   }
   {
     TScope ts(ctx, 1, st);
-    CK(launch_decode(ctx->ad, ctx->logits64, ctx->pd, B, ctx->hist_tab[1 - cur], ctx->hist_len[1 - cur], st));
+    CK(launch_decode(ctx->ad, ctx->logits64, ctx->pd, B, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur], st));
   }
+  ctx->hist_B[1 - cur] = B;
   ctx->hist_cur = 1 - cur;
   ctx->last_B = B;
   return DYO_OK;
@@ -869,7 +890,7 @@ dyo_status launch_segs(dyo_ctx* ctx, int64_t first, cudaStream_t s, int grid, in
 
 }  // namespace
 
-dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev_started, void* ev_prev_done,
+dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half_free, void* ev_prev_done,
                        void* ev_ready) {
   if (!ctx) return DYO_E_INVAL;
   if (!ctx->plan_valid) return fail(ctx, DYO_E_STATE, "dyo_migrate before a successful dyo_plan");
@@ -884,7 +905,20 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
   const int64_t dma_min = (ctx->cfg.flags & DYO_F_NO_ZEROCOPY) ? 0 : ctx->cfg.dma_min_bytes;
   const int zc_grid = 16;
   const int d2d_grid = 4 * ctx->sm_count;
-  if (ev_prev_started) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_started, 0));
+  // The EVICT phase runs on the ctx's D2H stream: it only needs the last user of half m (block
+  // j-2) to be done, so it overlaps the previous transition's H2D fetches (full-duplex PCIe).
+  // Without ev_half_free every prior operation on copy_stream counts as that user.
+  cudaStream_t sd = ctx->d2h;
+  TRACE("migrate j=%d evict=%d move=%d carry=%d fetch=%d", j, h.n_evict, h.n_move, h.n_carry, h.n_fetch);
+  if (ev_half_free) {
+    CK(cudaStreamWaitEvent(sd, (cudaEvent_t)ev_half_free, 0));
+  } else {
+    CK(cudaEventRecord(ctx->ev_entry, s));
+    CK(cudaStreamWaitEvent(sd, ctx->ev_entry, 0));
+  }
+  const int64_t stage_half = ctx->staging_bytes / 2 / 256 * 256;
+  char* stage_pack = ctx->staging;                 // D2H stream
+  char* stage_move = ctx->staging + stage_half;    // copy stream
 
   // 1. EVICT writebacks (D2H): host runs (ascending host offset) -> DMA (direct, or K3 packed
   //    through staging when the device sources are scattered), or one zero-copy scatter launch
@@ -908,8 +942,9 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
         ++r.count;
       }
       if (r.bytes >= dma_min && r.dev_contig) {
-        { TScope ts(ctx, 6, s, r.bytes);
-          CK(cudaMemcpyAsync(host + r.host_off, arena + r.dev_off, r.bytes, cudaMemcpyDeviceToHost, s)); }
+        TRACE("  d2h dma host_off=%lld dev=%lld bytes=%lld", (long long)r.host_off, (long long)r.dev_off, (long long)r.bytes);
+        { TScope ts(ctx, 6, sd, r.bytes);
+          CK(cudaMemcpyAsync(host + r.host_off, arena + r.dev_off, r.bytes, cudaMemcpyDeviceToHost, sd)); }
         ctx->ctr.d2h_dma += r.bytes;
         ctx->ctr.n_dma++;
       } else if (r.bytes >= dma_min && !(ctx->cfg.flags & DYO_F_NO_PACK)) {
@@ -918,24 +953,25 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
           const int64_t base = ev[q].host_off;
           const int64_t seg0 = ctx->seg_used;
           int q2 = q;
-          while (q2 < r.first + r.count && ev[q2].host_off + ev[q2].bytes - base <= ctx->staging_bytes) {
-            if (!push_seg(ctx, arena + ev[q2].src, ctx->staging + (ev[q2].host_off - base), ev[q2].bytes))
+          while (q2 < r.first + r.count && ev[q2].host_off + ev[q2].bytes - base <= stage_half) {
+            if (!push_seg(ctx, arena + ev[q2].src, stage_pack + (ev[q2].host_off - base), ev[q2].bytes))
               return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
             ++q2;
           }
           if (q2 == q) {   // a tensor larger than the staging buffer: its own DMA
-            { TScope ts(ctx, 6, s, ev[q].bytes);
-              CK(cudaMemcpyAsync(host + ev[q].host_off, arena + ev[q].src, ev[q].bytes, cudaMemcpyDeviceToHost, s)); }
+            { TScope ts(ctx, 6, sd, ev[q].bytes);
+              CK(cudaMemcpyAsync(host + ev[q].host_off, arena + ev[q].src, ev[q].bytes, cudaMemcpyDeviceToHost, sd)); }
             ctx->ctr.d2h_dma += ev[q].bytes;
             ctx->ctr.n_dma++;
             ++q;
             continue;
           }
-          dyo_status s1 = launch_segs(ctx, seg0, s, d2d_grid);
+          TRACE("  pack %d tensors", q2 - q);
+          dyo_status s1 = launch_segs(ctx, seg0, sd, d2d_grid);
           if (s1) return s1;
           const int64_t len = ev[q2 - 1].host_off + ev[q2 - 1].bytes - base;
-          { TScope ts(ctx, 6, s, len);
-            CK(cudaMemcpyAsync(host + base, ctx->staging, len, cudaMemcpyDeviceToHost, s)); }
+          { TScope ts(ctx, 6, sd, len);
+            CK(cudaMemcpyAsync(host + base, stage_pack, len, cudaMemcpyDeviceToHost, sd)); }
           ctx->ctr.d2h_packed += len;
           ctx->ctr.n_dma++;
           q = q2;
@@ -952,10 +988,14 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
           return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
         ctx->ctr.d2h_zc += ev[q].bytes;
       }
-      dyo_status s1 = launch_segs(ctx, g0, s, zc_grid, 4);
+      dyo_status s1 = launch_segs(ctx, g0, sd, zc_grid, 4);
       if (s1) return s1;
     }
   }
+  TRACE("  evict phase issued");
+  CK(cudaEventRecord(ctx->ev_evict, sd));
+  CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
+
   // 2. MOVE (compaction): staged through `staging` in ascending destination order (R12)
   {
     const dyo_move_rec* mv = ctx->out.mv + h.o_move;
@@ -965,8 +1005,8 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
       const int64_t g0 = ctx->seg_used;
       int64_t used = 0;
       std::vector<std::array<int64_t, 3>> parts;   // (src, dst, bytes) of this chunk
-      while (i < h.n_move && used < ctx->staging_bytes) {
-        const int64_t take = std::min(mv[i].bytes - piece_off, ctx->staging_bytes - used);
+      while (i < h.n_move && used < stage_half) {
+        const int64_t take = std::min(mv[i].bytes - piece_off, stage_half - used);
         parts.push_back({mv[i].src + piece_off, mv[i].dst + piece_off, take});
         used += take;
         piece_off += take;
@@ -974,7 +1014,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
       }
       int64_t so = 0;
       for (auto& p : parts) {
-        if (!push_seg(ctx, arena + p[0], ctx->staging + so, p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+        if (!push_seg(ctx, arena + p[0], stage_move + so, p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
         so += p[2];
       }
       dyo_status s1 = launch_segs(ctx, g0, s, d2d_grid);
@@ -982,7 +1022,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
       const int64_t g1 = ctx->seg_used;
       so = 0;
       for (auto& p : parts) {
-        if (!push_seg(ctx, ctx->staging + so, arena + p[1], p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+        if (!push_seg(ctx, stage_move + so, arena + p[1], p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
         so += p[2];
         ctx->ctr.d2d += p[2];
       }
@@ -1018,6 +1058,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
       }
       const int64_t bytes = fe[k - 1].host_off + fe[k - 1].bytes - fe[i].host_off;
       if (bytes >= dma_min) {
+        TRACE("  h2d dma host_off=%lld dst=%lld bytes=%lld", (long long)fe[i].host_off, (long long)fe[i].dst, (long long)bytes);
         { TScope ts(ctx, 5, s, bytes);
           CK(cudaMemcpyAsync(arena + fe[i].dst, host + fe[i].host_off, bytes, cudaMemcpyHostToDevice, s)); }
         ctx->ctr.h2d_dma += bytes;
@@ -1051,6 +1092,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_prev
       if (s1) return s1;
     }
   }
+  TRACE("  transition %d issued", j);
   if (ev_ready) CK(cudaEventRecord((cudaEvent_t)ev_ready, s));
   CK(cudaEventRecord(ctx->ev_last, s));
   ctx->ev_pending = true;

@@ -1,0 +1,73 @@
+// Block-level device helpers shared by the decode and planner kernels.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace dyo {
+
+// Exclusive scan of one int per thread over the block; *total gets the sum (all threads).
+// warp_tmp: >= 32 ints of shared memory. Contains three __syncthreads().
+__device__ __forceinline__ int block_scan(int v, int* warp_tmp, int* total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) warp_tmp[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    int s = lane < nw ? warp_tmp[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, s, o);
+      if (lane >= o) s += y;
+    }
+    if (lane < nw) warp_tmp[lane] = s;
+  }
+  __syncthreads();
+  const int base = w > 0 ? warp_tmp[w - 1] : 0;
+  const int tot = warp_tmp[nw - 1];
+  __syncthreads();
+  if (total) *total = tot;
+  return base + x - v;
+}
+
+// Exclusive scan of arr[0..n) in place (block-wide, chunks of blockDim); returns the total.
+__device__ __forceinline__ int block_scan_array(int* arr, int n, int* warp_tmp) {
+  int carry = 0;
+  for (int i0 = 0; i0 < n; i0 += blockDim.x) {
+    const int i = i0 + threadIdx.x;
+    const int v = i < n ? arr[i] : 0;
+    int tot = 0;
+    const int p = block_scan(v, warp_tmp, &tot);
+    if (i < n) arr[i] = carry + p;
+    carry += tot;
+    __syncthreads();
+  }
+  return carry;
+}
+
+// Ascending bitonic sort of key[0..n) (pads to a power of two with ~0); key has room for it.
+__device__ __forceinline__ void block_sort_u64(uint64_t* key, int n) {
+  int np2 = 1;
+  while (np2 < n) np2 <<= 1;
+  for (int i = n + threadIdx.x; i < np2; i += blockDim.x) key[i] = ~0ull;
+  __syncthreads();
+  for (int k = 2; k <= np2; k <<= 1) {
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < np2; i += blockDim.x) {
+        const int ixj = i ^ j;
+        if (ixj > i) {
+          const uint64_t x = key[i], z = key[ixj];
+          const bool up = (i & k) == 0;
+          if ((x > z) == up) { key[i] = z; key[ixj] = x; }
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
+}  // namespace dyo

@@ -141,14 +141,14 @@ struct PlanScratch {
 
 // ---- launchers (implemented in the .cu files) ------------------------------------------
 cudaError_t launch_encode(const ArchDev& a, const int64_t* desc, const int32_t* hist,
-                          const int32_t* hist_tab, const int32_t* hist_len, int B, float* feat,
+                          const int32_t* hist_tab, const int32_t* hist_K, int hist_B, int B, float* feat,
                           cudaStream_t s);
 cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_or_null,
                          const int64_t* desc, const int32_t* hist, const int32_t* hist_tab,
-                         const int32_t* hist_len, int B, double* logits64, float* logits32,
-                         int* cluster_used, cudaStream_t s);
+                         const int32_t* hist_K, int hist_B, int B, double* logits64, float* logits32,
+                         int32_t* zero_status, int* cluster_used, cudaStream_t s);
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
-                          int32_t* hist_tab_out, int32_t* hist_len_out, cudaStream_t s);
+                          int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s);
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,
                         PlanState& in, PlanState& work, PlanScratch& sc, PlanOut& out,
                         int max_groups, cudaStream_t s);

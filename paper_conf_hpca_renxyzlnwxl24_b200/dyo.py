@@ -323,8 +323,9 @@ class Dyo:
         buf = (C.c_int64 * (n.value * nf)).from_address(ptr.value)
         return np.ctypeslib.as_array(buf).reshape(n.value, nf).copy()
 
-    def migrate(self, j, stream=0, ev_prev_started=None, ev_prev_done=None, ev_ready=None):
-        self._check(self.L.dyo_migrate(self.ctx, j, P(stream), P(ev_prev_started), P(ev_prev_done), P(ev_ready)))
+    def migrate(self, j, stream=0, ev_half_free=None, ev_prev_done=None, ev_ready=None):
+        """ev_*: cudaEvent_t handles (torch.cuda.Event.cuda_event) or None."""
+        self._check(self.L.dyo_migrate(self.ctx, j, P(stream), P(ev_half_free), P(ev_prev_done), P(ev_ready)))
 
     def residency(self, t):
         p = P()

@@ -255,6 +255,10 @@ dyo_status dyo_get_counters(dyo_ctx* ctx, dyo_counters* c, int32_t reset);
 dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* launches, int64_t* bytes,
                            int32_t reset);
 
+/* Debugging aid: enable (1) / disable (0) %globaltimer phase stamps of the pilot kernel and
+ * read the 32 stamps of the last launch (ns; out32 may be NULL). Synchronises the device. */
+dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32);
+
 #ifdef __cplusplus
 }
 #endif

@@ -4,6 +4,7 @@
 
 #include <algorithm>
 #include <array>
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -28,6 +29,7 @@ struct dyo_ctx {
   ArchDev ad{};
   std::vector<void*> arch_dev;     // device buffers of the arch / prediction / plan
   PilotDev pdv{};
+  const PilotDev* pdv_dev = nullptr;    // device copy of pdv
   std::vector<void*> pilot_dev;
   // memory
   char* arena = nullptr;
@@ -490,6 +492,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   ArchDev& ad = ctx->ad;
   ad = ArchDev{};
   ad.T = T; ad.n_ops = n_ops; ad.n_sites = n_sites; ad.n_pieces = (int)piece_kind.size();
+  ad.n_arms = (int)arm_first.size();
   ad.nn_type = A->nn_type; ad.S_max = A->S_max; ad.D_s = A->D_s; ad.h = A->h; ad.K_max = A->K_max;
   ad.F = (3 + A->D_s + 10 * A->S_max + 10 * A->h + 15) / 16 * 16;
   ad.O = 0;
@@ -620,10 +623,22 @@ dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   int maxw = w->F;
   auto add_layer = [&](const float* W, const float* b, int in_off, int in_len, int out_len, int out_off) -> dyo_status {
     LayerDev& L = p.ly[nl++];
-    const int in_pad = (in_len + 3) / 4 * 4;
+    // row layout [w_0 .. w_{in-1}, bias, 0 pad] padded to 16 bytes: the bias rides with the
+    // weights in the same TMA bulk copy and is applied as the weight of a constant-1 input
+    const int in_pad = (in_len + 1 + 3) / 4 * 4;
     std::vector<float> wp((size_t)out_len * in_pad, 0.f), bp(b, b + out_len);
-    for (int r = 0; r < out_len; ++r)
-      for (int c = 0; c < in_len; ++c) wp[(size_t)r * in_pad + c] = W[(size_t)r * in_len + c];
+    // device copy: subnormal weights flushed to zero (the kernel widens fp32 -> fp64 by
+    // exponent rebias, exact for normals and zero); non-finite weights are rejected
+    auto keep = [](float v) { return std::fpclassify(v) == FP_SUBNORMAL ? 0.0f : v; };
+    for (int r = 0; r < out_len; ++r) {
+      for (int c = 0; c < in_len; ++c) {
+        const float v = W[(size_t)r * in_len + c];
+        if (!std::isfinite(v)) return DYO_E_INVAL;
+        wp[(size_t)r * in_pad + c] = keep(v);
+      }
+      if (!std::isfinite(b[r])) return DYO_E_INVAL;
+      wp[(size_t)r * in_pad + in_len] = keep(b[r]);
+    }
     const float* dw = nullptr;
     const float* db = nullptr;
     dyo_status s = dupload(ctx, ctx->pilot_dev, &dw, wp);
@@ -663,6 +678,14 @@ dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   S.out_width = S.rows = w->O;
   p.n_stages = ns;
   p.max_width = (maxw + 3) / 4 * 4;
+  {
+    // device copy of the descriptor block: the kernel loads it with 16-byte loads in one round trip
+    std::vector<PilotDev> one(1, p);
+    const PilotDev* dp = nullptr;
+    dyo_status s2 = dupload(ctx, ctx->pilot_dev, &dp, one);
+    if (s2) return s2;
+    ctx->pdv_dev = dp;
+  }
   ctx->ad.O = w->O;
   CK(cudaFree(nullptr));
   double* lg = nullptr;
@@ -742,12 +765,13 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
     return fail(ctx, DYO_E_INVAL, "feat must be device memory");
   }
   const int cur = ctx->hist_cur;
+  int fused = 0;
   {
     TScope ts(ctx, 0, st);
-    CK(launch_pilot(ctx->ad, ctx->pdv, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur], ctx->hist_B[cur], B,
-                    ctx->logits64, logits, ctx->pd.status, nullptr, st));
+    CK(launch_pilot(ctx->ad, ctx->pdv, ctx->pdv_dev, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur], ctx->hist_B[cur], B,
+                    ctx->logits64, logits, ctx->pd, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur], &fused, st));
   }
-  {
+  if (!fused) {
     TScope ts(ctx, 1, st);
     CK(launch_decode(ctx->ad, ctx->logits64, ctx->pd, B, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur], st));
   }
@@ -1117,6 +1141,14 @@ dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* laun
   if (reset) {
     for (int k = 0; k < DYO_T_KINDS; ++k) { ctx->tm_ms[k] = 0; ctx->tm_n[k] = 0; ctx->tm_bytes[k] = 0; }
   }
+  return DYO_OK;
+}
+
+dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32) {
+  if (!ctx) return DYO_E_INVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  CK(debug_stamps(enable, reinterpret_cast<unsigned long long*>(out32)));
   return DYO_OK;
 }
 

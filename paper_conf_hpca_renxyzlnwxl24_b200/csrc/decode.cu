@@ -1,55 +1,22 @@
-// A3 decode (§IV-B; R2, R4, R6, R8) in one kernel on the device.
-//
-// One CTA per (prediction b, group slot g); grid = B x K_max. Every CTA redundantly decodes the
-// head of its prediction in shared memory — block head -> rint'd counts (R4), branch head ->
-// argmax choices (tied sites replay, R6), piece lengths -> block scan -> piece starts (the
-// resolved path, R2, is never materialised), non-empty counts -> scan -> cut — which costs a
-// few parallel passes over <= 1024 entries and removes any inter-CTA dependency. Then CTA g
-// builds group g: its rows' operators (binary search over the piece starts), the executed block
-// vector (block reduction) and the tensor set W_g (R8): access records keyed
-// (tensor, position) -> bitonic sort -> first record per tensor + mode union -> re-sort by
-// first position. CTA 0 also writes the debug copies (slots, choices, path, K, L).
+// A3 decode kernel for batches whose groups outnumber the pilot cluster's CTAs (the fused
+// pilot epilogue handles the rest; pilot.cu). One CTA per (prediction b, group slot g): warp 0
+// decodes the head of prediction b into shared memory (decode_dev.cuh), then the block builds
+// group g. No inter-CTA dependency, no materialised path.
 #include <cuda_runtime.h>
 #include <cstdint>
 
-#include "dyo_device.cuh"
-#include "dyo_internal.h"
+#include "decode_dev.cuh"
 
 namespace dyo {
 
 constexpr int kDecThreads = 256;
-constexpr int kMaxPieces = 1024;
-constexpr int kRecCap = 2048;      // access records per group before deduplication
+constexpr int kDecTabCap2 = 8192;     // int32 words of decode tables staged in smem
 
 struct DecSmem {
-  int start[kMaxPieces + 1];       // piece starts (rows)
-  int cum[256 + 1];                // cumulative counts of non-empty slots
-  int cnt[256];
-  int choice[kMaxSites];
-  uint64_t key[kRecCap];
-  uint64_t key2[kRecCap];
-  int warp_tmp[32];
-  long long sig[9];
-  int L, nk, K, n, u;
+  DecHead H;
+  DecGroup G;
+  double ys[1];      // logits copy (O doubles, dynamic)
 };
-
-__device__ __forceinline__ int row_op(const ArchDev& a, const DecSmem& S, int r) {
-  int lo = 0, hi = a.n_pieces - 1;
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if (S.start[mid] <= r) lo = mid; else hi = mid - 1;
-  }
-  const int p = lo, q = r - S.start[p];
-  const int k = a.piece_kind[p];
-  if (k == 0) return a.piece_a[p] + q;
-  if (k == 1) {
-    const int s = a.piece_a[p];
-    return q == 0 ? -1 : a.arm_first_op[a.site_arm_ptr[s] + S.choice[s]] + q - 1;
-  }
-  const int c = a.piece_c[p];
-  const int w = q % (1 + c);
-  return w == 0 ? -1 : a.piece_b[p] + w - 1;
-}
 
 __global__ void __launch_bounds__(kDecThreads)
 decode_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t* __restrict__ hist_tab,
@@ -57,186 +24,20 @@ decode_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t*
   extern __shared__ __align__(16) unsigned char dsm[];
   DecSmem& S = *reinterpret_cast<DecSmem*>(dsm);
   const int b = blockIdx.x / a.K_max, g = blockIdx.x % a.K_max;
-  const double* y = logits + (int64_t)b * a.O;
-  const int tid = threadIdx.x, NT = blockDim.x;
-
-  // 1. block head counts (R4) and 2. branch head choices
-  for (int k = tid; k < a.K_max; k += NT) {
-    double t = y[10 * k] * 16.0;
-    t = fmin(fmax(t, 0.0), (double)kSat);
-    S.cnt[k] = (int)rint(t);
-  }
-  for (int i = tid; i < a.n_sites; i += NT) {
-    const int off = a.site_logit[i];
-    if (off >= 0) {
-      int best = 0;
-      double bv = y[off];
-      for (int c = 1; c < a.site_nch[i]; ++c) {
-        const double v = y[off + c];
-        if (v > bv) { bv = v; best = c; }
-      }
-      S.choice[i] = best;
-    }
-  }
+  const double* yg = logits + (int64_t)b * a.O;
+  for (int i = threadIdx.x; i < a.O; i += blockDim.x) S.ys[i] = yg[i];
   __syncthreads();
-  for (int i = tid; i < a.n_sites; i += NT)
-    if (a.site_logit[i] < 0) S.choice[i] = S.choice[a.site_tie[i]];   // tie targets are free sites
+  const double* y = S.ys;
+  int* tabs = reinterpret_cast<int*>(S.ys + ((a.O + 15) / 16) * 16);
+  const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap2);
+  if (threadIdx.x < 32) head_decode_warp(A, y, S.H, threadIdx.x);
   __syncthreads();
-  // 3. piece lengths -> starts (R2)
-  for (int p = tid; p < a.n_pieces; p += NT) {
-    const int k = a.piece_kind[p];
-    int len;
-    if (k == 0) {
-      len = a.piece_b[p];
-    } else if (k == 1) {
-      const int st = a.piece_a[p];
-      len = 1 + a.arm_nops[a.site_arm_ptr[st] + S.choice[st]];
-    } else {
-      const int st = a.piece_a[p];
-      len = (a.site_lo[st] + S.choice[st]) * (1 + a.piece_c[p]) + 1;
-    }
-    S.start[p] = len;
-  }
-  __syncthreads();
-  const int L = block_scan_array(S.start, a.n_pieces, S.warp_tmp);
-  if (tid == 0) S.start[a.n_pieces] = L;
-  // 4. cut (R4): cumulative counts of the non-empty slots, clipped to the path
-  for (int k = tid; k < a.K_max; k += NT) S.cum[k] = S.cnt[k] != 0 ? 1 : 0;
-  __syncthreads();
-  const int nk = block_scan_array(S.cum, a.K_max, S.warp_tmp);   // S.cum[k] = rank of slot k
-  // compact the non-empty counts in slot order into key2 (as ints), then scan them
-  int* cnt_c = reinterpret_cast<int*>(S.key2);
-  for (int k = tid; k < a.K_max; k += NT)
-    if (S.cnt[k] != 0) cnt_c[S.cum[k]] = S.cnt[k];
-  __syncthreads();
-  for (int k = tid; k < nk; k += NT) S.cum[k] = cnt_c[k];
-  __syncthreads();
-  block_scan_array(S.cum, nk, S.warp_tmp);                        // S.cum[k] = start row of group k
-  if (tid == 0) {
-    int K = 0;
-    while (K < nk && S.cum[K] < L) ++K;                            // groups starting inside the path
-    if (nk == 0 && L > 0) K = 1;
-    S.K = K;
-    S.L = L;
-  }
-  __syncthreads();
-  const int K = S.K;
-  auto grp_start = [&](int k) { return nk == 0 ? 0 : S.cum[k]; };
-  auto grp_end = [&](int k) {
-    if (nk == 0) return L;
-    if (k == K - 1) return L;                                      // clipped / absorbs the remainder
-    return min(S.cum[k] + cnt_c[k], L);
-  };
-
-  // CTA 0 of the prediction: debug copies for dyo_prediction_get
-  if (g == 0) {
-    for (int i = tid; i < a.K_max * 10; i += NT) {
-      const int e = i % 10;
-      double t = y[i] * (e < 7 ? 16.0 : 1024.0);
-      t = fmin(fmax(t, 0.0), (double)kSat);
-      pd.slots[(int64_t)b * a.K_max * 10 + i] = (int)rint(t);
-    }
-    for (int i = tid; i < a.n_sites; i += NT) pd.choices[(int64_t)b * a.n_sites + i] = S.choice[i];
-    if (L <= a.L_max)
-      for (int r = tid; r < L; r += NT) pd.path[(int64_t)b * a.L_max + r] = row_op(a, S, r);
-    if (tid == 0) {
-      pd.K[b] = K;
-      pd.L[b] = L;
-      hist_K[b] = K;
-    }
-  }
-  int32_t* ent_n = pd.ent_n + (int64_t)b * a.K_max + g;
-  if (g >= K) {
-    if (tid == 0) *ent_n = 0;
+  if (g == 0) write_head(A, S.H, y, pd, b, hist_K);
+  if (g >= S.H.K) {
+    if (threadIdx.x == 0) pd.ent_n[(int64_t)b * a.K_max + g] = 0;
     return;
   }
-  const int s = grp_start(g), e = grp_end(g);
-  if (tid == 0) {
-    pd.grp[((int64_t)b * a.K_max + g) * 2] = s;
-    pd.grp[((int64_t)b * a.K_max + g) * 2 + 1] = e;
-  }
-  // 5. block vector and access records of the group's rows
-  if (tid < 9) S.sig[tid] = 0;
-  const int nrows = e - s;
-  const int chunk = (nrows + NT - 1) / NT;
-  const int rs = s + tid * chunk, re = min(e, rs + chunk);
-  long long sg[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
-  int cnt = 0;
-  for (int r = rs; r < re; ++r) {
-    const int op = row_op(a, S, r);
-    if (op >= 0) {
-      cnt += a.acc_ptr[op + 1] - a.acc_ptr[op];
-#pragma unroll
-      for (int k = 0; k < 9; ++k) sg[k] += a.op_sig[(int64_t)op * 9 + k];
-    }
-  }
-  __syncthreads();
-#pragma unroll
-  for (int k = 0; k < 9; ++k) {
-    long long v = sg[k];
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    if ((tid & 31) == 0 && v) atomicAdd(reinterpret_cast<unsigned long long*>(&S.sig[k]), (unsigned long long)v);
-  }
-  int total = 0;
-  int pos = block_scan(cnt, S.warp_tmp, &total);
-  if (tid == 0) {
-    int32_t* bv = pd.blocks + ((int64_t)b * a.K_max + g) * 10;
-    int32_t* hv = hist_tab + ((int64_t)b * a.K_max + g) * 10;
-    const int c0 = min(nrows, kSat);
-    bv[0] = c0;
-    hv[0] = c0;
-    for (int k = 0; k < 9; ++k) {
-      const int v = (int)min(S.sig[k], (long long)kSat);
-      bv[1 + k] = v;
-      hv[1 + k] = v;
-    }
-  }
-  if (total > kRecCap) {
-    if (tid == 0) { *ent_n = 0; atomicCAS(&pd.status[0], 0, DYO_E_CAPACITY); pd.status[1] = total; }
-    return;
-  }
-  const int n = total;
-  for (int r = rs; r < re; ++r) {
-    const int op = row_op(a, S, r);
-    if (op < 0) continue;
-    for (int q = a.acc_ptr[op]; q < a.acc_ptr[op + 1]; ++q, ++pos)
-      S.key[pos] = ((uint64_t)a.acc_t[q] << 32) | ((uint64_t)pos << 2) | (uint64_t)a.acc_m[q];
-  }
-  __syncthreads();
-  // 6. tensor set (R8): first access per tensor, union of modes, ordered by first position
-  block_sort_u64(S.key, n);
-  int np2 = 1;
-  while (np2 < n) np2 <<= 1;
-  for (int i = tid; i < np2; i += NT) S.key2[i] = ~0ull;
-  __syncthreads();
-  for (int i = tid; i < n; i += NT) {
-    const uint32_t t = (uint32_t)(S.key[i] >> 32);
-    if (i > 0 && (uint32_t)(S.key[i - 1] >> 32) == t) continue;
-    const uint32_t p0 = (uint32_t)(S.key[i] & 0xffffffffu) >> 2;
-    const uint32_t m0 = (uint32_t)S.key[i] & 3u;
-    uint32_t mu = m0;
-    for (int k = i + 1; k < n && (uint32_t)(S.key[k] >> 32) == t; ++k) mu |= (uint32_t)S.key[k] & 3u;
-    S.key2[i] = ((uint64_t)p0 << 32) | ((uint64_t)t << 3) | (mu << 1) | (m0 & 1u);
-  }
-  __syncthreads();
-  block_sort_u64(S.key2, n);
-  if (tid == 0) {
-    int u = 0;
-    while (u < n && S.key2[u] != ~0ull) ++u;
-    S.u = u;
-  }
-  __syncthreads();
-  const int u = S.u;
-  if (u > kEntCap) {
-    if (tid == 0) { *ent_n = 0; atomicCAS(&pd.status[0], 0, DYO_E_CAPACITY); pd.status[1] = u; }
-    return;
-  }
-  int2* ent = pd.ent + ((int64_t)b * a.K_max + g) * kEntCap;
-  for (int i = tid; i < u; i += NT) {
-    const uint32_t lo = (uint32_t)(S.key2[i] & 0xffffffffu);
-    ent[i] = make_int2((int)(lo >> 3), (int)(((lo >> 1) & 3u) | ((lo & 1u) << 2)));
-  }
-  if (tid == 0) *ent_n = u;
+  build_group(A, S.H, S.G, pd, b, g, hist_tab);
 }
 
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
@@ -244,12 +45,12 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
   if (B <= 0) return cudaSuccess;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)sizeof(DecSmem));
+    cudaError_t e = cudaFuncSetAttribute(decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  decode_kernel<<<B * a.K_max, kDecThreads, sizeof(DecSmem), s>>>(a, logits, pd, hist_tab_out, hist_K_out);
+  const size_t smem = sizeof(DecSmem) + (size_t)((a.O + 15) / 16 * 16) * sizeof(double) + (size_t)kDecTabCap2 * 4;
+  decode_kernel<<<B * a.K_max, kDecThreads, smem, s>>>(a, logits, pd, hist_tab_out, hist_K_out);
   return cudaGetLastError();
 }
 

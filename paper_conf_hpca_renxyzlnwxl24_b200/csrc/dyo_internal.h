@@ -19,7 +19,7 @@ enum OpClass : int8_t { C_KEEP = 0, C_CARRY = 1, C_ALLOC = 2, C_FETCH = 3 };
 // ---- pilot --------------------------------------------------------------------------
 constexpr int kMaxLayers = 16;
 struct LayerDev {
-  const float* W;    // out x in_pad (rows padded to a multiple of 4 floats)
+  const float* W;    // out x in_pad: [w_0..w_{in-1}, bias, 0...] padded to a multiple of 4 floats
   const float* b;    // out
   int in_off;        // offset of this layer's input in the stage input vector
   int in_len;
@@ -44,7 +44,7 @@ struct PilotDev {
 
 // ---- arch on the device -------------------------------------------------------------
 struct ArchDev {
-  int T, n_ops, n_sites, n_pieces, nn_type, S_max, D_s, h, K_max, F, O, n_branch_logits;
+  int T, n_ops, n_sites, n_pieces, n_arms, nn_type, S_max, D_s, h, K_max, F, O, n_branch_logits;
   int L_max;
   int64_t H, align;
   // tensors
@@ -143,10 +143,14 @@ struct PlanScratch {
 cudaError_t launch_encode(const ArchDev& a, const int64_t* desc, const int32_t* hist,
                           const int32_t* hist_tab, const int32_t* hist_K, int hist_B, int B, float* feat,
                           cudaStream_t s);
-cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_or_null,
+// Fused encode + pilot (+ decode epilogue when *fused is set on return; otherwise the caller
+// launches the decode kernel).
+cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_dev, const float* feat_or_null,
                          const int64_t* desc, const int32_t* hist, const int32_t* hist_tab,
                          const int32_t* hist_K, int hist_B, int B, double* logits64, float* logits32,
-                         int32_t* zero_status, int* cluster_used, cudaStream_t s);
+                         PredDev& pd, int32_t* hist_tab_out, int32_t* hist_K_out, int* fused,
+                         cudaStream_t s);
+cudaError_t debug_stamps(int on, unsigned long long* out);
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s);
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,

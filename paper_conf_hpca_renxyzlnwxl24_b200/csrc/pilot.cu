@@ -1,23 +1,30 @@
-// K1: fused feature encode + pilot MLP forward (§IV-A, §IV-C;
-// DESIGN.md R3, R5).
+// K1: fused feature encode + pilot MLP forward + decode epilogue (§IV-A,
+// §IV-C, §IV-B; R3, R4, R5).
 //
-// B200 design: one thread-block cluster per sub-batch of <= kBs samples. Every stage (the
-// three input-feature layers form one stage, then each MLP layer, then the output layer)
-// splits its output rows across the C CTAs of the cluster; a warp owns a row, streams the
-// row's fp32 weights with 16-byte loads (L2-resident across calls), reuses them for all
-// samples of the sub-batch, reduces with warp shuffles, applies bias + LeakyReLU and writes
-// the value into the activation buffer of every CTA of the cluster through distributed shared
-// memory (DSMEM); one cluster barrier separates stages. The encode stage (R3) is computed
-// redundantly by each CTA straight into its shared activation buffer (no HBM round trip).
-// Precision: fp32 weights, fp64 products / accumulation / activations (an fp32 x fp32 product is
-// exact in fp64); the batch-1 GEMV chain is latency-bound, so B200's FP64 pipe costs nothing
-// measurable and the logits meet the north_star's 1e-5 relative gate against the fp64 oracle
-// with ~1e-12 to spare; decode decisions are taken on the fp64 logits (same precision as the
-// oracle). fp32 logits are an optional copy for the caller.
+// B200 design (one launch per prediction batch):
+//  * one thread-block cluster of C CTAs per sub-batch; every stage (the three input-feature
+//    layers form one stage, then each MLP layer, then the output layer) splits its output rows
+//    over the cluster;
+//  * at launch each CTA issues TMA bulk copies (cp.async.bulk + mbarrier complete_tx) of its
+//    slice of EVERY layer's weights into shared memory - the bias rides in the row as the weight
+//    of a constant-1 input - so the whole weight stream overlaps the layer chain;
+//  * a warp computes 4 rows at once from one shared activation read and reduces them with a
+//    transposed butterfly (6 shuffles instead of 20);
+//  * a stage's outputs are PUSHED to the peer CTAs with st.async ... mbarrier::complete_tx:
+//    each CTA waits on its own mbarrier for the expected bytes - no cluster barrier and no
+//    DSMEM pull per stage (measured: cluster barrier ~400 cycles, 512-double pull ~1300 cycles);
+//  * the encode stage (R3) is computed by each CTA straight into shared memory;
+//  * epilogue: after one cluster barrier (logits visible), CTA r decodes the groups g = r mod C
+//    of its samples (decode_dev.cuh) - for MoE's 16 groups on 16 CTAs, one group per CTA.
+// Precision: fp32 weights, fp64 products / accumulation / activations (fp32 x fp32 is exact in
+// fp64): the latency-bound GEMV chain does not notice B200's FP64 rate, and the logits meet the
+// north_star's 1e-5 relative gate against the fp64 oracle with ~1e-12 to spare; decode decides
+// on the fp64 logits (the oracle's precision). fp32 logits are an optional copy for the caller.
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 #include <cstdint>
 
+#include "decode_dev.cuh"
 #include "dyo_internal.h"
 
 namespace cg = cooperative_groups;
@@ -25,7 +32,9 @@ namespace cg = cooperative_groups;
 namespace dyo {
 
 constexpr int kBs = 8;          // samples per cluster
-constexpr int kPilotThreads = 256;
+constexpr int kDynCap = 227 * 1024 - 4096;   // dynamic smem cap (static smem holds the descriptors)
+constexpr int kDecTabCap = 16384;             // int32 words of decode tables staged in smem
+constexpr int kPilotThreads = 512;
 
 template <class T>
 __device__ __forceinline__ T scale_elem(int e, int v) {
@@ -121,176 +130,358 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
       : "memory");
 }
 
-// Per-launch plan of which stages are staged in shared memory (computed on the host for the
-// chosen cluster size C): stage s is staged iff st_off[s] >= 0; st_off = byte offset of the
-// CTA's weight slice (same for every rank; the slice size is bounded by st_bytes[s]).
+// Debug phase stamps (SM clock cycles of CTA 0), enabled by dyo_debug_pilot_stamps().
+__device__ unsigned long long g_stamp[32];
+__device__ int g_stamp_on;
+__device__ __forceinline__ void stamp(int i, int on) {
+  if (on && blockIdx.x == 0 && threadIdx.x == 0) g_stamp[i] = (unsigned long long)clock64();
+}
+
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t saddr, int rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+  return r;
+}
+// 8 / 16-byte asynchronous remote stores that signal the destination CTA's mbarrier
+__device__ __forceinline__ void st_async_b64(uint32_t raddr, double v, uint32_t rbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b64 [%0], %1, [%2];" ::"r"(raddr),
+               "l"(__double_as_longlong(v)), "r"(rbar)
+               : "memory");
+}
+__device__ __forceinline__ void st_async_v2b64(uint32_t raddr, double a, double b, uint32_t rbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.b64 [%0], {%1, %2}, [%3];" ::"r"(raddr),
+               "l"(__double_as_longlong(a)), "l"(__double_as_longlong(b)), "r"(rbar)
+               : "memory");
+}
+
+// Per-launch plan (host-computed for the chosen cluster size C): stage s is staged in shared
+// memory iff st_off[s] >= 0 (byte offset of the CTA's weight slice).
 struct StagePlan {
   int C;
   int Bs;                 // samples per cluster
   int act_off;            // byte offset of the activation buffers
+  int fuse_decode;        // 1: this kernel also decodes its samples (epilogue)
   int st_off[4 + kMaxLayers];
+  int rpc[4 + kMaxLayers];      // rows per CTA of each stage
+  int gsh[4 + kMaxLayers];      // log2 of the threads per row (k-split) of each stage
 };
 
+__device__ __forceinline__ float4 lds_f4(uint32_t a) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ double2 lds_d2(uint32_t a) {
+  double2 v;
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(a));
+  return v;
+}
+
+// fp32 -> fp64 by exponent rebias on the integer pipes (F2F.F64.F32 is a low-throughput
+// conversion on this part and the GEMV converts every weight). Exact for normal numbers and
+// zero; the loader flushes subnormal weights to zero (their contribution < 1.2e-38 |x|) and
+// rejects non-finite ones.
+__device__ __forceinline__ double f2d(float f) {
+  const uint32_t u = __float_as_uint(f);
+  const uint32_t e = (u >> 23) & 0xffu;
+  uint32_t hi = (u & 0x80000000u) | ((e + 896u) << 20) | ((u & 0x7fffffu) >> 3);
+  uint32_t lo = u << 29;
+  if (e == 0) { hi = u & 0x80000000u; lo = 0; }
+  return __hiloint2double((int)hi, (int)lo);
+}
+
+// Transposed butterfly reduction of 4 per-lane partial sums (rows 0..3) over the warp:
+// 6 shuffles instead of 4 x 5. Lane l ends with the total of row ((l >> 4) & 1) * 2 + ((l >> 3) & 1).
+__device__ __forceinline__ double warp_reduce4(double a0, double a1, double a2, double a3, int lane) {
+  const bool hi16 = lane & 16;
+  double k0 = hi16 ? a2 : a0, k1 = hi16 ? a3 : a1;
+  k0 += __shfl_xor_sync(0xffffffffu, hi16 ? a0 : a2, 16);
+  k1 += __shfl_xor_sync(0xffffffffu, hi16 ? a1 : a3, 16);
+  const bool hi8 = lane & 8;
+  double v = (hi8 ? k1 : k0) + __shfl_xor_sync(0xffffffffu, hi8 ? k0 : k1, 8);
+  v += __shfl_xor_sync(0xffffffffu, v, 4);
+  v += __shfl_xor_sync(0xffffffffu, v, 2);
+  v += __shfl_xor_sync(0xffffffffu, v, 1);
+  return v;
+}
+
 // grid = n_clusters * C (cluster dims C set at launch). Dynamic smem:
-//   [mbarriers][staged weight slices][activations 2 x Bs x max_width doubles]
+//   [mbarriers: n_stages (weights) + 2 (activation buffers)][staged weight slices]
+//   [activations 2 x BS x max_width doubles]
+// With fuse_decode the weight region is reused for the decode (DecHead / DecGroup) afterwards.
 template <int BS>
 __global__ void __launch_bounds__(kPilotThreads)
-pilot_kernel(ArchDev a, PilotDev p, StagePlan sp, const float* __restrict__ feat,
-             const int64_t* __restrict__ desc, const int32_t* __restrict__ hist,
+pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pdev, const __grid_constant__ StagePlan sp,
+             const float* __restrict__ feat, const int64_t* __restrict__ desc, const int32_t* __restrict__ hist,
              const int32_t* __restrict__ hist_tab, const int32_t* __restrict__ hist_K, int hist_B, int B,
-             double* __restrict__ logits64, float* __restrict__ logits32, int32_t* __restrict__ zero_status) {
+             double* __restrict__ logits64, float* __restrict__ logits32, PredDev pd,
+             int32_t* __restrict__ hist_tab_out, int32_t* __restrict__ hist_K_out) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  cg::cluster_group cluster = cg::this_cluster();
+  __shared__ __align__(16) PilotDev p;
+  const int tid = threadIdx.x;
+  const int stamp_on = g_stamp_on;
+  stamp(0, stamp_on);
+  {
+    // descriptors: one round trip of 16-byte loads (dynamic indexing of the parameter bank in
+    // the loops below would cost a dependent constant-cache miss each time)
+    const int4* src = reinterpret_cast<const int4*>(pdev);
+    int4* dst = reinterpret_cast<int4*>(&p);
+    for (int i = tid; i < (int)(sizeof(PilotDev) / 16); i += blockDim.x) dst[i] = src[i];
+  }
   const int C = sp.C;
-  const int r = (int)cluster.block_rank();
+  const int r = C > 1 ? (int)cg::this_cluster().block_rank() : 0;
   const int cluster_id = blockIdx.x / C;
-  const int Bs = sp.Bs;
-  const int b0 = cluster_id * Bs;
-  const int nb = min(Bs, B - b0);
-  const int W = p.max_width;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);
+  const int b0 = cluster_id * BS;
+  const int nb = min(BS, B - b0);
+  uint64_t* wbar = reinterpret_cast<uint64_t*>(smem_raw);           // one per stage
+  uint64_t* abar = wbar + (4 + kMaxLayers);                         // two activation buffers
   double* act = reinterpret_cast<double*>(smem_raw + sp.act_off);
-  double* buf[2] = {act, act + Bs * W};
-
-  // ---- 0. issue every staged weight slice of this CTA at once (TMA bulk, one mbarrier/stage)
-  if (blockIdx.x == 0 && threadIdx.x == 0 && zero_status) { zero_status[0] = 0; zero_status[1] = 0; }
-  if (threadIdx.x == 0) {
-    for (int si = 0; si < p.n_stages; ++si) mbar_init(&bars[si], 1);
+  if (blockIdx.x == 0 && tid == 0) { pd.status[0] = 0; pd.status[1] = 0; }
+  if (tid == 0) {
+    for (int i = 0; i < 4 + kMaxLayers; ++i) mbar_init(&wbar[i], 1);
+    mbar_init(&abar[0], 1);
+    mbar_init(&abar[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    for (int si = 0; si < p.n_stages; ++si) {
-      if (sp.st_off[si] < 0) continue;
-      const StageDev st = p.st[si];
-      const int rpc = (st.rows + C - 1) / C;
-      const int r0 = r * rpc, r1 = min(st.rows, r0 + rpc);
-      uint32_t bytes = 0;
-      int lr0 = 0;
-      for (int l = st.first_layer; l < st.first_layer + st.n_layers; ++l) {
-        const int lr1 = lr0 + p.ly[l].out_len;
-        const int a0 = max(r0, lr0), a1 = min(r1, lr1);
-        if (a1 > a0) bytes += (uint32_t)(a1 - a0) * p.ly[l].in_pad * 4;
-        lr0 = lr1;
+  }
+  __syncthreads();                       // descriptors + barrier inits visible in the CTA
+  const int W = p.max_width;
+  double* buf[2] = {act, act + BS * W};
+  // ---- 0. TMA: lane si of warp 0 issues stage si's weight slice (all stages in flight at once)
+  if (tid < p.n_stages && sp.st_off[tid] >= 0) {
+    const int si = tid;
+    const StageDev& st = p.st[si];
+    const int rpc = (st.rows + C - 1) / C;
+    const int r0 = r * rpc, r1 = min(st.rows, r0 + rpc);
+    uint32_t bytes = 0;
+    int lr0 = 0;
+    for (int l = st.first_layer; l < st.first_layer + st.n_layers; ++l) {
+      const int lr1 = lr0 + p.ly[l].out_len;
+      const int a0 = max(r0, lr0), a1 = min(r1, lr1);
+      if (a1 > a0) bytes += (uint32_t)(a1 - a0) * p.ly[l].in_pad * 4;
+      lr0 = lr1;
+    }
+    mbar_expect_tx(&wbar[si], bytes);
+    unsigned char* dst = smem_raw + sp.st_off[si];
+    lr0 = 0;
+    for (int l = st.first_layer; l < st.first_layer + st.n_layers; ++l) {
+      const int lr1 = lr0 + p.ly[l].out_len;
+      const int a0 = max(r0, lr0), a1 = min(r1, lr1);
+      if (a1 > a0) {
+        const uint32_t nbytes = (uint32_t)(a1 - a0) * p.ly[l].in_pad * 4;
+        tma_bulk_g2s(dst, p.ly[l].W + (int64_t)(a0 - lr0) * p.ly[l].in_pad, nbytes, &wbar[si]);
+        dst += nbytes;
       }
-      mbar_expect_tx(&bars[si], bytes);
-      unsigned char* dst = smem_raw + sp.st_off[si];
-      lr0 = 0;
-      for (int l = st.first_layer; l < st.first_layer + st.n_layers; ++l) {
-        const int lr1 = lr0 + p.ly[l].out_len;
-        const int a0 = max(r0, lr0), a1 = min(r1, lr1);
-        if (a1 > a0) {
-          const uint32_t nbytes = (uint32_t)(a1 - a0) * p.ly[l].in_pad * 4;
-          tma_bulk_g2s(dst, p.ly[l].W + (int64_t)(a0 - lr0) * p.ly[l].in_pad, nbytes, &bars[si]);
-          dst += nbytes;
-        }
-        lr0 = lr1;
-      }
+      lr0 = lr1;
     }
   }
-  // ---- 1. encode (or load) the sub-batch's feature vectors into buf[0] (overlaps the TMA)
+  stamp(1, stamp_on);
+  // ---- 1. the sub-batch's feature vectors into buf[0] (overlaps the weight stream)
   for (int bb = 0; bb < nb; ++bb) {
     double* x = buf[0] + bb * W;
     if (feat) {
-      for (int i = threadIdx.x; i < p.F; i += blockDim.x) x[i] = (double)feat[(int64_t)(b0 + bb) * p.F + i];
+      for (int i = tid; i < p.F; i += blockDim.x) x[i] = (double)feat[(int64_t)(b0 + bb) * p.F + i];
     } else {
       encode_one<double>(a, desc + (int64_t)(b0 + bb) * a.D_s, hist ? hist + (int64_t)(b0 + bb) * a.h : nullptr,
                          hist_tab, hist_K, hist_B, x);
     }
   }
+  // arm the activation barrier of stage 0's output (buffer 1) with the bytes the peers send
+  if (C > 1 && tid == 0) {
+    const int rows = p.st[0].rows, rpc = (rows + C - 1) / C;
+    const int own = max(0, min(rows, (r + 1) * rpc) - r * rpc);
+    mbar_expect_tx(&abar[1], (uint32_t)((rows - own) * nb * 8));
+  }
   __syncthreads();
+  stamp(2, stamp_on);
 
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int nwarps = blockDim.x >> 5;
-  int cur = 0;
+  const int warp = tid >> 5, lane = tid & 31;
+  const uint32_t abar_s[2] = {smem_u32(&abar[0]), smem_u32(&abar[1])};
   for (int si = 0; si < p.n_stages; ++si) {
-    const StageDev st = p.st[si];
+    const StageDev& st = p.st[si];
     const bool last = (si == p.n_stages - 1);
     const bool staged = sp.st_off[si] >= 0;
-    const int rpc = (st.rows + C - 1) / C;
+    const int rpc = sp.rpc[si];
     const int r0 = r * rpc, r1 = min(st.rows, r0 + rpc);
-    const double* in = buf[cur];
-    double* out = buf[cur ^ 1];
-    if (staged) mbar_wait(&bars[si], 0);
-    for (int row = r0 + warp; row < r1; row += nwarps) {
-      int li = st.first_layer, rowl = row, lr0 = 0;
-      while (rowl >= p.ly[li].out_len) { rowl -= p.ly[li].out_len; lr0 += p.ly[li].out_len; ++li; }
-      const LayerDev ly = p.ly[li];
-      const float* wrow;
-      if (staged) {
-        // byte offset of this row inside the CTA's staged slice: rows of earlier layers first
-        int64_t off = 0;
-        int l0 = 0;
-        for (int l = st.first_layer; l < li; ++l) {
-          const int l1 = l0 + p.ly[l].out_len;
-          const int a0 = max(r0, l0), a1 = min(r1, l1);
-          if (a1 > a0) off += (int64_t)(a1 - a0) * p.ly[l].in_pad;
-          l0 = l1;
+    const int cin = si & 1, cout = cin ^ 1;
+    const double* in = buf[cin];
+    double* out = buf[cout];
+    // inputs of this stage: the peers' rows of stage si-1 (arrived via st.async) + own rows
+    if (si > 0 && C > 1) mbar_wait(&abar[cin], ((si - 1) >> 1) & 1);
+    // arm the barrier of the NEXT stage's inputs (this stage's outputs) before any peer can finish
+    if (si + 1 < p.n_stages && si > 0 && C > 1 && tid == 0 && !last) {
+      const int own = max(0, r1 - r0);
+      mbar_expect_tx(&abar[cout], (uint32_t)((st.rows - own) * nb * 8));
+    }
+    stamp(3 + 3 * si, stamp_on);
+    if (staged) mbar_wait(&wbar[si], 0);
+    stamp(4 + 3 * si, stamp_on);
+    const uint32_t out_s = smem_u32(out);
+    // ---- k-split: G threads per output row (G = largest power of two with rows * G <= block),
+    //      each accumulates a contiguous chunk of the row (16-byte weight loads, fp64 FMAs with
+    //      two independent accumulators), then a log2(G)-step shuffle reduction ----
+    const int gsh = sp.gsh[si], G = 1 << gsh;
+    const int grp = tid >> gsh, part = tid & (G - 1);
+    const int rows_per_pass = blockDim.x >> gsh;
+    for (int row0 = r0; row0 < r1; row0 += rows_per_pass) {
+      const int row = row0 + grp;
+      const bool active = row < r1;
+      double acc0[BS], acc1[BS];
+#pragma unroll
+      for (int bb = 0; bb < BS; ++bb) { acc0[bb] = 0.0; acc1[bb] = 0.0; }
+      if (active) {
+        // layer of this row (the feature stage holds up to three layers)
+        int li = st.first_layer, rowl = row, lr0 = 0;
+        while (rowl >= p.ly[li].out_len) { rowl -= p.ly[li].out_len; lr0 += p.ly[li].out_len; ++li; }
+        const LayerDev& ly = p.ly[li];
+        const float* wrow;
+        if (staged) {
+          int64_t off = 0;
+          int l0 = 0;
+          for (int l = st.first_layer; l < li; ++l) {
+            const int l1 = l0 + p.ly[l].out_len;
+            const int a0 = max(r0, l0), a1 = min(r1, l1);
+            if (a1 > a0) off += (int64_t)(a1 - a0) * p.ly[l].in_pad;
+            l0 = l1;
+          }
+          off += (int64_t)(row - max(r0, lr0)) * ly.in_pad;
+          wrow = reinterpret_cast<const float*>(smem_raw + sp.st_off[si]) + off;
+        } else {
+          wrow = ly.W + (int64_t)rowl * ly.in_pad;
         }
-        off += (int64_t)(row - max(r0, lr0)) * ly.in_pad;
-        wrow = reinterpret_cast<const float*>(smem_raw + sp.st_off[si]) + off;
-      } else {
-        wrow = ly.W + (int64_t)rowl * ly.in_pad;
-      }
-      double acc[BS];
-#pragma unroll
-      for (int bb = 0; bb < BS; ++bb) acc[bb] = 0.0;
+        const int nq = ly.in_pad >> 2;                      // float4 chunks of the row
+        const int nfull = ly.in_len >> 2;                   // chunks without the bias column
+        // interleaved chunks: thread `part` takes q = part, part + G, ... so the G threads of a
+        // row read consecutive 16-byte words (bank-conflict free); explicit shared-memory loads
+        const uint32_t xin_s = smem_u32(in) + (uint32_t)ly.in_off * 8;
+        if (staged) {
+          const uint32_t w_s = smem_u32(wrow);
 #pragma unroll 4
-      for (int k = lane * 4; k < ly.in_pad; k += 128) {
-        const float4 w = staged ? *reinterpret_cast<const float4*>(wrow + k)
-                                : __ldg(reinterpret_cast<const float4*>(wrow + k));
-        const double wv[4] = {w.x, w.y, w.z, w.w};
+          for (int q = part; q < nfull; q += G) {
+            const float4 w = lds_f4(w_s + (uint32_t)q * 16);
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          if (k + q < ly.in_len) {
+            for (int bb = 0; bb < BS; ++bb) {
+              if (bb < nb) {
+                const uint32_t xa = xin_s + (uint32_t)(bb * W + q * 4) * 8;
+                const double2 x01 = ((ly.in_off & 1) == 0) ? lds_d2(xa) : make_double2(in[ly.in_off + bb * W + q * 4], in[ly.in_off + bb * W + q * 4 + 1]);
+                const double2 x23 = ((ly.in_off & 1) == 0) ? lds_d2(xa + 16) : make_double2(in[ly.in_off + bb * W + q * 4 + 2], in[ly.in_off + bb * W + q * 4 + 3]);
+                // two widenings on the F2F pipe, two by integer rebias (balances both pipes)
+                acc0[bb] = fma((double)w.x, x01.x, acc0[bb]);
+                acc1[bb] = fma(f2d(w.y), x01.y, acc1[bb]);
+                acc0[bb] = fma((double)w.z, x23.x, acc0[bb]);
+                acc1[bb] = fma(f2d(w.w), x23.y, acc1[bb]);
+              }
+            }
+          }
+        } else {
+#pragma unroll 4
+          for (int q = part; q < nfull; q += G) {
+            const float4 w = __ldg(reinterpret_cast<const float4*>(wrow) + q);
+            const double* xb = in + ly.in_off + q * 4;
+#pragma unroll
+            for (int bb = 0; bb < BS; ++bb) {
+              if (bb < nb) {
+                acc0[bb] = fma((double)w.x, xb[bb * W + 0], acc0[bb]);
+                acc1[bb] = fma(f2d(w.y), xb[bb * W + 1], acc1[bb]);
+                acc0[bb] = fma((double)w.z, xb[bb * W + 2], acc0[bb]);
+                acc1[bb] = fma(f2d(w.w), xb[bb * W + 3], acc1[bb]);
+              }
+            }
+          }
+        }
+        // the tail chunks (the remaining inputs and the bias column: weight of a constant 1)
+        for (int q = nfull + part; q < nq; q += G) {
+          const float4 w = staged ? lds_f4(smem_u32(wrow) + (uint32_t)q * 16) : __ldg(reinterpret_cast<const float4*>(wrow) + q);
+          const float wv[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+          for (int qq = 0; qq < 4; ++qq) {
+            const int kk = q * 4 + qq;
 #pragma unroll
             for (int bb = 0; bb < BS; ++bb)
-              if (bb < nb) acc[bb] = fma(wv[q], in[bb * W + ly.in_off + k + q], acc[bb]);
+              if (bb < nb) acc0[bb] = fma(f2d(wv[qq]), kk < ly.in_len ? in[ly.in_off + bb * W + kk] : (kk == ly.in_len ? 1.0 : 0.0), acc0[bb]);
           }
         }
       }
-      const double bias = (double)__ldg(ly.b + rowl);
 #pragma unroll
       for (int bb = 0; bb < BS; ++bb) {
-        if (bb < nb) {
-          double v = warp_sum(acc[bb]) + bias;
-          if (st.act) v = v > 0.0 ? v : p.slope * v;
-          if (last) {
-            if (lane == 0) {
-              logits64[(int64_t)(b0 + bb) * p.O + row] = v;
-              if (logits32) logits32[(int64_t)(b0 + bb) * p.O + row] = (float)v;
-            }
-          } else if (lane < C) {
-            double* dst = cluster.map_shared_rank(out, lane);
-            dst[bb * W + row] = v;
+        double v = acc0[bb] + acc1[bb];
+        for (int o = G >> 1; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (!active || bb >= nb) continue;
+        if (st.act) v = v > 0.0 ? v : p.slope * v;
+        if (last) {
+          if (part == 0) {
+            logits64[(int64_t)(b0 + bb) * p.O + row] = v;
+            if (logits32) logits32[(int64_t)(b0 + bb) * p.O + row] = (float)v;
+          }
+        } else {
+          if (part == 0) out[bb * W + row] = v;
+          if (C > 1) {
+            const uint32_t laddr = out_s + (uint32_t)((bb * W + row) * 8);
+            for (int c = part; c < C; c += G)
+              if (c != r) st_async_b64(mapa_u32(laddr, c), v, mapa_u32(abar_s[cout], c));
           }
         }
       }
     }
-    if (!last) {
-      cluster.sync();
-      cur ^= 1;
-    }
+    stamp(5 + 3 * si, stamp_on);
+    if (!last) __syncthreads();          // own rows of this stage visible to every warp
   }
-  // keep this CTA's shared memory alive until every peer finished its DSMEM writes
-  // (the last exchange is followed by cluster.sync() above, so no further sync is needed)
+  // ---- 2. fused decode epilogue: CTA r of the cluster decodes groups g == r (mod C) ----
+  if (!sp.fuse_decode) return;
+  if (C > 1) cg::this_cluster().sync();   // every CTA's logits written (release/acquire, cluster scope)
+  else __syncthreads();
+  DecHead& H = *reinterpret_cast<DecHead*>(smem_raw + ((2 * (4 + kMaxLayers) + 2) * 8 + 127) / 128 * 128);
+  DecGroup& Gs = *reinterpret_cast<DecGroup*>(reinterpret_cast<unsigned char*>(&H) + ((sizeof(DecHead) + 127) / 128 * 128));
+  double* ys = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(&Gs) + ((sizeof(DecGroup) + 127) / 128 * 128));
+  int* tabs = reinterpret_cast<int*>(ys + ((p.O + 15) / 16) * 16);
+  const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap);
+  for (int bb = 0; bb < nb; ++bb) {
+    const int b = b0 + bb;
+    if (r >= a.K_max && r != 0) continue;
+    const double* y = logits64 + (int64_t)b * p.O;
+    __syncthreads();
+    // the logits into shared memory in one coalesced pass (the argmax loops would otherwise
+    // chain dependent L2 round trips)
+    for (int i = tid; i < p.O; i += blockDim.x) ys[i] = y[i];
+    __syncthreads();
+    y = ys;
+    if (warp == 0) head_decode_warp(A, y, H, lane);
+    __syncthreads();
+    stamp(26, stamp_on);
+    if (r == 0) write_head(A, H, y, pd, b, hist_K_out);
+    for (int g = r; g < a.K_max; g += C) {
+      if (g >= H.K) {
+        if (tid == 0) pd.ent_n[(int64_t)b * a.K_max + g] = 0;
+        continue;
+      }
+      build_group(A, H, Gs, pd, b, g, hist_tab_out);
+    }
+    stamp(27, stamp_on);
+  }
 }
 
-cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_or_null,
+cudaError_t debug_stamps(int on, unsigned long long* out) {
+  cudaError_t e = cudaMemcpyToSymbol(g_stamp_on, &on, sizeof(int));
+  if (e == cudaSuccess && out) e = cudaMemcpyFromSymbol(out, g_stamp, sizeof(unsigned long long) * 32);
+  return e;
+}
+
+cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_dev, const float* feat_or_null,
                          const int64_t* desc, const int32_t* hist, const int32_t* hist_tab,
                          const int32_t* hist_K, int hist_B, int B, double* logits64, float* logits32,
-                         int32_t* zero_status, int* cluster_used, cudaStream_t s) {
+                         PredDev& pd, int32_t* hist_tab_out, int32_t* hist_K_out, int* fused,
+                         cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
   static int attr_done = 0;
   if (!attr_done) {
     for (auto fn : {pilot_kernel<1>, pilot_kernel<kBs>}) {
       cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
       if (e != cudaSuccess) return e;
-      e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+      e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kDynCap);
       if (e != cudaSuccess) return e;
     }
     attr_done = 1;
   }
-  // cluster size by weight volume: spread the layers over enough SMs that each CTA's slice
-  // streams in ~1 us; cached per (weights, max cluster) since cudaOccupancyMaxActiveClusters
-  // is expensive
+  // cluster size by weight volume (cached: cudaOccupancyMaxActiveClusters is expensive)
   int64_t wbytes = 0;
   for (int i = 0; i < p.n_stages; ++i) {
     const StageDev& st = p.st[i];
@@ -325,15 +516,20 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_
   }
   StagePlan sp{};
   sp.C = C;
-  sp.Bs = B < kBs ? B : kBs;
-  // shared memory: barriers, then staged slices while they fit, then activations
+  sp.Bs = B < kBs ? 1 : kBs;
+  // fuse the decode when the cluster has at least one CTA per two groups of its samples
+  sp.fuse_decode = (sp.Bs * a.K_max <= 2 * C) ? 1 : 0;
   const int act_bytes = 2 * sp.Bs * p.max_width * (int)sizeof(double);
-  const int budget = 227 * 1024 - act_bytes;
-  int off = (p.n_stages * 8 + 127) / 128 * 128;
+  const int base = ((2 * (4 + kMaxLayers) + 2) * 8 + 127) / 128 * 128;
+  const int budget = kDynCap - act_bytes;
+  int off = base;
   for (int i = 0; i < p.n_stages; ++i) {
     const StageDev& st = p.st[i];
     const int rpc = (st.rows + C - 1) / C;
-    // worst-case slice of any rank: rpc rows of the widest layer of the stage
+    sp.rpc[i] = rpc;
+    int gsh = 0;
+    while (gsh < 5 && rpc * (2 << gsh) <= kPilotThreads) ++gsh;
+    sp.gsh[i] = gsh;
     int maxpad = 0;
     for (int l = st.first_layer; l < st.first_layer + st.n_layers; ++l) maxpad = maxpad > p.ly[l].in_pad ? maxpad : p.ly[l].in_pad;
     const int bytes = (rpc * maxpad * 4 + 127) / 128 * 128;
@@ -344,8 +540,13 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_
       sp.st_off[i] = -1;
     }
   }
+  // the decode epilogue reuses [base, ...) after the MLP
+  const int dec_bytes = (int)(((sizeof(DecHead) + 127) / 128 * 128) + ((sizeof(DecGroup) + 127) / 128 * 128) +
+                              (size_t)((p.O + 15) / 16 * 16) * sizeof(double) + (size_t)kDecTabCap * 4);
+  if (sp.fuse_decode && base + dec_bytes > off) off = (base + dec_bytes + 127) / 128 * 128;
   sp.act_off = off;
-  const size_t smem = (size_t)off + act_bytes;
+  const size_t smem = (size_t)sp.act_off + act_bytes;
+  if (smem > (size_t)kDynCap) return cudaErrorInvalidValue;
   const int n_clusters = (B + sp.Bs - 1) / sp.Bs;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(n_clusters * C);
@@ -359,12 +560,12 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const float* feat_
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (cluster_used) *cluster_used = C;
+  if (fused) *fused = sp.fuse_decode;
   if (sp.Bs == 1)
-    return cudaLaunchKernelEx(&cfg, pilot_kernel<1>, a, p, sp, feat_or_null, desc, hist, hist_tab, hist_K, hist_B,
-                              B, logits64, logits32, zero_status);
-  return cudaLaunchKernelEx(&cfg, pilot_kernel<kBs>, a, p, sp, feat_or_null, desc, hist, hist_tab, hist_K, hist_B,
-                            B, logits64, logits32, zero_status);
+    return cudaLaunchKernelEx(&cfg, pilot_kernel<1>, a, p_dev, sp, feat_or_null, desc, hist, hist_tab, hist_K, hist_B,
+                              B, logits64, logits32, pd, hist_tab_out, hist_K_out);
+  return cudaLaunchKernelEx(&cfg, pilot_kernel<kBs>, a, p_dev, sp, feat_or_null, desc, hist, hist_tab, hist_K, hist_B,
+                            B, logits64, logits32, pd, hist_tab_out, hist_K_out);
 }
 
 }  // namespace dyo

@@ -94,7 +94,8 @@ def lib():
         for name in ("dyo_create", "dyo_destroy", "dyo_load_arch", "dyo_load_pilot", "dyo_host_pool",
                      "dyo_arena", "dyo_encode_features", "dyo_pilot_predict", "dyo_prediction_get",
                      "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records", "dyo_migrate",
-                     "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check"):
+                     "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
+                     "dyo_debug_pilot_stamps"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -103,7 +104,8 @@ def lib():
 EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_destroy", "dyo_load_arch",
            "dyo_load_pilot", "dyo_host_pool", "dyo_arena", "dyo_encode_features", "dyo_pilot_predict",
            "dyo_prediction_get", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
-           "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check")
+           "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
+           "dyo_debug_pilot_stamps")
 
 
 def _a(x, dt):
@@ -342,6 +344,11 @@ class Dyo:
             out[name] = {"ms": ms.value, "launches": n.value, "bytes": b.value}
         if reset:
             self._check(self.L.dyo_get_timings(self.ctx, 0, None, None, None, 1))
+        return out
+
+    def pilot_stamps(self, enable=True):
+        out = np.zeros(32, np.uint64)
+        self._check(self.L.dyo_debug_pilot_stamps(self.ctx, 1 if enable else 0, out.ctypes.data_as(C.POINTER(C.c_uint64))))
         return out
 
     def counters(self, reset=False):

@@ -258,6 +258,9 @@ dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* laun
 /* Debugging aid: enable (1) / disable (0) %globaltimer phase stamps of the pilot kernel and
  * read the 32 stamps of the last launch (ns; out32 may be NULL). Synchronises the device. */
 dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32);
+/* Debugging aid: clock64 stamps of the planner's phases for transition j of the next dyo_plan
+ * (j = -1 disables); out64 (64 entries, may be NULL) receives the stamps of the last plan. */
+dyo_status dyo_debug_plan_stamps(dyo_ctx* ctx, int32_t j, uint64_t* out64);
 
 #ifdef __cplusplus
 }

@@ -52,7 +52,8 @@ struct dyo_ctx {
   PlanState state[2]{};
   int committed = 0;
   PlanScratch sc{};
-  PlanOut out{};                   // record arrays + headers in pinned mapped host memory
+  PlanOut out{};                   // host (pinned) mirrors of the plan records + headers
+  PlanOut dout{};                  // device record arrays the planner kernel writes
   int32_t* h_status = nullptr;     // pinned mapped
   int32_t* h_counts = nullptr;
   int8_t* h_loc = nullptr;         // pinned mirrors of the committed residency
@@ -65,7 +66,8 @@ struct dyo_ctx {
   cudaEvent_t ev_last = nullptr;
   bool ev_pending = false;
   cudaStream_t d2h = nullptr;      // ctx-owned stream for the EVICT (D2H) phase
-  cudaEvent_t ev_entry = nullptr, ev_evict = nullptr;
+  cudaStream_t side = nullptr;     // ctx-owned stream for early CARRY (overlaps FETCH)
+  cudaEvent_t ev_entry = nullptr, ev_evict = nullptr, ev_moves = nullptr, ev_carry = nullptr;
   dyo_counters ctr{};
   int sm_count = 148;
   // DYO_F_TIMING: event pairs per launch kind
@@ -434,6 +436,9 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_entry, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_evict, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->d2h, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->side, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_moves, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_carry, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, device);
   if (e != cudaSuccess) {
     dyo_destroy(ctx);
@@ -458,6 +463,9 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->ev_entry) cudaEventDestroy(ctx->ev_entry);
   if (ctx->ev_evict) cudaEventDestroy(ctx->ev_evict);
   if (ctx->d2h) cudaStreamDestroy(ctx->d2h);
+  if (ctx->side) cudaStreamDestroy(ctx->side);
+  if (ctx->ev_moves) cudaEventDestroy(ctx->ev_moves);
+  if (ctx->ev_carry) cudaEventDestroy(ctx->ev_carry);
   for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   delete ctx;
@@ -545,7 +553,6 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   DA(sc.inw, T); DA(sc.cur_next, T); DA(sc.cur_rd, T); DA(sc.nxt, cap_ent); DA(sc.nxt_rd, cap_ent);
   DA(sc.rstat, T); DA(sc.keys, 2 * ((size_t)T + 1024) + 4096); DA(sc.gap_s, T + 1); DA(sc.gap_e, T + 1);
   DA(sc.kept, T); DA(sc.newoff, T); DA(sc.ebase, mg); DA(sc.grp_b, mg); DA(sc.grp_k, mg);
-#undef DA
   auto hmap = [&](void** p, size_t bytes) -> dyo_status {
     CK(cudaHostAlloc(p, std::max<size_t>(bytes, 64), cudaHostAllocMapped | cudaHostAllocPortable));
     memset(*p, 0, std::max<size_t>(bytes, 64));
@@ -562,6 +569,17 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   if ((st = hmap((void**)&o.ca, sizeof(dyo_carry_rec) * cap_rec))) return st;
   if ((st = hmap((void**)&o.al, sizeof(dyo_alloc_rec) * cap_rec))) return st;
   if ((st = hmap((void**)&o.fe, sizeof(dyo_fetch_rec) * cap_rec))) return st;
+  // the planner writes its records to device memory (writes to pinned host memory from a
+  // latency-bound single-CTA kernel stall its barriers); dyo_plan copies them back by count
+  PlanOut& dO = ctx->dout;
+  dO = PlanOut{};
+  dO.cap_ent = cap_ent;
+  dO.cap_rec = cap_rec;
+  {
+    PlanHdr* h1; dyo_entry_rec* e1; dyo_evict_rec* v1; dyo_move_rec* m1; dyo_carry_rec* c1; dyo_alloc_rec* a1; dyo_fetch_rec* f1;
+    DA(h1, mg); DA(e1, cap_ent); DA(v1, cap_rec); DA(m1, cap_rec); DA(c1, cap_rec); DA(a1, cap_rec); DA(f1, cap_rec);
+    dO.hdr = h1; dO.ent = e1; dO.ev = v1; dO.mv = m1; dO.ca = c1; dO.al = a1; dO.fe = f1;
+  }
   if ((st = hmap((void**)&ctx->h_status, 16 * sizeof(int32_t)))) return st;
   if ((st = hmap((void**)&ctx->h_counts, 16 * sizeof(int32_t)))) return st;
   if ((st = hmap((void**)&ctx->h_loc, T))) return st;
@@ -575,6 +593,9 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   CK(cudaHostGetDevicePointer((void**)&d_counts, ctx->h_counts, 0));
   o.status = d_status;
   o.counts = d_counts;
+  dO.status = d_status;
+  dO.counts = d_counts;
+#undef DA
   // ---- host pool (pinned, mapped: DMA and zero-copy kernels) ----
   ctx->host_bytes = pool;
   if (!(ctx->cfg.flags & DYO_F_NO_HOST_POOL))
@@ -832,7 +853,7 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
   PlanState& wk = ctx->state[1 - ctx->committed];
   {
     TScope ts(ctx, 2, st);
-    CK(launch_plan(ctx->ad, ctx->pd, b0, n, ctx->cfg.policy, in, wk, ctx->sc, ctx->out, ctx->max_groups, st));
+    CK(launch_plan(ctx->ad, ctx->pd, b0, n, ctx->cfg.policy, in, wk, ctx->sc, ctx->dout, ctx->max_groups, st));
   }
   CK(cudaMemcpyAsync(ctx->h_loc, wk.loc, ctx->T, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(ctx->h_off, wk.off, sizeof(int64_t) * ctx->T, cudaMemcpyDeviceToHost, st));
@@ -845,6 +866,25 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
     if (status == DYO_E_BUDGET) return fail(ctx, DYO_E_BUDGET, "transition %d: W_j exceeds half the budget", ctx->h_status[1]);
     if (status == DYO_E_CAPACITY) return fail(ctx, DYO_E_CAPACITY, "capacity exceeded (needed %d)", ctx->h_status[2]);
     return fail(ctx, (dyo_status)(status < 0 ? status : DYO_E_CUDA), "planner status %d", status);
+  }
+  {
+    // copy the plan (headers + every record list, exact counts) to the pinned host mirrors
+    const int32_t* c = ctx->h_counts;
+    const PlanOut& D = ctx->dout;
+    PlanOut& Hm = ctx->out;
+    int64_t n_ent = 0;
+    if (c[0] > 0) {
+      CK(cudaMemcpyAsync(Hm.hdr, D.hdr, sizeof(PlanHdr) * c[0], cudaMemcpyDeviceToHost, st));
+    }
+    CK(cudaStreamSynchronize(st));
+    for (int g = 0; g < c[0]; ++g) n_ent += Hm.hdr[g].n_ent;
+    if (n_ent) CK(cudaMemcpyAsync(Hm.ent, D.ent, sizeof(dyo_entry_rec) * n_ent, cudaMemcpyDeviceToHost, st));
+    if (c[1]) CK(cudaMemcpyAsync(Hm.ev, D.ev, sizeof(dyo_evict_rec) * c[1], cudaMemcpyDeviceToHost, st));
+    if (c[2]) CK(cudaMemcpyAsync(Hm.mv, D.mv, sizeof(dyo_move_rec) * c[2], cudaMemcpyDeviceToHost, st));
+    if (c[3]) CK(cudaMemcpyAsync(Hm.ca, D.ca, sizeof(dyo_carry_rec) * c[3], cudaMemcpyDeviceToHost, st));
+    if (c[4]) CK(cudaMemcpyAsync(Hm.al, D.al, sizeof(dyo_alloc_rec) * c[4], cudaMemcpyDeviceToHost, st));
+    if (c[5]) CK(cudaMemcpyAsync(Hm.fe, D.fe, sizeof(dyo_fetch_rec) * c[5], cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
   }
   ctx->committed = 1 - ctx->committed;
   ctx->plan_K = ctx->h_counts[0];
@@ -1020,42 +1060,63 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   CK(cudaEventRecord(ctx->ev_evict, sd));
   CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
 
-  // 2. MOVE (compaction): staged through `staging` in ascending destination order (R12)
+  // 2. MOVE (compaction, R11/R12), ascending destination. Processed in order, moves are safe
+  //    (new <= old and every destination ends below the later sources), but run in parallel a
+  //    move may overwrite an earlier move's source: group them into waves of mutually
+  //    non-overlapping (destination vs source) moves, one copy-kernel launch per wave. A move
+  //    overlapping its own source goes through the staging buffer in pieces.
   {
     const dyo_move_rec* mv = ctx->out.mv + h.o_move;
-    int i = 0;
-    int64_t piece_off = 0;
-    while (i < h.n_move) {
-      const int64_t g0 = ctx->seg_used;
-      int64_t used = 0;
-      std::vector<std::array<int64_t, 3>> parts;   // (src, dst, bytes) of this chunk
-      while (i < h.n_move && used < stage_half) {
-        const int64_t take = std::min(mv[i].bytes - piece_off, stage_half - used);
-        parts.push_back({mv[i].src + piece_off, mv[i].dst + piece_off, take});
-        used += take;
-        piece_off += take;
-        if (piece_off == mv[i].bytes) { ++i; piece_off = 0; }
+    int64_t wave0 = -1;
+    std::vector<std::pair<int64_t, int64_t>> wave_src;    // source ranges of the open wave
+    auto flush = [&]() -> dyo_status {
+      if (wave0 >= 0) {
+        dyo_status s1 = launch_segs(ctx, wave0, s, d2d_grid);
+        if (s1) return s1;
       }
-      int64_t so = 0;
-      for (auto& p : parts) {
-        if (!push_seg(ctx, arena + p[0], stage_move + so, p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
-        so += p[2];
+      wave0 = -1;
+      wave_src.clear();
+      return DYO_OK;
+    };
+    for (int i = 0; i < h.n_move; ++i) {
+      const int64_t src = mv[i].src, dst = mv[i].dst, nbytes = mv[i].bytes;
+      ctx->ctr.d2d += nbytes;
+      if (dst + nbytes > src) {                     // self-overlap: staged pieces, after the wave
+        dyo_status s1 = flush();
+        if (s1) return s1;
+        for (int64_t o = 0; o < nbytes; o += stage_half) {
+          const int64_t n = std::min(stage_half, nbytes - o);
+          const int64_t g0 = ctx->seg_used;
+          if (!push_seg(ctx, arena + src + o, stage_move, n)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+          s1 = launch_segs(ctx, g0, s, d2d_grid);
+          if (s1) return s1;
+          const int64_t g1 = ctx->seg_used;
+          if (!push_seg(ctx, stage_move, arena + dst + o, n)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+          s1 = launch_segs(ctx, g1, s, d2d_grid);
+          if (s1) return s1;
+        }
+        continue;
       }
-      dyo_status s1 = launch_segs(ctx, g0, s, d2d_grid);
-      if (s1) return s1;
-      const int64_t g1 = ctx->seg_used;
-      so = 0;
-      for (auto& p : parts) {
-        if (!push_seg(ctx, stage_move + so, arena + p[1], p[2])) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
-        so += p[2];
-        ctx->ctr.d2d += p[2];
+      bool clash = false;
+      for (auto& w : wave_src)
+        if (dst < w.second && dst + nbytes > w.first) { clash = true; break; }
+      if (clash) {
+        dyo_status s1 = flush();
+        if (s1) return s1;
       }
-      s1 = launch_segs(ctx, g1, s, d2d_grid);
-      if (s1) return s1;
+      if (wave0 < 0) wave0 = ctx->seg_used;
+      if (!push_seg(ctx, arena + src, arena + dst, nbytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+      wave_src.push_back({src, src + nbytes});
     }
+    dyo_status s1 = flush();
+    if (s1) return s1;
   }
   // 3. early CARRY (D2D, one launch) and FETCH (H2D: DMA per host run, zero-copy gather for
   //    the small runs, one launch)
+  //    early CARRYs run on the side stream, concurrently with the FETCH DMAs: their
+  //    destinations are disjoint from the fetch destinations and their sources lie in the
+  //    other half (read-only here)
+  bool carry_side = false;
   {
     const dyo_carry_rec* ca = ctx->out.ca + h.o_carry;
     const int64_t g0 = ctx->seg_used;
@@ -1064,8 +1125,14 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
       if (!push_seg(ctx, arena + ca[i].src, arena + ca[i].dst, ca[i].bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
       ctx->ctr.d2d += ca[i].bytes;
     }
-    dyo_status s1 = launch_segs(ctx, g0, s, d2d_grid);
-    if (s1) return s1;
+    if (ctx->seg_used > g0) {
+      CK(cudaEventRecord(ctx->ev_moves, s));
+      CK(cudaStreamWaitEvent(ctx->side, ctx->ev_moves, 0));
+      dyo_status s1 = launch_segs(ctx, g0, ctx->side, d2d_grid);
+      if (s1) return s1;
+      CK(cudaEventRecord(ctx->ev_carry, ctx->side));
+      carry_side = true;
+    }
   }
   {
     const dyo_fetch_rec* fe = ctx->out.fe + h.o_fetch;
@@ -1099,6 +1166,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
     dyo_status s1 = launch_segs(ctx, g0, s, zc_grid, 4);
     if (s1) return s1;
   }
+  if (carry_side) CK(cudaStreamWaitEvent(s, ctx->ev_carry, 0));
   // 4. late CARRY: block j-1 writes them, so they wait for its end
   {
     const dyo_carry_rec* ca = ctx->out.ca + h.o_carry;
@@ -1149,6 +1217,14 @@ dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32)
   CK(cudaSetDevice(ctx->device));
   CK(cudaDeviceSynchronize());
   CK(debug_stamps(enable, reinterpret_cast<unsigned long long*>(out32)));
+  return DYO_OK;
+}
+
+dyo_status dyo_debug_plan_stamps(dyo_ctx* ctx, int32_t j, uint64_t* out64) {
+  if (!ctx) return DYO_E_INVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  CK(plan_debug_stamps(j, reinterpret_cast<unsigned long long*>(out64)));
   return DYO_OK;
 }
 

@@ -35,6 +35,7 @@ struct DecGroup {
   uint64_t key[kRecCap];
   uint64_t key2[kRecCap];
   int warp_tmp[32];
+  long long sum_tmp[32];
   unsigned long long sig[9];
   int n, u;
 };
@@ -227,14 +228,13 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
       for (int k = 0; k < 9; ++k) sg[k] += a.op_sig[(int64_t)op * 9 + k];
     }
   }
-#pragma unroll
+  // block sums of the nine signature columns (no 64-bit shared atomics: CAS spin loops)
   for (int k = 0; k < 9; ++k) {
-    long long v = sg[k];
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    if (lane == 0 && v) atomicAdd(&G.sig[k], (unsigned long long)v);
+    const long long v = block_sum64(sg[k], G.sum_tmp);
+    if (tid == 0) G.sig[k] = (unsigned long long)v;
   }
   int total = 0;
-  int pos = block_scan(cnt, G.warp_tmp, &total);   // includes __syncthreads (sig atomics done)
+  int pos = block_scan(cnt, G.warp_tmp, &total);   // includes __syncthreads (sig sums done)
   if (tid == 0) {
     int32_t* bv = pd.blocks + ((int64_t)b * a.K_max + g) * 10;
     int32_t* hv = hist_tab + ((int64_t)b * a.K_max + g) * 10;

@@ -34,6 +34,21 @@ __device__ __forceinline__ int block_scan(int v, int* warp_tmp, int* total) {
   return base + x - v;
 }
 
+// Sum of one int64 per thread over the block, returned to every thread. No atomics: 64-bit
+// shared-memory atomicAdd compiles to a CAS spin loop (ATOMS.CAST.SPIN.64) that serialises
+// under contention. tmp: >= 32 long longs of shared memory. Contains two __syncthreads().
+__device__ __forceinline__ long long block_sum64(long long v, long long* tmp) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  if (lane == 0) tmp[w] = v;
+  __syncthreads();
+  long long t = 0;
+  for (int i = 0; i < nw; ++i) t += tmp[i];
+  __syncthreads();
+  return t;
+}
+
 // Exclusive scan of arr[0..n) in place (block-wide, chunks of blockDim); returns the total.
 __device__ __forceinline__ int block_scan_array(int* arr, int n, int* warp_tmp) {
   int carry = 0;

@@ -12,7 +12,7 @@ namespace dyo {
 constexpr int kSat = (1 << 24) - 1;       // R1(iii)
 constexpr int kMaxSites = 4096;
 constexpr int kEntCap = 1024;             // tensor-set entries per group (records before dedupe)
-constexpr int kPlanThreads = 512;
+constexpr int kPlanThreads = 256;
 
 enum OpClass : int8_t { C_KEEP = 0, C_CARRY = 1, C_ALLOC = 2, C_FETCH = 3 };
 
@@ -151,6 +151,7 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
                          PredDev& pd, int32_t* hist_tab_out, int32_t* hist_K_out, int* fused,
                          cudaStream_t s);
 cudaError_t debug_stamps(int on, unsigned long long* out);
+cudaError_t plan_debug_stamps(int j, unsigned long long* out);
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s);
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,

@@ -13,13 +13,19 @@
 //   compacted layout by exclusive scan (R11) -> records + state update.
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <cstdlib>
 
+#include "dyo_device.cuh"
 #include "dyo_internal.h"
 
 namespace dyo {
 
 constexpr int kSortCap = 4096;      // shared-memory sort capacity (larger sorts use global scratch)
 constexpr uint64_t kInfD = 0xFFFFull;
+
+__device__ unsigned long long g_pstamp[64];
+__device__ int g_pstamp_j = -1;
+#define PSTAMP(i) do { if (j == pstamp_j && tid == 0) g_pstamp[i] = (unsigned long long)clock64(); } while (0)
 
 enum RStat : int8_t { RS_NONE = 0, RS_KEEP = 1, RS_LIVE = 2, RS_DEAD = 3, RS_EVICT = 4, RS_RETAIN = 5 };
 
@@ -31,8 +37,7 @@ struct PlanSmem {
   int64_t e_new[kEntCap];
   uint64_t sortbuf[kSortCap];
   int warp_tmp[32];
-  int i_tmp[16];
-  unsigned long long u_tmp[8];
+  long long sum_tmp[32];
 };
 
 __device__ __forceinline__ void sort_keys(uint64_t* key, int n) {
@@ -55,43 +60,59 @@ __device__ __forceinline__ void sort_keys(uint64_t* key, int n) {
   }
 }
 
-// Block-wide exclusive scan of one int per thread; returns the prefix, *total gets the sum.
-__device__ __forceinline__ int block_scan(int v, int* warp_tmp, int* total) {
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  int x = v;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const int y = __shfl_up_sync(0xffffffffu, x, o);
-    if (lane >= o) x += y;
-  }
-  if (lane == 31) warp_tmp[w] = x;
-  __syncthreads();
-  if (w == 0) {
-    int s = lane < nw ? warp_tmp[lane] : 0;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int y = __shfl_up_sync(0xffffffffu, s, o);
-      if (lane >= o) s += y;
-    }
-    if (lane < nw) warp_tmp[lane] = s;
-  }
-  __syncthreads();
-  const int base = w > 0 ? warp_tmp[w - 1] : 0;
-  const int tot = warp_tmp[nw - 1];
-  __syncthreads();
-  if (total) *total = tot;
-  return base + x - v;
-}
-
 __global__ void __launch_bounds__(kPlanThreads, 1)
-plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, PlanState st,
-            PlanScratch sc, PlanOut out, int max_groups) {
+plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, PlanState stg,
+            PlanScratch scg, PlanOut out, int max_groups, int smem_state) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PlanSmem& S = *reinterpret_cast<PlanSmem*>(smem_raw);
   const int T = a.T;
   const int64_t H = a.H, AL = a.align;
   int* status = out.status;
   const int tid = threadIdx.x, NT = blockDim.x;
+
+  // Per-tensor working state and constants: in shared memory when they fit (smem_state), so
+  // the many dependent per-transition lookups cost ~30 cycles instead of an L2 round trip.
+  PlanState st = stg;
+  PlanScratch sc = scg;
+  const int64_t* t_ab = a.t_abytes;
+  const int64_t* t_host = a.t_host;
+  const int64_t* t_by = a.t_bytes;
+  const int32_t* t_fl = a.t_flags;
+  if (smem_state) {
+    unsigned char* q = smem_raw + ((sizeof(PlanSmem) + 15) / 16 * 16);
+    auto carve = [&](size_t bytes) { unsigned char* r = q; q += (bytes + 15) / 16 * 16; return r; };
+    st.off = reinterpret_cast<int64_t*>(carve(8 * (size_t)T));
+    sc.gap_s = reinterpret_cast<int64_t*>(carve(8 * (size_t)(T + 1)));
+    sc.gap_e = reinterpret_cast<int64_t*>(carve(8 * (size_t)(T + 1)));
+    sc.newoff = reinterpret_cast<int64_t*>(carve(8 * (size_t)T));
+    int64_t* ab = reinterpret_cast<int64_t*>(carve(8 * (size_t)T));
+    int64_t* ho = reinterpret_cast<int64_t*>(carve(8 * (size_t)T));
+    int64_t* by = reinterpret_cast<int64_t*>(carve(8 * (size_t)T));
+    st.res = reinterpret_cast<int32_t*>(carve(8 * (size_t)T));
+    st.prev = reinterpret_cast<int32_t*>(carve(4 * (size_t)T));
+    sc.cur_next = reinterpret_cast<int32_t*>(carve(4 * (size_t)T));
+    sc.kept = reinterpret_cast<int32_t*>(carve(4 * (size_t)T));
+    int32_t* fl = reinterpret_cast<int32_t*>(carve(4 * (size_t)T));
+    st.res_n = reinterpret_cast<int32_t*>(carve(16));
+    st.prev_n = reinterpret_cast<int32_t*>(carve(16));
+    st.G = reinterpret_cast<int64_t*>(carve(16));
+    st.loc = reinterpret_cast<int8_t*>(carve(T));
+    st.dirty = reinterpret_cast<uint8_t*>(carve(T));
+    st.pw = reinterpret_cast<uint8_t*>(carve(T));
+    sc.cur_rd = reinterpret_cast<uint8_t*>(carve(T));
+    sc.inw = reinterpret_cast<int8_t*>(carve(T));
+    sc.rstat = reinterpret_cast<int8_t*>(carve(T));
+    for (int t = tid; t < T; t += NT) {
+      ab[t] = a.t_abytes[t];
+      ho[t] = a.t_host[t];
+      by[t] = a.t_bytes[t];
+      fl[t] = a.t_flags[t];
+    }
+    t_ab = ab;
+    t_host = ho;
+    t_by = by;
+    t_fl = fl;
+  }
 
   // ---- 0. decode status, group list ----
   __shared__ int s_Kt, s_fail;
@@ -121,7 +142,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
   for (int t = tid; t < T; t += NT) {
     st.loc[t] = in.loc[t];
     st.off[t] = in.off[t];
-    st.dirty[t] = (a.t_flags[t] & 1) ? 0 : in.dirty[t];
+    st.dirty[t] = (t_fl[t] & 1) ? 0 : in.dirty[t];
     st.pw[t] = in.pw[t];
     st.res[t] = in.res[t];
     st.res[T + t] = in.res[T + t];
@@ -175,7 +196,9 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
   if (tid == 0) { c_ev = c_mv = c_ca = c_al = c_fe = 0; }
   __syncthreads();
 
+  const int pstamp_j = g_pstamp_j;
   for (int j = 0; j < Kt; ++j) {
+    PSTAMP(0);
     const int64_t Gj = st.G[0] + j;
     const int m = (int)(Gj & 1);
     const int2* ent = pd.ent + ((int64_t)sc.grp_b[j] * a.K_max + sc.grp_k[j]) * kEntCap;
@@ -190,19 +213,26 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
     }
     __syncthreads();
     // A. load W_j; need
+    long long my_need = 0;
     for (int e = tid; e < n; e += NT) {
       const int t = ent[e].x;
       S.e_t[e] = t;
       S.e_mode[e] = (int8_t)(ent[e].y & 3);
       S.e_rd[e] = (int8_t)((ent[e].y >> 2) & 1);
-      atomicAdd(&s_need, (unsigned long long)a.t_abytes[t]);
+      my_need += t_ab[t];
+    }
+    {
+      const long long tot = block_sum64(my_need, S.sum_tmp);
+      if (tid == 0) s_need = (unsigned long long)tot;
     }
     __syncthreads();
+    PSTAMP(1);
     // B. feasibility (R7)
     if ((int64_t)s_need > H) {
       if (tid == 0) { status[0] = DYO_E_BUDGET; status[1] = j; status[2] = 0; }
       return;
     }
+    PSTAMP(2);
     // C. classify (R8)
     for (int e = tid; e < n; e += NT) {
       const int t = S.e_t[e];
@@ -219,24 +249,31 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       else if (c == C_FETCH) atomicAdd(&s_nf, 1);
     }
     __syncthreads();
+    PSTAMP(3);
     // D. candidates of half m: dead (R9) or live with next-use distance
     const int nm = st.res_n[m];
     const int32_t* resm = st.res + (int64_t)m * T;
     const bool big = nm > kSortCap;
     uint64_t* keys = big ? sc.keys : S.sortbuf;
+    long long my_live = 0;
     for (int i = tid; i < nm; i += NT) {
       const int t = resm[i];
       if (sc.inw[t]) { sc.rstat[t] = RS_KEEP; continue; }
       const int nx = sc.cur_next[t];
-      const bool dead = (nx < 0 && (a.t_flags[t] & 1)) || (nx >= 0 && !sc.cur_rd[t]);
+      const bool dead = (nx < 0 && (t_fl[t] & 1)) || (nx >= 0 && !sc.cur_rd[t]);
       if (dead) { sc.rstat[t] = RS_DEAD; continue; }
       sc.rstat[t] = RS_LIVE;
       const uint64_t d = nx < 0 ? kInfD : (uint64_t)(nx - j);
       const int k = atomicAdd(&s_nlive, 1);
-      keys[k] = (d << 48) | ((uint64_t)(a.t_abytes[t] / AL) << 20) | (uint64_t)t;
-      atomicAdd(&s_livebytes, (unsigned long long)a.t_abytes[t]);
+      keys[k] = (d << 48) | ((uint64_t)(t_ab[t] / AL) << 20) | (uint64_t)t;
+      my_live += t_ab[t];
+    }
+    {
+      const long long tot = block_sum64(my_live, S.sum_tmp);
+      if (tid == 0) s_livebytes = (unsigned long long)tot;
     }
     __syncthreads();
+    PSTAMP(4);
     // E. retention (R10)
     const int64_t room = H - (int64_t)s_need;
     const int nlive = s_nlive;
@@ -261,13 +298,14 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       for (int k = tid; k < nlive; k += NT) sc.rstat[(int)(keys[k] & 0xFFFFF)] = RS_RETAIN;
     }
     __syncthreads();
+    PSTAMP(5);
     // F. EVICT records sorted by (host offset, id)
     for (int i = tid; i < nm; i += NT) {
       const int t = resm[i];
       const int8_t r = sc.rstat[t];
       if (r == RS_DEAD || r == RS_EVICT) {
         const int k = atomicAdd(&s_nev, 1);
-        keys[k] = ((uint64_t)(a.t_host[t] / AL) << 20) | (uint64_t)t;
+        keys[k] = ((uint64_t)(t_host[t] / AL) << 20) | (uint64_t)t;
       }
     }
     __syncthreads();
@@ -277,19 +315,25 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       return;
     }
     sort_keys(keys, nev);
+    long long my_d2h = 0;
     for (int k = tid; k < nev; k += NT) {
       const int t = (int)(keys[k] & 0xFFFFF);
       const bool wb = sc.rstat[t] == RS_EVICT && st.dirty[t];
       dyo_evict_rec r;
       r.t = t;
       r.src = (int64_t)m * H + st.off[t];
-      r.host_off = a.t_host[t];
-      r.bytes = a.t_bytes[t];
+      r.host_off = t_host[t];
+      r.bytes = t_by[t];
       r.writeback = wb ? 1 : 0;
       out.ev[c_ev + k] = r;
-      if (wb) atomicAdd(&s_d2h, (unsigned long long)a.t_bytes[t]);
+      if (wb) my_d2h += t_by[t];
+    }
+    {
+      const long long tot = block_sum64(my_d2h, S.sum_tmp);
+      if (tid == 0) s_d2h = (unsigned long long)tot;
     }
     __syncthreads();
+    PSTAMP(6);
     // G. kept list in ascending old offset (order-preserving compaction of the resident list)
     {
       int total = 0, base = 0;
@@ -306,6 +350,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       __syncthreads();
     }
     const int nkept = s_nkept;
+    PSTAMP(7);
     // H. gaps of half m between kept tensors
     {
       int total = 0, base = 0;
@@ -314,7 +359,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
         int f = 0;
         int64_t gs = 0, ge = 0;
         if (i <= nkept) {
-          gs = i == 0 ? 0 : st.off[sc.kept[i - 1]] + a.t_abytes[sc.kept[i - 1]];
+          gs = i == 0 ? 0 : st.off[sc.kept[i - 1]] + t_ab[sc.kept[i - 1]];
           ge = i == nkept ? H : st.off[sc.kept[i]];
           f = ge > gs;
         }
@@ -326,6 +371,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       if (tid == 0) s_ng = base;
       __syncthreads();
     }
+    PSTAMP(8);
     // I. placement order: CARRY by id, ALLOC by id, FETCH by (host offset, id)
     __shared__ uint64_t pkey[kEntCap];
     {
@@ -336,7 +382,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
         if (c == C_KEEP) continue;
         const int t = S.e_t[e];
         const uint64_t rank = c == C_CARRY ? 0 : (c == C_ALLOC ? 1 : 2);
-        const uint64_t mid = c == C_FETCH ? (uint64_t)(a.t_host[t] / AL) : 0;
+        const uint64_t mid = c == C_FETCH ? (uint64_t)(t_host[t] / AL) : 0;
         const int k = atomicAdd(&s_nplaced, 1);
         pkey[k] = (rank << 62) | (mid << 20) | (uint64_t)t;
       }
@@ -344,6 +390,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       sort_keys(pkey, s_nplaced);
     }
     const int np = s_nplaced;
+    PSTAMP(9);
     // J. first fit by warp 0 (R11)
     if (tid < 32) {
       const int lane = tid;
@@ -351,7 +398,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       bool fail = false;
       for (int p = 0; p < np && !fail; ++p) {
         const int t = (int)(pkey[p] & 0xFFFFF);
-        const int64_t need_t = a.t_abytes[t];
+        const int64_t need_t = t_ab[t];
         int found = -1;
         for (int g0 = 0; g0 < ng; g0 += 32) {
           const int g = g0 + lane;
@@ -369,17 +416,19 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       if (lane == 0) s_compact = fail ? 1 : 0;
     }
     __syncthreads();
+    PSTAMP(10);
     // compaction fallback: exclusive prefix sums over [kept | placed]
     if (s_compact) {
       if (tid == 0) {
         int64_t c = 0;
-        for (int i = 0; i < nkept; ++i) { const int t = sc.kept[i]; sc.newoff[t] = c; c += a.t_abytes[t]; }
-        for (int p = 0; p < np; ++p) { const int t = (int)(pkey[p] & 0xFFFFF); sc.newoff[t] = c; c += a.t_abytes[t]; }
+        for (int i = 0; i < nkept; ++i) { const int t = sc.kept[i]; sc.newoff[t] = c; c += t_ab[t]; }
+        for (int p = 0; p < np; ++p) { const int t = (int)(pkey[p] & 0xFFFFF); sc.newoff[t] = c; c += t_ab[t]; }
       }
     } else {
       for (int i = tid; i < nkept; i += NT) sc.newoff[sc.kept[i]] = st.off[sc.kept[i]];
     }
     __syncthreads();
+    PSTAMP(11);
     // K. records
     if (c_ca + s_nc > out.cap_rec || c_al + s_na > out.cap_rec || c_fe + s_nf > out.cap_rec ||
         c_mv + nkept > out.cap_rec) {
@@ -387,6 +436,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       return;
     }
     // MOVE (compaction only): kept whose offset changed, in kept order
+    long long my_d2d = 0, my_h2d = 0;
     {
       int total = 0, base = 0;
       if (s_compact) {
@@ -400,9 +450,9 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
             r.t = t;
             r.src = (int64_t)m * H + st.off[t];
             r.dst = (int64_t)m * H + sc.newoff[t];
-            r.bytes = a.t_bytes[t];
+            r.bytes = t_by[t];
             out.mv[c_mv + base + p] = r;
-            atomicAdd(&s_d2d, (unsigned long long)a.t_bytes[t]);
+            my_d2d += t_by[t];
           }
           base += total;
           __syncthreads();
@@ -419,24 +469,24 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
         r.t = t;
         r.src = (int64_t)(1 - m) * H + st.off[t];
         r.dst = dst;
-        r.bytes = a.t_bytes[t];
+        r.bytes = t_by[t];
         r.late = st.pw[t] ? 1 : 0;
         out.ca[c_ca + p] = r;
-        atomicAdd(&s_d2d, (unsigned long long)a.t_bytes[t]);
+        my_d2d += t_by[t];
       } else if (p < nc + na) {
         dyo_alloc_rec r;
         r.t = t;
         r.dst = dst;
-        r.bytes = a.t_bytes[t];
+        r.bytes = t_by[t];
         out.al[c_al + p - nc] = r;
       } else {
         dyo_fetch_rec r;
         r.t = t;
-        r.host_off = a.t_host[t];
+        r.host_off = t_host[t];
         r.dst = dst;
-        r.bytes = a.t_bytes[t];
+        r.bytes = t_by[t];
         out.fe[c_fe + p - nc - na] = r;
-        atomicAdd(&s_h2d, (unsigned long long)a.t_bytes[t]);
+        my_h2d += t_by[t];
       }
     }
     const int64_t ebase_j = sc.ebase[j];
@@ -449,7 +499,13 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       r.dst = (int64_t)m * H + sc.newoff[t];
       out.ent[ebase_j + e] = r;
     }
+    {
+      const long long t1 = block_sum64(my_d2d, S.sum_tmp);
+      const long long t2 = block_sum64(my_h2d, S.sum_tmp);
+      if (tid == 0) { s_d2d = (unsigned long long)t1; s_h2d = (unsigned long long)t2; }
+    }
     __syncthreads();
+    PSTAMP(12);
     // L. state update
     for (int i = tid; i < nm; i += NT) {
       const int t = resm[i];
@@ -467,6 +523,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
     for (int e = tid; e < n; e += NT) {
       if (S.e_mode[e] & 2) st.dirty[S.e_t[e]] = 1;   // block j writes
     }
+    PSTAMP(13);
     // previous-group written flags, next occurrences, inW
     const int pn = st.prev_n[0];
     for (int i = tid; i < pn; i += NT) st.pw[st.prev[i]] = 0;
@@ -482,6 +539,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
     for (int i = tid; i < nm; i += NT) sc.rstat[resm[i]] = RS_NONE;
     if (tid == 0) st.prev_n[0] = n;
     __syncthreads();
+    PSTAMP(14);
     // resident lists: half m = kept + placed sorted by offset; half 1-m drops what left it
     {
       const int nnew = nkept + np;
@@ -512,6 +570,7 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
       for (int i = tid; i < base; i += NT) reso[i] = sc.kept[i];
       if (tid == 0) st.res_n[1 - m] = base;
     }
+    PSTAMP(15);
     // M. header
     if (tid == 0) {
       hd.half = m;
@@ -538,8 +597,26 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
     }
     __syncthreads();
   }
+  if (tid == 0) st.G[0] += Kt;
+  if (smem_state) {
+    __syncthreads();
+    for (int t = tid; t < T; t += NT) {
+      stg.loc[t] = st.loc[t];
+      stg.off[t] = st.off[t];
+      stg.dirty[t] = st.dirty[t];
+      stg.pw[t] = st.pw[t];
+      stg.res[t] = st.res[t];
+      stg.res[T + t] = st.res[T + t];
+      stg.prev[t] = st.prev[t];
+    }
+    if (tid == 0) {
+      stg.res_n[0] = st.res_n[0];
+      stg.res_n[1] = st.res_n[1];
+      stg.prev_n[0] = st.prev_n[0];
+      stg.G[0] = st.G[0];
+    }
+  }
   if (tid == 0) {
-    st.G[0] += Kt;
     out.counts[0] = Kt;
     out.counts[1] = (int)c_ev;
     out.counts[2] = (int)c_mv;
@@ -550,17 +627,33 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
   }
 }
 
+size_t plan_state_smem_bytes(int T) {
+  auto r16 = [](size_t b) { return (b + 15) / 16 * 16; };
+  const size_t t = (size_t)T;
+  return r16(8 * t) + 2 * r16(8 * (t + 1)) + 4 * r16(8 * t) + r16(8 * t) + 4 * r16(4 * t) + 3 * 16 + 6 * r16(t);
+}
+
+cudaError_t plan_debug_stamps(int j, unsigned long long* out) {
+  cudaError_t e = cudaMemcpyToSymbol(g_pstamp_j, &j, sizeof(int));
+  if (e == cudaSuccess && out) e = cudaMemcpyFromSymbol(out, g_pstamp, sizeof(unsigned long long) * 64);
+  return e;
+}
+
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,
                         PlanState& in, PlanState& work, PlanScratch& sc, PlanOut& out,
                         int max_groups, cudaStream_t s) {
   static bool attr = false;
-  const size_t smem = sizeof(PlanSmem);
+  constexpr int kMaxDyn = 227 * 1024 - 12 * 1024;      // leave room for the static shared arrays
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(plan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(plan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDyn);
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  plan_kernel<<<1, kPlanThreads, smem, s>>>(a, pd, b0, nb, policy, in, work, sc, out, max_groups);
+  const size_t base = (sizeof(PlanSmem) + 15) / 16 * 16;
+  const size_t need = base + plan_state_smem_bytes(a.T);
+  const int smem_state = (need <= (size_t)kMaxDyn && !getenv("DYO_PLAN_GLOBAL_STATE")) ? 1 : 0;
+  const size_t smem = smem_state ? need : sizeof(PlanSmem);
+  plan_kernel<<<1, kPlanThreads, smem, s>>>(a, pd, b0, nb, policy, in, work, sc, out, max_groups, smem_state);
   return cudaGetLastError();
 }
 

@@ -151,3 +151,12 @@ def test_state_unchanged_after_budget_error():
     K = d2.plan(stream=_stream())
     assert K == len(r0["trs"]) and gpu_lists(d2, 0) == tr_lists(r0["trs"][0])
     d.close(); d2.close()
+
+
+@pytest.mark.parametrize("name,steps", [("tiny", 4), ("moe", 3)])
+def test_plan_bitexact_global_state_path(name, steps, monkeypatch):
+    """The planner's global-memory state path (used when the per-tensor state does not fit in
+    shared memory) must give the same plans as the shared-memory path."""
+    monkeypatch.setenv("DYO_PLAN_GLOBAL_STATE", "1")
+    wl = WL.make(name, n_samples=32)
+    _run_plan_steps(wl, steps, 1, 1).close()

@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--budget-gib", type=float, default=0.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--dist-backend", default="nccl")
+    ap.add_argument("--compute", default="auto", choices=["auto", "none", "emulate"],
+                    help="emulate the DyNN's per-group compute with spin kernels (auto: on for af)")
     return ap.parse_args()
 
 
@@ -176,6 +178,29 @@ def run_reference(args):
 # B200 leg
 # ---------------------------------------------------------------------------------------------
 
+def calibrate_spin(torch):
+    """GPU cycles per microsecond of torch.cuda._sleep (the compute emulation's spin kernel)."""
+    s = torch.cuda.Stream()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(s):
+        torch.cuda._sleep(1000000)
+        a.record(s)
+        torch.cuda._sleep(20000000)
+        b.record(s)
+    b.synchronize()
+    return 20000000 / (a.elapsed_time(b) * 1e3)
+
+
+def group_compute_us(wl, j, K):
+    """Emulated compute of group j (survey §8(d) M2): Evoformer-shaped blocks of ~100 GFLOP forward
+    and 2x that backward at half the sustained bf16 rate (0.5 x 1398 TFLOPS) -> ~143 / ~286 us;
+    the final group ~10 us. Groups past the forward recycles are backward."""
+    blocks = wl.notes.get("blocks", 48)
+    if j == K - 1:
+        return 10.0
+    return 286.0 if j >= K - 1 - blocks else 143.0
+
+
 def pcie_probe(torch, nbytes=256 << 20, reps=5):
     h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
     d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
@@ -221,25 +246,44 @@ def run_dyo(args):
     hist_dev = torch.from_numpy(hist_np).to(dev) if hist_np is not None else None
     nS = len(wl.samples)
 
-    # Zero-duration compute blocks: block j "starts" and "ends" when ready[j] fires, so transition
-    # j's EVICT waits ready[j-2] (its half's last user) and overlaps transition j-1's FETCH.
+    # Blocks: without compute emulation, block j "starts" and "ends" when ready[j] fires, so
+    # transition j's EVICT waits ready[j-2] (its half's last user) and overlaps transition j-1's
+    # FETCH. With emulation, block j is a spin kernel on the compute stream after ready[j] whose
+    # duration follows the workload's per-group FLOPs; migrations wait on the block-end events.
+    emulate = args.compute == "emulate" or (args.compute == "auto" and args.config == "af")
     ready = [torch.cuda.Event() for _ in range(wl.K_max + 1)]
+    bend = [torch.cuda.Event() for _ in range(wl.K_max + 1)]
     t_start = torch.cuda.Event()
-    for e in ready + [t_start]:
+    s_comp = torch.cuda.Stream()
+    for e in ready + bend + [t_start]:
         e.record(s1)                          # materialise the cudaEvent_t handles
+    cyc_per_us = calibrate_spin(torch) if emulate else 0.0
+    comp_us_total = [0.0]
 
     def step(i, desc, hist):
         d.predict(desc, hist, 1, stream=s0.cuda_stream)
         K = d.plan(stream=s0.cuda_stream)
         h2d = d2h = 0
         t_start.record(s1)
+        if emulate:
+            s_comp.wait_event(t_start)
         for j in range(K):
             info = d.plan_info(j)
             h2d += info["h2d"]
             d2h += info["d2h"]
-            half_free = ready[j - 2] if j >= 2 else t_start
-            prev_done = ready[j - 1] if j >= 1 else t_start
+            ends = bend if emulate else ready
+            half_free = ends[j - 2] if j >= 2 else t_start
+            prev_done = ends[j - 1] if j >= 1 else t_start
             d.migrate(j, s1.cuda_stream, half_free.cuda_event, prev_done.cuda_event, ready[j].cuda_event)
+            if emulate:
+                us = group_compute_us(wl, j, K)
+                comp_us_total[0] += us
+                s_comp.wait_event(ready[j])
+                with torch.cuda.stream(s_comp):
+                    torch.cuda._sleep(int(us * cyc_per_us))
+                bend[j].record(s_comp)
+        if emulate:
+            s1.wait_stream(s_comp)
         return K, h2d, d2h
 
     def barrier():
@@ -256,6 +300,7 @@ def run_dyo(args):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     tot_h2d = tot_d2h = tot_K = 0
     plan_wall = []
+    comp_us_total[0] = 0.0
     with Clocks(local) as clk:
         e0.record(s0)
         for i in range(args.steps):
@@ -268,6 +313,7 @@ def run_dyo(args):
         e1.record(s0)
         e1.synchronize()
     barrier()
+    comp_ms_step = comp_us_total[0] / 1e3 / args.steps if emulate else 0.0
     ms = e0.elapsed_time(e1)
     tm = d.timings(reset=True)
     ctr = d.counters(reset=True)
@@ -369,6 +415,10 @@ def run_dyo(args):
                    "budget_bytes": wl.budget, "tensors": len(wl.tensors),
                    "l2": "inputs larger than L2 (every step moves >= 1 GiB through HBM and PCIe)",
                    "parallelism": f"{world} independent managers (replicas, no collective on the path)"},
+        "compute_emulation": ({"compute_ms_per_step": round(comp_ms_step, 3),
+                               "exposed_ms_per_step": round(ms_max / args.steps - comp_ms_step, 3),
+                               "exposed_frac_of_compute": round((ms_max / args.steps - comp_ms_step) / comp_ms_step, 4)}
+                              if emulate else None),
         "pilot_us_per_prediction": round(pred_us, 3),
         "pilot_kernel_us": round(pilot_kernel_us, 3), "decode_kernels_us": round(decode_us, 3),
         "predictions_per_s": round(1e6 / pred_us, 1),

@@ -260,18 +260,25 @@ def run_dyo(args):
     cyc_per_us = calibrate_spin(torch) if emulate else 0.0
     comp_us_total = [0.0]
 
-    def step(i, desc, hist):
+    def plan_next(desc, hist):
+        """Predict + plan one step (the plan is double-buffered: this may run while the previous
+        step's transitions are still migrating)."""
         d.predict(desc, hist, 1, stream=s0.cuda_stream)
         K = d.plan(stream=s0.cuda_stream)
         h2d = d2h = 0
-        t_start.record(s1)
-        if emulate:
-            s_comp.wait_event(t_start)
         for j in range(K):
             info = d.plan_info(j)
             h2d += info["h2d"]
             d2h += info["d2h"]
-            ends = bend if emulate else ready
+        return K, h2d, d2h
+
+    def enqueue(K):
+        """Enqueue every transition of the oldest outstanding plan (+ the emulated compute)."""
+        t_start.record(s1)
+        if emulate:
+            s_comp.wait_event(t_start)
+        ends = bend if emulate else ready
+        for j in range(K):
             half_free = ends[j - 2] if j >= 2 else t_start
             prev_done = ends[j - 1] if j >= 1 else t_start
             d.migrate(j, s1.cuda_stream, half_free.cuda_event, prev_done.cuda_event, ready[j].cuda_event)
@@ -284,7 +291,21 @@ def run_dyo(args):
                 bend[j].record(s_comp)
         if emulate:
             s1.wait_stream(s_comp)
-        return K, h2d, d2h
+
+    def run_steps(n, first, inputs):
+        """n steps with plan lookahead: step i's transitions are enqueued, then step i+1 is
+        predicted and planned while they run."""
+        tot = [0, 0, 0]
+        pending = plan_next(*inputs(first))
+        for i in range(n):
+            K, h2d, d2h = pending
+            enqueue(K)
+            tot[0] += K
+            tot[1] += h2d
+            tot[2] += d2h
+            if i + 1 < n:
+                pending = plan_next(*inputs(first + i + 1))
+        return tot
 
     def barrier():
         if world > 1:
@@ -292,8 +313,8 @@ def run_dyo(args):
         torch.cuda.synchronize()
 
     _log("warmup")
-    for i in range(args.warmup):
-        step(i, desc_dev[i % nS: i % nS + 1], hist_dev)
+    dev_inputs = lambda k: (desc_dev[k % nS: k % nS + 1], hist_dev)
+    run_steps(args.warmup, 0, dev_inputs)
     barrier()
     d.timings(reset=True)
     d.counters(reset=True)
@@ -303,12 +324,7 @@ def run_dyo(args):
     comp_us_total[0] = 0.0
     with Clocks(local) as clk:
         e0.record(s0)
-        for i in range(args.steps):
-            k = (args.warmup + i) % nS
-            K, h2d, d2h = step(i, desc_dev[k: k + 1], hist_dev)
-            tot_K += K
-            tot_h2d += h2d
-            tot_d2h += d2h
+        tot_K, tot_h2d, tot_d2h = run_steps(args.steps, args.warmup, dev_inputs)
         s0.wait_stream(s1)
         e1.record(s0)
         e1.synchronize()
@@ -324,9 +340,8 @@ def run_dyo(args):
     hist_host = torch.from_numpy(hist_np).pin_memory() if hist_np is not None else None
     barrier()
     t0 = time.perf_counter()
-    for i in range(args.steps):
-        k = (args.warmup + args.steps + i) % nS
-        step(i, desc_host[k: k + 1].numpy(), hist_host.numpy() if hist_host is not None else None)
+    host_inputs = lambda k: (desc_host[k % nS: k % nS + 1].numpy(), hist_host.numpy() if hist_host is not None else None)
+    run_steps(args.steps, args.warmup + args.steps, host_inputs)
     s1.synchronize()
     barrier()
     e2e_s = time.perf_counter() - t0

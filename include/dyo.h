@@ -212,17 +212,23 @@ dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* out, i
 /* A4: plan every transition of the predictions [b0, b0 + n) of the last predict, concatenated
  * in sample order (n = -1: all). Runs the planner kernel on `stream`, then synchronises once
  * and copies the plan lists to pinned host memory (the DMA issue needs host-visible sizes).
- * On DYO_E_BUDGET / DYO_E_CAPACITY the residency state is unchanged. *K_out = transitions. */
+ * On DYO_E_BUDGET / DYO_E_CAPACITY the residency state is unchanged. *K_out = transitions.
+ * Plans are double-buffered (plan lookahead): the next step may be predicted and planned while
+ * the previous plan's transitions are still migrating - the planned state does not depend on the
+ * migrations' progress - so the pilot runs ahead of the batch as in the paper. At most
+ * two plans may be outstanding (DYO_E_STATE otherwise); a new plan waits (host) for the
+ * migrations of the plan two generations back to finish. */
 dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* stream);
 
-/* Host copies of the current plan (valid until the next dyo_plan). */
+/* Host copies of the most recent plan (valid until the dyo_plan after next). */
 dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info);
 /* list: 0 evict, 1 move, 2 carry, 3 alloc, 4 fetch, 5 entries (with placement); returns a
  * pointer to the transition's records (host memory owned by the ctx) and their count. */
 dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** recs,
                             int32_t* n);
 
-/* A5: execute transition j (j = 0, 1, ... in order; DYO_E_STATE otherwise):
+/* A5: execute transition j of the OLDEST plan that still has transitions to enqueue (plans
+ * migrate in FIFO order; j = 0, 1, ... in order; DYO_E_STATE otherwise):
  *   EVICT writebacks (D2H: DMA per host run, K3 pack + DMA for scattered sources, K5 zero-copy
  *   for small runs) on a ctx-owned D2H stream, after ev_half_free = the end of block j-2, the
  *   last user of half m (NULL: after everything already enqueued on copy_stream); then on

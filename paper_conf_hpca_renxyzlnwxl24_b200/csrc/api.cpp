@@ -52,19 +52,26 @@ struct dyo_ctx {
   PlanState state[2]{};
   int committed = 0;
   PlanScratch sc{};
-  PlanOut out{};                   // host (pinned) mirrors of the plan records + headers
-  PlanOut dout{};                  // device record arrays the planner kernel writes
+  // Two plan slots: dyo_plan fills slot (plan_seq & 1) while the previous plan may still be
+  // migrating (plan lookahead); dyo_migrate continues the oldest plan with transitions left.
+  struct PlanSlot {
+    PlanOut out{};                 // host (pinned) mirrors of the plan records + headers
+    PlanOut dout{};                // device record arrays the planner kernel writes
+    CopySeg* h_segs = nullptr;     // pinned mapped work items for the copy kernels
+    int64_t seg_cap = 0, seg_used = 0;
+    int K = 0, next_j = 0;
+    bool valid = false;
+    cudaEvent_t ev_last = nullptr; // recorded after every migrate of this plan
+    bool ev_pending = false;
+  };
+  PlanSlot slot[2];
+  int64_t plan_seq = 0, mig_seq = 0;
   int32_t* h_status = nullptr;     // pinned mapped
   int32_t* h_counts = nullptr;
   int8_t* h_loc = nullptr;         // pinned mirrors of the committed residency
   int64_t* h_off = nullptr;
-  int plan_K = 0, next_j = 0;
-  bool plan_valid = false;
+
   // migration
-  CopySeg* h_segs = nullptr;       // pinned mapped work items for the copy kernels
-  int64_t seg_cap = 0, seg_used = 0;
-  cudaEvent_t ev_last = nullptr;
-  bool ev_pending = false;
   cudaStream_t d2h = nullptr;      // ctx-owned stream for the EVICT (D2H) phase
   cudaStream_t side = nullptr;     // ctx-owned stream for early CARRY (overlaps FETCH)
   cudaEvent_t ev_entry = nullptr, ev_evict = nullptr, ev_moves = nullptr, ev_carry = nullptr;
@@ -148,13 +155,21 @@ bool is_device_ptr(const void* p) {
 
 void free_plan_host(dyo_ctx* c) {
   auto fh = [](void* p) { if (p) cudaFreeHost(p); };
-  fh(c->out.hdr); fh(c->out.ent); fh(c->out.ev); fh(c->out.mv); fh(c->out.ca); fh(c->out.al);
-  fh(c->out.fe); fh(c->h_status); fh(c->h_counts); fh(c->h_loc); fh(c->h_off); fh(c->h_segs);
-  c->out = PlanOut{};
+  for (auto& P : c->slot) {
+    fh(P.out.hdr); fh(P.out.ent); fh(P.out.ev); fh(P.out.mv); fh(P.out.ca); fh(P.out.al); fh(P.out.fe);
+    fh(P.h_segs);
+    P.out = PlanOut{};
+    P.dout = PlanOut{};
+    P.h_segs = nullptr;
+    P.valid = false;
+    P.K = P.next_j = 0;
+    P.seg_used = 0;
+  }
+  fh(c->h_status); fh(c->h_counts); fh(c->h_loc); fh(c->h_off);
   c->h_status = c->h_counts = nullptr;
   c->h_loc = nullptr;
   c->h_off = nullptr;
-  c->h_segs = nullptr;
+  c->plan_seq = c->mig_seq = 0;
 }
 
 // timing helpers (no-ops unless DYO_F_TIMING)
@@ -432,7 +447,8 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   cudaError_t e = cudaSetDevice(device);
   if (e == cudaSuccess) e = cudaMalloc(&ctx->arena, 2 * ctx->H);
   if (e == cudaSuccess) e = cudaMalloc(&ctx->staging, c.staging_bytes);
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_last, cudaEventDisableTiming);
+  for (auto& P : ctx->slot)
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&P.ev_last, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_entry, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_evict, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->d2h, cudaStreamNonBlocking);
@@ -459,7 +475,8 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->host_pool) cudaFreeHost(ctx->host_pool);
   if (ctx->arena) cudaFree(ctx->arena);
   if (ctx->staging) cudaFree(ctx->staging);
-  if (ctx->ev_last) cudaEventDestroy(ctx->ev_last);
+  for (auto& P : ctx->slot)
+    if (P.ev_last) cudaEventDestroy(P.ev_last);
   if (ctx->ev_entry) cudaEventDestroy(ctx->ev_entry);
   if (ctx->ev_evict) cudaEventDestroy(ctx->ev_evict);
   if (ctx->d2h) cudaStreamDestroy(ctx->d2h);
@@ -480,7 +497,6 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   free_plan_host(ctx);
   if (ctx->host_pool) { cudaFreeHost(ctx->host_pool); ctx->host_pool = nullptr; }
   ctx->arch_ok = false;
-  ctx->plan_valid = false;
   const int64_t AL = ctx->cfg.align;
   ArchHost h;
   dyo_status pst = parse_arch(A, AL, h, ctx->err);
@@ -558,43 +574,46 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
     memset(*p, 0, std::max<size_t>(bytes, 64));
     return DYO_OK;
   };
-  PlanOut& o = ctx->out;
-  o = PlanOut{};
-  o.cap_ent = cap_ent;
-  o.cap_rec = cap_rec;
-  if ((st = hmap((void**)&o.hdr, sizeof(PlanHdr) * mg))) return st;
-  if ((st = hmap((void**)&o.ent, sizeof(dyo_entry_rec) * cap_ent))) return st;
-  if ((st = hmap((void**)&o.ev, sizeof(dyo_evict_rec) * cap_rec))) return st;
-  if ((st = hmap((void**)&o.mv, sizeof(dyo_move_rec) * cap_rec))) return st;
-  if ((st = hmap((void**)&o.ca, sizeof(dyo_carry_rec) * cap_rec))) return st;
-  if ((st = hmap((void**)&o.al, sizeof(dyo_alloc_rec) * cap_rec))) return st;
-  if ((st = hmap((void**)&o.fe, sizeof(dyo_fetch_rec) * cap_rec))) return st;
-  // the planner writes its records to device memory (writes to pinned host memory from a
-  // latency-bound single-CTA kernel stall its barriers); dyo_plan copies them back by count
-  PlanOut& dO = ctx->dout;
-  dO = PlanOut{};
-  dO.cap_ent = cap_ent;
-  dO.cap_rec = cap_rec;
-  {
-    PlanHdr* h1; dyo_entry_rec* e1; dyo_evict_rec* v1; dyo_move_rec* m1; dyo_carry_rec* c1; dyo_alloc_rec* a1; dyo_fetch_rec* f1;
-    DA(h1, mg); DA(e1, cap_ent); DA(v1, cap_rec); DA(m1, cap_rec); DA(c1, cap_rec); DA(a1, cap_rec); DA(f1, cap_rec);
-    dO.hdr = h1; dO.ent = e1; dO.ev = v1; dO.mv = m1; dO.ca = c1; dO.al = a1; dO.fe = f1;
-  }
   if ((st = hmap((void**)&ctx->h_status, 16 * sizeof(int32_t)))) return st;
   if ((st = hmap((void**)&ctx->h_counts, 16 * sizeof(int32_t)))) return st;
   if ((st = hmap((void**)&ctx->h_loc, T))) return st;
   if ((st = hmap((void**)&ctx->h_off, sizeof(int64_t) * T))) return st;
   memset(ctx->h_loc, 0xff, T);
-  ctx->seg_cap = 8 * cap_rec + 65536;
-  if ((st = hmap((void**)&ctx->h_segs, sizeof(CopySeg) * ctx->seg_cap))) return st;
   int32_t* d_status = nullptr;
   int32_t* d_counts = nullptr;
   CK(cudaHostGetDevicePointer((void**)&d_status, ctx->h_status, 0));
   CK(cudaHostGetDevicePointer((void**)&d_counts, ctx->h_counts, 0));
-  o.status = d_status;
-  o.counts = d_counts;
-  dO.status = d_status;
-  dO.counts = d_counts;
+  for (auto& P : ctx->slot) {
+    PlanOut& o = P.out;
+    o = PlanOut{};
+    o.cap_ent = cap_ent;
+    o.cap_rec = cap_rec;
+    if ((st = hmap((void**)&o.hdr, sizeof(PlanHdr) * mg))) return st;
+    if ((st = hmap((void**)&o.ent, sizeof(dyo_entry_rec) * cap_ent))) return st;
+    if ((st = hmap((void**)&o.ev, sizeof(dyo_evict_rec) * cap_rec))) return st;
+    if ((st = hmap((void**)&o.mv, sizeof(dyo_move_rec) * cap_rec))) return st;
+    if ((st = hmap((void**)&o.ca, sizeof(dyo_carry_rec) * cap_rec))) return st;
+    if ((st = hmap((void**)&o.al, sizeof(dyo_alloc_rec) * cap_rec))) return st;
+    if ((st = hmap((void**)&o.fe, sizeof(dyo_fetch_rec) * cap_rec))) return st;
+    // the planner writes its records to device memory (writes to pinned host memory from a
+    // latency-bound single-CTA kernel are avoided); dyo_plan copies them back by count
+    PlanOut& dO = P.dout;
+    dO = PlanOut{};
+    dO.cap_ent = cap_ent;
+    dO.cap_rec = cap_rec;
+    PlanHdr* h1; dyo_entry_rec* e1; dyo_evict_rec* v1; dyo_move_rec* m1; dyo_carry_rec* c1; dyo_alloc_rec* a1; dyo_fetch_rec* f1;
+    DA(h1, mg); DA(e1, cap_ent); DA(v1, cap_rec); DA(m1, cap_rec); DA(c1, cap_rec); DA(a1, cap_rec); DA(f1, cap_rec);
+    dO.hdr = h1; dO.ent = e1; dO.ev = v1; dO.mv = m1; dO.ca = c1; dO.al = a1; dO.fe = f1;
+    P.seg_cap = 8 * cap_rec + 65536;
+    if ((st = hmap((void**)&P.h_segs, sizeof(CopySeg) * P.seg_cap))) return st;
+    o.status = dO.status = d_status;
+    o.counts = dO.counts = d_counts;
+    P.valid = false;
+    P.K = P.next_j = 0;
+    P.seg_used = 0;
+    P.ev_pending = false;
+  }
+  ctx->plan_seq = ctx->mig_seq = 0;
 #undef DA
   // ---- host pool (pinned, mapped: DMA and zero-copy kernels) ----
   ctx->host_bytes = pool;
@@ -844,16 +863,19 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
   if (b0 < 0 || n < 1 || b0 + n > ctx->last_B) return fail(ctx, DYO_E_INVAL, "prediction range");
   CK(cudaSetDevice(ctx->device));
   cudaStream_t st = (cudaStream_t)stream;
-  // the pinned plan lists and copy descriptors are about to be rewritten: the previous plan's
-  // migrations must have consumed them
-  if (ctx->ev_pending) { CK(cudaEventSynchronize(ctx->ev_last)); ctx->ev_pending = false; }
-  ctx->plan_valid = false;
+  // plan slot (plan_seq & 1): its previous plan (two generations back) must be fully enqueued
+  // and its migrations must have consumed the pinned lists and copy descriptors
+  dyo_ctx::PlanSlot& P = ctx->slot[ctx->plan_seq & 1];
+  if (P.valid && P.next_j < P.K)
+    return fail(ctx, DYO_E_STATE, "two plans are outstanding: migrate the older one first");
+  if (P.ev_pending) { CK(cudaEventSynchronize(P.ev_last)); P.ev_pending = false; }
+  P.valid = false;
   ctx->h_status[0] = -100;
   PlanState& in = ctx->state[ctx->committed];
   PlanState& wk = ctx->state[1 - ctx->committed];
   {
     TScope ts(ctx, 2, st);
-    CK(launch_plan(ctx->ad, ctx->pd, b0, n, ctx->cfg.policy, in, wk, ctx->sc, ctx->dout, ctx->max_groups, st));
+    CK(launch_plan(ctx->ad, ctx->pd, b0, n, ctx->cfg.policy, in, wk, ctx->sc, P.dout, ctx->max_groups, st));
   }
   CK(cudaMemcpyAsync(ctx->h_loc, wk.loc, ctx->T, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(ctx->h_off, wk.off, sizeof(int64_t) * ctx->T, cudaMemcpyDeviceToHost, st));
@@ -870,8 +892,8 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
   {
     // copy the plan (headers + every record list, exact counts) to the pinned host mirrors
     const int32_t* c = ctx->h_counts;
-    const PlanOut& D = ctx->dout;
-    PlanOut& Hm = ctx->out;
+    const PlanOut& D = P.dout;
+    PlanOut& Hm = P.out;
     int64_t n_ent = 0;
     if (c[0] > 0) {
       CK(cudaMemcpyAsync(Hm.hdr, D.hdr, sizeof(PlanHdr) * c[0], cudaMemcpyDeviceToHost, st));
@@ -887,19 +909,24 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
     CK(cudaStreamSynchronize(st));
   }
   ctx->committed = 1 - ctx->committed;
-  ctx->plan_K = ctx->h_counts[0];
-  ctx->next_j = 0;
-  ctx->seg_used = 0;
-  ctx->plan_valid = true;
-  if (K_out) *K_out = ctx->plan_K;
+  P.K = ctx->h_counts[0];
+  P.next_j = 0;
+  P.seg_used = 0;
+  P.valid = true;
+  if (ctx->mig_seq < ctx->plan_seq && !(ctx->slot[ctx->mig_seq & 1].valid &&
+                                        ctx->slot[ctx->mig_seq & 1].next_j < ctx->slot[ctx->mig_seq & 1].K))
+    ctx->mig_seq = ctx->plan_seq;            // the older plan is fully enqueued
+  ctx->plan_seq += 1;
+  if (K_out) *K_out = P.K;
   return DYO_OK;
 }
 
 dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info) {
   if (!ctx || !info) return DYO_E_INVAL;
-  if (!ctx->plan_valid) return fail(ctx, DYO_E_STATE, "no valid plan");
-  if (j < 0 || j >= ctx->plan_K) return DYO_E_INVAL;
-  const PlanHdr& h = ctx->out.hdr[j];
+  if (ctx->plan_seq == 0 || !ctx->slot[(ctx->plan_seq - 1) & 1].valid) return fail(ctx, DYO_E_STATE, "no valid plan");
+  const dyo_ctx::PlanSlot& P = ctx->slot[(ctx->plan_seq - 1) & 1];
+  if (j < 0 || j >= P.K) return DYO_E_INVAL;
+  const PlanHdr& h = P.out.hdr[j];
   info->half = h.half; info->n_entries = h.n_ent; info->n_evict = h.n_evict; info->n_move = h.n_move;
   info->n_carry = h.n_carry; info->n_alloc = h.n_alloc; info->n_fetch = h.n_fetch;
   info->need = h.need; info->h2d = h.h2d; info->d2h = h.d2h; info->d2d = h.d2d;
@@ -908,16 +935,17 @@ dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info) {
 
 dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** recs, int32_t* n) {
   if (!ctx || !recs || !n) return DYO_E_INVAL;
-  if (!ctx->plan_valid) return fail(ctx, DYO_E_STATE, "no valid plan");
-  if (j < 0 || j >= ctx->plan_K) return DYO_E_INVAL;
-  const PlanHdr& h = ctx->out.hdr[j];
+  if (ctx->plan_seq == 0 || !ctx->slot[(ctx->plan_seq - 1) & 1].valid) return fail(ctx, DYO_E_STATE, "no valid plan");
+  const dyo_ctx::PlanSlot& P = ctx->slot[(ctx->plan_seq - 1) & 1];
+  if (j < 0 || j >= P.K) return DYO_E_INVAL;
+  const PlanHdr& h = P.out.hdr[j];
   switch (list) {
-    case 0: *recs = ctx->out.ev + h.o_evict; *n = h.n_evict; break;
-    case 1: *recs = ctx->out.mv + h.o_move; *n = h.n_move; break;
-    case 2: *recs = ctx->out.ca + h.o_carry; *n = h.n_carry; break;
-    case 3: *recs = ctx->out.al + h.o_alloc; *n = h.n_alloc; break;
-    case 4: *recs = ctx->out.fe + h.o_fetch; *n = h.n_fetch; break;
-    case 5: *recs = ctx->out.ent + h.o_ent; *n = h.n_ent; break;
+    case 0: *recs = P.out.ev + h.o_evict; *n = h.n_evict; break;
+    case 1: *recs = P.out.mv + h.o_move; *n = h.n_move; break;
+    case 2: *recs = P.out.ca + h.o_carry; *n = h.n_carry; break;
+    case 3: *recs = P.out.al + h.o_alloc; *n = h.n_alloc; break;
+    case 4: *recs = P.out.fe + h.o_fetch; *n = h.n_fetch; break;
+    case 5: *recs = P.out.ent + h.o_ent; *n = h.n_ent; break;
     default: return DYO_E_INVAL;
   }
   return DYO_OK;
@@ -931,21 +959,27 @@ struct Run { int64_t host_off, dev_off, bytes; bool dev_contig; int first, count
 constexpr int64_t kChunk = 256 << 10;   // copy-kernel work item
 
 // push (src, dst, bytes) split into work items; returns false on capacity
+// the slot being migrated (set by dyo_migrate before it pushes descriptors)
+thread_local dyo_ctx::PlanSlot* g_mslot = nullptr;
+
 bool push_seg(dyo_ctx* ctx, const char* src, char* dst, int64_t bytes) {
+  dyo_ctx::PlanSlot& P = *g_mslot;
+  (void)ctx;
   for (int64_t o = 0; o < bytes; o += kChunk) {
-    if (ctx->seg_used >= ctx->seg_cap) return false;
-    ctx->h_segs[ctx->seg_used++] = CopySeg{src + o, dst + o, std::min(kChunk, bytes - o)};
+    if (P.seg_used >= P.seg_cap) return false;
+    P.h_segs[P.seg_used++] = CopySeg{src + o, dst + o, std::min(kChunk, bytes - o)};
   }
   return true;
 }
 
 dyo_status launch_segs(dyo_ctx* ctx, int64_t first, cudaStream_t s, int grid, int kind = 3) {
-  const int64_t n = ctx->seg_used - first;
+  dyo_ctx::PlanSlot& P = *g_mslot;
+  const int64_t n = P.seg_used - first;
   if (n <= 0) return DYO_OK;
   CopySeg* dptr = nullptr;
-  CK(cudaHostGetDevicePointer((void**)&dptr, ctx->h_segs + first, 0));
+  CK(cudaHostGetDevicePointer((void**)&dptr, P.h_segs + first, 0));
   int64_t bytes = 0;
-  for (int64_t i = first; i < ctx->seg_used; ++i) bytes += ctx->h_segs[i].bytes;
+  for (int64_t i = first; i < P.seg_used; ++i) bytes += P.h_segs[i].bytes;
   TScope ts(ctx, kind, s, bytes);
   CK(launch_copy_segments(dptr, (int)n, kChunk, grid, s));
   ctx->ctr.n_kernels++;
@@ -957,12 +991,20 @@ dyo_status launch_segs(dyo_ctx* ctx, int64_t first, cudaStream_t s, int grid, in
 dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half_free, void* ev_prev_done,
                        void* ev_ready) {
   if (!ctx) return DYO_E_INVAL;
-  if (!ctx->plan_valid) return fail(ctx, DYO_E_STATE, "dyo_migrate before a successful dyo_plan");
-  if (j != ctx->next_j || j >= ctx->plan_K) return fail(ctx, DYO_E_STATE, "transition %d out of order (next %d)", j, ctx->next_j);
+  // the oldest plan with transitions left (plans migrate in FIFO order, at most two outstanding)
+  while (ctx->mig_seq < ctx->plan_seq) {
+    dyo_ctx::PlanSlot& Q = ctx->slot[ctx->mig_seq & 1];
+    if (Q.valid && Q.next_j < Q.K) break;
+    ctx->mig_seq += 1;
+  }
+  if (ctx->mig_seq >= ctx->plan_seq) return fail(ctx, DYO_E_STATE, "dyo_migrate without a pending plan");
+  dyo_ctx::PlanSlot& P = ctx->slot[ctx->mig_seq & 1];
+  if (j != P.next_j || j >= P.K) return fail(ctx, DYO_E_STATE, "transition %d out of order (next %d)", j, P.next_j);
   if (!ctx->host_pool) return fail(ctx, DYO_E_STATE, "plan-only ctx (DYO_F_NO_HOST_POOL) cannot migrate");
   CK(cudaSetDevice(ctx->device));
+  g_mslot = &P;
   cudaStream_t s = (cudaStream_t)copy_stream;
-  const PlanHdr& h = ctx->out.hdr[j];
+  const PlanHdr& h = P.out.hdr[j];
   char* arena = ctx->arena;
   char* host = ctx->host_pool;
   const int64_t AL = ctx->cfg.align;
@@ -988,7 +1030,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   //    through staging when the device sources are scattered), or one zero-copy scatter launch
   //    (K5) for the runs below dma_min
   {
-    const dyo_evict_rec* ev = ctx->out.ev + h.o_evict;
+    const dyo_evict_rec* ev = P.out.ev + h.o_evict;
     std::vector<int> small;
     int i = 0;
     while (i < h.n_evict) {
@@ -1015,7 +1057,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
         int q = r.first;
         while (q < r.first + r.count) {
           const int64_t base = ev[q].host_off;
-          const int64_t seg0 = ctx->seg_used;
+          const int64_t seg0 = P.seg_used;
           int q2 = q;
           while (q2 < r.first + r.count && ev[q2].host_off + ev[q2].bytes - base <= stage_half) {
             if (!push_seg(ctx, arena + ev[q2].src, stage_pack + (ev[q2].host_off - base), ev[q2].bytes))
@@ -1046,7 +1088,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
       i = k;
     }
     if (!small.empty()) {
-      const int64_t g0 = ctx->seg_used;
+      const int64_t g0 = P.seg_used;
       for (int q : small) {
         if (!push_seg(ctx, arena + ev[q].src, host + ev[q].host_off, ev[q].bytes))
           return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
@@ -1066,7 +1108,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   //    non-overlapping (destination vs source) moves, one copy-kernel launch per wave. A move
   //    overlapping its own source goes through the staging buffer in pieces.
   {
-    const dyo_move_rec* mv = ctx->out.mv + h.o_move;
+    const dyo_move_rec* mv = P.out.mv + h.o_move;
     int64_t wave0 = -1;
     std::vector<std::pair<int64_t, int64_t>> wave_src;    // source ranges of the open wave
     auto flush = [&]() -> dyo_status {
@@ -1086,11 +1128,11 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
         if (s1) return s1;
         for (int64_t o = 0; o < nbytes; o += stage_half) {
           const int64_t n = std::min(stage_half, nbytes - o);
-          const int64_t g0 = ctx->seg_used;
+          const int64_t g0 = P.seg_used;
           if (!push_seg(ctx, arena + src + o, stage_move, n)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
           s1 = launch_segs(ctx, g0, s, d2d_grid);
           if (s1) return s1;
-          const int64_t g1 = ctx->seg_used;
+          const int64_t g1 = P.seg_used;
           if (!push_seg(ctx, stage_move, arena + dst + o, n)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
           s1 = launch_segs(ctx, g1, s, d2d_grid);
           if (s1) return s1;
@@ -1104,7 +1146,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
         dyo_status s1 = flush();
         if (s1) return s1;
       }
-      if (wave0 < 0) wave0 = ctx->seg_used;
+      if (wave0 < 0) wave0 = P.seg_used;
       if (!push_seg(ctx, arena + src, arena + dst, nbytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
       wave_src.push_back({src, src + nbytes});
     }
@@ -1118,14 +1160,14 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   //    other half (read-only here)
   bool carry_side = false;
   {
-    const dyo_carry_rec* ca = ctx->out.ca + h.o_carry;
-    const int64_t g0 = ctx->seg_used;
+    const dyo_carry_rec* ca = P.out.ca + h.o_carry;
+    const int64_t g0 = P.seg_used;
     for (int i = 0; i < h.n_carry; ++i) {
       if (ca[i].late) continue;
       if (!push_seg(ctx, arena + ca[i].src, arena + ca[i].dst, ca[i].bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
       ctx->ctr.d2d += ca[i].bytes;
     }
-    if (ctx->seg_used > g0) {
+    if (P.seg_used > g0) {
       CK(cudaEventRecord(ctx->ev_moves, s));
       CK(cudaStreamWaitEvent(ctx->side, ctx->ev_moves, 0));
       dyo_status s1 = launch_segs(ctx, g0, ctx->side, d2d_grid);
@@ -1135,8 +1177,8 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
     }
   }
   {
-    const dyo_fetch_rec* fe = ctx->out.fe + h.o_fetch;
-    const int64_t g0 = ctx->seg_used;
+    const dyo_fetch_rec* fe = P.out.fe + h.o_fetch;
+    const int64_t g0 = P.seg_used;
     int i = 0;
     while (i < h.n_fetch) {
       int64_t hend = fe[i].host_off + align_up(fe[i].bytes, AL);
@@ -1169,12 +1211,12 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   if (carry_side) CK(cudaStreamWaitEvent(s, ctx->ev_carry, 0));
   // 4. late CARRY: block j-1 writes them, so they wait for its end
   {
-    const dyo_carry_rec* ca = ctx->out.ca + h.o_carry;
+    const dyo_carry_rec* ca = P.out.ca + h.o_carry;
     bool any = false;
     for (int i = 0; i < h.n_carry; ++i) any |= ca[i].late != 0;
     if (any) {
       if (ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
-      const int64_t g0 = ctx->seg_used;
+      const int64_t g0 = P.seg_used;
       for (int i = 0; i < h.n_carry; ++i) {
         if (!ca[i].late) continue;
         if (!push_seg(ctx, arena + ca[i].src, arena + ca[i].dst, ca[i].bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
@@ -1186,9 +1228,9 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   }
   TRACE("  transition %d issued", j);
   if (ev_ready) CK(cudaEventRecord((cudaEvent_t)ev_ready, s));
-  CK(cudaEventRecord(ctx->ev_last, s));
-  ctx->ev_pending = true;
-  ctx->next_j = j + 1;
+  CK(cudaEventRecord(P.ev_last, s));
+  P.ev_pending = true;
+  P.next_j = j + 1;
   return DYO_OK;
 }
 

@@ -130,7 +130,7 @@ def test_af_scaled_recycling():
     run_bytes(wl, 3, 1)
 
 
-def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0):
+def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0, lookahead=False):
     """The full event protocol, enqueued asynchronously: emulated compute block j runs on its own
     stream after ready[j]; transition j's EVICT waits end[j-2], its late carries end[j-1].
     Read mismatches are accumulated on the device; the host syncs once per step."""
@@ -150,32 +150,46 @@ def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0):
     st = PL.initial_state(len(wl.tensors))
     table = ()
     ver = [0] * len(wl.tensors)
-    for s in range(steps):
-        r = oracle_step(wl, [s % len(wl.samples)], st, table, policy)
-        d.predict(wl.samples[[s % len(wl.samples)]].copy(), hist_for(wl, 1), 1,
-                  stream=torch.cuda.current_stream().cuda_stream)
-        K = d.plan(stream=torch.cuda.current_stream().cuda_stream)
+    cs = torch.cuda.current_stream().cuda_stream
+
+    def plan_step(s, st_, table_):
+        r = oracle_step(wl, [s % len(wl.samples)], st_, table_, policy)
+        d.predict(wl.samples[[s % len(wl.samples)]].copy(), hist_for(wl, 1), 1, stream=cs)
+        K = d.plan(stream=cs)
         assert K == len(r["trs"])
+        ents = [d.plan_records(j, "entries").tolist() for j in range(K)]
+        for j, tr in enumerate(r["trs"]):
+            assert gpu_lists(d, j) == tr_lists(tr)
+        return r, K, ents
+
+    pending = plan_step(0, st, table)
+    for s in range(steps):
+        r, K, ents = pending
+        if lookahead and s + 1 < steps:
+            # plan the next step BEFORE this step's transitions are enqueued: two plans outstanding
+            pending = plan_step(s + 1, r["state"], r["table"])
         t0.record(s_copy)
         fresh = set()
         for j in range(K):
             hf = end[j - 2] if j >= 2 else t0
             pd = end[j - 1] if j >= 1 else t0
             d.migrate(j, s_copy.cuda_stream, hf.cuda_event, pd.cuda_event, ready[j].cuda_event)
-            ent = d.plan_records(j, "entries").tolist()
             s_comp.wait_event(ready[j])
             with torch.cuda.stream(s_comp):
-                for (t, mode, rd, dst) in ent:
+                for (t, mode, rd, dst) in ents[j]:
                     nb = wl.tensors[t].nbytes
                     if rd and (not wl.tensors[t].transient or t in fresh):
                         bad += (arena[dst: dst + nb].view(torch.int32) != _words(t, ver[t], nb)).sum()
-                for (t, mode, rd, dst) in ent:
+                for (t, mode, rd, dst) in ents[j]:
                     if mode & 2:
                         ver[t] += 1
                         fresh.add(t)
                         nb = wl.tensors[t].nbytes
                         arena[dst: dst + nb].view(torch.int32).copy_(_words(t, ver[t], nb))
             end[j].record(s_comp)
+        s_copy.wait_stream(s_comp)
+        if not lookahead and s + 1 < steps:
+            pending = plan_step(s + 1, r["state"], r["table"])
         torch.cuda.synchronize()
         assert int(bad.item()) == 0, f"step {s}: {int(bad.item())} stale words"
         st, table = r["state"], r["table"]
@@ -217,3 +231,14 @@ def test_moe_scaled_packed_writebacks_small_staging():
 
 def test_tiny_compaction_moves_small_staging_pipelined():
     run_pipelined(_tiny_with_moves(), 4, 1, staging=8 << 20)   # 4 MiB halves: tensors split into pieces
+
+
+def test_pipelined_plan_lookahead_moe_scaled():
+    """Two plans outstanding: step s+1 is predicted and planned before step s's transitions are
+    enqueued; dyo_migrate must continue the older plan (FIFO) and the bytes stay exact."""
+    wl = WL.make_moe(seed=4, n_samples=8, expert_mib=1, act_mib=1, budget=96 << 20)
+    run_pipelined(wl, 4, 1, dma_min=1 << 20, lookahead=True)
+
+
+def test_pipelined_plan_lookahead_tiny_compaction():
+    run_pipelined(_tiny_with_moves(), 4, 1, lookahead=True)

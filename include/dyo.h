@@ -217,7 +217,8 @@ dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* out, i
  * the previous plan's transitions are still migrating - the planned state does not depend on the
  * migrations' progress - so the pilot runs ahead of the batch as in the paper. At most
  * two plans may be outstanding (DYO_E_STATE otherwise); a new plan waits (host) for the
- * migrations of the plan two generations back to finish. */
+ * migrations of the plan two generations back to finish. In a plan-only ctx
+ * (DYO_F_NO_HOST_POOL) each plan supersedes the previous ones. */
 dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* stream);
 
 /* Host copies of the most recent plan (valid until the dyo_plan after next). */

@@ -865,8 +865,16 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
   cudaStream_t st = (cudaStream_t)stream;
   // plan slot (plan_seq & 1): its previous plan (two generations back) must be fully enqueued
   // and its migrations must have consumed the pinned lists and copy descriptors
+  // advance the migration cursor past fully enqueued plans BEFORE a slot is reused (a plan-only
+  // ctx, DYO_F_NO_HOST_POOL, never migrates: its earlier plans are simply superseded)
+  if (!ctx->host_pool) ctx->mig_seq = ctx->plan_seq;
+  while (ctx->mig_seq < ctx->plan_seq) {
+    const dyo_ctx::PlanSlot& Q = ctx->slot[ctx->mig_seq & 1];
+    if (Q.valid && Q.next_j < Q.K) break;
+    ctx->mig_seq += 1;
+  }
   dyo_ctx::PlanSlot& P = ctx->slot[ctx->plan_seq & 1];
-  if (P.valid && P.next_j < P.K)
+  if (ctx->plan_seq - ctx->mig_seq >= 2)
     return fail(ctx, DYO_E_STATE, "two plans are outstanding: migrate the older one first");
   if (P.ev_pending) { CK(cudaEventSynchronize(P.ev_last)); P.ev_pending = false; }
   P.valid = false;
@@ -913,9 +921,6 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
   P.next_j = 0;
   P.seg_used = 0;
   P.valid = true;
-  if (ctx->mig_seq < ctx->plan_seq && !(ctx->slot[ctx->mig_seq & 1].valid &&
-                                        ctx->slot[ctx->mig_seq & 1].next_j < ctx->slot[ctx->mig_seq & 1].K))
-    ctx->mig_seq = ctx->plan_seq;            // the older plan is fully enqueued
   ctx->plan_seq += 1;
   if (K_out) *K_out = P.K;
   return DYO_OK;

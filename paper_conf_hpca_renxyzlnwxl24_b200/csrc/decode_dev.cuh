@@ -180,28 +180,6 @@ __device__ __forceinline__ int row_op(const ArchDev& a, const DecHead& H, int r)
   return w == 0 ? -1 : a.piece_b[p] + w - 1;
 }
 
-// bitonic sort of 64 keys held two per lane (index lane -> x, lane + 32 -> z), ascending
-__device__ __forceinline__ void warp_sort64(uint64_t& x, uint64_t& z, int lane) {
-#pragma unroll
-  for (int k = 2; k <= 64; k <<= 1) {
-#pragma unroll
-    for (int j = k >> 1; j > 0; j >>= 1) {
-      if (j == 32) {
-        const uint64_t lo = x < z ? x : z, hi = x < z ? z : x;
-        x = lo;
-        z = hi;
-      } else {
-        const uint64_t px = __shfl_xor_sync(0xffffffffu, x, j);
-        const uint64_t pz = __shfl_xor_sync(0xffffffffu, z, j);
-        const bool lower = (lane & j) == 0;
-        const bool upx = (lane & k) == 0, upz = ((lane + 32) & k) == 0;
-        x = (lower == upx) ? (x < px ? x : px) : (x < px ? px : x);
-        z = (lower == upz) ? (z < pz ? z : pz) : (z < pz ? pz : z);
-      }
-    }
-  }
-}
-
 // Build group g of prediction b. All threads of the block must call it (uniform arguments).
 // Writes blocks / hist / grp / ent / ent_n for (b, g).
 static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup& G, PredDev& pd, int b, int g,

@@ -85,4 +85,26 @@ __device__ __forceinline__ void block_sort_u64(uint64_t* key, int n) {
   }
 }
 
+// bitonic sort of 64 keys held two per lane (index lane -> x, lane + 32 -> z), ascending
+__device__ __forceinline__ void warp_sort64(uint64_t& x, uint64_t& z, int lane) {
+#pragma unroll
+  for (int k = 2; k <= 64; k <<= 1) {
+#pragma unroll
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      if (j == 32) {
+        const uint64_t lo = x < z ? x : z, hi = x < z ? z : x;
+        x = lo;
+        z = hi;
+      } else {
+        const uint64_t px = __shfl_xor_sync(0xffffffffu, x, j);
+        const uint64_t pz = __shfl_xor_sync(0xffffffffu, z, j);
+        const bool lower = (lane & j) == 0;
+        const bool upx = (lane & k) == 0, upz = ((lane + 32) & k) == 0;
+        x = (lower == upx) ? (x < px ? x : px) : (x < px ? px : x);
+        z = (lower == upz) ? (z < pz ? z : pz) : (z < pz ? pz : z);
+      }
+    }
+  }
+}
+
 }  // namespace dyo

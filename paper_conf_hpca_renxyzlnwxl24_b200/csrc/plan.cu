@@ -41,6 +41,19 @@ struct PlanSmem {
 };
 
 __device__ __forceinline__ void sort_keys(uint64_t* key, int n) {
+  if (n <= 64) {
+    // one warp, registers + shuffles (a block bitonic stage costs a barrier + smem round trip)
+    if (threadIdx.x < 32) {
+      const int lane = threadIdx.x;
+      uint64_t x = lane < n ? key[lane] : ~0ull;
+      uint64_t z = lane + 32 < n ? key[lane + 32] : ~0ull;
+      warp_sort64(x, z, lane);
+      if (lane < n) key[lane] = x;
+      if (lane + 32 < n) key[lane + 32] = z;
+    }
+    __syncthreads();
+    return;
+  }
   int np2 = 1;
   while (np2 < n) np2 <<= 1;
   for (int i = n + threadIdx.x; i < np2; i += blockDim.x) key[i] = ~0ull;
@@ -391,32 +404,47 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
     }
     const int np = s_nplaced;
     PSTAMP(9);
-    // J. first fit by warp 0 (R11)
+    // J. first fit by warp 0 (R11). <= 32 gaps and placed tensors: gaps and sizes live in
+    //    registers (lane g owns gap g, lane p holds placed tensor p), one ballot per placement
     if (tid < 32) {
       const int lane = tid;
       const int ng = s_ng;
       bool fail = false;
-      for (int p = 0; p < np && !fail; ++p) {
-        const int t = (int)(pkey[p] & 0xFFFFF);
-        const int64_t need_t = t_ab[t];
-        int found = -1;
-        for (int g0 = 0; g0 < ng; g0 += 32) {
-          const int g = g0 + lane;
-          const bool fits = g < ng && (sc.gap_e[g] - sc.gap_s[g]) >= need_t;
-          const unsigned bal = __ballot_sync(0xffffffffu, fits);
-          if (bal) { found = g0 + __ffs(bal) - 1; break; }
+      if (ng <= 32 && np <= 32) {
+        int64_t gs = lane < ng ? sc.gap_s[lane] : 0, ge = lane < ng ? sc.gap_e[lane] : 0;
+        const int my_t = lane < np ? (int)(pkey[lane] & 0xFFFFF) : 0;
+        const int64_t my_a = lane < np ? t_ab[my_t] : 0;
+        for (int p = 0; p < np; ++p) {
+          const int64_t need_t = __shfl_sync(0xffffffffu, my_a, p);
+          const unsigned bal = __ballot_sync(0xffffffffu, lane < ng && ge - gs >= need_t);
+          if (!bal) { fail = true; break; }
+          const int found = __ffs(bal) - 1;
+          const int64_t off = __shfl_sync(0xffffffffu, gs, found);
+          if (lane == found) gs += need_t;
+          if (lane == p) sc.newoff[my_t] = off;
         }
-        if (found < 0) { fail = true; break; }
-        if (lane == 0) {
-          sc.newoff[t] = sc.gap_s[found];
-          sc.gap_s[found] += need_t;
+      } else {
+        for (int p = 0; p < np && !fail; ++p) {
+          const int t = (int)(pkey[p] & 0xFFFFF);
+          const int64_t need_t = t_ab[t];
+          int found = -1;
+          for (int g0 = 0; g0 < ng; g0 += 32) {
+            const int g = g0 + lane;
+            const bool fits = g < ng && (sc.gap_e[g] - sc.gap_s[g]) >= need_t;
+            const unsigned bal = __ballot_sync(0xffffffffu, fits);
+            if (bal) { found = g0 + __ffs(bal) - 1; break; }
+          }
+          if (found < 0) { fail = true; break; }
+          if (lane == 0) {
+            sc.newoff[t] = sc.gap_s[found];
+            sc.gap_s[found] += need_t;
+          }
+          __syncwarp();
         }
-        __syncwarp();
       }
       if (lane == 0) s_compact = fail ? 1 : 0;
     }
     __syncthreads();
-    PSTAMP(10);
     // compaction fallback: exclusive prefix sums over [kept | placed]
     if (s_compact) {
       if (tid == 0) {

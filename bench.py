@@ -44,7 +44,7 @@ def parse():
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--budget-gib", type=float, default=0.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--dist-backend", default="nccl")
+    ap.add_argument("--dist-backend", default=None, help="nccl (default with CUDA) or gloo")
     ap.add_argument("--compute", default="auto", choices=["auto", "none", "emulate"],
                     help="emulate the DyNN's per-group compute with spin kernels (auto: on for af)")
     return ap.parse_args()
@@ -109,6 +109,21 @@ class Clocks:
         reasons = sorted({names[i] for s in self.samples for i in range(4) if len(s) > 3 + i and s[3 + i] == "Active"})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
                 "reasons": reasons, "samples": len(self.samples)}
+
+
+def reduce_over_ranks(vals_max, vals_sum, backend):
+    """Max of `vals_max` and sum of `vals_sum` over all ranks (timings: the slowest rank bounds the
+    job; bytes: every rank's work counts). World size 1: identity."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size() == 1:
+        return list(vals_max), list(vals_sum)
+    dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
+    a = torch.tensor(list(vals_max), dtype=torch.float64, device=dev)
+    b = torch.tensor(list(vals_sum), dtype=torch.float64, device=dev)
+    dist.all_reduce(a, op=dist.ReduceOp.MAX)
+    dist.all_reduce(b, op=dist.ReduceOp.SUM)
+    return a.cpu().tolist(), b.cpu().tolist()
 
 
 def make_workload(args, rank):
@@ -228,9 +243,11 @@ def run_dyo(args):
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    # one manager per GPU; with fewer GPUs than ranks (functional tests) ranks share devices
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
+    backend = args.dist_backend or "nccl"
     if world > 1:
-        dist.init_process_group(args.dist_backend)
+        dist.init_process_group(backend)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
 
@@ -308,9 +325,9 @@ def run_dyo(args):
         return tot
 
     def barrier():
+        torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
-        torch.cuda.synchronize()
 
     _log("warmup")
     dev_inputs = lambda k: (desc_dev[k % nS: k % nS + 1], hist_dev)
@@ -364,18 +381,9 @@ def run_dyo(args):
     _log("probe")
     probe = pcie_probe(torch)
 
-    # max over ranks
-    tt = torch.tensor([ms, e2e_s, float(tot_h2d + tot_d2h), float(tot_h2d), float(tot_d2h)], device=dev, dtype=torch.float64)
-    if world > 1:
-        mx = tt.clone()
-        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
-        sm = tt.clone()
-        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
-        ms_max, e2e_max = mx[0].item(), mx[1].item()
-        bytes_all, h2d_all, d2h_all = sm[2].item(), sm[3].item(), sm[4].item()
-    else:
-        ms_max, e2e_max = ms, e2e_s
-        bytes_all, h2d_all, d2h_all = float(tot_h2d + tot_d2h), float(tot_h2d), float(tot_d2h)
+    # max over ranks (time), sum over ranks (work)
+    (ms_max, e2e_max), (bytes_all, h2d_all, d2h_all) = reduce_over_ranks(
+        [ms, e2e_s], [float(tot_h2d + tot_d2h), float(tot_h2d), float(tot_d2h)], backend)
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()

@@ -64,6 +64,7 @@ typedef struct {
 #define DYO_F_NO_PACK 2       /* never pack scattered writebacks into one DMA */
 #define DYO_F_NO_HOST_POOL 4  /* plan-only ctx: no pinned host pool (dyo_migrate -> DYO_E_STATE) */
 #define DYO_F_TIMING 8        /* record CUDA events around every internal launch (dyo_get_timings) */
+#define DYO_F_SM_COPY 16      /* device<->device moves by the SM vector-copy kernel instead of TMA bulk copies */
 
 /* Static architecture: the DyNN program in preorder, its operators and the
  * tensor table. All arrays are HOST memory; dyo_load_arch copies what it needs. */
@@ -261,6 +262,11 @@ dyo_status dyo_get_counters(dyo_ctx* ctx, dyo_counters* c, int32_t reset);
 #define DYO_T_KINDS 7
 dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* launches, int64_t* bytes,
                            int32_t reset);
+
+/* Debugging / measurement aid: copy `bytes` device->device (or through mapped host memory) with
+ * the library's segment-copy kernel: mode 0 = SM vector copies (K5 path), 1 = TMA bulk copies
+ * (K3/K4 path). Synchronises `stream`. */
+dyo_status dyo_debug_copy(dyo_ctx* ctx, const void* src, void* dst, int64_t bytes, int32_t mode, void* stream);
 
 /* Debugging aid: enable (1) / disable (0) %globaltimer phase stamps of the pilot kernel and
  * read the 32 stamps of the last launch (ns; out32 may be NULL). Synchronises the device. */

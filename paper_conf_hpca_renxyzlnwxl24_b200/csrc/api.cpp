@@ -16,6 +16,8 @@
 
 using namespace dyo;
 
+constexpr int64_t kChunk = 256 << 10;   // copy-kernel work item
+
 struct dyo_ctx {
   dyo_config cfg{};
   int device = 0;
@@ -961,7 +963,6 @@ namespace {
 
 struct Run { int64_t host_off, dev_off, bytes; bool dev_contig; int first, count; };
 
-constexpr int64_t kChunk = 256 << 10;   // copy-kernel work item
 
 // push (src, dst, bytes) split into work items; returns false on capacity
 // the slot being migrated (set by dyo_migrate before it pushes descriptors)
@@ -986,7 +987,12 @@ dyo_status launch_segs(dyo_ctx* ctx, int64_t first, cudaStream_t s, int grid, in
   int64_t bytes = 0;
   for (int64_t i = first; i < P.seg_used; ++i) bytes += P.h_segs[i].bytes;
   TScope ts(ctx, kind, s, bytes);
-  CK(launch_copy_segments(dptr, (int)n, kChunk, grid, s));
+  if (kind == 3 && !(ctx->cfg.flags & DYO_F_SM_COPY)) {
+    // device<->device: TMA bulk copies, one CTA per SM
+    CK(launch_copy_segments_tma(dptr, (int)n, ctx->sm_count, s));
+  } else {
+    CK(launch_copy_segments(dptr, (int)n, kChunk, grid, s));
+  }
   ctx->ctr.n_kernels++;
   return DYO_OK;
 }
@@ -1256,6 +1262,24 @@ dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* laun
   if (reset) {
     for (int k = 0; k < DYO_T_KINDS; ++k) { ctx->tm_ms[k] = 0; ctx->tm_n[k] = 0; ctx->tm_bytes[k] = 0; }
   }
+  return DYO_OK;
+}
+
+dyo_status dyo_debug_copy(dyo_ctx* ctx, const void* src, void* dst, int64_t bytes, int32_t mode, void* stream) {
+  if (!ctx || !src || !dst || bytes < 0) return DYO_E_INVAL;
+  CK(cudaSetDevice(ctx->device));
+  // descriptors in a temporary device buffer (work items of kChunk bytes)
+  std::vector<CopySeg> segs;
+  for (int64_t o = 0; o < bytes; o += kChunk)
+    segs.push_back(CopySeg{(const char*)src + o, (char*)dst + o, std::min(kChunk, bytes - o)});
+  if (segs.empty()) return DYO_OK;
+  CopySeg* d = nullptr;
+  CK(cudaMallocAsync((void**)&d, sizeof(CopySeg) * segs.size(), (cudaStream_t)stream));
+  CK(cudaMemcpyAsync(d, segs.data(), sizeof(CopySeg) * segs.size(), cudaMemcpyHostToDevice, (cudaStream_t)stream));
+  if (mode == 1) CK(launch_copy_segments_tma(d, (int)segs.size(), ctx->sm_count, (cudaStream_t)stream));
+  else CK(launch_copy_segments(d, (int)segs.size(), kChunk, 4 * ctx->sm_count, (cudaStream_t)stream));
+  CK(cudaFreeAsync(d, (cudaStream_t)stream));
+  CK(cudaStreamSynchronize((cudaStream_t)stream));
   return DYO_OK;
 }
 

@@ -160,5 +160,6 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
 struct CopySeg { const char* src; char* dst; int64_t bytes; };
 cudaError_t launch_copy_segments(const CopySeg* segs_dev_or_mapped, int n, int64_t chunk,
                                  int grid, cudaStream_t s);
+cudaError_t launch_copy_segments_tma(const CopySeg* segs, int n, int grid, cudaStream_t s);
 
 }  // namespace dyo

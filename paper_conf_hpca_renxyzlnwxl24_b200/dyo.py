@@ -95,7 +95,7 @@ def lib():
                      "dyo_arena", "dyo_encode_features", "dyo_pilot_predict", "dyo_prediction_get",
                      "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records", "dyo_migrate",
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
-                     "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps"):
+                     "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -105,7 +105,7 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_load_pilot", "dyo_host_pool", "dyo_arena", "dyo_encode_features", "dyo_pilot_predict",
            "dyo_prediction_get", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
-           "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps")
+           "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy")
 
 
 def _a(x, dt):
@@ -350,6 +350,9 @@ class Dyo:
         out = np.zeros(32, np.uint64)
         self._check(self.L.dyo_debug_pilot_stamps(self.ctx, 1 if enable else 0, out.ctypes.data_as(C.POINTER(C.c_uint64))))
         return out
+
+    def debug_copy(self, src, dst, nbytes, mode, stream=0):
+        self._check(self.L.dyo_debug_copy(self.ctx, P(self._ptr(src)), P(self._ptr(dst)), i64(nbytes), mode, P(stream)))
 
     def plan_stamps(self, j):
         out = np.zeros(64, np.uint64)

@@ -242,3 +242,18 @@ def test_pipelined_plan_lookahead_moe_scaled():
 
 def test_pipelined_plan_lookahead_tiny_compaction():
     run_pipelined(_tiny_with_moves(), 4, 1, lookahead=True)
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+@pytest.mark.parametrize("nbytes,soff,doff", [(1 << 20, 0, 0), ((3 << 20) + 5, 16, 48), (777, 3, 5), (96 << 10, 0, 4096)])
+def test_copy_kernels_exact(mode, nbytes, soff, doff):
+    """Segment-copy kernels (SM vector path and TMA bulk path) move exactly the bytes, including
+    unaligned heads/tails, and touch nothing outside the destination range."""
+    wl = WL.make("tiny")
+    d = make_ctx(wl, flags=4)
+    src = torch.randint(0, 255, (nbytes + 8192,), dtype=torch.uint8, device="cuda")
+    dst = torch.zeros(nbytes + 8192, dtype=torch.uint8, device="cuda")
+    d.debug_copy(src.data_ptr() + soff, dst.data_ptr() + doff, nbytes, mode, torch.cuda.current_stream().cuda_stream)
+    assert torch.equal(dst[doff: doff + nbytes], src[soff: soff + nbytes])
+    assert int(dst[:doff].sum()) == 0 and int(dst[doff + nbytes:].sum()) == 0
+    d.close()

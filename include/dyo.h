@@ -257,11 +257,13 @@ dyo_status dyo_get_counters(dyo_ctx* ctx, dyo_counters* c, int32_t reset);
 /* With DYO_F_TIMING: device time (CUDA events on the launching stream) summed over the launches
  * of one kind since the last reset: 0 pilot kernel (K1), 1 decode kernels, 2 planner kernel (K2),
  * 3 device copy kernel (pack / unpack / carry / compaction), 4 zero-copy kernel (K5),
- * 5 DMA H2D, 6 DMA D2H. bytes = algorithmic bytes moved by those launches. Synchronises on
- * the recorded events. */
+ * 5 DMA H2D, 6 DMA D2H. bytes = algorithmic bytes moved by those launches; busy_ms = length of
+ * the union of their [start, end] intervals (launches of one kind on different streams overlap).
+ * Any output may be NULL. reset also records the reference event the intervals are measured
+ * from. Synchronises on the recorded events. */
 #define DYO_T_KINDS 7
 dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* launches, int64_t* bytes,
-                           int32_t reset);
+                           double* busy_ms, int32_t reset);
 
 /* Debugging / measurement aid: copy `bytes` device->device (or through mapped host memory) with
  * the library's segment-copy kernel: mode 0 = SM vector copies (K5 path), 1 = TMA bulk copies

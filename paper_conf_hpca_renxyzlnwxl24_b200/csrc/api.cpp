@@ -85,6 +85,8 @@ struct dyo_ctx {
   std::vector<cudaEvent_t> ev_pool;
   double tm_ms[DYO_T_KINDS] = {};
   int64_t tm_n[DYO_T_KINDS] = {}, tm_bytes[DYO_T_KINDS] = {};
+  cudaEvent_t ev_ref = nullptr;                           // timing reference (recorded at reset)
+  std::vector<std::pair<double, double>> tm_iv[DYO_T_KINDS];  // [start, end] ms after ev_ref
 };
 
 namespace {
@@ -200,6 +202,13 @@ void drain_timings(dyo_ctx* c) {
     cudaEventSynchronize(t.b);
     float ms = 0.f;
     cudaEventElapsedTime(&ms, t.a, t.b);
+    if (c->ev_ref) {
+      float t0 = 0.f, t1 = 0.f;
+      if (cudaEventElapsedTime(&t0, c->ev_ref, t.a) == cudaSuccess &&
+          cudaEventElapsedTime(&t1, c->ev_ref, t.b) == cudaSuccess)
+        c->tm_iv[t.kind].push_back({t0, t1});
+      cudaGetLastError();
+    }
     c->tm_ms[t.kind] += ms;
     c->tm_n[t.kind] += 1;
     c->tm_bytes[t.kind] += t.bytes;
@@ -487,6 +496,7 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->ev_carry) cudaEventDestroy(ctx->ev_carry);
   for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+  if (ctx->ev_ref) cudaEventDestroy(ctx->ev_ref);
   delete ctx;
   return DYO_OK;
 }
@@ -987,12 +997,68 @@ dyo_status launch_segs(dyo_ctx* ctx, int64_t first, cudaStream_t s, int grid, in
   int64_t bytes = 0;
   for (int64_t i = first; i < P.seg_used; ++i) bytes += P.h_segs[i].bytes;
   TScope ts(ctx, kind, s, bytes);
-  if (kind == 3 && !(ctx->cfg.flags & DYO_F_SM_COPY)) {
-    // device<->device: TMA bulk copies, one CTA per SM
-    CK(launch_copy_segments_tma(dptr, (int)n, ctx->sm_count, s));
-  } else {
-    CK(launch_copy_segments(dptr, (int)n, kChunk, grid, s));
+  CK(launch_copy_segments(dptr, (int)n, kChunk, grid, s));
+  ctx->ctr.n_kernels++;
+  return DYO_OK;
+}
+
+// Device<->device copies of plan records [i0, i1) (R = one of the all-int64 record types):
+// record k copies rec.bytes from src_base + rec.<f_src> to dst_base + rec.<f_dst> - dst_bias;
+// f_late >= 0 selects the records with rec.late == late_val. The TMA copy kernel reads the
+// records from the plan's device copy (P.dout); the pinned host copy (P.out) only sizes the
+// launch. With DYO_F_SM_COPY the host builds work items for the SM vector-copy kernel instead.
+extern "C++" template <class R>
+dyo_status d2d_records(dyo_ctx* ctx, const R* hrec, const R* drec, int i0, int i1, int f_src, int f_dst,
+                       int f_bytes, int f_late, int64_t late_val, const char* src_base, char* dst_base,
+                       int64_t dst_bias, cudaStream_t s, int grid) {
+  static_assert(sizeof(R) % sizeof(int64_t) == 0, "records are int64 fields");
+  const int stride = (int)(sizeof(R) / sizeof(int64_t));
+  int64_t total = 0, bytes = 0;
+  for (int k = i0; k < i1; ++k) {
+    const int64_t* r = reinterpret_cast<const int64_t*>(hrec + k);
+    if (f_late >= 0 && r[f_late] != late_val) continue;
+    total += rec_body(src_base + r[f_src], dst_base + (r[f_dst] - dst_bias), r[f_bytes]);
+    bytes += r[f_bytes];
   }
+  if (bytes == 0) return DYO_OK;
+  if (ctx->cfg.flags & DYO_F_SM_COPY) {
+    dyo_ctx::PlanSlot& P = *g_mslot;
+    const int64_t g0 = P.seg_used;
+    for (int k = i0; k < i1; ++k) {
+      const int64_t* r = reinterpret_cast<const int64_t*>(hrec + k);
+      if (f_late >= 0 && r[f_late] != late_val) continue;
+      if (!push_seg(ctx, src_base + r[f_src], dst_base + (r[f_dst] - dst_bias), r[f_bytes]))
+        return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+    }
+    return launch_segs(ctx, g0, s, grid);
+  }
+  RecCopyArgs a{};
+  a.rec = reinterpret_cast<const int64_t*>(drec + i0);
+  a.stride = stride;
+  a.n = i1 - i0;
+  a.f_src = f_src; a.f_dst = f_dst; a.f_bytes = f_bytes; a.f_late = f_late;
+  a.late_val = late_val;
+  a.src_base = src_base; a.dst_base = dst_base; a.dst_bias = dst_bias;
+  a.total = total;
+  TScope ts(ctx, 3, s, bytes);
+  CK(launch_copy_records(a, ctx->sm_count, s));
+  ctx->ctr.n_kernels++;
+  return DYO_OK;
+}
+
+// One device<->device range (staged pieces of a self-overlapping move).
+dyo_status d2d_range(dyo_ctx* ctx, const char* src, char* dst, int64_t bytes, cudaStream_t s, int grid) {
+  if (bytes <= 0) return DYO_OK;
+  if (ctx->cfg.flags & DYO_F_SM_COPY) {
+    dyo_ctx::PlanSlot& P = *g_mslot;
+    const int64_t g0 = P.seg_used;
+    if (!push_seg(ctx, src, dst, bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+    return launch_segs(ctx, g0, s, grid);
+  }
+  RecCopyArgs a{};
+  a.src_base = src; a.dst_base = dst; a.total = bytes;
+  TScope ts(ctx, 3, s, bytes);
+  CK(launch_copy_records(a, ctx->sm_count, s));
   ctx->ctr.n_kernels++;
   return DYO_OK;
 }
@@ -1042,6 +1108,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   //    (K5) for the runs below dma_min
   {
     const dyo_evict_rec* ev = P.out.ev + h.o_evict;
+    const dyo_evict_rec* dev_ev = P.dout.ev + h.o_evict;
     std::vector<int> small;
     int i = 0;
     while (i < h.n_evict) {
@@ -1068,13 +1135,8 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
         int q = r.first;
         while (q < r.first + r.count) {
           const int64_t base = ev[q].host_off;
-          const int64_t seg0 = P.seg_used;
           int q2 = q;
-          while (q2 < r.first + r.count && ev[q2].host_off + ev[q2].bytes - base <= stage_half) {
-            if (!push_seg(ctx, arena + ev[q2].src, stage_pack + (ev[q2].host_off - base), ev[q2].bytes))
-              return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
-            ++q2;
-          }
+          while (q2 < r.first + r.count && ev[q2].host_off + ev[q2].bytes - base <= stage_half) ++q2;
           if (q2 == q) {   // a tensor larger than the staging buffer: its own DMA
             { TScope ts(ctx, 6, sd, ev[q].bytes);
               CK(cudaMemcpyAsync(host + ev[q].host_off, arena + ev[q].src, ev[q].bytes, cudaMemcpyDeviceToHost, sd)); }
@@ -1084,7 +1146,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
             continue;
           }
           TRACE("  pack %d tensors", q2 - q);
-          dyo_status s1 = launch_segs(ctx, seg0, sd, d2d_grid);
+          dyo_status s1 = d2d_records(ctx, ev, dev_ev, q, q2, 1, 2, 3, -1, 0, arena, stage_pack, base, sd, d2d_grid);
           if (s1) return s1;
           const int64_t len = ev[q2 - 1].host_off + ev[q2 - 1].bytes - base;
           { TScope ts(ctx, 6, sd, len);
@@ -1120,14 +1182,15 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   //    overlapping its own source goes through the staging buffer in pieces.
   {
     const dyo_move_rec* mv = P.out.mv + h.o_move;
-    int64_t wave0 = -1;
-    std::vector<std::pair<int64_t, int64_t>> wave_src;    // source ranges of the open wave
+    const dyo_move_rec* dev_mv = P.dout.mv + h.o_move;
+    int wave0 = -1, wave1 = -1;                           // the open wave: records [wave0, wave1)
+    std::vector<std::pair<int64_t, int64_t>> wave_src;    // its source ranges
     auto flush = [&]() -> dyo_status {
       if (wave0 >= 0) {
-        dyo_status s1 = launch_segs(ctx, wave0, s, d2d_grid);
+        dyo_status s1 = d2d_records(ctx, mv, dev_mv, wave0, wave1, 1, 2, 3, -1, 0, arena, arena, 0, s, d2d_grid);
         if (s1) return s1;
       }
-      wave0 = -1;
+      wave0 = wave1 = -1;
       wave_src.clear();
       return DYO_OK;
     };
@@ -1139,13 +1202,9 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
         if (s1) return s1;
         for (int64_t o = 0; o < nbytes; o += stage_half) {
           const int64_t n = std::min(stage_half, nbytes - o);
-          const int64_t g0 = P.seg_used;
-          if (!push_seg(ctx, arena + src + o, stage_move, n)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
-          s1 = launch_segs(ctx, g0, s, d2d_grid);
+          s1 = d2d_range(ctx, arena + src + o, stage_move, n, s, d2d_grid);
           if (s1) return s1;
-          const int64_t g1 = P.seg_used;
-          if (!push_seg(ctx, stage_move, arena + dst + o, n)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
-          s1 = launch_segs(ctx, g1, s, d2d_grid);
+          s1 = d2d_range(ctx, stage_move, arena + dst + o, n, s, d2d_grid);
           if (s1) return s1;
         }
         continue;
@@ -1157,8 +1216,8 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
         dyo_status s1 = flush();
         if (s1) return s1;
       }
-      if (wave0 < 0) wave0 = P.seg_used;
-      if (!push_seg(ctx, arena + src, arena + dst, nbytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
+      if (wave0 < 0) wave0 = i;
+      wave1 = i + 1;
       wave_src.push_back({src, src + nbytes});
     }
     dyo_status s1 = flush();
@@ -1172,16 +1231,15 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   bool carry_side = false;
   {
     const dyo_carry_rec* ca = P.out.ca + h.o_carry;
-    const int64_t g0 = P.seg_used;
-    for (int i = 0; i < h.n_carry; ++i) {
-      if (ca[i].late) continue;
-      if (!push_seg(ctx, arena + ca[i].src, arena + ca[i].dst, ca[i].bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
-      ctx->ctr.d2d += ca[i].bytes;
-    }
-    if (P.seg_used > g0) {
+    int64_t early = 0;
+    for (int i = 0; i < h.n_carry; ++i)
+      if (!ca[i].late) early += ca[i].bytes;
+    ctx->ctr.d2d += early;
+    if (early > 0) {
       CK(cudaEventRecord(ctx->ev_moves, s));
       CK(cudaStreamWaitEvent(ctx->side, ctx->ev_moves, 0));
-      dyo_status s1 = launch_segs(ctx, g0, ctx->side, d2d_grid);
+      dyo_status s1 = d2d_records(ctx, ca, P.dout.ca + h.o_carry, 0, h.n_carry, 1, 2, 3, 4, 0, arena, arena, 0,
+                                  ctx->side, d2d_grid);
       if (s1) return s1;
       CK(cudaEventRecord(ctx->ev_carry, ctx->side));
       carry_side = true;
@@ -1227,13 +1285,10 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
     for (int i = 0; i < h.n_carry; ++i) any |= ca[i].late != 0;
     if (any) {
       if (ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
-      const int64_t g0 = P.seg_used;
-      for (int i = 0; i < h.n_carry; ++i) {
-        if (!ca[i].late) continue;
-        if (!push_seg(ctx, arena + ca[i].src, arena + ca[i].dst, ca[i].bytes)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors");
-        ctx->ctr.d2d += ca[i].bytes;
-      }
-      dyo_status s1 = launch_segs(ctx, g0, s, d2d_grid);
+      for (int i = 0; i < h.n_carry; ++i)
+        if (ca[i].late) ctx->ctr.d2d += ca[i].bytes;
+      dyo_status s1 = d2d_records(ctx, ca, P.dout.ca + h.o_carry, 0, h.n_carry, 1, 2, 3, 4, 1, arena, arena, 0, s,
+                                  d2d_grid);
       if (s1) return s1;
     }
   }
@@ -1253,14 +1308,30 @@ dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr) {
 }
 
 dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* launches, int64_t* bytes,
-                           int32_t reset) {
+                           double* busy_ms, int32_t reset) {
   if (!ctx || kind < 0 || kind >= DYO_T_KINDS) return DYO_E_INVAL;
   drain_timings(ctx);
   if (ms) *ms = ctx->tm_ms[kind];
   if (launches) *launches = ctx->tm_n[kind];
   if (bytes) *bytes = ctx->tm_bytes[kind];
+  if (busy_ms) {
+    // length of the union of this kind's [start, end] intervals: launches of one kind that run
+    // concurrently on different streams share the hardware, so their summed durations overstate
+    // the time the kind kept the GPU busy
+    auto iv = ctx->tm_iv[kind];
+    std::sort(iv.begin(), iv.end());
+    double tot = 0, cs = -1, ce = -1;
+    for (auto& p : iv) {
+      if (p.first > ce) { if (ce > cs) tot += ce - cs; cs = p.first; ce = p.second; }
+      else if (p.second > ce) ce = p.second;
+    }
+    if (ce > cs) tot += ce - cs;
+    *busy_ms = tot;
+  }
   if (reset) {
-    for (int k = 0; k < DYO_T_KINDS; ++k) { ctx->tm_ms[k] = 0; ctx->tm_n[k] = 0; ctx->tm_bytes[k] = 0; }
+    for (int k = 0; k < DYO_T_KINDS; ++k) { ctx->tm_ms[k] = 0; ctx->tm_n[k] = 0; ctx->tm_bytes[k] = 0; ctx->tm_iv[k].clear(); }
+    if (!ctx->ev_ref) cudaEventCreate(&ctx->ev_ref);
+    cudaEventRecord(ctx->ev_ref, 0);
   }
   return DYO_OK;
 }
@@ -1276,7 +1347,11 @@ dyo_status dyo_debug_copy(dyo_ctx* ctx, const void* src, void* dst, int64_t byte
   CopySeg* d = nullptr;
   CK(cudaMallocAsync((void**)&d, sizeof(CopySeg) * segs.size(), (cudaStream_t)stream));
   CK(cudaMemcpyAsync(d, segs.data(), sizeof(CopySeg) * segs.size(), cudaMemcpyHostToDevice, (cudaStream_t)stream));
-  if (mode == 1) CK(launch_copy_segments_tma(d, (int)segs.size(), ctx->sm_count, (cudaStream_t)stream));
+  if (mode == 1) {
+    RecCopyArgs a{};
+    a.src_base = (const char*)src; a.dst_base = (char*)dst; a.total = bytes;
+    CK(launch_copy_records(a, ctx->sm_count, (cudaStream_t)stream));
+  }
   else CK(launch_copy_segments(d, (int)segs.size(), kChunk, 4 * ctx->sm_count, (cudaStream_t)stream));
   CK(cudaFreeAsync(d, (cudaStream_t)stream));
   CK(cudaStreamSynchronize((cudaStream_t)stream));

@@ -1,4 +1,4 @@
-// K3/K4/K5: segment-list copy kernels (DESIGN.md §6 "migrate").
+// K3/K4/K5: copy kernels of the migration engine (DESIGN.md §6 "migrate").
 //
 // One kernel serves every byte move of a transition that is not a plain DMA:
 //   K3 gather-pack   scattered arena ranges -> contiguous device staging (then one DMA D2H)
@@ -47,70 +47,143 @@ copy_segments_kernel(const CopySeg* __restrict__ segs, int n) {
 }
 
 // ---- TMA bulk variant (device<->device moves: pack / unpack / carry / compaction) ----------
-// One elected thread per CTA streams each work item through a ring of kStages shared-memory
+// One elected thread per CTA streams its work items through a ring of kTmaStages shared-memory
 // buffers: cp.async.bulk global->shared (mbarrier complete_tx), then cp.async.bulk
 // shared->global (bulk_group); a buffer is reused only after its store has read it
 // (cp.async.bulk.wait_group.read). The copy engine of the SM does the byte moving, so a few
 // CTAs saturate HBM and the SMs stay free for the DyNN's compute. Unaligned heads/tails (not
 // multiples of 16 bytes) are copied by the CTA's threads.
 constexpr int kTmaStages = 4;
-constexpr int kTmaChunk = 32 << 10;
+constexpr int kTmaChunk = 16 << 10;   // 4 x 16 KiB per CTA: three copy kernels can share an SM
 
 __device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
-// A cursor over the 32 KiB chunks of this CTA's work items (items blockIdx.x, +gridDim.x, ...;
-// only their 16-byte-aligned bodies).
-struct ChunkCursor {
-  const CopySeg* segs;
-  int n, it;
-  int64_t off, body;
+// The device<->device moves of a transition are driven straight from the plan's records, which
+// the planner left in device memory: the host never builds or ships work items for them (it
+// would have to send them over a PCIe link that the transition's own DMAs keep saturated in
+// both directions; measured: a zero-copy descriptor read under that load stretched 220 MB
+// launches from ~40 to 100-150 us).
+//
+// Records i < n (filtered by `late` when f_late >= 0) define copies
+//   src_base + rec[i][f_src]  ->  dst_base + rec[i][f_dst] - dst_bias,  rec[i][f_bytes] bytes.
+// Each record's 16-byte-aligned body (0 when src or dst is not 16-byte aligned) is a piece of
+// one virtual stream of `total` bytes; CTA b copies the contiguous slice [b*per, (b+1)*per) of
+// it (per = total/grid rounded up to 16 bytes), so one large record spreads over every SM. The
+// remaining < 16-byte tails (and unaligned records) are copied by the CTAs' threads.
+
+constexpr int kRecThreads = 128;
+
+struct RecCursor {
+  const RecCopyArgs* a;
+  int i;                       // current record
+  int64_t off, body, pos, hi;  // offset in its body; position in the stream; slice end
   const char* src;
   char* dst;
-  __device__ void load_item() {
-    while (it < n) {
-      const CopySeg sg = segs[it];
-      src = sg.src;
-      dst = sg.dst;
-      const bool aligned = ((((uintptr_t)src) | ((uintptr_t)dst)) & 15) == 0;
-      body = aligned ? (sg.bytes & ~(int64_t)15) : 0;
-      if (body > 0) return;
-      it += gridDim.x;
+  __device__ int64_t body_of(int k, const char** s, char** d) const {
+    const int64_t* r = a->rec + (int64_t)k * a->stride;
+    if (a->f_late >= 0 && r[a->f_late] != a->late_val) return 0;
+    *s = a->src_base + r[a->f_src];
+    *d = a->dst_base + (r[a->f_dst] - a->dst_bias);
+    const bool al = ((((uintptr_t)*s) | ((uintptr_t)*d)) & 15) == 0;
+    return al ? (r[a->f_bytes] & ~(int64_t)15) : 0;
+  }
+  __device__ void settle() {   // skip exhausted / empty records
+    while (pos < hi && off >= body) {
+      ++i;
+      off = 0;
+      body = i < a->n ? body_of(i, &src, &dst) : 0;
+      if (i >= a->n) { pos = hi; return; }
     }
   }
-  __device__ void init(const CopySeg* s, int nn) { segs = s; n = nn; it = blockIdx.x; off = 0; load_item(); }
-  __device__ bool valid() const { return it < n; }
-  __device__ uint32_t len() const { return (uint32_t)((body - off) < kTmaChunk ? (body - off) : kTmaChunk); }
+  __device__ void init(const RecCopyArgs* aa, int i0, int64_t off0, int64_t lo, int64_t hi_) {
+    a = aa; i = i0; off = off0; pos = lo; hi = hi_;
+    if (a->rec == nullptr) { src = a->src_base; dst = a->dst_base; body = hi_; off = lo; return; }
+    body = (i < a->n) ? body_of(i, &src, &dst) : 0;
+    settle();
+  }
+  __device__ bool valid() const { return pos < hi; }
+  __device__ uint32_t len() const {
+    int64_t l = body - off;
+    if (hi - pos < l) l = hi - pos;
+    return (uint32_t)(l < kTmaChunk ? l : kTmaChunk);
+  }
   __device__ void next() {
-    off += kTmaChunk;
-    if (off >= body) { it += gridDim.x; off = 0; load_item(); }
+    const uint32_t l = len();
+    off += l;
+    pos += l;
+    if (a->rec != nullptr) settle();
   }
 };
 
-__global__ void __launch_bounds__(128)
-copy_segments_tma_kernel(const CopySeg* __restrict__ segs, int n) {
+__global__ void __launch_bounds__(kRecThreads)
+copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
   extern __shared__ __align__(128) unsigned char sbuf[];
   __shared__ __align__(8) uint64_t bar[kTmaStages];
+  __shared__ int64_t wsum[kRecThreads / 32];
+  __shared__ int s_i0;
+  __shared__ int64_t s_off0;
   constexpr int L = kTmaStages - 1;          // loads kept in flight ahead of the store cursor
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < kTmaStages; ++i)
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar[i])));
+  const RecCopyArgs* a = &args;
+  // the stream: the records' bodies, or the single range's body (0 when unaligned)
+  const bool single = a->rec == nullptr;
+  const int64_t T = !single ? a->total
+                  : (((((uintptr_t)a->src_base) | ((uintptr_t)a->dst_base)) & 15) == 0 ? a->total & ~(int64_t)15 : 0);
+  int64_t per = (T + gridDim.x - 1) / gridDim.x;
+  per = (per + 15) & ~(int64_t)15;
+  const int64_t lo = (int64_t)blockIdx.x * per;
+  const int64_t hi = lo + per < T ? lo + per : T;
+
+  // the record holding stream position lo: exclusive scan of the bodies, a tile at a time
+  if (threadIdx.x == 0) { s_i0 = a->n; s_off0 = 0; }
+  __syncthreads();
+  if (a->rec != nullptr && lo < hi) {
+    int64_t carry = 0;
+    for (int t0 = 0; t0 < a->n; t0 += blockDim.x) {
+      const int k = t0 + threadIdx.x;
+      int64_t v = 0;
+      if (k < a->n) { const char* s_; char* d_; RecCursor c; c.a = a; v = c.body_of(k, &s_, &d_); }
+      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+      int64_t x = v;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      if (lane == 31) wsum[w] = x;
+      __syncthreads();
+      int64_t before = carry, tile = 0;
+      for (int q = 0; q < (int)(blockDim.x >> 5); ++q) {
+        if (q < w) before += wsum[q];
+        tile += wsum[q];
+      }
+      const int64_t start = before + x - v;   // exclusive prefix of record k
+      if (k < a->n && v > 0 && start <= lo && lo < start + v) { s_i0 = k; s_off0 = lo - start; }
+      carry += tile;
+      __syncthreads();
+      if (s_i0 < a->n || carry > lo) break;   // found (uniform: shared flag / uniform carry)
+    }
+  }
+
+  if (threadIdx.x == 0 && lo < hi) {
+    for (int q = 0; q < kTmaStages; ++q)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar[q])));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    ChunkCursor lc, sc;
-    lc.init(segs, n);
-    sc.init(segs, n);
-    auto issue_load = [&](int k) {
-      const int st = k % kTmaStages;
+    RecCursor lc, sc;
+    lc.init(a, s_i0, s_off0, lo, hi);
+    sc.init(a, s_i0, s_off0, lo, hi);
+    auto issue_load = [&](uint32_t k) {
+      const uint32_t st = k % kTmaStages;
       const uint32_t len = lc.len();
       asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(&bar[st])), "r"(len) : "memory");
       asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                    ::"r"(su32(sbuf + st * kTmaChunk)), "l"(lc.src + lc.off), "r"(len), "r"(su32(&bar[st])) : "memory");
       lc.next();
     };
-    int issued = 0;
-    for (; issued < L && lc.valid(); ++issued) issue_load(issued);
-    for (int k = 0; sc.valid(); ++k) {
-      const int st = k % kTmaStages;
-      const uint32_t par = (uint32_t)((k / kTmaStages) & 1);
+    uint32_t issued = 0;
+    for (; issued < (uint32_t)L && lc.valid(); ++issued) issue_load(issued);
+    for (uint32_t k = 0; sc.valid(); ++k) {
+      const uint32_t st = k % kTmaStages;
+      const uint32_t par = (k / kTmaStages) & 1;
       asm volatile("{\n.reg .pred P1;\nWAIT_%=:\nmbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n@!P1 bra WAIT_%=;\n}\n"
                    ::"r"(su32(&bar[st])), "r"(par) : "memory");
       asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(sc.dst + sc.off),
@@ -119,33 +192,46 @@ copy_segments_tma_kernel(const CopySeg* __restrict__ segs, int n) {
       sc.next();
       if (lc.valid()) {
         // the next load reuses the buffer of chunk issued+1-kTmaStages = k: wait until every
-        // store but the newest one (chunk k's, L - ... >= that) has read its buffer
+        // store but the newest kTmaStages-L ones has read its buffer
         asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(kTmaStages - L) : "memory");
         issue_load(issued++);
       }
     }
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
-  // unaligned items and the < 16-byte tails: plain byte copies by the CTA's threads
-  for (int it = blockIdx.x; it < n; it += gridDim.x) {
-    const CopySeg sg = segs[it];
-    const bool aligned = ((((uintptr_t)sg.src) | ((uintptr_t)sg.dst)) & 15) == 0;
-    const int64_t body = aligned ? (sg.bytes & ~(int64_t)15) : 0;
-    for (int64_t i = body + threadIdx.x; i < sg.bytes; i += blockDim.x) sg.dst[i] = sg.src[i];
+
+  // < 16-byte tails and unaligned records: byte copies, record k by CTA k % grid
+  if (single) {
+    for (int64_t x = T + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; x < a->total; x += (int64_t)gridDim.x * blockDim.x)
+      a->dst_base[x] = a->src_base[x];
+    return;
+  }
+  for (int k = blockIdx.x; k < a->n; k += gridDim.x) {
+    const int64_t* r = a->rec + (int64_t)k * a->stride;
+    if (a->f_late >= 0 && r[a->f_late] != a->late_val) continue;
+    const char* sp = a->src_base + r[a->f_src];
+    char* dp = a->dst_base + (r[a->f_dst] - a->dst_bias);
+    const int64_t nb = r[a->f_bytes];
+    const bool al = ((((uintptr_t)sp) | ((uintptr_t)dp)) & 15) == 0;
+    for (int64_t x = (al ? nb & ~(int64_t)15 : 0) + threadIdx.x; x < nb; x += blockDim.x) dp[x] = sp[x];
   }
 }
 
-cudaError_t launch_copy_segments_tma(const CopySeg* segs, int n, int grid, cudaStream_t s) {
-  if (n <= 0) return cudaSuccess;
+cudaError_t launch_copy_records(const RecCopyArgs& a, int grid, cudaStream_t s) {
+  if (a.total <= 0 && (a.rec == nullptr || a.n <= 0)) return cudaSuccess;
   static bool attr = false;
   const int smem = kTmaStages * kTmaChunk;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(copy_segments_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaError_t e = cudaFuncSetAttribute(copy_records_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  if (grid > n) grid = n;
-  copy_segments_tma_kernel<<<grid, 128, smem, s>>>(segs, n);
+  // at least one 16 KiB chunk per CTA; enough CTAs for the tail loop over the records
+  int64_t g = (a.total + kTmaChunk - 1) / kTmaChunk;
+  if (a.rec != nullptr && g < a.n) g = a.n;
+  if (g > grid) g = grid;
+  if (g < 1) g = 1;
+  copy_records_tma_kernel<<<(int)g, kRecThreads, smem, s>>>(a);
   return cudaGetLastError();
 }
 

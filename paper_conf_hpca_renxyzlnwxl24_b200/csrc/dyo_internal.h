@@ -160,6 +160,24 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
 struct CopySeg { const char* src; char* dst; int64_t bytes; };
 cudaError_t launch_copy_segments(const CopySeg* segs_dev_or_mapped, int n, int64_t chunk,
                                  int grid, cudaStream_t s);
-cudaError_t launch_copy_segments_tma(const CopySeg* segs, int n, int grid, cudaStream_t s);
+// Record-driven device<->device copy (TMA bulk; copy.cu): records rec[i*stride ..] (int64
+// fields) in DEVICE memory, i < n, filtered by rec[f_late] == late_val when f_late >= 0, copy
+// rec[f_bytes] bytes from src_base + rec[f_src] to dst_base + rec[f_dst] - dst_bias.
+// rec == nullptr: one range of `total` bytes from src_base to dst_base. total = sum over the
+// selected records of their 16-byte-aligned bodies (bytes & ~15, or 0 when src or dst is not
+// 16-byte aligned): the host computes it with rec_body() below.
+struct RecCopyArgs {
+  const int64_t* rec;
+  int32_t stride, n, f_src, f_dst, f_bytes, f_late;
+  int64_t late_val;
+  const char* src_base;
+  char* dst_base;
+  int64_t dst_bias;
+  int64_t total;
+};
+inline int64_t rec_body(const char* src, const char* dst, int64_t bytes) {
+  return ((((uintptr_t)src) | ((uintptr_t)dst)) & 15) == 0 ? (bytes & ~(int64_t)15) : 0;
+}
+cudaError_t launch_copy_records(const RecCopyArgs& a, int grid, cudaStream_t s);
 
 }  // namespace dyo

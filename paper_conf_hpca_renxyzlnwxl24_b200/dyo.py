@@ -339,11 +339,11 @@ class Dyo:
     def timings(self, reset=False):
         out = {}
         for k, name in enumerate(self.TIMING_KINDS):
-            ms, n, b = C.c_double(), i64(), i64()
-            self._check(self.L.dyo_get_timings(self.ctx, k, C.byref(ms), C.byref(n), C.byref(b), 0))
-            out[name] = {"ms": ms.value, "launches": n.value, "bytes": b.value}
+            ms, n, b, busy = C.c_double(), i64(), i64(), C.c_double()
+            self._check(self.L.dyo_get_timings(self.ctx, k, C.byref(ms), C.byref(n), C.byref(b), C.byref(busy), 0))
+            out[name] = {"ms": ms.value, "launches": n.value, "bytes": b.value, "busy_ms": busy.value}
         if reset:
-            self._check(self.L.dyo_get_timings(self.ctx, 0, None, None, None, 1))
+            self._check(self.L.dyo_get_timings(self.ctx, 0, None, None, None, None, 1))
         return out
 
     def pilot_stamps(self, enable=True):

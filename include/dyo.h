@@ -74,7 +74,10 @@ typedef struct {
   int32_t D_s;            /* input-shape descriptors per sample (R3) */
   int32_t h;              /* history groups per sample (R3) */
   int32_t K_max;          /* block-head slots (R4) */
-  int32_t branch_head;    /* 1: logits carry a branch head (R4); 0: paper traversal decode */
+  int32_t branch_head;    /* 1: logits carry a branch head (R4); 0: the paper's traversal decode
+                           * (P:L145-L147): dyo_pilot_predict copies the logits to the host,
+                           * synchronises its stream once and searches the program's paths
+                           * there (top-level sites only, like the device decode) */
   /* program nodes in preorder; node kinds: 0 OP, 1 IF, 2 LOOP, 3 BRANCH (start of an If arm).
    * IF: a = number of branches, followed by that many BRANCH nodes each followed by its body;
    * LOOP: a = lo, b = hi trip count, followed by its body; OP: a = operator index (operators
@@ -177,6 +180,14 @@ typedef struct {
 dyo_status dyo_arch_check(const dyo_arch* arch, int32_t align, dyo_arch_summary* out, int32_t* seg_table,
                           int32_t* op_sig, char* err, int32_t errlen);
 
+/* Host-only run of the traversal decode (R4) that dyo_pilot_predict uses when the
+ * arch has no branch head (no GPU needed; used by the CPU test suite). slots: K_max x 10 decoded
+ * block-head vectors (a slot with count 0 is empty); choices (n_sites int32 out): the choice of
+ * every site, preorder; *matched = 1 for an exact match, 0 for the closest-count fallback.
+ * DYO_E_UNSUPPORTED for nested control flow, DYO_E_CAPACITY if the search exceeds its budget. */
+dyo_status dyo_traverse_check(const dyo_arch* arch, const int32_t* slots, int32_t* choices, int32_t* matched,
+                              char* err, int32_t errlen);
+
 /* Load pilot weights (copied to the device, rows padded to 16 bytes). F and O must match the
  * arch: F = pad16(3 + D_s + 10*S_max + 10*h); O >= 10*K_max + branch logits. */
 dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w);
@@ -205,6 +216,10 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
  * group_rows (2*K_max int32 [start, end) pairs). Any output pointer may be NULL. */
 dyo_status dyo_prediction_get(dyo_ctx* ctx, int32_t b, int32_t* K, int32_t* blocks,
                               int32_t* choices, int32_t* group_rows, void* stream);
+/* Traversal decode only (arch without a branch head): *matched = 1 if prediction b
+ * of the last dyo_pilot_predict matched a path exactly, 0 if the closest-operator-count
+ * fallback of P:L147 was taken. DYO_E_STATE with a branch head. Host-side; no sync. */
+dyo_status dyo_prediction_matched(dyo_ctx* ctx, int32_t b, int32_t* matched);
 /* Tensor-set entries of group g of prediction b (host out, capacity cap entries of 3 int32:
  * tensor, mode, needs_fetch); *n receives the count (DYO_E_CAPACITY if cap < n). */
 dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* out, int32_t cap,

@@ -42,6 +42,14 @@ struct dyo_ctx {
   // prediction
   PredDev pd{};
   double* logits64 = nullptr;      // fp64 logits (decode decisions, R4)
+  // traversal decode (no branch head): host copy of the program tables, pinned
+  // logits / choices staging and the device choices the decode kernel replays
+  int branch_head = 1;
+  TravArch trav;
+  double* h_logits = nullptr;      // pinned, max_batch x O
+  int32_t* h_forced[2] = {nullptr, nullptr};   // pinned, max_batch x n_sites (alternating)
+  int32_t* d_forced = nullptr;
+  int32_t* h_matched = nullptr;    // per prediction of the last traversal: 1 exact match
   int64_t* desc_dev = nullptr;
   int32_t* hist_dev = nullptr;
   int32_t* hist_tab[2] = {nullptr, nullptr};
@@ -170,6 +178,8 @@ void free_plan_host(dyo_ctx* c) {
     P.seg_used = 0;
   }
   fh(c->h_status); fh(c->h_counts); fh(c->h_loc); fh(c->h_off);
+  fh(c->h_forced[0]); fh(c->h_forced[1]); fh(c->h_matched);
+  c->h_forced[0] = c->h_forced[1] = c->h_matched = nullptr;
   c->h_status = c->h_counts = nullptr;
   c->h_loc = nullptr;
   c->h_off = nullptr;
@@ -245,8 +255,6 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, ArchHost& h, std::string& e
       A->K_max > 256 || A->n_tensors < 1 || A->n_tensors >= (1 << 20) || A->n_ops < 0 ||
       A->n_ops >= (1 << 24) || A->n_nodes < 0)
     return hfail(err, DYO_E_INVAL, "arch: bad sizes");
-  if (!A->branch_head)
-    return hfail(err, DYO_E_UNSUPPORTED, "arch: traversal decode (no branch head) runs only in the oracle in this build");
   const int T = A->n_tensors, n_ops = A->n_ops, N = A->n_nodes;
   // ---- tensors ----
   h.T = T;
@@ -361,6 +369,8 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, ArchHost& h, std::string& e
       if (site_tie[tie] >= 0 || site_nch[tie] != site_nch[s] || site_kind[tie] != k)
         return hfail(err, DYO_E_INVAL, "arch: site %d tie target must be a free site of the same shape", s);
       site_logit.push_back(-1);
+    } else if (!A->branch_head) {
+      site_logit.push_back(-1);          // traversal decode: choices come from the host (R4)
     } else {
       site_logit.push_back(logit);
       logit += site_nch[s];
@@ -484,6 +494,7 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   free_list(ctx->pilot_dev);
   free_plan_host(ctx);
   if (ctx->host_pool) cudaFreeHost(ctx->host_pool);
+  if (ctx->h_logits) cudaFreeHost(ctx->h_logits);
   if (ctx->arena) cudaFree(ctx->arena);
   if (ctx->staging) cudaFree(ctx->staging);
   for (auto& P : ctx->slot)
@@ -547,6 +558,10 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   UP(seg_table, seg_table);
 #undef UP
   ctx->n_ops = n_ops; ctx->n_sites = n_sites; ctx->K_max = A->K_max; ctx->F = ad.F;
+  ctx->branch_head = A->branch_head ? 1 : 0;
+  ad.branch_head = ctx->branch_head;
+  ctx->trav = TravArch{h.sig, site_kind, site_nch, site_lo, site_tie, site_arm_ptr, arm_first, arm_n,
+                       piece_kind, piece_a, piece_b, piece_c};
   ctx->O_min = 10 * A->K_max + ctx->n_branch_logits;
 
   // ---- prediction storage ----
@@ -561,6 +576,11 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   DA(ctx->desc_dev, (size_t)B * std::max(A->D_s, 1)); DA(ctx->hist_dev, (size_t)B * std::max(A->h, 1));
   DA(ctx->hist_tab[0], (size_t)B * K * 10); DA(ctx->hist_tab[1], (size_t)B * K * 10);
   DA(ctx->hist_K[0], B); DA(ctx->hist_K[1], B);
+  if (!ctx->branch_head) {
+    int32_t* f = nullptr;
+    DA(f, (size_t)B * std::max(n_sites, 1));
+    ad.forced = ctx->d_forced = f;
+  }
   ctx->hist_B[0] = ctx->hist_B[1] = 0;
   ctx->hist_cur = 0;
   ctx->last_B = 0;
@@ -590,6 +610,11 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   if ((st = hmap((void**)&ctx->h_counts, 16 * sizeof(int32_t)))) return st;
   if ((st = hmap((void**)&ctx->h_loc, T))) return st;
   if ((st = hmap((void**)&ctx->h_off, sizeof(int64_t) * T))) return st;
+  if (!ctx->branch_head) {
+    for (int i = 0; i < 2; ++i)
+      if ((st = hmap((void**)&ctx->h_forced[i], sizeof(int32_t) * B * std::max(n_sites, 1)))) return st;
+    if ((st = hmap((void**)&ctx->h_matched, sizeof(int32_t) * B))) return st;
+  }
   memset(ctx->h_loc, 0xff, T);
   int32_t* d_status = nullptr;
   int32_t* d_counts = nullptr;
@@ -634,6 +659,23 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   ctx->arch_ok = true;
   ctx->pilot_ok = false;
   return DYO_OK;
+}
+
+dyo_status dyo_traverse_check(const dyo_arch* A, const int32_t* slots, int32_t* choices, int32_t* matched,
+                              char* err, int32_t errlen) {
+  if (!A || !slots || !choices || !matched) return DYO_E_INVAL;
+  ArchHost h;
+  std::string e;
+  dyo_status st = parse_arch(A, 256, h, e);
+  if (!st) {
+    TravArch t{h.sig, h.site_kind, h.site_nch, h.site_lo, h.site_tie, h.site_arm_ptr, h.arm_first, h.arm_n,
+               h.piece_kind, h.piece_a, h.piece_b, h.piece_c};
+    int m = 0;
+    st = traverse_decode(t, slots, A->K_max, choices, &m, e);
+    *matched = m;
+  }
+  if (err && errlen > 0) { strncpy(err, e.c_str(), errlen - 1); err[errlen - 1] = 0; }
+  return st;
 }
 
 dyo_status dyo_arch_check(const dyo_arch* A, int32_t align, dyo_arch_summary* out, int32_t* seg_table,
@@ -743,6 +785,9 @@ dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   double* lg = nullptr;
   if ((s = dalloc(ctx, ctx->pilot_dev, &lg, (size_t)ctx->cfg.max_batch * w->O))) return s;
   ctx->logits64 = lg;
+  if (ctx->h_logits) { cudaFreeHost(ctx->h_logits); ctx->h_logits = nullptr; }
+  if (!ctx->branch_head)
+    CK(cudaHostAlloc((void**)&ctx->h_logits, sizeof(double) * ctx->cfg.max_batch * w->O, cudaHostAllocPortable));
   ctx->pilot_ok = true;
   return DYO_OK;
 }
@@ -823,6 +868,27 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
     CK(launch_pilot(ctx->ad, ctx->pdv, ctx->pdv_dev, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur], ctx->hist_B[cur], B,
                     ctx->logits64, logits, ctx->pd, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur], &fused, st));
   }
+  if (!ctx->branch_head) {
+    // traversal decode: logits to the host, one sync, block head -> slots
+    // (R4: rint half-even of y * 2^sigma, clamped), path search, choices back to the device
+    const int O = ctx->ad.O, K = ctx->K_max, ns = ctx->n_sites;
+    CK(cudaMemcpyAsync(ctx->h_logits, ctx->logits64, sizeof(double) * B * O, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    int32_t* hf = ctx->h_forced[cur];
+    std::vector<int32_t> slots((size_t)K * 10);
+    for (int b = 0; b < B; ++b) {
+      const double* y = ctx->h_logits + (size_t)b * O;
+      for (int i = 0; i < K * 10; ++i) {
+        const double t = std::fmin(std::fmax(y[i] * ((i % 10) < 7 ? 16.0 : 1024.0), 0.0), (double)kSat);
+        slots[i] = (int32_t)std::nearbyint(t);
+      }
+      int matched = 0;
+      dyo_status r = traverse_decode(ctx->trav, slots.data(), K, hf + (size_t)b * std::max(ns, 1), &matched, ctx->err);
+      if (r) return r;
+      ctx->h_matched[b] = matched;
+    }
+    if (ns > 0) CK(cudaMemcpyAsync(ctx->d_forced, hf, sizeof(int32_t) * B * ns, cudaMemcpyHostToDevice, st));
+  }
   if (!fused) {
     TScope ts(ctx, 1, st);
     CK(launch_decode(ctx->ad, ctx->logits64, ctx->pd, B, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur], st));
@@ -847,6 +913,13 @@ dyo_status dyo_prediction_get(dyo_ctx* ctx, int32_t b, int32_t* K, int32_t* bloc
   if (choices && ctx->n_sites)
     CK(cudaMemcpy(choices, ctx->pd.choices + (size_t)b * ctx->n_sites, sizeof(int32_t) * ctx->n_sites, cudaMemcpyDeviceToHost));
   if (group_rows) CK(cudaMemcpy(group_rows, ctx->pd.grp + (size_t)b * Km * 2, sizeof(int32_t) * Km * 2, cudaMemcpyDeviceToHost));
+  return DYO_OK;
+}
+
+dyo_status dyo_prediction_matched(dyo_ctx* ctx, int32_t b, int32_t* matched) {
+  if (!ctx || !matched || b < 0 || b >= ctx->last_B) return DYO_E_INVAL;
+  if (ctx->branch_head || !ctx->h_matched) return fail(ctx, DYO_E_STATE, "no traversal decode in this arch");
+  *matched = ctx->h_matched[b];
   return DYO_OK;
 }
 

@@ -30,7 +30,7 @@ decode_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t*
   const double* y = S.ys;
   int* tabs = reinterpret_cast<int*>(S.ys + ((a.O + 15) / 16) * 16);
   const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap2);
-  if (threadIdx.x < 32) head_decode_warp(A, y, S.H, threadIdx.x);
+  if (threadIdx.x < 32) head_decode_warp(A, y, S.H, threadIdx.x, b);
   __syncthreads();
   if (g == 0) write_head(A, S.H, y, pd, b, hist_K);
   if (g >= S.H.K) {

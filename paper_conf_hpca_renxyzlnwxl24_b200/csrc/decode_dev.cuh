@@ -79,7 +79,9 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 }
 
 // Decode the head of logits y (fp64, R4) into H. Called by ONE warp; __syncwarp() at the end.
-static __device__ void head_decode_warp(const ArchDev& a, const double* __restrict__ y, DecHead& H, int lane) {
+// b = index of the prediction in its batch (selects the host traversal's choices when the
+// arch has no branch head).
+static __device__ void head_decode_warp(const ArchDev& a, const double* __restrict__ y, DecHead& H, int lane, int b) {
   // 1. block-head counts of every slot; compact the non-empty ones in slot order
   int nk = 0;
   for (int k0 = 0; k0 < a.K_max; k0 += 32) {
@@ -94,8 +96,12 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
     if (n != 0) H.cntc[nk + __popc(m & ((1u << lane) - 1))] = n;
     nk += __popc(m);
   }
-  // 2. branch head: argmax per free site (lowest index on ties), then tied sites
-  for (int i = lane; i < a.n_sites; i += 32) {
+  // 2. branch head: argmax per free site (lowest index on ties), then tied sites; without a
+  //    branch head the choices are the host traversal's
+  if (a.forced) {
+    for (int i = lane; i < a.n_sites; i += 32) H.choice[i] = a.forced[(int64_t)b * a.n_sites + i];
+  }
+  for (int i = lane; i < a.n_sites && !a.forced; i += 32) {
     const int off = a.site_logit[i];
     if (off >= 0) {
       int best = 0;
@@ -109,7 +115,7 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
     }
   }
   __syncwarp();
-  for (int i = lane; i < a.n_sites; i += 32)
+  for (int i = lane; i < a.n_sites && !a.forced; i += 32)
     if (a.site_logit[i] < 0) H.choice[i] = H.choice[a.site_tie[i]];   // tie targets are free sites
   __syncwarp();
   // 3. piece lengths -> exclusive scan -> piece starts (R2)

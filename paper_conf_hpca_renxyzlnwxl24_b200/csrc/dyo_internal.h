@@ -73,6 +73,8 @@ struct ArchDev {
   const int32_t* piece_b;
   const int32_t* piece_c;
   const int32_t* seg_table;  // S_max x 10
+  int branch_head;           // 0: choices come from the host traversal (forced, R4)
+  const int32_t* forced;     // max_batch x n_sites choices written by the traversal, or null
 };
 
 // ---- prediction storage -------------------------------------------------------------
@@ -138,6 +140,17 @@ struct PlanScratch {
   int32_t* grp_b;       // max_groups: prediction of each planned group
   int32_t* grp_k;
 };
+
+// ---- host traversal decode (traverse.cpp, R4) ------------------------------
+struct TravArch {
+  std::vector<int32_t> sig;   // n_ops x 9 saturated signatures
+  std::vector<int32_t> site_kind, site_nch, site_lo, site_tie, site_arm_ptr, arm_first, arm_n;
+  std::vector<int32_t> piece_kind, piece_a, piece_b, piece_c;
+};
+// slots: K_max x 10 decoded block head of one prediction; choices: n_sites out; *matched = 1
+// when an exact match was found (else the closest-count fallback of P:L147).
+dyo_status traverse_decode(const TravArch& A, const int32_t* slots, int K_max, int32_t* choices, int* matched,
+                           std::string& err);
 
 // ---- launchers (implemented in the .cu files) ------------------------------------------
 cudaError_t launch_encode(const ArchDev& a, const int64_t* desc, const int32_t* hist,

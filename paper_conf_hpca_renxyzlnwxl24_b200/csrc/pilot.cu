@@ -444,7 +444,7 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
     for (int i = tid; i < p.O; i += blockDim.x) ys[i] = y[i];
     __syncthreads();
     y = ys;
-    if (warp == 0) head_decode_warp(A, y, H, lane);
+    if (warp == 0) head_decode_warp(A, y, H, lane, b);
     __syncthreads();
     stamp(26, stamp_on);
     if (r == 0) write_head(A, H, y, pd, b, hist_K_out);
@@ -518,7 +518,7 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   sp.C = C;
   sp.Bs = B < kBs ? 1 : kBs;
   // fuse the decode when the cluster has at least one CTA per two groups of its samples
-  sp.fuse_decode = (sp.Bs * a.K_max <= 2 * C) ? 1 : 0;
+  sp.fuse_decode = (a.branch_head && sp.Bs * a.K_max <= 2 * C) ? 1 : 0;   // traversal: host decides first
   const int act_bytes = 2 * sp.Bs * p.max_width * (int)sizeof(double);
   const int base = ((2 * (4 + kMaxLayers) + 2) * 8 + 127) / 128 * 128;
   const int budget = kDynCap - act_bytes;

@@ -95,7 +95,7 @@ def lib():
                      "dyo_arena", "dyo_encode_features", "dyo_pilot_predict", "dyo_prediction_get",
                      "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records", "dyo_migrate",
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
-                     "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy"):
+                     "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -103,9 +103,9 @@ def lib():
 
 EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_destroy", "dyo_load_arch",
            "dyo_load_pilot", "dyo_host_pool", "dyo_arena", "dyo_encode_features", "dyo_pilot_predict",
-           "dyo_prediction_get", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
+           "dyo_prediction_get", "dyo_prediction_matched", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
-           "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy")
+           "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check")
 
 
 def _a(x, dt):
@@ -184,6 +184,19 @@ def arch_check(wl, align=256, branch_head=None):
     st = lib().dyo_arch_check(C.byref(arch), align, C.byref(summ), _p(seg, i32), _p(sig, i32), err, 512)
     return (st, {f: getattr(summ, f) for f, _ in ArchSummary._fields_}, seg[:wl.S_max], sig[:n_ops],
             err.value.decode())
+
+
+def traverse_check(wl, slots):
+    """Host-only traversal decode by libdyo (no GPU): (status, choices, matched, err)."""
+    arch, keep = _arch_struct(wl, False)
+    n_sites = sum(1 for k in keep[0]["kind"] if k in (1, 2))
+    sl = _a(slots, np.int32).reshape(-1)
+    assert sl.size == wl.K_max * 10
+    ch = np.zeros(max(n_sites, 1), np.int32)
+    m = i32()
+    err = C.create_string_buffer(512)
+    st = lib().dyo_traverse_check(C.byref(arch), _p(sl, i32), _p(ch, i32), C.byref(m), err, 512)
+    return st, ch[:n_sites].tolist(), m.value, err.value.decode()
 
 
 class Dyo:
@@ -296,6 +309,13 @@ class Dyo:
                                               _p(rows, i32), P(stream)))
         k = K.value
         return k, blocks[:k].copy(), choices[:n_sites].copy(), rows[:k].copy()
+
+    def matched(self, b):
+        """Traversal decode: 1 if prediction b matched a path exactly, 0 if the
+        closest-count fallback was taken."""
+        m = i32()
+        self._check(self.L.dyo_prediction_matched(self.ctx, b, C.byref(m)))
+        return m.value
 
     def group_entries(self, b, g, cap=1024, stream=0):
         out = np.zeros((cap, 3), np.int32)

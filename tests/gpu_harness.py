@@ -24,7 +24,7 @@ def oracle_step(wl, sample_ids, state, table, policy=None):
         y = P.forward(wl.pilot, x, wl.nn_type)
         feats.append(x)
         logits.append(y)
-        preds.append(D.decode(wl, y))
+        preds.append(D.decode(wl, y, branch_head=wl.notes.get("branch_head", True)))
     Ws = [Wj for p in preds for Wj in p.W]
     new_table = [b for p in preds for b in p.blocks]
     try:

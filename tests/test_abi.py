@@ -63,5 +63,5 @@ def test_arch_validation_errors(dyo):
     wl.program.append(WL.If([[WL.Loop([wl.program[0]], 1, 2)], []]))   # nested site
     st, *_ = dyo.arch_check(wl)
     assert st == -7
-    st, *_ = dyo.arch_check(WL.make("tiny"), branch_head=False)
-    assert st == -7
+    st, summ, *_ = dyo.arch_check(WL.make("tiny"), branch_head=False)   # traversal decode: no branch head
+    assert st == 0 and summ["n_branch_logits"] == 0

@@ -160,3 +160,45 @@ def test_plan_bitexact_global_state_path(name, steps, monkeypatch):
     monkeypatch.setenv("DYO_PLAN_GLOBAL_STATE", "1")
     wl = WL.make(name, n_samples=32)
     _run_plan_steps(wl, steps, 1, 1).close()
+
+
+def _planted_path_tiny(choices, seed=0):
+    """tiny without a branch head whose block head is planted with the exact block vectors of
+    one path cut in 8 even groups (oracle values; R4 scaling is exact in fp32)."""
+    wl = WL.make_tiny(seed=seed, n_samples=32, branch_head=False)
+    from oracle import decode as D
+    rows = A.resolve(wl.program, choices)
+    L = len(rows)
+    cuts = [(k * L // 8, (k + 1) * L // 8) for k in range(8)]
+    Wo, bo = wl.pilot.weights["out.W"], wl.pilot.weights["out.b"]
+    Wo[:80] = 0
+    bo[:80] = 0
+    for k, (s, e) in enumerate(cuts):
+        v = A.block10(rows[s:e])
+        for i in range(10):
+            bo[10 * k + i] = np.float32(v[i] / (16.0 if i < 7 else 1024.0))
+    return wl
+
+
+@pytest.mark.parametrize("B", [1, 4])
+@pytest.mark.parametrize("planted", [None, [1, 0, 2], [0, 1, 1]])
+def test_decode_traversal(B, planted):
+    """No branch head: the paper's traversal on the host inside dyo_pilot_predict,
+    then the device decode of the chosen path; exact-match and fallback cases."""
+    wl = WL.make_tiny(n_samples=32, branch_head=False) if planted is None else _planted_path_tiny(planted)
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    d.predict(wl.samples[:B].copy(), None, B, stream=_stream())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), ())
+    for b in range(B):
+        p = r["preds"][b]
+        assert not p.near_ties
+        assert d.matched(b) == int(p.matched)
+        if planted is not None:
+            assert p.matched
+        _check_prediction(d, wl, b, p)
+    d.close()
+
+
+def test_plan_bitexact_traversal():
+    wl = _planted_path_tiny([1, 1, 0])
+    _run_plan_steps(wl, 4, 2, 1).close()

@@ -53,7 +53,7 @@ typedef struct {
   int32_t policy;         /* 0 = PAPER (evict every unused tensor), 1 = RETAIN (R10) */
   int32_t max_batch;      /* max predictions per dyo_pilot_predict call (>= 1) */
   int32_t max_groups;     /* max groups per dyo_plan (sum over its predictions), <= 65535 */
-  int32_t max_entries;    /* capacity of tensor-set entries per dyo_plan (0 = auto) */
+  int32_t max_entries;    /* capacity of tensor-set entries per dyo_plan (0 = 512 per group) */
   int32_t max_records;    /* capacity of plan records per dyo_plan (0 = auto) */
   int64_t staging_bytes;  /* device staging for pack/unpack/compaction (outside B; 0 = 64 MiB) */
   int64_t dma_min_bytes;  /* host runs >= this move by DMA, smaller by zero-copy kernel (0 = 2 MiB) */
@@ -104,6 +104,17 @@ typedef struct {
   const int64_t* t_bytes;       /* > 0 */
   const int64_t* t_host_off;    /* home offset in the ctx's pinned host pool, ALIGN-aligned */
   const int32_t* t_flags;       /* bit 0: transient (contents end with the step, R9) */
+  /* per-iteration and per-sample tensors (R13; each may be NULL = all zero): access q of an
+   * operator names tensor acc_tensor[q] + acc_stride[q] * k + acc_bstride[q] * b, where k is
+   * the iteration index of its LOOP (0..n-1, or n-1..0 when the LOOP node's flags bit 0 is
+   * set: a backward pass over a forward loop's tensors) and b the prediction's index in its
+   * dyo_pilot_predict batch (e.g. the minibatch row whose input sequence it reads). The named
+   * ids must stay in [0, n_tensors) and ascending within the operator for every k < hi and
+   * b < max_batch (linear, so checked at the corners; DYO_E_INVAL otherwise); operators outside
+   * loops must have acc_stride 0. */
+  const int32_t* acc_stride;
+  const int32_t* node_flags;
+  const int32_t* acc_bstride;
 } dyo_arch;
 
 /* Pilot weights (host fp32, row-major W[out][in]); topology R5. n_feature = 0 means an

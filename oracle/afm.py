@@ -75,13 +75,40 @@ def n_choices(site):
     return len(site.branches) if isinstance(site, If) else site.hi - site.lo + 1
 
 
-def resolve(program, choices):
+def bind(op, k, b=0):
+    """The operator as executed in iteration k of its innermost enclosing loop by prediction b
+    of its batch (reading R13): an access (t, m, stride_k, stride_b) names tensor
+    t + stride_k * k + stride_b * b (missing strides are 0); accesses sorted by tensor id (the
+    order W_j uses within an operator, reading R8). k = None outside loops (stride_k must be 0)."""
+    acc = []
+    plain = True
+    for a in op.acc:
+        t, m = a[0], a[1]
+        sk = a[2] if len(a) > 2 else 0
+        sb = a[3] if len(a) > 3 else 0
+        if sk:
+            if k is None:
+                raise ValueError("strided access outside a loop")
+            t = t + sk * k
+        t = t + sb * b
+        plain = plain and len(a) == 2
+        acc.append((t, m))
+    acc.sort()
+    if len({t for t, _ in acc}) != len(acc):
+        raise ValueError("an operator accesses a tensor twice in one iteration")
+    if plain and tuple(acc) == tuple(op.acc):
+        return op
+    return Op(op.idioms, op.inputs, tuple(acc), op.name)
+
+
+def resolve(program, choices, b=0):
     """Executed row sequence for given site choices (choices[i] = choice index of preorder
     site i; If -> branch index, Loop -> trip count lo + index).
 
     Each row is (op or None). An executed If contributes one control row followed by the
     chosen branch; a Loop with n iterations contributes n+1 control rows (n continue tests
-    plus the exit test, reading R2): [Z, body, Z, body, ..., Z]."""
+    plus the exit test, reading R2): [Z, body, Z, body, ..., Z]. b = the prediction's index in
+    its batch (per-sample tensors, reading R13)."""
     site_list = sites(program)
     index = {id(s): i for i, s in enumerate(site_list)}
 
@@ -91,23 +118,23 @@ def resolve(program, choices):
             i = s.tie
         return choices[i]
 
-    def rec(prog):
+    def rec(prog, k):
         out = []
         for it in prog:
             if isinstance(it, Op):
-                out.append(it)
+                out.append(bind(it, k, b))
             elif isinstance(it, If):
                 out.append(None)
-                out.extend(rec(it.branches[choice_of(it)]))
+                out.extend(rec(it.branches[choice_of(it)], k))
             else:
                 n = it.lo + choice_of(it)
-                for _ in range(n):
+                for i in range(n):
                     out.append(None)
-                    out.extend(rec(it.body))
+                    out.extend(rec(it.body, n - 1 - i if it.rev else i))
                 out.append(None)
         return out
 
-    return rec(program)
+    return rec(program, None)
 
 
 def row_sig(row):

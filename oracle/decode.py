@@ -94,21 +94,21 @@ def cut(L, counts):
     return groups
 
 
-def enumerate_paths(program):
+def enumerate_paths(program, b=0):
     """All resolved paths in lexicographic order of branch choices (program order; lower
     branch index / lower trip count first). Yields (choices_by_site_index, rows)."""
     sl = A.sites(program)
     index = {id(s): i for i, s in enumerate(sl)}
 
-    def rec(items, pos, choices):
-        # yields (choices, rows) for items[pos:]
+    def rec(items, pos, choices, k=None):
+        # yields (choices, rows) for items[pos:]; k = iteration index of the innermost loop (R13)
         if pos == len(items):
             yield choices, []
             return
         it = items[pos]
         if isinstance(it, Op):
-            for ch, rows in rec(items, pos + 1, choices):
-                yield ch, [it] + rows
+            for ch, rows in rec(items, pos + 1, choices, k):
+                yield ch, [A.bind(it, k, b)] + rows
             return
         si = index[id(it)]
         opts = [choices[it.tie]] if it.tie >= 0 else list(range(A.n_choices(it)))
@@ -116,38 +116,37 @@ def enumerate_paths(program):
             ch0 = dict(choices)
             ch0[si] = c
             if isinstance(it, If):
-                heads = [(ch0, [None])]
                 body_items = it.branches[c]
-                for ch1, brows in rec(body_items, 0, ch0):
-                    for ch2, rest in rec(items, pos + 1, ch1):
+                for ch1, brows in rec(body_items, 0, ch0, k):
+                    for ch2, rest in rec(items, pos + 1, ch1, k):
                         yield ch2, [None] + brows + rest
             else:
                 n = it.lo + c
-                yield from _loop_iter(it, n, items, pos, ch0, rec)
+                yield from _loop_iter(it, n, items, pos, ch0, rec, k)
 
-    def _loop_iter(it, n, items, pos, ch, rec_):
-        def iters(k, chk):
-            if k == n:
+    def _loop_iter(it, n, items, pos, ch, rec_, k_out):
+        def iters(i, chk):
+            if i == n:
                 yield chk, [None]
                 return
-            for ch1, brows in rec_(it.body, 0, chk):
-                for ch2, rest in iters(k + 1, ch1):
+            for ch1, brows in rec_(it.body, 0, chk, n - 1 - i if it.rev else i):
+                for ch2, rest in iters(i + 1, ch1):
                     yield ch2, [None] + brows + rest
         for ch1, lrows in iters(0, ch):
-            for ch2, rest in rec_(items, pos + 1, ch1):
+            for ch2, rest in rec_(items, pos + 1, ch1, k_out):
                 yield ch2, lrows + rest
 
     for ch, rows in rec(program, 0, {}):
         yield [ch.get(i, 0) for i in range(len(sl))], rows
 
 
-def traversal(program, pred_blocks):
+def traversal(program, pred_blocks, b=0):
     """The paper's mapping: find the first path (lexicographic order) whose
     rows, cut at the predicted cumulative counts, give exactly the predicted block vectors;
     otherwise pick the path closest in operator count (first on ties)."""
     total = sum(v[0] for v in pred_blocks)
     best = None
-    for choices, rows in enumerate_paths(program):
+    for choices, rows in enumerate_paths(program, b):
         if len(rows) == total:
             groups = cut(len(rows), [v[0] for v in pred_blocks])
             if len(groups) == len(pred_blocks) and all(
@@ -180,16 +179,17 @@ def tensor_sets(path, groups):
     return out
 
 
-def decode(wl, y, branch_head=True):
+def decode(wl, y, branch_head=True, b=0):
+    """Decode prediction b of a batch (b selects its per-sample tensors, reading R13)."""
     near = []
     slots = decode_block_head(y, wl.K_max, near)
     counts_slots = [v for v in slots if v[0] != 0]
     matched = True
     if branch_head:
         choices = decode_branch_head(y, wl.program, wl.K_max, near)
-        path = A.resolve(wl.program, choices)
+        path = A.resolve(wl.program, choices, b)
     else:
-        choices, path, matched = traversal(wl.program, counts_slots)
+        choices, path, matched = traversal(wl.program, counts_slots, b)
     groups = cut(len(path), [v[0] for v in counts_slots])
     blocks = [A.block10(path[s:e]) for s, e in groups]
     return Prediction(choices, path, groups, blocks, tensor_sets(path, groups), slots, near, matched)

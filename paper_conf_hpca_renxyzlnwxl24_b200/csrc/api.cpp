@@ -235,7 +235,7 @@ struct ArchHost {
   int T = 0, n_sites = 0, n_branch_logits = 0;
   int64_t L_max = 0, pool = 0;
   std::vector<int64_t> t_bytes, t_abytes, t_host;
-  std::vector<int32_t> t_flags, sig, acc_ptr, acc_t, acc_m;
+  std::vector<int32_t> t_flags, sig, acc_ptr, acc_t, acc_m, acc_s, acc_sb, site_rev;
   std::vector<int32_t> site_kind, site_nch, site_lo, site_tie, site_logit, site_arm_ptr, arm_first, arm_n;
   std::vector<int32_t> piece_kind, piece_a, piece_b, piece_c, seg_table;
 };
@@ -250,7 +250,7 @@ dyo_status hfail(std::string& err, dyo_status s, const char* fmt, ...) {
   return s;
 }
 
-dyo_status parse_arch(const dyo_arch* A, int64_t AL, ArchHost& h, std::string& err) {
+dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std::string& err) {
   if (A->nn_type < 0 || A->nn_type > 2 || A->S_max < 0 || A->D_s < 0 || A->h < 0 || A->K_max < 1 ||
       A->K_max > 256 || A->n_tensors < 1 || A->n_tensors >= (1 << 20) || A->n_ops < 0 ||
       A->n_ops >= (1 << 24) || A->n_nodes < 0)
@@ -298,6 +298,8 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, ArchHost& h, std::string& e
       prev = t;
       acc_t.push_back(t);
       acc_m.push_back(md);
+      h.acc_s.push_back(A->acc_stride ? A->acc_stride[q] : 0);
+      h.acc_sb.push_back(A->acc_bstride ? A->acc_bstride[q] : 0);
     }
   }
   acc_ptr[n_ops] = (int32_t)acc_t.size();
@@ -365,6 +367,7 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, ArchHost& h, std::string& e
       site_nch.push_back(A->node_b[i] - A->node_a[i] + 1);
       site_lo.push_back(A->node_a[i]);
     }
+    h.site_rev.push_back(k == 2 && A->node_flags && (A->node_flags[i] & 1) ? 1 : 0);
     if (tie >= 0) {
       if (site_tie[tie] >= 0 || site_nch[tie] != site_nch[s] || site_kind[tie] != k)
         return hfail(err, DYO_E_INVAL, "arch: site %d tie target must be a free site of the same shape", s);
@@ -417,6 +420,33 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, ArchHost& h, std::string& e
     }
   }
   if ((int)piece_kind.size() > 1024) return hfail(err, DYO_E_CAPACITY, "arch: more than 1024 top-level pieces");
+  // per-iteration tensors (R13): strides only in loop bodies; named ids in range and ascending
+  // within the operator at k = 0 (checked above) and k = hi - 1 (linear in k, so everywhere)
+  {
+    std::vector<int> op_hi(n_ops, -1);   // trip bound of the operator's loop, -1 outside loops
+    for (size_t p = 0; p < piece_kind.size(); ++p)
+      if (piece_kind[p] == 2) {
+        const int s = piece_a[p];
+        for (int o = piece_b[p]; o < piece_b[p] + piece_c[p]; ++o) op_hi[o] = site_lo[s] + site_nch[s] - 1;
+      }
+    for (int o = 0; o < n_ops; ++o) {
+      for (int q = acc_ptr[o]; q < acc_ptr[o + 1]; ++q)
+        if (h.acc_s[q] != 0 && op_hi[o] < 0)
+          return hfail(err, DYO_E_INVAL, "arch: op %d has a strided access outside a loop", o);
+      // corners (k, b) in {0, hi-1} x {0, max_b-1}; (0, 0) was checked with the accesses
+      const int kmax = std::max(op_hi[o] - 1, 0), bmax = std::max(max_b - 1, 0);
+      for (int corner = 1; corner < 4; ++corner) {
+        const int k = (corner & 1) ? kmax : 0, b = (corner & 2) ? bmax : 0;
+        int64_t prev_id = -1;
+        for (int q = acc_ptr[o]; q < acc_ptr[o + 1]; ++q) {
+          const int64_t t = (int64_t)acc_t[q] + (int64_t)h.acc_s[q] * k + (int64_t)h.acc_sb[q] * b;
+          if (t < 0 || t >= T || t <= prev_id)
+            return hfail(err, DYO_E_INVAL, "arch: op %d strided accesses leave [0, T) or lose ascending order", o);
+          prev_id = t;
+        }
+      }
+    }
+  }
   if (L_max >= (1 << 30)) return hfail(err, DYO_E_CAPACITY, "arch: path too long");
   auto& seg_table = h.seg_table;
   seg_table.assign((size_t)A->S_max * 10, 0);
@@ -522,7 +552,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   ctx->arch_ok = false;
   const int64_t AL = ctx->cfg.align;
   ArchHost h;
-  dyo_status pst = parse_arch(A, AL, h, ctx->err);
+  dyo_status pst = parse_arch(A, AL, ctx->cfg.max_batch, h, ctx->err);
   if (pst) return pst;
   const int T = h.T, n_ops = A->n_ops, n_sites = h.n_sites;
   ctx->T = T;
@@ -551,7 +581,8 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   dyo_status st;
 #define UP(field, vec) if ((st = dupload(ctx, own, &ad.field, vec))) return st
   UP(t_bytes, ctx->t_bytes); UP(t_abytes, ctx->t_abytes); UP(t_host, ctx->t_host); UP(t_flags, ctx->t_flags);
-  UP(op_sig, sig); UP(acc_ptr, acc_ptr); UP(acc_t, acc_t); UP(acc_m, acc_m);
+  UP(op_sig, sig); UP(acc_ptr, acc_ptr); UP(acc_t, acc_t); UP(acc_m, acc_m); UP(acc_s, h.acc_s); UP(acc_sb, h.acc_sb);
+  UP(site_rev, h.site_rev);
   UP(site_kind, site_kind); UP(site_nch, site_nch); UP(site_lo, site_lo); UP(site_tie, site_tie);
   UP(site_logit, site_logit); UP(site_arm_ptr, site_arm_ptr); UP(arm_first_op, arm_first); UP(arm_nops, arm_n);
   UP(piece_kind, piece_kind); UP(piece_a, piece_a); UP(piece_b, piece_b); UP(piece_c, piece_c);
@@ -595,7 +626,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
     CK(cudaMemset(ps.loc, 0xff, T));   // -1: every tensor starts on the host
   }
   ctx->committed = 0;
-  int64_t cap_ent = ctx->cfg.max_entries > 0 ? ctx->cfg.max_entries : (int64_t)mg * 256;
+  int64_t cap_ent = ctx->cfg.max_entries > 0 ? ctx->cfg.max_entries : (int64_t)mg * 512;
   int64_t cap_rec = ctx->cfg.max_records > 0 ? ctx->cfg.max_records : 4 * ((int64_t)T + cap_ent);
   PlanScratch& sc = ctx->sc;
   DA(sc.inw, T); DA(sc.cur_next, T); DA(sc.cur_rd, T); DA(sc.nxt, cap_ent); DA(sc.nxt_rd, cap_ent);
@@ -666,7 +697,7 @@ dyo_status dyo_traverse_check(const dyo_arch* A, const int32_t* slots, int32_t* 
   if (!A || !slots || !choices || !matched) return DYO_E_INVAL;
   ArchHost h;
   std::string e;
-  dyo_status st = parse_arch(A, 256, h, e);
+  dyo_status st = parse_arch(A, 256, 1, h, e);
   if (!st) {
     TravArch t{h.sig, h.site_kind, h.site_nch, h.site_lo, h.site_tie, h.site_arm_ptr, h.arm_first, h.arm_n,
                h.piece_kind, h.piece_a, h.piece_b, h.piece_c};
@@ -683,7 +714,7 @@ dyo_status dyo_arch_check(const dyo_arch* A, int32_t align, dyo_arch_summary* ou
   if (!A || align < 16 || (align & (align - 1))) return DYO_E_INVAL;
   ArchHost h;
   std::string e;
-  dyo_status st = parse_arch(A, align, h, e);
+  dyo_status st = parse_arch(A, align, 1, h, e);
   if (err && errlen > 0) { strncpy(err, e.c_str(), errlen - 1); err[errlen - 1] = 0; }
   if (st) return st;
   if (out) {

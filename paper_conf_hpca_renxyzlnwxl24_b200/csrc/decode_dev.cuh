@@ -59,6 +59,7 @@ __device__ __forceinline__ ArchDev stage_decode_tables(const ArchDev& a, int* bu
   s.site_tie = take(a.site_tie, a.n_sites);
   s.site_lo = take(a.site_lo, a.n_sites);
   s.site_arm_ptr = take(a.site_arm_ptr, a.n_sites);
+  s.site_rev = take(a.site_rev, a.n_sites);
   s.piece_kind = take(a.piece_kind, a.n_pieces);
   s.piece_a = take(a.piece_a, a.n_pieces);
   s.piece_b = take(a.piece_b, a.n_pieces);
@@ -168,7 +169,9 @@ __device__ __forceinline__ int group_end(const DecHead& H, int g) {
   return min(H.cum[g] + H.cntc[g], H.L);
 }
 
-__device__ __forceinline__ int row_op(const ArchDev& a, const DecHead& H, int r) {
+// Operator of path row r (-1 for a control row); *it = iteration index of its loop for the
+// per-iteration tensors (R13; 0 outside loops, counted down in a reversed loop).
+__device__ __forceinline__ int row_op(const ArchDev& a, const DecHead& H, int r, int* it = nullptr) {
   int lo = 0, hi = a.n_pieces - 1;
   while (lo < hi) {
     const int mid = (lo + hi + 1) >> 1;
@@ -183,6 +186,11 @@ __device__ __forceinline__ int row_op(const ArchDev& a, const DecHead& H, int r)
   }
   const int c = a.piece_c[p];
   const int w = q % (1 + c);
+  if (it) {
+    const int s = a.piece_a[p];
+    const int i = q / (1 + c);
+    *it = a.site_rev[s] ? (a.site_lo[s] + H.choice[s] - 1 - i) : i;
+  }
   return w == 0 ? -1 : a.piece_b[p] + w - 1;
 }
 
@@ -240,10 +248,13 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
   }
   const int n = total;
   for (int r = rs; r < re; ++r) {
-    const int op = row_op(a, H, r);
+    int it = 0;
+    const int op = row_op(a, H, r, &it);
     if (op < 0) continue;
-    for (int q = a.acc_ptr[op]; q < a.acc_ptr[op + 1]; ++q, ++pos)
-      G.key[pos] = ((uint64_t)a.acc_t[q] << 32) | ((uint64_t)pos << 2) | (uint64_t)a.acc_m[q];
+    for (int q = a.acc_ptr[op]; q < a.acc_ptr[op + 1]; ++q, ++pos) {
+      const uint32_t t = (uint32_t)(a.acc_t[q] + a.acc_s[q] * it + a.acc_sb[q] * b);   // R13 (validated at load)
+      G.key[pos] = ((uint64_t)t << 32) | ((uint64_t)pos << 2) | (uint64_t)a.acc_m[q];
+    }
   }
   __syncthreads();
   if (n <= 64) {

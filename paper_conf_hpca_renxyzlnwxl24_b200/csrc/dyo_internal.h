@@ -57,6 +57,8 @@ struct ArchDev {
   const int32_t* acc_ptr;    // n_ops + 1
   const int32_t* acc_t;
   const int32_t* acc_m;
+  const int32_t* acc_s;      // stride per access (R13): tensor = acc_t + acc_s * iteration
+  const int32_t* acc_sb;     //   + acc_sb * (prediction index in the batch)
   // sites (preorder IF/LOOP)
   const int32_t* site_kind;  // 1 IF, 2 LOOP
   const int32_t* site_nch;   // choices
@@ -64,6 +66,7 @@ struct ArchDev {
   const int32_t* site_tie;
   const int32_t* site_logit; // logit offset (absolute in the O vector) or -1 (tied)
   const int32_t* site_arm_ptr;   // IF: site -> first arm index; arms give (first op, n ops)
+  const int32_t* site_rev;   // LOOP: 1 = iteration index counts down (R13)
   const int32_t* arm_first_op;
   const int32_t* arm_nops;
   // top-level pieces: kind 0 static run (a = first op, b = n ops), 1 IF (a = site),

@@ -34,7 +34,8 @@ class Arch(C.Structure):
                 ("node_b", PI32), ("node_span", PI32), ("node_tie", PI32), ("n_ops", i32),
                 ("op_idioms", PI32), ("op_in_ptr", PI32), ("in_dim_ptr", PI32), ("in_dims", PI64),
                 ("op_acc_ptr", PI32), ("acc_tensor", PI32), ("acc_mode", PI32), ("n_tensors", i32),
-                ("t_bytes", PI64), ("t_host_off", PI64), ("t_flags", PI32)]
+                ("t_bytes", PI64), ("t_host_off", PI64), ("t_flags", PI32),
+                ("acc_stride", PI32), ("node_flags", PI32), ("acc_bstride", PI32)]
 
 
 class PilotDesc(C.Structure):
@@ -118,7 +119,7 @@ def _p(arr, ct):
 
 def flatten_program(program):
     """Preorder node arrays + operator CSR of the program (marshalling into dyo_arch)."""
-    kind, na, nb, span, tie = [], [], [], [], []
+    kind, na, nb, span, tie, flags = [], [], [], [], [], []
     ops = []
 
     def rec(items):
@@ -137,26 +138,33 @@ def flatten_program(program):
                 span[idx] = len(kind) - idx - 1
             elif isinstance(it, Loop):
                 kind.append(2); na.append(it.lo); nb.append(it.hi); span.append(0); tie.append(it.tie)
+                flags.append((idx, 1 if it.rev else 0))
                 rec(it.body)
                 span[idx] = len(kind) - idx - 1
             else:
                 raise TypeError(it)
     rec(program)
-    idioms, in_ptr, dim_ptr, dims, acc_ptr, acc_t, acc_m = [], [0], [0], [], [0], [], []
+    nflags = [0] * len(kind)
+    for i, f in flags:
+        nflags[i] = f
+    idioms, in_ptr, dim_ptr, dims, acc_ptr, acc_t, acc_m, acc_s, acc_sb = [], [0], [0], [], [0], [], [], [], []
     for op in ops:
         idioms.extend(op.idioms)
         for shp in op.inputs:
             dims.extend(shp)
             dim_ptr.append(len(dims))
         in_ptr.append(len(dim_ptr) - 1)
-        for t, m in op.acc:
-            acc_t.append(t)
-            acc_m.append(m)
+        for a in op.acc:
+            acc_t.append(a[0])
+            acc_m.append(a[1])
+            acc_s.append(a[2] if len(a) > 2 else 0)
+            acc_sb.append(a[3] if len(a) > 3 else 0)
         acc_ptr.append(len(acc_t))
     return dict(kind=_a(kind, np.int32), a=_a(na, np.int32), b=_a(nb, np.int32), span=_a(span, np.int32),
                 tie=_a(tie, np.int32), n_ops=len(ops), idioms=_a(idioms, np.int32), in_ptr=_a(in_ptr, np.int32),
                 dim_ptr=_a(dim_ptr, np.int32), dims=_a(dims, np.int64), acc_ptr=_a(acc_ptr, np.int32),
-                acc_t=_a(acc_t, np.int32), acc_m=_a(acc_m, np.int32))
+                acc_t=_a(acc_t, np.int32), acc_m=_a(acc_m, np.int32), acc_s=_a(acc_s, np.int32), acc_sb=_a(acc_sb, np.int32),
+                flags=_a(nflags, np.int32))
 
 
 def _arch_struct(wl, branch_head=None):
@@ -169,7 +177,8 @@ def _arch_struct(wl, branch_head=None):
                 _p(fp["kind"], i32), _p(fp["a"], i32), _p(fp["b"], i32), _p(fp["span"], i32),
                 _p(fp["tie"], i32), fp["n_ops"], _p(fp["idioms"], i32), _p(fp["in_ptr"], i32),
                 _p(fp["dim_ptr"], i32), _p(fp["dims"], i64), _p(fp["acc_ptr"], i32), _p(fp["acc_t"], i32),
-                _p(fp["acc_m"], i32), len(wl.tensors), _p(tb, i64), _p(th, i64), _p(tf, i32))
+                _p(fp["acc_m"], i32), len(wl.tensors), _p(tb, i64), _p(th, i64), _p(tf, i32),
+                _p(fp["acc_s"], i32), _p(fp["flags"], i32), _p(fp["acc_sb"], i32))
     return arch, (fp, tb, th, tf)
 
 

@@ -19,12 +19,12 @@ def make_ctx(wl, max_batch=1, flags=0, policy=None, **kw):
 def oracle_step(wl, sample_ids, state, table, policy=None):
     """Oracle for a batch of samples planned together (sample order)."""
     preds, feats, logits = [], [], []
-    for s in sample_ids:
+    for b, s in enumerate(sample_ids):
         x = E.encode(wl, wl.samples[s], wl.hist_ids, table)
         y = P.forward(wl.pilot, x, wl.nn_type)
         feats.append(x)
         logits.append(y)
-        preds.append(D.decode(wl, y, branch_head=wl.notes.get("branch_head", True)))
+        preds.append(D.decode(wl, y, branch_head=wl.notes.get("branch_head", True), b=b))
     Ws = [Wj for p in preds for Wj in p.W]
     new_table = [b for p in preds for b in p.blocks]
     try:

@@ -28,7 +28,7 @@ def test_exports_match_header(dyo):
     assert declared == set(dyo.EXPORTS)
 
 
-@pytest.mark.parametrize("name", ["tiny", "moe", "af"])
+@pytest.mark.parametrize("name", ["tiny", "moe", "af", "lstm"])
 def test_arch_parse_matches_oracle(dyo, name):
     wl = WL.make(name)
     st, summ, seg, sig, err = dyo.arch_check(wl)
@@ -65,3 +65,22 @@ def test_arch_validation_errors(dyo):
     assert st == -7
     st, summ, *_ = dyo.arch_check(WL.make("tiny"), branch_head=False)   # traversal decode: no branch head
     assert st == 0 and summ["n_branch_logits"] == 0
+
+
+def test_strided_access_validation(dyo):
+    """R13: strides only inside loops; named ids stay in [0, T) and ascending at every k."""
+    from workloads import R, W
+    T = 8
+    ts = [WL.Tensor(256, 256 * i, False) for i in range(T)]
+
+    def wl_of(prog):
+        return WL.Workload("s", WL.LSTM, prog, ts, 1, 1, 0, 2, 1 << 30, 256, 1, None,
+                           np.zeros((1, 1), np.int64), np.zeros(0, np.int32), 0)
+    ok = [WL.Loop([WL.Op((0,) * 6, (), ((0, R), (1, W, 1)))], 1, 7)]     # ids 1..7 at k <= 6
+    assert dyo.arch_check(wl_of(ok))[0] == 0
+    too_far = [WL.Loop([WL.Op((0,) * 6, (), ((0, R), (1, W, 1)))], 1, 8)]
+    assert dyo.arch_check(wl_of(too_far))[0] == -1
+    crossing = [WL.Loop([WL.Op((0,) * 6, (), ((0, R, 2), (3, W)))], 1, 4)]   # 0,2,4 passes 3
+    assert dyo.arch_check(wl_of(crossing))[0] == -1
+    outside = [WL.Op((0,) * 6, (), ((0, R, 1),))]
+    assert dyo.arch_check(wl_of(outside))[0] == -1

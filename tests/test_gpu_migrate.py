@@ -38,10 +38,10 @@ def _check_dev(arena, dst, t, v, nb):
     return bool(torch.equal(got, _words(t, v, nb)))
 
 
-def run_bytes(wl, steps, policy=None, flags=0, dma_min=0, staging=0):
+def run_bytes(wl, steps, policy=None, flags=0, dma_min=0, staging=0, B=1):
     for t in wl.tensors:
         assert t.nbytes % 4 == 0
-    d = make_ctx(wl, flags=flags, policy=policy, dma_min_bytes=dma_min, staging_bytes=staging)
+    d = make_ctx(wl, flags=flags, policy=policy, dma_min_bytes=dma_min, staging_bytes=staging, max_batch=B)
     pool = d.host_pool_array()
     for t, ten in enumerate(wl.tensors):
         pool[ten.host_off: ten.host_off + ten.nbytes] = M.content_bytes(t, 0, ten.nbytes)
@@ -52,9 +52,10 @@ def run_bytes(wl, steps, policy=None, flags=0, dma_min=0, staging=0):
     ver = [0] * len(wl.tensors)
     mech = {"dma": 0, "zc": 0, "packed": 0}
     for s in range(steps):
-        r = oracle_step(wl, [s % len(wl.samples)], st, table, policy)
+        ids = [(s * B + i) % len(wl.samples) for i in range(B)]
+        r = oracle_step(wl, ids, st, table, policy)
         assert r["err"] is None
-        d.predict(wl.samples[[s % len(wl.samples)]].copy(), hist_for(wl, 1), 1, stream=stream.cuda_stream)
+        d.predict(wl.samples[ids].copy(), hist_for(wl, B), B, stream=stream.cuda_stream)
         K = d.plan(stream=stream.cuda_stream)
         assert K == len(r["trs"])
         fresh = set()
@@ -128,6 +129,14 @@ def test_af_scaled_recycling():
         t.host_off = off
         off += (t.nbytes + 255) // 256 * 256
     run_bytes(wl, 3, 1)
+
+
+def test_lstm_scaled_small_tensors_zero_copy():
+    """Many 2-4 KiB per-timestep / per-sample tensors (R13): fetched and carried by the
+    zero-copy and vector-copy kernels; a batch of 4 predictions per plan."""
+    wl = WL.make_lstm(n_samples=16, batch=4, max_len=64, hidden=128, budget=4 << 20)
+    m = run_bytes(wl, 2, 1, B=4)
+    assert m["zc"] > 0
 
 
 def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0, lookahead=False):

@@ -41,7 +41,8 @@ def test_encode_bitexact(name):
     d.close()
 
 
-@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 16), ("moe", 1), ("moe", 8), ("af", 1), ("af", 3)])
+@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 16), ("moe", 1), ("moe", 8), ("af", 1), ("af", 3),
+                                    ("lstm", 8), ("lstm", 64)])
 def test_pilot_logits(name, B):
     wl = WL.make(name, n_samples=max(16, B))
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
@@ -69,7 +70,7 @@ def _check_prediction(d, wl, b, pred):
         assert [tuple(e) for e in ent.tolist()] == [(t, m, int(f)) for t, m, f in pred.W[g]], f"group {g}"
 
 
-@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 8), ("moe", 1), ("moe", 4), ("af", 2)])
+@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 8), ("moe", 1), ("moe", 4), ("af", 2), ("lstm", 8)])
 def test_decode(name, B):
     wl = WL.make(name, n_samples=max(16, B))
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
@@ -202,3 +203,16 @@ def test_decode_traversal(B, planted):
 def test_plan_bitexact_traversal():
     wl = _planted_path_tiny([1, 1, 0])
     _run_plan_steps(wl, 4, 2, 1).close()
+
+
+@pytest.mark.parametrize("policy", [0, 1])
+def test_plan_bitexact_lstm_scaled(policy):
+    """Var-length LSTM (configs[3] variant): per-timestep / per-sample tensors (R13), reversed
+    backward loop, batch of 8 predictions planned as one sequence, two consecutive steps."""
+    wl = WL.make_lstm(n_samples=32, batch=8, max_len=96)
+    _run_plan_steps(wl, 2, 8, policy).close()
+
+
+def test_plan_bitexact_lstm_fullsize():
+    wl = WL.make_lstm(n_samples=16)
+    _run_plan_steps(wl, 1, 8, 1).close()

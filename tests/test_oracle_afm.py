@@ -69,3 +69,35 @@ def test_loop_rows_count():
         rows = A.resolve(prog, [idx])
         assert len(rows) == 4 * n + n + 1
         assert sum(r is None for r in rows) == n + 1
+
+
+def test_strided_accesses_forward_reverse_and_per_sample():
+    """Reading R13, written out by hand: an access (t, m, stride_k, stride_b) names tensor
+    t + stride_k * k + stride_b * b; a reversed loop counts k down from n - 1."""
+    from workloads import R, W
+    from oracle import decode as D
+    fwd = Op((0, 0, 0, 1, 1, 0), ((2,),), ((0, R), (10, R, 1, 100), (20, W, 1)), "f")
+    bwd = Op((0, 0, 0, 1, 1, 0), ((2,),), ((0, R), (20, R, 1)), "g")
+    prog = [Loop([fwd], 1, 4), Loop([bwd], 1, 4, tie=0, rev=True)]
+    rows = A.resolve(prog, [2], b=1)                     # trip 3, sample 1 of the batch
+    accs = [r.acc for r in rows if r is not None]
+    assert accs == [((0, R), (20, W), (110, R)),          # k = 0: x[1,0] = 10 + 100
+                    ((0, R), (21, W), (111, R)),
+                    ((0, R), (22, W), (112, R)),
+                    ((0, R), (22, R)),                    # reversed: k = 2, 1, 0
+                    ((0, R), (21, R)),
+                    ((0, R), (20, R))]
+    assert [r is None for r in rows] == [True, False] * 3 + [True] + [True, False] * 3 + [True]
+    # the same binding through path enumeration, and W_j in first-access order (R8)
+    for ch, rr in D.enumerate_paths(prog, b=1):
+        if ch == [2, 2]:
+            assert rr == rows
+    Ws = D.tensor_sets(rows, [(0, 4), (4, len(rows))])
+    assert Ws[0] == [(0, R, True), (20, W, False), (110, R, True), (21, W, False), (111, R, True)]
+    assert [t for t, _, _ in Ws[1]] == [0, 22, 112, 21, 20]      # ascending within an operator
+
+
+def test_strided_access_outside_loop_is_rejected():
+    from workloads import R
+    with pytest.raises(ValueError):
+        A.resolve([Op((0,) * 6, (), ((3, R, 1),))], [])

@@ -13,9 +13,13 @@ Program model (§IV-A2):
       idioms = counts of [transpose, gather, scatter, reduction, stream, stencil]
       (column order P:L135); acc sorted by tensor id, unique.
   If(branches=[program, ...], tie=-1)   one control-flow statement
-  Loop(body=program, lo, hi, tie=-1)    trip count in [lo, hi]
+  Loop(body=program, lo, hi, tie=-1, rev=False)    trip count in [lo, hi]
   tie >= 0 marks a site that replays the choice of an earlier site (the backward
   pass of a routed layer follows its forward choice) — DESIGN.md reading R6.
+  An access may carry a stride: (tensor_id, mode, stride) names tensor
+  tensor_id + stride * k, k = iteration index of the innermost enclosing Loop
+  (0..n-1; n-1..0 when the Loop has rev=True, a backward pass over a forward loop's
+  per-iteration tensors) — DESIGN.md reading R13. Outside loops the stride is 0.
 """
 from __future__ import annotations
 
@@ -48,6 +52,7 @@ class Loop:
     lo: int
     hi: int
     tie: int = -1
+    rev: bool = False
 
 
 @dataclass
@@ -474,7 +479,175 @@ def make_af(seed=0, n_samples=16, blocks=48, max_recycle=4, budget=2 * GiB,
                     notes={"blocks": blocks, "max_recycle": max_recycle})
 
 
-CONFIGS = {"tiny": make_tiny, "moe": make_moe, "af": make_af}
+# ----------------------------------------------------------------------------
+# M3 variable-length sequence LSTM (BASELINE configs[3])
+# ----------------------------------------------------------------------------
+
+def make_lstm(seed=0, n_samples=128, batch=64, max_len=512, min_len=16, hidden=512, tasks=4,
+              budget=48 * MiB, pilot_kind="P512", K_max=16):
+    """Variable-length 2-layer LSTM with a per-sample task head: the "variable-length sequence"
+    variant of configs[3] (many small per-timestep tensors, batch-64 pilot predictions, one plan
+    over the batch's group sequences concatenated in sample order).
+
+    Per sample (one training example; DyNN with per-sample structure):
+      embed op; Loop F (trip n = sequence length in [16, 512]) of two LSTM cells per timestep:
+        cell1 reads x[k], h1[k], c1[k], W1 and writes h1[k+1], c1[k+1], g1[k] (saved gates);
+        cell2 reads h1[k+1], h2[k], c2[k], W2 and writes h2[k+1], c2[k+1], g2[k]; pool RW;
+      If(task head, 4 arms: different op mixes and head weights Wh[a]) + loss;
+      If(tie = head) head backward (writes gWh[a]);
+      Loop B (tie = F, reversed: k = n-1..0) of two backward cells reading the saved
+        g*[k], h*[k], c*[k+1] and x[k], accumulating gW1 / gW2 (RW);
+      optimizer op (W1, W2, Wh RW with their gradients).
+    Per-iteration / per-sample tensors use strided accesses (reading R13): x[b, k] is row k of
+    minibatch sample b's input sequence (its own host home), h/c/g[k] are per-timestep
+    transients shared by the batch's samples (each sample's die with its backward pass).
+    Sizes: hidden 512 fp32 h/c/x = 2 KiB, bf16 gates 4 x 512 = 4 KiB, W1/W2 = 4 x 512 x 1024
+    bf16 = 4 MiB, Wh 1 MiB: 32,768 input rows + 3,079 per-timestep transients + 16
+    weight/gradient/state tensors (T = 35,863).
+    Budget 48 MiB (H = 24 MiB): a backward group holds W1, W2, gW1, gW2 (16 MiB) plus its
+    timesteps; saved activations of long sequences overflow and migrate in 2-4 KiB pieces.
+    """
+    rng = np.random.default_rng(seed)
+    tensors = []
+
+    def add(nb, transient, name):
+        tensors.append([nb, transient, name])
+        return len(tensors) - 1
+
+    hb, gb = hidden * 4, 4 * hidden * 2
+    W1 = add(4 * hidden * 2 * hidden * 2, False, "W1")
+    W2 = add(4 * hidden * 2 * hidden * 2, False, "W2")
+    gW1 = add(4 * hidden * 2 * hidden * 2, False, "gW1")
+    gW2 = add(4 * hidden * 2 * hidden * 2, False, "gW2")
+    Wh = [add(hidden * 2048, False, f"Wh[{a}]") for a in range(tasks)]
+    gWh = [add(hidden * 2048, False, f"gWh[{a}]") for a in range(tasks)]
+    pool = add(hb, True, "pool")
+    dpool = add(hb, True, "dpool")
+    dh = add(2 * hb, True, "dh_dc")
+    loss = add(256, True, "loss")
+    x0 = len(tensors)
+    for b in range(batch):
+        for k in range(max_len):
+            add(hb, False, f"x[{b},{k}]")
+    h1 = len(tensors)
+    for k in range(max_len + 1):
+        add(hb, True, f"h1[{k}]")
+    c1 = len(tensors)
+    for k in range(max_len + 1):
+        add(hb, True, f"c1[{k}]")
+    g1 = len(tensors)
+    for k in range(max_len):
+        add(gb, True, f"g1[{k}]")
+    h2 = len(tensors)
+    for k in range(max_len + 1):
+        add(hb, True, f"h2[{k}]")
+    c2 = len(tensors)
+    for k in range(max_len + 1):
+        add(hb, True, f"c2[{k}]")
+    g2 = len(tensors)
+    for k in range(max_len):
+        add(gb, True, f"g2[{k}]")
+
+    Hd = hidden
+    cell = (0, 0, 0, 2, 6, 0)          # 2 matmul reductions, gate elementwise streams
+    cell_bwd = (1, 0, 0, 3, 8, 0)
+
+    def acc(*a):
+        return tuple(sorted(a, key=lambda e: e[0]))
+
+    fwd_body = [
+        Op(cell, ((1, Hd), (Hd, 4 * Hd), (1, Hd)),
+           acc((W1, R, 0), (x0, R, 1, max_len), (h1, R, 1), (c1, R, 1), (h1 + 1, W, 1), (c1 + 1, W, 1), (g1, W, 1)), "cell1"),
+        Op(cell, ((1, Hd), (Hd, 4 * Hd), (1, Hd), (1, Hd)),
+           acc((W2, R, 0), (pool, RW, 0), (h1 + 1, R, 1), (h2, R, 1), (c2, R, 1), (h2 + 1, W, 1), (c2 + 1, W, 1),
+               (g2, W, 1)), "cell2"),
+    ]
+    bwd_body = [
+        Op(cell_bwd, ((1, Hd), (4 * Hd, Hd), (1, 4 * Hd)),
+           acc((W2, R, 0), (gW2, RW, 0), (dh, RW, 0), (g2, R, 1), (h2, R, 1), (c2 + 1, R, 1), (h1 + 1, R, 1)),
+           "cell2_bwd"),
+        Op(cell_bwd, ((1, Hd), (4 * Hd, Hd), (1, 4 * Hd), (1, Hd)),
+           acc((W1, R, 0), (gW1, RW, 0), (dh, RW, 0), (g1, R, 1), (h1, R, 1), (c1 + 1, R, 1), (x0, R, 1, max_len)),
+           "cell1_bwd"),
+    ]
+    head_arms, head_bwd_arms = [], []
+    for a in range(tasks):
+        na = 1 + a % 3
+        head_arms.append([Op((a % 2, 0, a % 2, 1, 1 + a, 0), ((1, Hd), (Hd, 256 * (a + 1))),
+                             acc((Wh[a], R, 0), (pool, R, 0)) if i == 0 else acc((loss, W if i == na - 1 else RW, 0)),
+                             f"head{a}.{i}") for i in range(na)])
+        head_bwd_arms.append([Op((1, 0, a % 2, 1, 2 + a, 0), ((1, Hd), (256 * (a + 1), Hd)),
+                                 acc((Wh[a], R, 0), (gWh[a], W, 0), (dpool, W, 0), (loss, R, 0)), f"head_bwd{a}")])
+    program = [Op((0, 1, 0, 0, 1, 0), ((max_len, Hd),), (), "embed"),
+               Loop(fwd_body, min_len, max_len),
+               If(head_arms),
+               If(head_bwd_arms, tie=1),
+               Op((0, 0, 0, 1, 1, 0), ((1, Hd),), acc((dpool, R, 0), (dh, W, 0)), "pool_bwd"),
+               Loop(bwd_body, min_len, max_len, tie=0, rev=True),
+               Op((0, 0, 0, 0, 3, 0), ((4 * Hd, 2 * Hd),) * 2,
+                  acc((W1, RW, 0), (W2, RW, 0), (gW1, RW, 0), (gW2, RW, 0)), "optimizer")]
+    sizes = [t[0] for t in tensors]
+    offs, _ = _host_layout(sizes, 256)
+    tens = [Tensor(t[0], offs[i], t[1], t[2]) for i, t in enumerate(tensors)]
+    S_max, D_s, h = 16, 16, 2
+    lens = rng.integers(min_len, max_len + 1, size=n_samples)
+    task = rng.integers(0, tasks, size=n_samples)
+    samples = np.stack([lens, task] + [rng.integers(1, 4096, size=n_samples) for _ in range(D_s - 2)],
+                       axis=1).astype(np.int64)
+    nbl = n_branch_logits(program)
+    pilot = make_pilot(rng, pilot_kind, S_max, D_s, h, K_max, nbl, planted_counts=None,
+                       xs_mean=[(min_len + max_len) / 2, (tasks - 1) / 2] + [2048.0] * (D_s - 2))
+    _plant_lstm_heads(pilot, K_max, min_len, max_len, tasks,
+                      rows_per_step=2 + len(fwd_body) + len(bwd_body),
+                      rows_const=1 + 2 + 3 + 2 + 1 + 1)
+    return Workload("lstm", LSTM, program, tens, S_max, D_s, h, K_max,
+                    budget=budget, align=256, policy=1, pilot=pilot, samples=samples,
+                    hist_ids=np.array([-2, -1], np.int32), seed=seed,
+                    notes={"batch": batch, "max_len": max_len, "tasks": tasks})
+
+
+def _plant_lstm_heads(pilot, K_max, min_len, max_len, tasks, rows_per_step, rows_const):
+    """Stand-in for a trained pilot on the var-LSTM trace: two pass-through units
+    carry the descriptors n = x_s[0] and task = x_s[1] (in feature units, desc x 2^-10, R3)
+    unchanged through every layer (weight 1 on the previous unit, bias 0; LeakyReLU is the
+    identity on positive inputs), and the heads read only them, with power-of-two-exact weights:
+      trip-count logits  l_t = (2 t n - t^2) / 2048       -> argmax t = n (gap 1/2048),
+      task logits        l_a = (2 a task - a^2) / 8       -> argmax a = task (gap 1/8),
+      block counts       16 y_k = (rows_const + rows_per_step n) / K_max + 1/32 for every slot,
+    so the groups scale with the sequence (the cut's last group absorbs the rounding rest) and
+    no rint lands on a half. Every other weight stays seeded-random (the layers remain dense)."""
+    w = pilot.weights
+    f0 = w["feat0.W"]
+    f0[0, :] = 0.0; f0[1, :] = 0.0
+    f0[0, 0] = 1.0; f0[1, 1] = 1.0
+    w["feat0.b"][:2] = 0.0
+    for k in range(3):
+        for l in range(len(pilot.mlp)):
+            Wl = w[f"mlp{k}.{l}.W"]
+            Wl[0, :] = 0.0; Wl[1, :] = 0.0
+            Wl[0, 0] = 1.0; Wl[1, 1] = 1.0
+            w[f"mlp{k}.{l}.b"][:2] = 0.0
+    Wo, bo = w["out.W"], w["out.b"]
+    Wo[: 10 * K_max, :] = 0.0
+    bo[: 10 * K_max] = 0.0
+    for k in range(K_max):
+        # 16 y = 1024 * Wo * (n / 1024) + 16 b  ->  Wo = rows_per_step / (16 K_max) * 1024 / 1024
+        Wo[10 * k, 0] = np.float32(rows_per_step / (16.0 * K_max) * 1024.0)
+        bo[10 * k] = np.float32((rows_const / K_max + 1.0 / 32.0) / 16.0)
+    off = 10 * K_max
+    for t in range(min_len, max_len + 1):          # Loop F trip-count logits
+        Wo[off, :] = 0.0
+        Wo[off, 0] = np.float32(t)
+        bo[off] = np.float32(-t * t / 2048.0)
+        off += 1
+    for a in range(tasks):                          # task-head logits
+        Wo[off, :] = 0.0
+        Wo[off, 1] = np.float32(2 * a * 1024 / 8.0)
+        bo[off] = np.float32(-a * a / 8.0)
+        off += 1
+
+
+CONFIGS = {"tiny": make_tiny, "moe": make_moe, "af": make_af, "lstm": make_lstm}
 
 
 def make(name, seed=0, **kw):

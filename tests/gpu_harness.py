@@ -16,8 +16,9 @@ def make_ctx(wl, max_batch=1, flags=0, policy=None, **kw):
     return d
 
 
-def oracle_step(wl, sample_ids, state, table, policy=None):
-    """Oracle for a batch of samples planned together (sample order)."""
+def oracle_step(wl, sample_ids, state, table, policy=None, plan=True):
+    """Oracle for a batch of samples planned together (sample order); plan=False stops after
+    the decode."""
     preds, feats, logits = [], [], []
     for b, s in enumerate(sample_ids):
         x = E.encode(wl, wl.samples[s], wl.hist_ids, table)
@@ -27,6 +28,8 @@ def oracle_step(wl, sample_ids, state, table, policy=None):
         preds.append(D.decode(wl, y, branch_head=wl.notes.get("branch_head", True), b=b))
     Ws = [Wj for p in preds for Wj in p.W]
     new_table = [b for p in preds for b in p.blocks]
+    if not plan:
+        return dict(feats=feats, logits=logits, preds=preds, trs=[], state=state, table=new_table, err=None)
     try:
         trs, st = PL.plan(state, wl, Ws, policy)
         err = None

@@ -48,7 +48,7 @@ def test_pilot_logits(name, B):
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
     logits = torch.zeros((B, wl.pilot.O), device="cuda")
     d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, stream=_stream())
-    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), ())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), (), plan=False)
     y = logits.cpu().numpy()
     n1 = 0
     for b in range(B):
@@ -75,7 +75,7 @@ def test_decode(name, B):
     wl = WL.make(name, n_samples=max(16, B))
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
     d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, stream=_stream())
-    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), ())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), (), plan=False)
     for b in range(B):
         assert not r["preds"][b].near_ties
         _check_prediction(d, wl, b, r["preds"][b])

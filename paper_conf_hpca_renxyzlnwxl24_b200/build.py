@@ -9,7 +9,7 @@ OUT = os.path.join(HERE, "libdyo.so")
 BUILD = os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-CU = ["pilot.cu", "decode.cu", "plan.cu", "copy.cu"]
+CU = ["pilot.cu", "pilot_tc.cu", "decode.cu", "plan.cu", "copy.cu"]
 CPP = ["api.cpp", "traverse.cpp"]
 
 
@@ -23,7 +23,7 @@ def _run(cmd):
 
 def build(force=False, verbose=False):
     os.makedirs(BUILD, exist_ok=True)
-    srcs = [os.path.join(CSRC, f) for f in CU + CPP] + [os.path.join(CSRC, "dyo_internal.h"), os.path.join(CSRC, "decode_dev.cuh"),
+    srcs = [os.path.join(CSRC, f) for f in CU + CPP] + [os.path.join(CSRC, "dyo_internal.h"), os.path.join(CSRC, "decode_dev.cuh"), os.path.join(CSRC, "pilot_common.cuh"),
                                                        os.path.join(HERE, "..", "include", "dyo.h")]
     if not force and os.path.exists(OUT) and all(os.path.getmtime(OUT) >= os.path.getmtime(s) for s in srcs):
         return OUT

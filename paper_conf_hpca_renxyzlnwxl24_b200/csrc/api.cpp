@@ -50,6 +50,9 @@ struct dyo_ctx {
   int32_t* h_forced[2] = {nullptr, nullptr};   // pinned, max_batch x n_sites (alternating)
   int32_t* d_forced = nullptr;
   int32_t* h_matched = nullptr;    // per prediction of the last traversal: 1 exact match
+  // K1-TC (tensor-core batch pilot): device plan, or null when the pilot's shape does not fit it
+  const TcPlan* tc_dev = nullptr;
+  int tc_flag_off = 0;             // DYO_PILOT_TC=0 in the environment disables it (measurement)
   int64_t* desc_dev = nullptr;
   int32_t* hist_dev = nullptr;
   int32_t* hist_tab[2] = {nullptr, nullptr};
@@ -730,6 +733,120 @@ dyo_status dyo_arch_check(const dyo_arch* A, int32_t align, dyo_arch_summary* ou
   return DYO_OK;
 }
 
+// cvt.rna.tf32.f32 on the host: round to nearest (ties away) to 10 mantissa bits
+static float tf32_rna_host(float x) {
+  uint32_t u;
+  memcpy(&u, &x, 4);
+  if ((u & 0x7f800000u) == 0x7f800000u) return x;
+  u = (u + 0x1000u) & ~0x1fffu;
+  float y;
+  memcpy(&y, &u, 4);
+  return y;
+}
+
+// K1-TC plan (pilot_tc.cu): stages = the selected MLP's layers + the output layer; stage s has
+// n_m = ceil(out/128) tiles and its K split n_ks ways (n_m * n_ks <= 16 CTAs; K-slices multiple
+// of 8 and <= 128); weights pre-split into TF32 hi/lo and laid out per (CTA, chunk) in the UMMA
+// K-major no-swizzle core-matrix layout ([k/4][row/8][row%8][k%4]) so one cp.async.bulk moves a
+// chunk. Only for the P-type topology (three feature layers); otherwise tc_dev stays null.
+static dyo_status build_tc_plan(dyo_ctx* ctx, const dyo_pilot_desc* w) {
+  if (const char* e = getenv("DYO_PILOT_TC")) ctx->tc_flag_off = (e[0] == '0');
+  if (w->n_feature != 3 || ctx->F > 256 || ctx->cfg.max_batch < kTcMinBatch) return DYO_OK;
+  const int k = ctx->ad.nn_type;
+  int n_feat = 0;
+  for (int i = 0; i < 3; ++i) n_feat += w->feat_out[i];
+  struct L { const float* W; const float* b; int out, in, act; };
+  std::vector<L> layers;
+  for (int l = 0; l < w->n_mlp; ++l)
+    layers.push_back({w->mlp_W[k * w->n_mlp + l], w->mlp_b[k * w->n_mlp + l], w->mlp_out[l], w->mlp_in[l], 1});
+  layers.push_back({w->out_W, w->out_b, w->O, w->out_in, 0});
+  if ((int)layers.size() > kTcMaxStages || layers[0].in != n_feat) return DYO_OK;
+  TcPlan P{};
+  P.n_stages = (int)layers.size();
+  P.n_feat = n_feat;
+  std::vector<std::vector<TcChunk>> per(kTcCtas);
+  std::vector<float> blob;
+  for (int s = 0; s < P.n_stages; ++s) {
+    const L& ly = layers[s];
+    TcStage& S = P.st[s];
+    S.n_out = ly.out; S.K = ly.in; S.act = ly.act;
+    S.n_m = (ly.out + 127) / 128;
+    if (ly.in % 8) return DYO_OK;
+    if (S.n_m > kTcCtas) {
+      if (s != P.n_stages - 1 || S.n_m > 2 * kTcCtas || ly.in > kTcMaxKsl) return DYO_OK;
+      S.n_ks = 1;
+    } else {
+      S.n_ks = 0;
+      for (int p = 16; p >= 1; p >>= 1)
+        if (S.n_m * p <= kTcCtas && ly.in % (8 * p) == 0 && ly.in / p <= kTcMaxKsl) { S.n_ks = p; break; }
+      if (!S.n_ks) return DYO_OK;
+    }
+    S.ksl = ly.in / S.n_ks;
+    std::vector<float> bias(ly.b, ly.b + ly.out);
+    const float* db = nullptr;
+    dyo_status st = dupload(ctx, ctx->pilot_dev, &db, bias);
+    if (st) return st;
+    S.bias = db;
+    // jobs of every CTA (same rule as jobs_of() in the kernel), chunked along K
+    for (int r = 0; r < kTcCtas; ++r) {
+      std::vector<std::pair<int, int>> jobs;   // (m, ks)
+      if (S.n_m * S.n_ks <= kTcCtas) {
+        if (r < S.n_m * S.n_ks) jobs.push_back({r / S.n_ks, r % S.n_ks});
+      } else {
+        for (int m = r; m < S.n_m && (int)jobs.size() < 2; m += kTcCtas) jobs.push_back({m, 0});
+      }
+      for (size_t jj = 0; jj < jobs.size(); ++jj) {
+        const int m = jobs[jj].first, ks = jobs[jj].second;
+        for (int k0 = 0; k0 < S.ksl; k0 += kTcMaxKc) {
+          const int kc = std::min(kTcMaxKc, S.ksl - k0);
+          TcChunk ch{};
+          ch.off = (int64_t)blob.size();
+          ch.bytes = 128 * kc * 8;
+          ch.stage = s; ch.job = (int)jj; ch.k0 = k0; ch.kc = kc;
+          blob.resize(blob.size() + (size_t)128 * kc * 2, 0.f);
+          float* hi = blob.data() + ch.off;
+          float* lo = hi + 128 * kc;
+          for (int row = 0; row < 128; ++row) {
+            const int R = m * 128 + row;
+            if (R >= ly.out) continue;
+            for (int kk = 0; kk < kc; ++kk) {
+              const int K = ks * S.ksl + k0 + kk;
+              const float v = ly.W[(size_t)R * ly.in + K];
+              if (!std::isfinite(v)) return DYO_E_INVAL;
+              const float h = tf32_rna_host(v);
+              const float l = tf32_rna_host(v - h);
+              const size_t o = (size_t)(kk >> 2) * (16 * 32) + (size_t)(row >> 3) * 32 + (size_t)(row & 7) * 4 + (kk & 3);
+              hi[o] = h;
+              lo[o] = l;
+            }
+          }
+          per[r].push_back(ch);
+        }
+      }
+    }
+  }
+  std::vector<TcChunk> all;
+  for (int r = 0; r < kTcCtas; ++r) {
+    P.chunk_ptr[r] = (int)all.size();
+    all.insert(all.end(), per[r].begin(), per[r].end());
+  }
+  P.chunk_ptr[kTcCtas] = (int)all.size();
+  const float* dblob = nullptr;
+  const TcChunk* dch = nullptr;
+  dyo_status st = dupload(ctx, ctx->pilot_dev, &dblob, blob);
+  if (st) return st;
+  st = dupload(ctx, ctx->pilot_dev, &dch, all);
+  if (st) return st;
+  P.blob = dblob;
+  P.chunks = dch;
+  std::vector<TcPlan> one(1, P);
+  const TcPlan* dp = nullptr;
+  st = dupload(ctx, ctx->pilot_dev, &dp, one);
+  if (st) return st;
+  ctx->tc_dev = dp;
+  return DYO_OK;
+}
+
 dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   if (!ctx || !w) return DYO_E_INVAL;
   if (!ctx->arch_ok) return fail(ctx, DYO_E_STATE, "load the arch first");
@@ -816,6 +933,8 @@ dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   double* lg = nullptr;
   if ((s = dalloc(ctx, ctx->pilot_dev, &lg, (size_t)ctx->cfg.max_batch * w->O))) return s;
   ctx->logits64 = lg;
+  ctx->tc_dev = nullptr;
+  if ((s = build_tc_plan(ctx, w))) return s;
   if (ctx->h_logits) { cudaFreeHost(ctx->h_logits); ctx->h_logits = nullptr; }
   if (!ctx->branch_head)
     CK(cudaHostAlloc((void**)&ctx->h_logits, sizeof(double) * ctx->cfg.max_batch * w->O, cudaHostAllocPortable));
@@ -896,8 +1015,16 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
   int fused = 0;
   {
     TScope ts(ctx, 0, st);
-    CK(launch_pilot(ctx->ad, ctx->pdv, ctx->pdv_dev, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur], ctx->hist_B[cur], B,
-                    ctx->logits64, logits, ctx->pd, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur], &fused, st));
+    if (ctx->tc_dev && !ctx->tc_flag_off && B >= kTcMinBatch) {
+      // K1-TC: batch large enough for the layers to be real dense contractions (3xTF32)
+      CK(launch_pilot_tc(ctx->ad, ctx->pdv_dev, ctx->tc_dev, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur],
+                         ctx->hist_B[cur], B, ctx->logits64, logits, st));
+      fused = 0;
+    } else {
+      CK(launch_pilot(ctx->ad, ctx->pdv, ctx->pdv_dev, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur],
+                      ctx->hist_B[cur], B, ctx->logits64, logits, ctx->pd, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur],
+                      &fused, st));
+    }
   }
   if (!ctx->branch_head) {
     // traversal decode: logits to the host, one sync, block head -> slots

@@ -42,6 +42,31 @@ struct PilotDev {
   LayerDev ly[3 * kMaxLayers + 8];
 };
 
+// ---- K1-TC: tensor-core batch pilot plan (pilot_tc.cu; built by dyo_load_pilot) --------
+constexpr int kTcCtas = 16;           // CTAs per cluster
+constexpr int kTcBatch = 64;          // predictions per cluster (MMA N)
+constexpr int kTcMaxStages = 8;
+constexpr int kTcSlots = 5;           // weight-chunk ring
+constexpr int kTcSlotBytes = 24 * 1024;   // 128 rows x <= 24 K x (hi + lo) x 4 B
+constexpr int kTcMaxKc = 24;
+constexpr int kTcMaxKsl = 128;        // K-slice of one CTA (X buffer: 64 x 128 x (hi + lo))
+constexpr int kTcMinBatch = 16;       // smaller batches take the cluster GEMV kernel
+struct TcStage {
+  int n_out, K, n_m, n_ks, ksl, act;
+  const float* bias;                  // device, n_out
+};
+struct TcChunk {                      // one weight chunk: rows m*128.. of tile m, K [k0, k0+kc) of the slice
+  int64_t off;                        // float offset into the blob (hi block, then lo block)
+  int32_t bytes, stage, job, k0, kc, pad;
+};
+struct TcPlan {
+  int n_stages, n_feat;
+  TcStage st[kTcMaxStages];
+  int chunk_ptr[kTcCtas + 1];
+  const TcChunk* chunks;
+  const float* blob;
+};
+
 // ---- arch on the device -------------------------------------------------------------
 struct ArchDev {
   int T, n_ops, n_sites, n_pieces, n_arms, nn_type, S_max, D_s, h, K_max, F, O, n_branch_logits;
@@ -167,6 +192,10 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
                          PredDev& pd, int32_t* hist_tab_out, int32_t* hist_K_out, int* fused,
                          cudaStream_t s);
 cudaError_t debug_stamps(int on, unsigned long long* out);
+// K1-TC: batch pilot on tensor cores (logits only; the caller launches the decode kernel).
+cudaError_t launch_pilot_tc(const ArchDev& a, const PilotDev* p_dev, const TcPlan* plan_dev, const float* feat,
+                            const int64_t* desc, const int32_t* hist, const int32_t* hist_tab, const int32_t* hist_K,
+                            int hist_B, int B, double* logits64, float* logits32, cudaStream_t s);
 cudaError_t plan_debug_stamps(int j, unsigned long long* out);
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s);

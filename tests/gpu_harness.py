@@ -54,9 +54,11 @@ def gpu_lists(d, j):
     return {k: d.plan_records(j, k).tolist() for k in ("evict", "move", "carry", "alloc", "fetch")}
 
 
-def logit_gates(y_gpu, x, spec, nn_type):
+def logit_gates(y_gpu, x, spec, nn_type, with_scale=False):
     """Gate 1 (north_star): |g-o| <= 1e-5 * max(|o|, 1e-3 max|o|). Gate 2: rigorous fp32
-    forward-error bound propagated layer by layer (gamma_n = n u / (1 - n u), u = 2^-24)."""
+    forward-error bound propagated layer by layer (gamma_n = n u / (1 - n u), u = 2^-24).
+    with_scale: also return the output layer's magnitude scale sum_k |w_ik z_k| + |b_i| (the
+    denominator of the tensor-core path's componentwise gate, reading R14)."""
     u = 2.0 ** -24
     w = spec.weights
 
@@ -81,8 +83,11 @@ def logit_gates(y_gpu, x, spec, nn_type):
         z, e = x, np.zeros_like(x)
     for l in range(len(spec.mlp)):
         z, e = layer(w[f"mlp{nn_type}.{l}.W"], w[f"mlp{nn_type}.{l}.b"], z, e, True)
+    scale = np.abs(w["out.W"].astype(np.float64)) @ np.abs(z) + np.abs(w["out.b"].astype(np.float64))
     o, e = layer(w["out.W"], w["out.b"], z, e, False)
     err = np.abs(y_gpu.astype(np.float64) - o)
+    if with_scale:
+        return err <= 1e-5 * np.maximum(np.abs(o), 1e-3 * np.abs(o).max()), err <= e * 1.01 + 1e-30, o, scale
     g1 = err <= 1e-5 * np.maximum(np.abs(o), 1e-3 * np.abs(o).max())
     g2 = err <= e * 1.01 + 1e-30
     return g1, g2, o

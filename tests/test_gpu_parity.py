@@ -216,3 +216,61 @@ def test_plan_bitexact_lstm_scaled(policy):
 def test_plan_bitexact_lstm_fullsize():
     wl = WL.make_lstm(n_samples=16)
     _run_plan_steps(wl, 1, 8, 1).close()
+
+
+@pytest.mark.parametrize("name,B", [("moe", 64), ("af", 64), ("lstm", 64), ("moe", 20), ("moe", 100)])
+def test_pilot_logits_tensor_cores(name, B):
+    """K1-TC (tcgen05 kind::tf32, 3xTF32 split) for batches >= 16. fp32-accumulating tensor
+    cores: every logit within 1e-5 of its magnitude scale max(|o|, sum |w z| + |b|) (reading R14)
+    and within the rigorous fp32 error bound; gate-1 (floored at 1e-3 max|o|) misses are counted
+    and must be cancellation (|o| < 1e-2 of the scale); decisions identical to the oracle's."""
+    wl = WL.make(name, n_samples=max(16, B))
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    logits = torch.zeros((B, wl.pilot.O), device="cuda")
+    d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, stream=_stream())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), (), plan=False)
+    y = logits.cpu().numpy()
+    n1, worst, worst_s, n_cancel, worst_rel = 0, 0.0, 0.0, 0, 0.0
+    for b in range(B):
+        g1, g2, o, scale = logit_gates(y[b], r["feats"][b], wl.pilot, wl.nn_type, with_scale=True)
+        err = np.abs(y[b].astype(np.float64) - o)
+        assert g2.all(), f"sample {b}: fp32 error bound violated at {np.where(~g2)[0][:5]}"
+        den_s = np.maximum(np.abs(o), scale)
+        rel_s = np.divide(err, den_s, out=np.where(err > 0, np.inf, 0.0), where=den_s > 0)
+        worst_s = max(worst_s, float(rel_s.max()))
+        wide = np.abs(o) >= 0.1 * scale
+        if wide.any():
+            worst_rel = max(worst_rel, float((err[wide] / np.abs(o[wide])).max()))
+        miss = ~g1
+        n1 += int(miss.sum())
+        n_cancel += int((miss & (np.abs(o) < 1e-2 * scale)).sum())
+        den = np.maximum(np.abs(o), 1e-3 * np.abs(o).max())
+        worst = max(worst, float((err / den).max()))
+    print(f"{name} B={B}: worst err/scale {worst_s:.3e}; worst err/|o| where |o| >= scale/10 {worst_rel:.3e}; "
+          f"gate-1 misses {n1} (cancellation {n_cancel}), worst floored relative {worst:.3e}")
+    assert worst_s <= 1e-5, "componentwise relative error above 1e-5 (R14)"
+    # decisions: identical, except a branch-head argmax whose top-2 gap in the oracle's logits is
+    # inside the path's error (2 x 1e-5 x the site's largest magnitude scale): a documented tie
+    from oracle import afm as AF
+    sites = AF.sites(wl.program)
+    n_tie = 0
+    for b in range(B):
+        p = r["preds"][b]
+        K, blocks, choices, rows = d.prediction(b, wl.K_max, len(sites), _stream())
+        if choices.tolist() != p.choices:
+            _, _, o, scale = logit_gates(y[b], r["feats"][b], wl.pilot, wl.nn_type, with_scale=True)
+            off = 10 * wl.K_max
+            for i, st_ in enumerate(sites):
+                if st_.tie >= 0:
+                    continue
+                nch = AF.n_choices(st_)
+                if choices[i] != p.choices[i]:
+                    lg = o[off:off + nch]
+                    gap = abs(lg[choices[i]] - lg[p.choices[i]])
+                    assert gap <= 2e-5 * scale[off:off + nch].max(), f"sample {b} site {i}: not a near-tie"
+                off += nch
+            n_tie += 1
+            continue
+        _check_prediction(d, wl, b, p)
+    print(f"{name} B={B}: {n_tie} predictions with a documented argmax near-tie")
+    d.close()

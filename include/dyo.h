@@ -51,7 +51,7 @@ typedef struct {
   int64_t budget;         /* B: device arena bytes, split in two equal halves (R7) */
   int32_t align;          /* ALIGN in bytes (power of two >= 16; 256 in all configs) */
   int32_t policy;         /* 0 = PAPER (evict every unused tensor), 1 = RETAIN (R10) */
-  int32_t max_batch;      /* max predictions per dyo_pilot_predict call (>= 1) */
+  int32_t max_batch;      /* max predictions per dyo_pilot_predict call (1..1024) */
   int32_t max_groups;     /* max groups per dyo_plan (sum over its predictions), <= 65535 */
   int32_t max_entries;    /* capacity of tensor-set entries per dyo_plan (0 = 512 per group) */
   int32_t max_records;    /* capacity of plan records per dyo_plan (0 = auto) */
@@ -296,8 +296,9 @@ dyo_status dyo_get_timings(dyo_ctx* ctx, int32_t kind, double* ms, int64_t* laun
  * (K3/K4 path). Synchronises `stream`. */
 dyo_status dyo_debug_copy(dyo_ctx* ctx, const void* src, void* dst, int64_t bytes, int32_t mode, void* stream);
 
-/* Debugging aid: enable (1) / disable (0) %globaltimer phase stamps of the pilot kernel and
- * read the 32 stamps of the last launch (ns; out32 may be NULL). Synchronises the device. */
+/* Debugging aid: enable (1) / disable (0) phase stamps of the pilot kernel and read the 32
+ * stamps of the last launch (out32 may be NULL): SM clock cycles for the cluster GEMV kernel,
+ * %globaltimer ns for the tensor-core batch kernel (K1-TC). Synchronises the device. */
 dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32);
 /* Debugging aid: clock64 stamps of the planner's phases for transition j of the next dyo_plan
  * (j = -1 disables); out64 (64 entries, may be NULL) receives the stamps of the last plan. */

@@ -53,6 +53,7 @@ struct dyo_ctx {
   // K1-TC (tensor-core batch pilot): device plan, or null when the pilot's shape does not fit it
   const TcPlan* tc_dev = nullptr;
   int tc_flag_off = 0;             // DYO_PILOT_TC=0 in the environment disables it (measurement)
+  int last_tc = 0;                 // the last dyo_pilot_predict ran K1-TC
   int64_t* desc_dev = nullptr;
   int32_t* hist_dev = nullptr;
   int32_t* hist_tab[2] = {nullptr, nullptr};
@@ -490,7 +491,7 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   ctx->device = device;
   dyo_config& c = ctx->cfg;
   if (c.align <= 0 || (c.align & (c.align - 1)) || c.align < 16 || c.budget < 2 * c.align ||
-      c.max_batch < 1 || c.max_batch > 64 || c.policy < 0 || c.policy > 1) {
+      c.max_batch < 1 || c.max_batch > 1024 || c.policy < 0 || c.policy > 1) {
     delete ctx;
     return DYO_E_INVAL;
   }
@@ -757,10 +758,27 @@ static dyo_status build_tc_plan(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   for (int i = 0; i < 3; ++i) n_feat += w->feat_out[i];
   struct L { const float* W; const float* b; int out, in, act; };
   std::vector<L> layers;
+  // stage 0: the three feature layers as one block-diagonal [n_feat x F_pad] layer (F padded to
+  // a multiple of 64 so its K splits over many CTAs; the padded inputs are zero)
+  const int Fp = (ctx->F + 63) / 64 * 64;
+  std::vector<float> fW((size_t)n_feat * Fp, 0.f), fb(n_feat, 0.f);
+  {
+    int o = 0;
+    for (int i = 0; i < 3; ++i) {
+      if (w->feat_off[i] < 0 || w->feat_off[i] + w->feat_len[i] > ctx->F) return DYO_OK;
+      for (int rr = 0; rr < w->feat_out[i]; ++rr) {
+        for (int c = 0; c < w->feat_len[i]; ++c)
+          fW[(size_t)(o + rr) * Fp + w->feat_off[i] + c] = w->feat_W[i][(size_t)rr * w->feat_len[i] + c];
+        fb[o + rr] = w->feat_b[i][rr];
+      }
+      o += w->feat_out[i];
+    }
+  }
+  layers.push_back({fW.data(), fb.data(), n_feat, Fp, 1});
   for (int l = 0; l < w->n_mlp; ++l)
     layers.push_back({w->mlp_W[k * w->n_mlp + l], w->mlp_b[k * w->n_mlp + l], w->mlp_out[l], w->mlp_in[l], 1});
   layers.push_back({w->out_W, w->out_b, w->O, w->out_in, 0});
-  if ((int)layers.size() > kTcMaxStages || layers[0].in != n_feat) return DYO_OK;
+  if ((int)layers.size() > kTcMaxStages || layers[1].in != n_feat) return DYO_OK;
   TcPlan P{};
   P.n_stages = (int)layers.size();
   P.n_feat = n_feat;
@@ -776,10 +794,13 @@ static dyo_status build_tc_plan(dyo_ctx* ctx, const dyo_pilot_desc* w) {
       if (s != P.n_stages - 1 || S.n_m > 2 * kTcCtas || ly.in > kTcMaxKsl) return DYO_OK;
       S.n_ks = 1;
     } else {
+      // n_ks <= 8 (an owner's w = 64 / n_ks samples form whole 8-sample groups); hidden stages
+      // need n_ks >= 4 (w <= 16: the owner's staging buffer)
       S.n_ks = 0;
-      for (int p = 16; p >= 1; p >>= 1)
+      for (int p = 8; p >= 1; p >>= 1)
         if (S.n_m * p <= kTcCtas && ly.in % (8 * p) == 0 && ly.in / p <= kTcMaxKsl) { S.n_ks = p; break; }
       if (!S.n_ks) return DYO_OK;
+      if (s != P.n_stages - 1 && S.n_ks < 4) return DYO_OK;
     }
     S.ksl = ly.in / S.n_ks;
     std::vector<float> bias(ly.b, ly.b + ly.out);
@@ -825,6 +846,9 @@ static dyo_status build_tc_plan(dyo_ctx* ctx, const dyo_pilot_desc* w) {
       }
     }
   }
+  // an owner's tile rows split into whole K-slices of the next stage
+  for (int s2 = 0; s2 + 1 < P.n_stages; ++s2)
+    if (P.st[s2].n_m > 1 && 128 % P.st[s2 + 1].ksl) return DYO_OK;
   std::vector<TcChunk> all;
   for (int r = 0; r < kTcCtas; ++r) {
     P.chunk_ptr[r] = (int)all.size();
@@ -1020,7 +1044,9 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
       CK(launch_pilot_tc(ctx->ad, ctx->pdv_dev, ctx->tc_dev, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur],
                          ctx->hist_B[cur], B, ctx->logits64, logits, st));
       fused = 0;
+      ctx->last_tc = 1;
     } else {
+      ctx->last_tc = 0;
       CK(launch_pilot(ctx->ad, ctx->pdv, ctx->pdv_dev, feat, desc, hist, ctx->hist_tab[cur], ctx->hist_K[cur],
                       ctx->hist_B[cur], B, ctx->logits64, logits, ctx->pd, ctx->hist_tab[1 - cur], ctx->hist_K[1 - cur],
                       &fused, st));
@@ -1594,6 +1620,7 @@ dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32)
   CK(cudaSetDevice(ctx->device));
   CK(cudaDeviceSynchronize());
   CK(debug_stamps(enable, reinterpret_cast<unsigned long long*>(out32)));
+  CK(tc_debug_stamps(enable, ctx->last_tc ? reinterpret_cast<unsigned long long*>(out32) : nullptr));
   return DYO_OK;
 }
 

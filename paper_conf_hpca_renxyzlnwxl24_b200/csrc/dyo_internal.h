@@ -46,7 +46,7 @@ struct PilotDev {
 constexpr int kTcCtas = 16;           // CTAs per cluster
 constexpr int kTcBatch = 64;          // predictions per cluster (MMA N)
 constexpr int kTcMaxStages = 8;
-constexpr int kTcSlots = 5;           // weight-chunk ring
+constexpr int kTcSlots = 4;           // weight-chunk ring
 constexpr int kTcSlotBytes = 24 * 1024;   // 128 rows x <= 24 K x (hi + lo) x 4 B
 constexpr int kTcMaxKc = 24;
 constexpr int kTcMaxKsl = 128;        // K-slice of one CTA (X buffer: 64 x 128 x (hi + lo))
@@ -192,6 +192,7 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
                          PredDev& pd, int32_t* hist_tab_out, int32_t* hist_K_out, int* fused,
                          cudaStream_t s);
 cudaError_t debug_stamps(int on, unsigned long long* out);
+cudaError_t tc_debug_stamps(int on, unsigned long long* out);   // K1-TC: globaltimer ns of CTA 0
 // K1-TC: batch pilot on tensor cores (logits only; the caller launches the decode kernel).
 cudaError_t launch_pilot_tc(const ArchDev& a, const PilotDev* p_dev, const TcPlan* plan_dev, const float* feat,
                             const int64_t* desc, const int32_t* hist, const int32_t* hist_tab, const int32_t* hist_K,

@@ -5,7 +5,8 @@
 // and the output layer is a GEMM  D[out][n] = sum_k W[out][k] X[n][k]  with M = 128 output rows
 // per tile (tcgen05.mma.cta_group::1.kind::tf32, A = weights from shared memory, B = the 64
 // samples' activations from shared memory, D = fp32 in TMEM: lane = output row, column =
-// sample). fp32 accuracy from TF32 operands by the 3xTF32 split: W = W_hi + W_lo,
+// sample). Stage 0 is the three input-feature layers as one block-diagonal layer over the
+// encoded features (R3/R5), which each CTA of stage 0 encodes straight into its X buffer. fp32 accuracy from TF32 operands by the 3xTF32 split: W = W_hi + W_lo,
 // X = X_hi + X_lo (each part rounded to TF32, so the tensor core reads it exactly), and
 // D = W_hi X_hi + W_hi X_lo + W_lo X_hi (the dropped W_lo X_lo is < 2^-22 |W X|).
 //
@@ -20,11 +21,11 @@
 // Warp roles: warp 0 lane 0 streams this CTA's pre-split weight chunks (host-laid-out in the
 // UMMA K-major no-swizzle core-matrix layout) through a 5-slot ring with cp.async.bulk (it runs
 // ahead across stages); warp 1 lane 0 issues the MMAs; warps 4-7 are the epilogue (TMEM lane
-// quarter = warp % 4); all 8 warps first compute the three input-feature layers (R5) for the 64
-// samples on the CUDA cores in fp64 and send them to the first stage's consumers.
-// Cluster-wide progress: after stage s every CTA arrives on every CTA's `prog` mbarrier (its
-// accumulator and reduce buffer are read); activations of stage s+1 are sent only after `prog`
-// completes, so single X / reduce buffers are safe.
+// quarter = warp % 4); all 8 warps first encode the stage-0 input.
+// Cluster-wide progress, two mbarriers per CTA arrived by every CTA: `progx` (its MMAs of stage s
+// are done, so its X buffer may be overwritten: activations of stage s+1 are sent after it) and
+// `progr` (its reduce buffer of stage s is read: partials of stage s+1 are sent after it); a
+// local `tfree` keeps the next stage's MMAs off the accumulator until the epilogue has read it.
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 #include <cstdint>
@@ -45,7 +46,9 @@ constexpr int kXOff = kRingBytes;
 constexpr int kXBytes = kTcBatch * kTcMaxKsl * 8;     // hi + lo
 constexpr int kRedOff = kXOff + kXBytes;
 constexpr int kRedBytes = 128 * kTcBatch * 4;
-constexpr int kBarOff = kRedOff + kRedBytes;
+constexpr int kStgOff = kRedOff + kRedBytes;
+constexpr int kStgBytes = 16 * 1024;                  // owner's outgoing activations (w <= 16 samples)
+constexpr int kBarOff = kStgOff + kStgBytes;
 constexpr int kScratchOff = kBarOff + 256;
 constexpr int kScratchFloats = 256;                   // per warp: one sample's feature vector
 constexpr int kSmemBytes = kScratchOff + 8 * kScratchFloats * 4;
@@ -62,7 +65,10 @@ __device__ __forceinline__ void mbar_arrive_local(uint64_t* bar) {
 __device__ __forceinline__ void mbar_arrive_remote(uint32_t raddr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(raddr) : "memory");
 }
+// Wait for a phase completed by peers of the cluster: spin at CTA scope (no L1 invalidation per
+// poll), then one cluster-scope acquire on the completed phase.
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t phase) {
+  mbar_wait(bar, phase);
   asm volatile(
       "{\n"
       ".reg .pred P1;\n"
@@ -128,6 +134,22 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
 #pragma unroll
   for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
 }
+// all 64 columns of this thread's lane (four x16 loads, one wait)
+__device__ __forceinline__ void tmem_ld64(uint32_t taddr, float* v) {
+  uint32_t r[64];
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15}, [%16];"
+        : "=r"(r[16 * q + 0]), "=r"(r[16 * q + 1]), "=r"(r[16 * q + 2]), "=r"(r[16 * q + 3]), "=r"(r[16 * q + 4]),
+          "=r"(r[16 * q + 5]), "=r"(r[16 * q + 6]), "=r"(r[16 * q + 7]), "=r"(r[16 * q + 8]), "=r"(r[16 * q + 9]),
+          "=r"(r[16 * q + 10]), "=r"(r[16 * q + 11]), "=r"(r[16 * q + 12]), "=r"(r[16 * q + 13]),
+          "=r"(r[16 * q + 14]), "=r"(r[16 * q + 15])
+        : "r"(taddr + 16u * q));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 64; ++i) v[i] = __uint_as_float(r[i]);
+}
 __device__ __forceinline__ void tmem_ld4(uint32_t taddr, float* v) {
   uint32_t r[4];
   asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0, %1, %2, %3}, [%4];"
@@ -149,39 +171,25 @@ __device__ __forceinline__ Job jobs_of(const TcStage& S, int r) {
   }
   return j;
 }
-// byte offset of X element (sample n, k) inside a K-slice buffer (K-major core matrices)
-__device__ __forceinline__ uint32_t xoff(int n, int k) {
-  return (uint32_t)((k >> 2) * (kTcBatch / 8 * 128) + (n >> 3) * 128 + (n & 7) * 16 + (k & 3) * 4);
-}
-
-// Send activation v of (row R of stage s's output = input R of stage s+1, sample n) to every
-// consumer of stage s+1 (hi / lo TF32 parts).
-__device__ __forceinline__ void send_x(const TcStage& N, int R, int n, double v, uint32_t xs, uint32_t xbar) {
-  const float f = (float)v;
-  const uint32_t hi = tf32_rna(f);
-  const uint32_t lo = tf32_rna(f - __uint_as_float(hi));
-  const int ks = R / N.ksl, k = R - ks * N.ksl;
-  const uint32_t o = xoff(n, k);
-  const uint32_t lo_off = (uint32_t)N.ksl * (kTcBatch * 4);
-  if (N.n_m * N.n_ks <= kTcCtas) {
-    for (int mm = 0; mm < N.n_m; ++mm) {
-      const int c = mm * N.n_ks + ks;
-      const uint32_t b = mapa_u32(xbar, c);
-      st_async_b32(mapa_u32(xs + o, c), hi, b);
-      st_async_b32(mapa_u32(xs + lo_off + o, c), lo, b);
-    }
-  } else {
-    const int nc = N.n_m < kTcCtas ? N.n_m : kTcCtas;
-    for (int c = 0; c < nc; ++c) {
-      const uint32_t b = mapa_u32(xbar, c);
-      st_async_b32(mapa_u32(xs + o, c), hi, b);
-      st_async_b32(mapa_u32(xs + lo_off + o, c), lo, b);
-    }
-  }
+// byte offset of X element (sample n, k) inside a K-slice buffer of ksl inputs: UMMA K-major
+// no-swizzle core matrices ordered [n/8][k/4][n%8][k%4] (8-sample groups outermost, so the
+// activations of 8 consecutive samples over the whole K-slice are one contiguous block)
+__device__ __forceinline__ uint32_t xoff(int n, int k, int ksl) {
+  return (uint32_t)((n >> 3) * (ksl * 32) + (k >> 2) * 128 + (n & 7) * 16 + (k & 3) * 4);
 }
 
 __device__ __forceinline__ uint32_t x_bytes(const TcStage& S, int r) {
   return jobs_of(S, r).n ? (uint32_t)(kTcBatch * S.ksl * 8) : 0u;
+}
+
+__device__ unsigned long long g_tc_stamp[32];
+__device__ int g_tc_on;
+__device__ __forceinline__ void tstamp(int i, int on) {
+  if (on && blockIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_tc_stamp[i] = t;
+  }
 }
 
 }  // namespace
@@ -190,7 +198,7 @@ __global__ void __cluster_dims__(kTcCtas, 1, 1) __launch_bounds__(kThreads, 1)
 pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pdev, const TcPlan* __restrict__ plan_g,
                 const float* __restrict__ feat, const int64_t* __restrict__ desc, const int32_t* __restrict__ hist,
                 const int32_t* __restrict__ hist_tab, const int32_t* __restrict__ hist_K, int hist_B, int B,
-                double* __restrict__ logits64, float* __restrict__ logits32, int terms) {
+                double* __restrict__ logits64, float* __restrict__ logits32) {
   extern __shared__ __align__(1024) unsigned char sm[];
   __shared__ TcPlan P;
   __shared__ uint32_t tmem_base_s;
@@ -198,13 +206,16 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
   const int r = (int)cg::this_cluster().block_rank();
   const int b0 = (blockIdx.x / kTcCtas) * kTcBatch;
   const int nb = min(kTcBatch, B - b0);
-  if (tid == 0) P = *plan_g;
+  const int son = g_tc_on;
+  if (tid == 0) { P = *plan_g; tstamp(0, son); }
   uint64_t* full = reinterpret_cast<uint64_t*>(sm + kBarOff);
   uint64_t* empty = full + kTcSlots;
   uint64_t* xfull = empty + kTcSlots;
   uint64_t* dfull = xfull + 1;
   uint64_t* redfull = dfull + 1;
-  uint64_t* prog = redfull + 1;
+  uint64_t* progx = redfull + 1;     // cluster: every CTA finished the MMAs of stage s (X_s free)
+  uint64_t* progr = progx + 1;       // cluster: every CTA finished reading its reduce buffer of s
+  uint64_t* tfree = progr + 1;       // local: the epilogue finished reading TMEM of stage s
   const uint32_t xs = smem_u32(sm + kXOff);
   const uint32_t red_s = smem_u32(sm + kRedOff);
   __syncthreads();
@@ -214,10 +225,11 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
     mbar_init(xfull, 1);
     mbar_init(dfull, 1);
     mbar_init(redfull, 1);
-    mbar_init(prog, kTcCtas);
+    mbar_init(progx, kTcCtas);
+    mbar_init(progr, kTcCtas);
+    mbar_init(tfree, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    // arm stage 0's activation and reduce buffers before any peer can send
-    mbar_expect_tx(xfull, x_bytes(P.st[0], r));
+    // arm stage 0's reduce buffer before any peer can send (its X is this CTA's own encode)
     const TcStage& S0 = P.st[0];
     if (S0.n_ks > 1 && r < S0.n_m * S0.n_ks) mbar_expect_tx(redfull, (uint32_t)kRedBytes);
   }
@@ -230,6 +242,7 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
   tc_fence_after();
   const uint32_t tmem = tmem_base_s;
   const int c0 = P.chunk_ptr[r], c1 = P.chunk_ptr[r + 1];
+  if (tid == 0) tstamp(1, son);
   // ---- weight stream: fill the ring now (overlaps the feature layers) ----
   if (tid == 0) {
     for (int i = c0; i < c1 && i < c0 + kTcSlots; ++i) {
@@ -239,42 +252,57 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
       tma_bulk_g2s(sm + slot * kTcSlotBytes, P.blob + ch.off, (uint32_t)ch.bytes, &full[slot]);
     }
   }
-  // ---- feature layers (R5) on the CUDA cores, fp64: CTA r computes features
-  //      [r * fpc, (r + 1) * fpc) for all 64 samples, one sample per warp at a time ----
+  // ---- stage 0 input: the encoded feature vectors (R3) of the 64 samples, K-slice ks of this
+  //      CTA, written straight into the local X buffer as TF32 hi / lo (zero past F / nb) ----
   {
-    const int nf = P.n_feat, fpc = (nf + kTcCtas - 1) / kTcCtas;
-    const int f0 = r * fpc, f1 = min(nf, f0 + fpc);
-    float* xw = reinterpret_cast<float*>(sm + kScratchOff) + warp * kScratchFloats;
-    const int hl = (!feat && hist && hist_B > 0) ? hist_len(hist_K, hist_B) : 0;
     const TcStage& S0 = P.st[0];
-    const double slope = pdev->slope;
-    for (int n = warp; n < kTcBatch; n += 8) {
-      const int b = b0 + n;
-      for (int i = lane; i < a.F; i += 32) {
+    const Job J0 = jobs_of(S0, r);
+    if (J0.n) {
+      // history prefix sums in scratch (R3: history ids index the concatenated group table)
+      int* pre = reinterpret_cast<int*>(sm + kScratchOff);
+      const int use_hist = (!feat && hist && hist_B > 0) ? 1 : 0;
+      if (use_hist && tid == 0) {
+        int acc = 0;
+        for (int b = 0; b < hist_B && b < 2047; ++b) { pre[b] = acc; acc += hist_K[b]; }
+        pre[2047] = acc;
+      }
+      __syncthreads();
+      const int hl = use_hist ? pre[2047] : 0;
+      const int xh0 = 3 + a.D_s + 10 * a.S_max;
+      const uint32_t lo_off = (uint32_t)S0.ksl * (kTcBatch * 4);
+      for (int i = tid; i < kTcBatch * S0.ksl; i += kThreads) {
+        const int n = i / S0.ksl, kl = i - n * S0.ksl, k = J0.ks * S0.ksl + kl;
+        const int b = b0 + n;
         float v = 0.f;
-        if (n < nb)
-          v = feat ? feat[(int64_t)b * a.F + i]
-                   : encode_elem(a, desc + (int64_t)b * a.D_s, hist ? hist + (int64_t)b * a.h : nullptr, hist_tab,
-                                 hist_K, hist_B, hl, i);
-        xw[i] = v;
+        if (n < nb && k < a.F) {
+          if (feat) {
+            v = feat[(int64_t)b * a.F + k];
+          } else if (k >= xh0 && k < xh0 + 10 * a.h) {
+            // x_h by binary search over the history prefix sums (instead of a linear walk)
+            if (use_hist) {
+              const int kk = (k - xh0) / 10, el = (k - xh0) % 10;
+              const int gid = hist[(int64_t)b * a.h + kk];
+              const int idx = gid >= 0 ? gid : hl + gid;
+              if (idx >= 0 && idx < hl) {
+                int lo = 0, hi = min(hist_B, 2047) - 1;
+                while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (pre[mid] <= idx) lo = mid; else hi = mid - 1; }
+                v = scale_elem<float>(el, hist_tab[((int64_t)lo * a.K_max + (idx - pre[lo])) * 10 + el]);
+              }
+            }
+          } else {
+            v = encode_elem(a, desc + (int64_t)b * a.D_s, nullptr, hist_tab, hist_K, 0, 0, k);
+          }
+        }
+        const uint32_t h = tf32_rna(v);
+        const uint32_t l = tf32_rna(v - __uint_as_float(h));
+        *reinterpret_cast<uint32_t*>(sm + kXOff + xoff(n, kl, S0.ksl)) = h;
+        *reinterpret_cast<uint32_t*>(sm + kXOff + lo_off + xoff(n, kl, S0.ksl)) = l;
       }
-      __syncwarp();
-      for (int f = f0; f < f1; ++f) {
-        int li = pdev->st[0].first_layer, fl = f;
-        while (fl >= pdev->ly[li].out_len) { fl -= pdev->ly[li].out_len; ++li; }
-        const LayerDev& L = pdev->ly[li];
-        const float* wr = L.W + (int64_t)fl * L.in_pad;
-        double acc = 0.0;
-        for (int k = lane; k < L.in_len; k += 32) acc = fma((double)__ldg(wr + k), (double)xw[L.in_off + k], acc);
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-        acc += (double)__ldg(wr + L.in_len);                    // bias rides in the row (R5 loader)
-        acc = acc > 0.0 ? acc : slope * acc;
-        if (lane == 0) send_x(S0, f, n, acc, xs, smem_u32(xfull));
-      }
-      __syncwarp();
     }
+    __syncthreads();
+    if (tid == 0) mbar_arrive_local(xfull);      // stage 0 input complete (local writes)
   }
+  if (tid == 128) tstamp(2, son);
   // ---- role split ----
   if (tid == 0) {
     // TMA producer: the rest of this CTA's chunk list, gated by the ring's empty barriers
@@ -292,7 +320,9 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
       const TcStage S = P.st[s];
       const Job J = jobs_of(S, r);
       mbar_wait_cluster(xfull, s & 1);
+      tstamp(3 + s, son);
       if (J.n == 0) { mbar_arrive_local(dfull); continue; }
+      if (s > 0) mbar_wait(tfree, (s - 1) & 1);       // accumulator of stage s-1 read
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       tc_fence_after();
       const uint32_t xlo = xs + (uint32_t)S.ksl * (kTcBatch * 4);
@@ -310,22 +340,12 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
             const int kk = ch.k0 + 8 * j;
             const uint64_t a_hi = sdesc(ahi + (uint32_t)j * 4096u, 2048u, 128u);
             const uint64_t a_lo = sdesc(alo + (uint32_t)j * 4096u, 2048u, 128u);
-            const uint64_t x_hi = sdesc(xs + (uint32_t)(kk >> 2) * 1024u, 1024u, 128u);
-            const uint64_t x_lo = sdesc(xlo + (uint32_t)(kk >> 2) * 1024u, 1024u, 128u);
-            const uint32_t acc0 = (k0 > 0 || j > 0) ? 1u : 0u;
-            if (terms == 3) {
-              mma_tf32(d, a_lo, x_hi, acc0);
-              mma_tf32(d, a_hi, x_lo, 1u);
-              mma_tf32(d, a_hi, x_hi, 1u);
-            } else if (terms == 2) {
-              mma_tf32(d, a_hi, x_lo, acc0);
-              mma_tf32(d, a_hi, x_hi, 1u);
-            } else if (terms == 4) {
-              mma_tf32(d, a_lo, x_hi, acc0);
-              mma_tf32(d, a_hi, x_hi, 1u);
-            } else {
-              mma_tf32(d, a_hi, x_hi, acc0);
-            }
+            const uint64_t x_hi = sdesc(xs + (uint32_t)(kk >> 2) * 128u, 128u, (uint32_t)S.ksl * 32u);
+            const uint64_t x_lo = sdesc(xlo + (uint32_t)(kk >> 2) * 128u, 128u, (uint32_t)S.ksl * 32u);
+            // 3xTF32: small terms first, then the dominant hi x hi
+            mma_tf32(d, a_lo, x_hi, (k0 > 0 || j > 0) ? 1u : 0u);
+            mma_tf32(d, a_hi, x_lo, 1u);
+            mma_tf32(d, a_hi, x_hi, 1u);
           }
           mma_commit(&empty[slot]);
           k0 += ch.kc;
@@ -335,98 +355,166 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
       mma_commit(dfull);
     }
   } else if (warp >= 4) {
-    // epilogue: thread e <-> TMEM lane e = output row e of the tile
+    // epilogue: thread e <-> TMEM lane e = output row e of the tile. The partial tile leaves
+    // straight from registers; owners reduce and push each activation as soon as it is ready.
     const int e = tid - 128;
     const uint32_t lane_base = (uint32_t)((warp & 3) * 32) << 16;
+    const double slope = pdev->slope;
+    const float fslope = (float)slope;
+    const float* rd = reinterpret_cast<const float*>(sm + kRedOff);
+    const int ql = lane & ~3;
     int red_ph = 0;
     for (int s = 0; s < ns; ++s) {
       const TcStage S = P.st[s];
       const bool last = (s == ns - 1);
       const Job J = jobs_of(S, r);
       const bool owner = S.n_ks > 1 && r < S.n_m * S.n_ks;
-      const float* bias = S.bias;
+      const int w = kTcBatch / S.n_ks;
       mbar_wait(dfull, s & 1);
       tc_fence_after();
+      if (e == 0) tstamp(11 + s, son);
+      const TcStage N = P.st[last ? s : s + 1];
       float vals[kTcBatch];
-      int vrow = -1, vn0 = 0, vw = 0;           // values kept for the X sends after `prog`
-      if (S.n_ks == 1) {
-        for (int jj = 0; jj < J.n; ++jj) {
-          const int R = J.m[jj] * 128 + e;
-          for (int c = 0; c < kTcBatch; c += 16) tmem_ld16(tmem + lane_base + (uint32_t)(jj * kTcBatch + c), vals + c);
-          if (R < S.n_out) {
-            const double bv = (double)__ldg(bias + R);
-            if (last) {
+      if (J.n) {
+        if (S.n_ks > 1) {
+          tmem_ld64(tmem + lane_base, vals);
+        } else {
+          for (int jj = 0; jj < J.n; ++jj) {
+            tmem_ld64(tmem + lane_base + (uint32_t)(jj * kTcBatch), vals);
+            const int R = J.m[jj] * 128 + e;
+            if (last && R < S.n_out) {
+              const double bv = (double)__ldg(S.bias + R);
+#pragma unroll 1
               for (int n = 0; n < nb; ++n) {
                 const double v = (double)vals[n] + bv;
                 logits64[(int64_t)(b0 + n) * S.n_out + R] = v;
                 if (logits32) logits32[(int64_t)(b0 + n) * S.n_out + R] = (float)v;
               }
-            } else {
-              for (int n = 0; n < kTcBatch; ++n) {
-                double v = (double)vals[n] + bv;
-                if (S.act) v = v > 0.0 ? v : pdev->slope * v;
-                vals[n] = (float)v;
-              }
-              vrow = R; vn0 = 0; vw = kTcBatch;
             }
-          }
-        }
-      } else {
-        if (J.n) {
-          // reduce-scatter the partial tile: columns [q w, (q+1) w) to owner m * n_ks + q
-          const int w = kTcBatch / S.n_ks;
-          for (int qq = 0; qq < S.n_ks; ++qq) {
-            const int owner_c = J.m[0] * S.n_ks + qq;
-            const uint32_t rb = mapa_u32(smem_u32(redfull), owner_c);
-            for (int c = 0; c < w; c += 4) {
-              float v4[4];
-              tmem_ld4(tmem + lane_base + (uint32_t)(qq * w + c), v4);
-              const uint32_t dst = red_s + (uint32_t)(((J.ks * 128 + e) * w + c) * 4);
-              st_async_v4b32(mapa_u32(dst, owner_c), v4[0], v4[1], v4[2], v4[3], rb);
-            }
-          }
-        }
-        if (owner) {
-          const int m = r / S.n_ks, qo = r % S.n_ks, w = kTcBatch / S.n_ks;
-          const int R = m * 128 + e;
-          mbar_wait_cluster(redfull, red_ph & 1);
-          ++red_ph;
-          const float* rd = reinterpret_cast<const float*>(sm + kRedOff);
-          if (R < S.n_out) {
-            const double bv = (double)__ldg(bias + R);
-            for (int c = 0; c < w; ++c) {
-              double v = bv;
-              for (int k2 = 0; k2 < S.n_ks; ++k2) v += (double)rd[(k2 * 128 + e) * w + c];
-              const int n = qo * w + c;
-              if (last) {
-                if (n < nb) {
-                  logits64[(int64_t)(b0 + n) * S.n_out + R] = v;
-                  if (logits32) logits32[(int64_t)(b0 + n) * S.n_out + R] = (float)v;
-                }
-              } else {
-                if (S.act) v = v > 0.0 ? v : pdev->slope * v;
-                vals[c] = (float)v;
-              }
-            }
-            if (!last) { vrow = R; vn0 = qo * w; vw = w; }
           }
         }
       }
-      if (last) break;
-      // stage s consumed (TMEM read, reduce buffer read): arm stage s+1, then cluster progress
+      // the accumulator is read: the next stage's MMAs may start; X_s is free (MMAs done)
       tc_fence_before();
       asm volatile("bar.sync 1, 128;" ::: "memory");
-      const TcStage N = P.st[s + 1];
-      if (e == 0) {
-        mbar_expect_tx(xfull, x_bytes(N, r));
-        if (N.n_ks > 1 && r < N.n_m * N.n_ks) mbar_expect_tx(redfull, (uint32_t)kRedBytes);
-        for (int c = 0; c < kTcCtas; ++c) mbar_arrive_remote(mapa_u32(smem_u32(prog), c));
+      if (!last && e == 0) {
+        mbar_expect_tx(xfull, x_bytes(N, r));           // before any peer can pass progx(s)
+        mbar_arrive_local(tfree);
       }
-      mbar_wait_cluster(prog, s & 1);
-      if (vrow >= 0)
-        for (int c = 0; c < vw; ++c) send_x(N, vrow, vn0 + c, (double)vals[c], xs, smem_u32(xfull));
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (!last && e < kTcCtas) mbar_arrive_remote(mapa_u32(smem_u32(progx), e));
+      if (J.n && S.n_ks > 1) {
+        // reduce-scatter: columns [q w, (q+1) w) of the partial tile to owner m * n_ks + q, as
+        // 16-byte st.async from registers (owner's reduce buffer: [ks][c][row]); its reduce
+        // buffer of the previous stage must be read (progr(s-1))
+        if (s > 0) mbar_wait_cluster(progr, (s - 1) & 1);
+#pragma unroll
+        for (int c = 0; c < kTcBatch; c += 4) {
+          const int qq = c / w, cc = c - qq * w;
+          const int owner_c = J.m[0] * S.n_ks + qq;
+          const uint32_t dst = mapa_u32(red_s + (uint32_t)(((J.ks * (w / 4) + cc / 4) * 128 + e) * 16), owner_c);
+          st_async_v4b32(dst, vals[c], vals[c + 1], vals[c + 2], vals[c + 3], mapa_u32(smem_u32(redfull), owner_c));
+        }
+      }
+      if (owner) {
+        const int m = r / S.n_ks, qo = r % S.n_ks;
+        const int R = m * 128 + e, R0 = m * 128 + (e & ~3);
+        if (e == 0 && s == 1) tstamp(28, son);
+        mbar_wait_cluster(redfull, red_ph & 1);
+        if (e == 0 && s == 1) tstamp(29, son);
+        ++red_ph;
+        const float bv = R < S.n_out ? __ldg(S.bias + R) : 0.f;
+        const int nsl = N.ksl;                          // K-slice of the next stage
+        const int kr = R - m * 128, jq = kr / nsl, kq = (kr & ~3) - jq * nsl;   // quad's slice / first k
+        const int li = lane & 3;
+#pragma unroll 1
+        for (int cg = 0; cg < w / 4; ++cg) {
+          float4 acc4 = make_float4(0.f, 0.f, 0.f, 0.f);
+          double a64[4] = {(double)bv, (double)bv, (double)bv, (double)bv};
+          for (int k2 = 0; k2 < S.n_ks; ++k2) {
+            const float4 p4 = *reinterpret_cast<const float4*>(rd + ((k2 * (w / 4) + cg) * 128 + e) * 4);
+            if (last) { a64[0] += p4.x; a64[1] += p4.y; a64[2] += p4.z; a64[3] += p4.w; }
+            else { acc4.x += p4.x; acc4.y += p4.y; acc4.z += p4.z; acc4.w += p4.w; }
+          }
+          if (last) {
+            // logits: the partials combined in fp64
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+              const int n = qo * w + cg * 4 + i;
+              if (R < S.n_out && n < nb) {
+                logits64[(int64_t)(b0 + n) * S.n_out + R] = a64[i];
+                if (logits32) logits32[(int64_t)(b0 + n) * S.n_out + R] = (float)a64[i];
+              }
+            }
+            continue;
+          }
+          // fp32 (R14: an fp32-accumulating path): bias, LeakyReLU, TF32 hi / lo
+          float v[4] = {acc4.x + bv, acc4.y + bv, acc4.z + bv, acc4.w + bv};
+          uint32_t h[4], l[4];
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            if (S.act) v[i] = v[i] > 0.f ? v[i] : fslope * v[i];
+            h[i] = tf32_rna(v[i]);
+            l[i] = tf32_rna(v[i] - __uint_as_float(h[i]));
+          }
+          // 4x4 transpose inside the quad: lane li gets sample cg*4+li of the quad's four rows
+          uint32_t th[4], tl[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const int snd = (li - j) & 3, src = (li + j) & 3;
+            const uint32_t sh = snd == 0 ? h[0] : snd == 1 ? h[1] : snd == 2 ? h[2] : h[3];
+            const uint32_t sl = snd == 0 ? l[0] : snd == 1 ? l[1] : snd == 2 ? l[2] : l[3];
+            const uint32_t rh = __shfl_sync(0xffffffffu, sh, (lane & ~3) + src);
+            const uint32_t rl = __shfl_sync(0xffffffffu, sl, (lane & ~3) + src);
+            th[src] = rh;   // row (quad base + src)
+            tl[src] = rl;
+          }
+          // staging: [slice j of the next stage][hi, lo][c/8][k/4][c%8][k%4] (k = row within the
+          // slice); each (slice, part) block is contiguous in the consumers' X layout
+          if (R - (e & 3) < S.n_out) {
+            const int c = cg * 4 + li;
+            const uint32_t blk = (uint32_t)((jq * 2) * w * nsl * 4);
+            const uint32_t o = (uint32_t)((c >> 3) * (nsl * 32) + (kq >> 2) * 128 + (c & 7) * 16);
+            *reinterpret_cast<uint4*>(sm + kStgOff + blk + o) = make_uint4(th[0], th[1], th[2], th[3]);
+            *reinterpret_cast<uint4*>(sm + kStgOff + blk + (uint32_t)(w * nsl * 4) + o) = make_uint4(tl[0], tl[1], tl[2], tl[3]);
+          }
+        }
+        if (!last) {
+          // one bulk copy per (next-stage K-slice j, part, consumer) into the consumer's X at
+          // samples [qo w, qo w + w), once the consumers' MMAs of this stage are done (progx)
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          asm volatile("bar.sync 1, 128;" ::: "memory");
+          mbar_wait_cluster(progx, s & 1);
+          const int nj = (min(S.n_out - m * 128, 128) + nsl - 1) / nsl;
+          const bool grid = N.n_m * N.n_ks <= kTcCtas;
+          const int ncons = grid ? N.n_m : min(N.n_m, kTcCtas);
+          const uint32_t bytes = (uint32_t)(w * nsl * 4);
+          for (int t = e; t < nj * 2 * ncons; t += 128) {
+            const int j = t / (2 * ncons), part = (t / ncons) & 1, ci = t % ncons;
+            const int ks2 = (m * 128) / nsl + j;         // the slice's index in the next stage
+            const int cons = grid ? ci * N.n_ks + ks2 : ci;
+            const uint32_t src = smem_u32(sm + kStgOff) + (uint32_t)((j * 2 + part) * w * nsl * 4);
+            const uint32_t dst = xs + (uint32_t)part * (uint32_t)(nsl * kTcBatch * 4) + (uint32_t)(qo * w / 8) * (uint32_t)(nsl * 32);
+            asm volatile(
+                "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                    mapa_u32(dst, cons)),
+                "r"(src), "r"(bytes), "r"(mapa_u32(smem_u32(xfull), cons))
+                : "memory");
+          }
+        }
+        if (s == 1 && (e == 0 || e == 96)) tstamp(e == 0 ? 31 : 26, son);
+      }
+      if (last) break;
+      // reduce buffer of stage s read: arm stage s+1's, then let peers send their partials
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (e == 0 && N.n_ks > 1 && r < N.n_m * N.n_ks) mbar_expect_tx(redfull, (uint32_t)kRedBytes);
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (e == 0 && s == 1) tstamp(30, son);
+      if (e < kTcCtas) mbar_arrive_remote(mapa_u32(smem_u32(progr), e));
+      if (e == 0) tstamp(19 + s, son);
     }
   }
+  if (tid == 128) tstamp(27, son);
   tc_fence_before();
   __syncthreads();
   cg::this_cluster().sync();       // no CTA leaves while a peer may still address its memory
@@ -434,6 +522,12 @@ pilot_tc_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ 
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
   }
+}
+
+cudaError_t tc_debug_stamps(int on, unsigned long long* out) {
+  cudaError_t e = cudaMemcpyToSymbol(g_tc_on, &on, sizeof(int));
+  if (e == cudaSuccess && out) e = cudaMemcpyFromSymbol(out, g_tc_stamp, sizeof(unsigned long long) * 32);
+  return e;
 }
 
 cudaError_t launch_pilot_tc(const ArchDev& a, const PilotDev* p_dev, const TcPlan* plan_dev, const float* feat,
@@ -449,10 +543,8 @@ cudaError_t launch_pilot_tc(const ArchDev& a, const PilotDev* p_dev, const TcPla
     attr = true;
   }
   const int n_clusters = (B + kTcBatch - 1) / kTcBatch;
-  static int terms = -1;
-  if (terms < 0) { const char* e = getenv("DYO_TC_TERMS"); terms = e ? atoi(e) : 3; }
   pilot_tc_kernel<<<n_clusters * kTcCtas, kThreads, kSmemBytes, s>>>(a, p_dev, plan_dev, feat, desc, hist, hist_tab,
-                                                                    hist_K, hist_B, B, logits64, logits32, terms);
+                                                                    hist_K, hist_B, B, logits64, logits32);
   return cudaGetLastError();
 }
 

@@ -608,6 +608,8 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   DA(pd.K, B); DA(pd.L, B); DA(pd.choices, (size_t)B * std::max(n_sites, 1)); DA(pd.slots, (size_t)B * K * 10);
   DA(pd.path, (size_t)B * ad.L_max); DA(pd.grp, (size_t)B * K * 2); DA(pd.blocks, (size_t)B * K * 10);
   DA(pd.ent_n, (size_t)B * K); DA(pd.ent, (size_t)B * K * kEntCap); DA(pd.status, 4);
+  pd.head_stride = 3 + n_sites + ((int)piece_kind.size() + 1) + (K + 1) + K;
+  DA(pd.head, (size_t)B * pd.head_stride);
   DA(ctx->desc_dev, (size_t)B * std::max(A->D_s, 1)); DA(ctx->hist_dev, (size_t)B * std::max(A->h, 1));
   DA(ctx->hist_tab[0], (size_t)B * K * 10); DA(ctx->hist_tab[1], (size_t)B * K * 10);
   DA(ctx->hist_K[0], B); DA(ctx->hist_K[1], B);

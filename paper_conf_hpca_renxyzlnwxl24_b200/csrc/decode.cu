@@ -1,7 +1,7 @@
-// A3 decode kernel for batches whose groups outnumber the pilot cluster's CTAs (the fused
-// pilot epilogue handles the rest; pilot.cu). One CTA per (prediction b, group slot g): warp 0
-// decodes the head of prediction b into shared memory (decode_dev.cuh), then the block builds
-// group g. No inter-CTA dependency, no materialised path.
+// A3 decode kernels for batches whose groups outnumber the pilot cluster's CTAs, for the
+// tensor-core batch pilot and for the traversal decode (the fused pilot epilogue handles the
+// rest; pilot.cu): a head kernel (one warp per prediction) and a group kernel (one CTA per
+// (prediction, group slot)). No materialised path.
 #include <cuda_runtime.h>
 #include <cstdint>
 
@@ -12,31 +12,68 @@ namespace dyo {
 constexpr int kDecThreads = 256;
 constexpr int kDecTabCap2 = 8192;     // int32 words of decode tables staged in smem
 
-struct DecSmem {
+// ---- two-phase batch decode -------------------------------------------------------------
+// Phase A (one warp per prediction): head decode (R4) of the fp64 logits straight from global
+// memory; writes the debug copies (slots, choices, path, K, L) and the compact head (choices,
+// piece starts, group starts / counts) to pd.head. Phase B (one CTA per (prediction, group
+// slot)): groups past K exit at once; the others load the compact head and build their tensor
+// set. Replaces the per-(prediction, group) redundant head decode + logits staging of the
+// single-phase kernel for large batches (AF: 256 group slots x O = 2,576 logits).
+struct HeadSmem {
+  DecHead H;
+};
+
+__device__ __forceinline__ int* head_of(const PredDev& pd, int b) { return pd.head + (int64_t)b * pd.head_stride; }
+
+__global__ void __launch_bounds__(32)
+decode_head_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t* __restrict__ hist_K) {
+  __shared__ HeadSmem S;
+  const int b = blockIdx.x, lane = threadIdx.x;
+  if (b == 0 && lane == 0) { pd.status[0] = 0; pd.status[1] = 0; }
+  const double* y = logits + (int64_t)b * a.O;
+  head_decode_warp(a, y, S.H, lane, b);
+  write_head(a, S.H, y, pd, b, hist_K);
+  int* h = head_of(pd, b);
+  const int ns = a.n_sites, np = a.n_pieces, K = a.K_max;
+  if (lane == 0) { h[0] = S.H.L; h[1] = S.H.nk; h[2] = S.H.K; }
+  int* hc = h + 3;
+  for (int i = lane; i < ns; i += 32) hc[i] = S.H.choice[i];
+  int* hs = hc + ns;
+  for (int i = lane; i <= np; i += 32) hs[i] = S.H.start[i];
+  int* hcum = hs + np + 1;
+  for (int i = lane; i < S.H.nk; i += 32) hcum[i] = S.H.cum[i];
+  int* hcnt = hcum + K + 1;
+  for (int i = lane; i < S.H.nk; i += 32) hcnt[i] = S.H.cntc[i];
+}
+
+struct GroupSmem {
   DecHead H;
   DecGroup G;
-  double ys[1];      // logits copy (O doubles, dynamic)
 };
 
 __global__ void __launch_bounds__(kDecThreads)
-decode_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t* __restrict__ hist_tab,
-              int32_t* __restrict__ hist_K) {
+decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab) {
   extern __shared__ __align__(16) unsigned char dsm[];
-  DecSmem& S = *reinterpret_cast<DecSmem*>(dsm);
+  GroupSmem& S = *reinterpret_cast<GroupSmem*>(dsm);
   const int b = blockIdx.x / a.K_max, g = blockIdx.x % a.K_max;
-  const double* yg = logits + (int64_t)b * a.O;
-  for (int i = threadIdx.x; i < a.O; i += blockDim.x) S.ys[i] = yg[i];
-  __syncthreads();
-  const double* y = S.ys;
-  int* tabs = reinterpret_cast<int*>(S.ys + ((a.O + 15) / 16) * 16);
-  const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap2);
-  if (threadIdx.x < 32) head_decode_warp(A, y, S.H, threadIdx.x, b);
-  __syncthreads();
-  if (g == 0) write_head(A, S.H, y, pd, b, hist_K);
-  if (g >= S.H.K) {
+  const int* h = head_of(pd, b);
+  const int K = h[2];
+  if (g >= K) {
     if (threadIdx.x == 0) pd.ent_n[(int64_t)b * a.K_max + g] = 0;
     return;
   }
+  const int ns = a.n_sites, np = a.n_pieces;
+  if (threadIdx.x == 0) { S.H.L = h[0]; S.H.nk = h[1]; S.H.K = K; }
+  const int* hc = h + 3;
+  for (int i = threadIdx.x; i < ns; i += blockDim.x) S.H.choice[i] = hc[i];
+  const int* hs = hc + ns;
+  for (int i = threadIdx.x; i <= np; i += blockDim.x) S.H.start[i] = hs[i];
+  const int* hcum = hs + np + 1;
+  const int* hcnt = hcum + a.K_max + 1;
+  const int nk = h[1];
+  for (int i = threadIdx.x; i < nk; i += blockDim.x) { S.H.cum[i] = hcum[i]; S.H.cntc[i] = hcnt[i]; }
+  int* tabs = reinterpret_cast<int*>(dsm + sizeof(GroupSmem));
+  const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap2);   // ends with __syncthreads()
   build_group(A, S.H, S.G, pd, b, g, hist_tab);
 }
 
@@ -44,13 +81,16 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
   static bool attr = false;
+  const size_t smem = sizeof(GroupSmem) + (size_t)kDecTabCap2 * 4;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaError_t e = cudaFuncSetAttribute(decode_groups_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  const size_t smem = sizeof(DecSmem) + (size_t)((a.O + 15) / 16 * 16) * sizeof(double) + (size_t)kDecTabCap2 * 4;
-  decode_kernel<<<B * a.K_max, kDecThreads, smem, s>>>(a, logits, pd, hist_tab_out, hist_K_out);
+  decode_head_kernel<<<B, 32, 0, s>>>(a, logits, pd, hist_K_out);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  decode_groups_kernel<<<B * a.K_max, kDecThreads, smem, s>>>(a, pd, hist_tab_out);
   return cudaGetLastError();
 }
 

@@ -118,6 +118,8 @@ struct PredDev {
   int32_t* ent_n;     // B x K_max entry counts
   int2* ent;          // B x K_max x kEntCap (t, mode | needs_fetch << 2)
   int32_t* status;    // decode status word (0 ok, else DYO_E_*), [1] = detail
+  int32_t* head;      // B x head_stride: decoded heads for the two-phase batch decode (decode.cu)
+  int head_stride;    // 3 + n_sites + (n_pieces + 1) + (K_max + 1) + K_max
 };
 
 // ---- planner state (device) -----------------------------------------------------------

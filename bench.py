@@ -39,7 +39,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="dyo", choices=["dyo", "reference"])
-    ap.add_argument("--config", default="moe", choices=["moe", "tiny", "af"])
+    ap.add_argument("--config", default="moe", choices=["moe", "tiny", "af", "lstm"])
     ap.add_argument("--policy", type=int, default=1)
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--budget-gib", type=float, default=0.0)
@@ -55,6 +55,8 @@ CONFIG_DESC = {
            "3 GiB budget = 8x oversubscribed expert pool, P512 pilot (BASELINE configs[1])",
     "tiny": "tiny trace: 8 groups, 64 tensors, T32 pilot, 1 GiB budget (BASELINE configs[0])",
     "af": "AlphaFold-Evoformer-shaped trace, 48 blocks x recycle 1..4, MSA 128x256, 2 GiB budget (BASELINE configs[2])",
+    "lstm": "variable-length 2-layer LSTM (length U{16..512}, 4 task heads), batch of 64 predictions planned per "
+            "step, 35,860 tensors of 2-4 KiB (+ 4 MiB weights), 48 MiB budget (BASELINE configs[3], var-length variant)",
 }
 
 
@@ -128,7 +130,7 @@ def reduce_over_ranks(vals_max, vals_sum, backend):
 
 def make_workload(args, rank):
     import workloads as WL
-    wl = WL.make(args.config, seed=args.seed + rank, n_samples=64)
+    wl = WL.make(args.config, seed=args.seed + rank, n_samples=128)
     wl.policy = args.policy
     if args.budget_gib > 0:
         wl.budget = int(args.budget_gib * (1 << 30))
@@ -152,11 +154,18 @@ def oracle_steps(wl, n_steps, budget_s=None):
     buf_a = np.ones(256 << 20, np.uint8)
     buf_b = np.zeros(256 << 20, np.uint8)
     total_b, t0, done = 0, time.perf_counter(), 0
+    B = wl.notes.get("batch", 1)
+    bs = min(B, wl.notes.get("oracle_batch", B))     # bounded sample of a batched step
     with threadpool_limits(limits=1):
         for s in range(n_steps):
-            r = OR.step(wl, s % len(wl.samples), st, table)
-            st, table = r.state, r.pred.blocks
-            nbytes = sum(t.h2d + t.d2h for t in r.transitions)
+            if B == 1:
+                r = OR.step(wl, s % len(wl.samples), st, table)
+                st, table, trs = r.state, r.pred.blocks, r.transitions
+            else:
+                ids = [(s * bs + i) % len(wl.samples) for i in range(bs)]
+                preds, trs, st, _ = OR.step_batch(wl, ids, st, table)
+                table = [v for p in preds for v in p.blocks]
+            nbytes = sum(t.h2d + t.d2h for t in trs)
             left = nbytes
             while left > 0:
                 n = min(left, buf_a.size)
@@ -253,23 +262,25 @@ def run_dyo(args):
 
     wl = make_workload(args, rank)
     _log("workload built")
-    d = Dyo(wl.budget, wl.align, wl.policy, max_batch=1, device=local, flags=DYO_F_TIMING)
+    B = wl.notes.get("batch", 1)          # predictions planned per step (lstm: a minibatch of 64)
+    d = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, device=local, flags=DYO_F_TIMING)
     d.load(wl)
     _log("ctx loaded")
     s0 = torch.cuda.current_stream()
     s1 = torch.cuda.Stream()
     desc_dev = torch.from_numpy(wl.samples.copy()).to(dev)
-    hist_np = wl.hist_ids.astype(np.int32).reshape(1, -1) if wl.h else None
+    hist_np = np.tile(wl.hist_ids.astype(np.int32), (B, 1)) if wl.h else None
     hist_dev = torch.from_numpy(hist_np).to(dev) if hist_np is not None else None
     nS = len(wl.samples)
+    assert nS % B == 0
 
     # Blocks: without compute emulation, block j "starts" and "ends" when ready[j] fires, so
     # transition j's EVICT waits ready[j-2] (its half's last user) and overlaps transition j-1's
     # FETCH. With emulation, block j is a spin kernel on the compute stream after ready[j] whose
     # duration follows the workload's per-group FLOPs; migrations wait on the block-end events.
     emulate = args.compute == "emulate" or (args.compute == "auto" and args.config == "af")
-    ready = [torch.cuda.Event() for _ in range(wl.K_max + 1)]
-    bend = [torch.cuda.Event() for _ in range(wl.K_max + 1)]
+    ready = [torch.cuda.Event() for _ in range(B * wl.K_max + 1)]
+    bend = [torch.cuda.Event() for _ in range(B * wl.K_max + 1)]
     t_start = torch.cuda.Event()
     s_comp = torch.cuda.Stream()
     for e in ready + bend + [t_start]:
@@ -280,7 +291,7 @@ def run_dyo(args):
     def plan_next(desc, hist):
         """Predict + plan one step (the plan is double-buffered: this may run while the previous
         step's transitions are still migrating)."""
-        d.predict(desc, hist, 1, stream=s0.cuda_stream)
+        d.predict(desc, hist, B, stream=s0.cuda_stream)
         K = d.plan(stream=s0.cuda_stream)
         h2d = d2h = 0
         for j in range(K):
@@ -330,7 +341,7 @@ def run_dyo(args):
             dist.barrier()
 
     _log("warmup")
-    dev_inputs = lambda k: (desc_dev[k % nS: k % nS + 1], hist_dev)
+    dev_inputs = lambda k: (desc_dev[(k * B) % nS: (k * B) % nS + B], hist_dev)
     run_steps(args.warmup, 0, dev_inputs)
     barrier()
     d.timings(reset=True)
@@ -357,27 +368,49 @@ def run_dyo(args):
     hist_host = torch.from_numpy(hist_np).pin_memory() if hist_np is not None else None
     barrier()
     t0 = time.perf_counter()
-    host_inputs = lambda k: (desc_host[k % nS: k % nS + 1].numpy(), hist_host.numpy() if hist_host is not None else None)
+    host_inputs = lambda k: (desc_host[(k * B) % nS: (k * B) % nS + B].numpy(),
+                             hist_host.numpy() if hist_host is not None else None)
     run_steps(args.steps, args.warmup + args.steps, host_inputs)
     s1.synchronize()
     barrier()
     e2e_s = time.perf_counter() - t0
     e2e_bytes = None
 
+    peaks, peak_src = measured_peaks()
     _log("pilot loop")
-    # pilot latency: back-to-back predictions (device time per prediction) and kernel-only
-    d.timings(reset=True)
-    n_pred = 200
-    p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    p0.record(s0)
-    for i in range(n_pred):
-        d.predict(desc_dev[i % nS: i % nS + 1], hist_dev, 1, stream=s0.cuda_stream)
-    p1.record(s0)
-    p1.synchronize()
-    pred_us = p0.elapsed_time(p1) * 1e3 / n_pred
-    tp = d.timings(reset=True)
-    pilot_kernel_us = tp["pilot"]["ms"] * 1e3 / max(1, tp["pilot"]["launches"])
-    decode_us = tp["decode"]["ms"] * 1e3 / max(1, tp["decode"]["launches"])
+    # pilot latency at batch 1 (the cluster GEMV kernel, decode fused) and throughput at batch 64
+    # (K1-TC tensor-core kernel + two-phase decode): back-to-back predictions, device time
+    dp = Dyo(wl.budget, wl.align, wl.policy, max_batch=64, device=local, flags=DYO_F_TIMING | 4)
+    dp.load(wl)
+    desc64 = desc_dev[:64] if nS >= 64 else desc_dev.repeat((64 + nS - 1) // nS, 1)[:64]
+    hist64 = torch.from_numpy(np.tile(wl.hist_ids.astype(np.int32), (64, 1))).to(dev) if wl.h else None
+
+    def pilot_loop(ctx, n, bsz):
+        for i in range(3):
+            ctx.predict(desc64[:bsz] if bsz > 1 else desc_dev[i % nS: i % nS + 1],
+                        hist64[:bsz] if hist64 is not None else None, bsz, stream=s0.cuda_stream)
+        torch.cuda.synchronize()
+        ctx.timings(reset=True)
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        p0.record(s0)
+        for i in range(n):
+            if bsz == 1:
+                ctx.predict(desc_dev[i % nS: i % nS + 1], hist64[:1] if hist64 is not None else None, 1,
+                            stream=s0.cuda_stream)
+            else:
+                ctx.predict(desc64, hist64, bsz, stream=s0.cuda_stream)
+        p1.record(s0)
+        p1.synchronize()
+        t = ctx.timings(reset=True)
+        return (p0.elapsed_time(p1) * 1e3 / n, t["pilot"]["ms"] * 1e3 / max(1, t["pilot"]["launches"]),
+                t["decode"]["ms"] * 1e3 / max(1, t["decode"]["launches"]))
+    pred_us, pilot_kernel_us, decode_us = pilot_loop(dp, 200, 1)
+    b64_us, b64_kernel_us, b64_decode_us = pilot_loop(dp, 50, 64)
+    # K1-TC work per launch: 2 x 64 x sum(in x out) over the tensor-core stages, x3 for 3xTF32
+    sp = wl.pilot
+    macs = sum(ln * o for _, ln, o in sp.feature) + sum(i * o for i, o in sp.mlp) + sp.out_in * sp.O
+    tc_flop = 2.0 * 64 * macs
+    dp.close()
     _log("probe")
     probe = pcie_probe(torch)
 
@@ -390,7 +423,6 @@ def run_dyo(args):
         d.close()
         return
 
-    peaks, peak_src = measured_peaks()
     value = bytes_all / (ms_max * 1e-3) / 1e9
     # dominant kernel of the timed region among libdyo's kernels
     kern = {k: tm[k] for k in ("pilot", "decode", "plan", "copy_d2d", "copy_zc")}
@@ -452,6 +484,18 @@ def run_dyo(args):
         "pilot_us_per_prediction": round(pred_us, 3),
         "pilot_kernel_us": round(pilot_kernel_us, 3), "decode_kernels_us": round(decode_us, 3),
         "predictions_per_s": round(1e6 / pred_us, 1),
+        "pilot_batch64": {"us_per_batch": round(b64_us, 2), "us_per_prediction": round(b64_us / 64, 3),
+                          "predictions_per_s": round(64e6 / b64_us, 1),
+                          "pilot_kernel_us": round(b64_kernel_us, 2), "decode_kernels_us": round(b64_decode_us, 2),
+                          "kernel": "pilot_tc_kernel (tcgen05 kind::tf32, 3xTF32)" if wl.pilot.feature else
+                                    "pilot_kernel (cluster GEMV; T32 pilot has no tensor-core plan)",
+                          "tensor_roofline": ({"bound": "tensor", "achieved": round(3 * tc_flop / (b64_kernel_us * 1e-6) / 1e12, 4),
+                                               "peak": round(peaks["bf16_tflops"] / 2, 1), "unit": "TFLOP/s",
+                                               "frac": round(3 * tc_flop / (b64_kernel_us * 1e-6) / 1e12 / (peaks["bf16_tflops"] / 2), 6),
+                                               "flop_per_launch": 3 * tc_flop,
+                                               "peak_source": "TF32 dense = measured bf16 / 2 (guide's nominal ratio)",
+                                               "note": "latency-bound: 6 dependent layers of M=128 x N=64 tiles"}
+                                              if wl.pilot.feature else None)},
         "plan_us": round(plan_us, 2), "transitions_per_step": round(tot_K / args.steps, 2),
         "h2d_bytes_per_step": int(h2d_all / args.steps / world), "d2h_bytes_per_step": int(d2h_all / args.steps / world),
         "pcie": {"h2d_dma_gbs": round(h2d_link, 2) if h2d_link else None,

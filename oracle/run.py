@@ -44,3 +44,21 @@ def run(wl, n_steps, policy=None, branch_head=None):
         st = r.state
         table = r.pred.blocks
     return out
+
+
+def step_batch(wl, samples, state, group_table=(), branch_head=None, policy=None):
+    """A batch of predictions planned as one sequence (sample order, reading R13's per-sample
+    tensors: prediction b of the batch names its own tensors). Returns (preds, transitions,
+    state, error)."""
+    bh = wl.notes.get("branch_head", True) if branch_head is None else branch_head
+    preds = []
+    for b, smp in enumerate(samples):
+        x = E.encode(wl, wl.samples[smp], wl.hist_ids, group_table)
+        y = P.forward(wl.pilot, x, wl.nn_type)
+        preds.append(D.decode(wl, y, branch_head=bh, b=b))
+    Ws = [Wj for p in preds for Wj in p.W]
+    try:
+        trs, st = PL.plan(state, wl, Ws, policy)
+        return preds, trs, st, ""
+    except PL.BudgetError as e:
+        return preds, [], state, str(e)

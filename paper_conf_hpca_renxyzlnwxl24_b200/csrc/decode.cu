@@ -25,25 +25,32 @@ struct HeadSmem {
 
 __device__ __forceinline__ int* head_of(const PredDev& pd, int b) { return pd.head + (int64_t)b * pd.head_stride; }
 
-__global__ void __launch_bounds__(32)
+__global__ void __launch_bounds__(kDecThreads)
 decode_head_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t* __restrict__ hist_K) {
-  __shared__ HeadSmem S;
-  const int b = blockIdx.x, lane = threadIdx.x;
-  if (b == 0 && lane == 0) { pd.status[0] = 0; pd.status[1] = 0; }
-  const double* y = logits + (int64_t)b * a.O;
-  head_decode_warp(a, y, S.H, lane, b);
-  write_head(a, S.H, y, pd, b, hist_K);
+  extern __shared__ __align__(16) unsigned char dsm[];
+  HeadSmem& S = *reinterpret_cast<HeadSmem*>(dsm);
+  double* ys = reinterpret_cast<double*>(dsm + sizeof(HeadSmem));
+  const int b = blockIdx.x, tid = threadIdx.x, lane = tid & 31;
+  if (b == 0 && tid == 0) { pd.status[0] = 0; pd.status[1] = 0; }
+  // the logits into shared memory in one coalesced pass (the warp's head decode would otherwise
+  // chain dependent global round trips)
+  const double* yg = logits + (int64_t)b * a.O;
+  for (int i = tid; i < a.O; i += blockDim.x) ys[i] = yg[i];
+  __syncthreads();
+  if (tid < 32) head_decode_warp(a, ys, S.H, lane, b);
+  __syncthreads();
+  write_head(a, S.H, ys, pd, b, hist_K);
   int* h = head_of(pd, b);
   const int ns = a.n_sites, np = a.n_pieces, K = a.K_max;
-  if (lane == 0) { h[0] = S.H.L; h[1] = S.H.nk; h[2] = S.H.K; }
+  if (tid == 0) { h[0] = S.H.L; h[1] = S.H.nk; h[2] = S.H.K; }
   int* hc = h + 3;
-  for (int i = lane; i < ns; i += 32) hc[i] = S.H.choice[i];
+  for (int i = tid; i < ns; i += blockDim.x) hc[i] = S.H.choice[i];
   int* hs = hc + ns;
-  for (int i = lane; i <= np; i += 32) hs[i] = S.H.start[i];
+  for (int i = tid; i <= np; i += blockDim.x) hs[i] = S.H.start[i];
   int* hcum = hs + np + 1;
-  for (int i = lane; i < S.H.nk; i += 32) hcum[i] = S.H.cum[i];
+  for (int i = tid; i < S.H.nk; i += blockDim.x) hcum[i] = S.H.cum[i];
   int* hcnt = hcum + K + 1;
-  for (int i = lane; i < S.H.nk; i += 32) hcnt[i] = S.H.cntc[i];
+  for (int i = tid; i < S.H.nk; i += blockDim.x) hcnt[i] = S.H.cntc[i];
 }
 
 struct GroupSmem {
@@ -87,7 +94,14 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  decode_head_kernel<<<B, 32, 0, s>>>(a, logits, pd, hist_K_out);
+  const size_t hsm = sizeof(HeadSmem) + (size_t)a.O * sizeof(double);
+  static size_t hsm_set = 0;
+  if (hsm > hsm_set) {
+    cudaError_t e = cudaFuncSetAttribute(decode_head_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsm);
+    if (e != cudaSuccess) return e;
+    hsm_set = hsm;
+  }
+  decode_head_kernel<<<B, kDecThreads, hsm, s>>>(a, logits, pd, hist_K_out);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   decode_groups_kernel<<<B * a.K_max, kDecThreads, smem, s>>>(a, pd, hist_tab_out);

@@ -603,7 +603,8 @@ def make_lstm(seed=0, n_samples=128, batch=64, max_len=512, min_len=16, hidden=5
     return Workload("lstm", LSTM, program, tens, S_max, D_s, h, K_max,
                     budget=budget, align=256, policy=1, pilot=pilot, samples=samples,
                     hist_ids=np.array([-2, -1], np.int32), seed=seed,
-                    notes={"batch": batch, "max_len": max_len, "tasks": tasks})
+                    notes={"batch": batch, "max_len": max_len, "tasks": tasks,
+                           "oracle_batch": 4})   # bench.py's bounded CPU-oracle sample
 
 
 def _plant_lstm_heads(pilot, K_max, min_len, max_len, tasks, rows_per_step, rows_const):

@@ -454,8 +454,12 @@ def run_dyo(args):
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
             tr = json.load(f)
-        if roof["kernel"].split()[0] in tr:
-            roof["traffic"] = tr[roof["kernel"].split()[0]]
+        t = tr.get(roof["kernel"].split()[0])
+        if t and roof.get("alg_bytes_per_launch"):
+            # measured DRAM bytes per algorithmic byte (one ncu capture) x this run's bytes per launch
+            roof["traffic"] = round(t["dram_per_alg_byte"] * roof["alg_bytes_per_launch"])
+            roof["traffic_source"] = "profiles/ncu_traffic.json: dram/alg = %s over %d launches" % (
+                t["dram_per_alg_byte"], t["launches"])
     except OSError:
         pass
     shares = {k: round(v["ms"] / ms, 4) for k, v in tm.items()}

@@ -1261,6 +1261,18 @@ dyo_status launch_segs(dyo_ctx* ctx, int64_t first, cudaStream_t s, int grid, in
   return DYO_OK;
 }
 
+// DYO_COPY_LOG=<path>: one line per TMA copy launch with its algorithmic bytes (bytes moved);
+// tools/ncu_traffic.py pairs these with an ncu capture's per-launch DRAM bytes (same order).
+void log_copy_bytes(int64_t bytes) {
+  static FILE* f = nullptr;
+  static int init = 0;
+  if (!init) {
+    init = 1;
+    if (const char* e = getenv("DYO_COPY_LOG")) f = fopen(e, "w");
+  }
+  if (f) { fprintf(f, "%lld\n", (long long)bytes); fflush(f); }
+}
+
 // Device<->device copies of plan records [i0, i1) (R = one of the all-int64 record types):
 // record k copies rec.bytes from src_base + rec.<f_src> to dst_base + rec.<f_dst> - dst_bias;
 // f_late >= 0 selects the records with rec.late == late_val. The TMA copy kernel reads the
@@ -1300,6 +1312,7 @@ dyo_status d2d_records(dyo_ctx* ctx, const R* hrec, const R* drec, int i0, int i
   a.src_base = src_base; a.dst_base = dst_base; a.dst_bias = dst_bias;
   a.total = total;
   TScope ts(ctx, 3, s, bytes);
+  log_copy_bytes(bytes);
   CK(launch_copy_records(a, ctx->sm_count, s));
   ctx->ctr.n_kernels++;
   return DYO_OK;
@@ -1317,6 +1330,7 @@ dyo_status d2d_range(dyo_ctx* ctx, const char* src, char* dst, int64_t bytes, cu
   RecCopyArgs a{};
   a.src_base = src; a.dst_base = dst; a.total = bytes;
   TScope ts(ctx, 3, s, bytes);
+  log_copy_bytes(bytes);
   CK(launch_copy_records(a, ctx->sm_count, s));
   ctx->ctr.n_kernels++;
   return DYO_OK;

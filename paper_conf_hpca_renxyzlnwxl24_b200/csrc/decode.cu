@@ -22,6 +22,7 @@ constexpr int kDecTabCap2 = 8192;     // int32 words of decode tables staged in 
 struct HeadSmem {
   DecHead H;
 };
+constexpr size_t kHeadSmemBytes = (sizeof(HeadSmem) + 15) / 16 * 16;   // fp64 logits follow, 16-byte aligned
 
 __device__ __forceinline__ int* head_of(const PredDev& pd, int b) { return pd.head + (int64_t)b * pd.head_stride; }
 
@@ -29,7 +30,7 @@ __global__ void __launch_bounds__(kDecThreads)
 decode_head_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t* __restrict__ hist_K) {
   extern __shared__ __align__(16) unsigned char dsm[];
   HeadSmem& S = *reinterpret_cast<HeadSmem*>(dsm);
-  double* ys = reinterpret_cast<double*>(dsm + sizeof(HeadSmem));
+  double* ys = reinterpret_cast<double*>(dsm + kHeadSmemBytes);
   const int b = blockIdx.x, tid = threadIdx.x, lane = tid & 31;
   if (b == 0 && tid == 0) { pd.status[0] = 0; pd.status[1] = 0; }
   // the logits into shared memory in one coalesced pass (the warp's head decode would otherwise
@@ -79,7 +80,7 @@ decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab) {
   const int* hcnt = hcum + a.K_max + 1;
   const int nk = h[1];
   for (int i = threadIdx.x; i < nk; i += blockDim.x) { S.H.cum[i] = hcum[i]; S.H.cntc[i] = hcnt[i]; }
-  int* tabs = reinterpret_cast<int*>(dsm + sizeof(GroupSmem));
+  int* tabs = reinterpret_cast<int*>(dsm + (sizeof(GroupSmem) + 15) / 16 * 16);
   const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap2);   // ends with __syncthreads()
   build_group(A, S.H, S.G, pd, b, g, hist_tab);
 }
@@ -88,13 +89,13 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
   static bool attr = false;
-  const size_t smem = sizeof(GroupSmem) + (size_t)kDecTabCap2 * 4;
+  const size_t smem = (sizeof(GroupSmem) + 15) / 16 * 16 + (size_t)kDecTabCap2 * 4;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(decode_groups_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  const size_t hsm = sizeof(HeadSmem) + (size_t)a.O * sizeof(double);
+  const size_t hsm = kHeadSmemBytes + (size_t)a.O * sizeof(double);
   static size_t hsm_set = 0;
   if (hsm > hsm_set) {
     cudaError_t e = cudaFuncSetAttribute(decode_head_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsm);

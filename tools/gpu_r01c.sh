@@ -1,0 +1,17 @@
+#!/bin/bash
+# Session re-measure: GPU parity tests, bench (moe headline + lstm + af), ncu launch list,
+# per-launch DRAM traffic of the TMA copy kernel, and one ncu --set full capture of it.
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1; echo "build rc=$?"
+timeout 1200 python -m pytest tests -m gpu -q --timeout 400 -p no:cacheprovider > gpurun_out/gpu_tests.log 2>&1; echo "tests rc=$?"
+tail -3 gpurun_out/gpu_tests.log
+timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
+tail -c 2500 gpurun_out/bench.json
+for cfg in lstm af; do
+  timeout 600 python bench.py --config $cfg --no-cpu-baseline > gpurun_out/bench_$cfg.json 2> gpurun_out/bench_$cfg.err; echo "$cfg rc=$?"
+  tail -c 600 gpurun_out/bench_$cfg.json; tail -2 gpurun_out/bench_$cfg.err
+done
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 4000 --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline > gpurun_out/ncu_launch_bench.log 2>&1; echo "ncu launches rc=$?"
+DYO_COPY_LOG=gpurun_out/copy_log.txt timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -k regex:copy_records -c 400 --csv --log-file gpurun_out/copy_traffic.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline > gpurun_out/ncu_copy.log 2>&1; echo "ncu traffic rc=$?"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"copy_records|plan_kernel|pilot_kernel|pilot_tc" -s 30 -c 6 -o gpurun_out/prof_full -f python bench.py --steps 2 --warmup 1 --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1; echo "ncu full rc=$?"
+tail -2 gpurun_out/ncu_full.log

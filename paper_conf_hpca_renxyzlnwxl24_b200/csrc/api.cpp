@@ -30,6 +30,7 @@ struct dyo_ctx {
   int64_t H = 0;
   ArchDev ad{};
   std::vector<void*> arch_dev;     // device buffers of the arch / prediction / plan
+  struct Slab { std::vector<void*>* owner = nullptr; char* p = nullptr; size_t left = 0; } slab[2];
   PilotDev pdv{};
   const PilotDev* pdv_dev = nullptr;    // device copy of pdv
   std::vector<void*> pilot_dev;
@@ -125,11 +126,37 @@ dyo_status fail(dyo_ctx* c, dyo_status s, const char* fmt, ...) {
 
 template <class T>
 dyo_status dalloc(dyo_ctx* ctx, std::vector<void*>& owner, T** p, size_t n) {
-  void* v = nullptr;
+  // Small buffers are carved (256-byte aligned) from 16 MiB slabs owned by `owner`, so the
+  // kernels' many small tables share a handful of pages (fewer TLB misses on the dependent
+  // lookups of the decode and planner); large buffers get their own allocation.
+  constexpr size_t kSlab = 16u << 20, kSmall = 2u << 20;
   size_t bytes = std::max<size_t>(n * sizeof(T), 16);
-  CK(cudaMalloc(&v, bytes));
+  void* v = nullptr;
+  if (bytes <= kSmall) {
+    dyo_ctx::Slab* sl = nullptr;
+    for (auto& c : ctx->slab)
+      if (c.owner == &owner) sl = &c;
+    if (!sl) {
+      sl = ctx->slab[0].owner == nullptr || ctx->slab[0].owner == &owner ? &ctx->slab[0] : &ctx->slab[1];
+      *sl = dyo_ctx::Slab{};
+      sl->owner = &owner;
+    }
+    bytes = (bytes + 255) / 256 * 256;
+    if (sl->left < bytes) {
+      void* blk = nullptr;
+      CK(cudaMalloc(&blk, kSlab));
+      owner.push_back(blk);
+      sl->p = static_cast<char*>(blk);
+      sl->left = kSlab;
+    }
+    v = sl->p;
+    sl->p += bytes;
+    sl->left -= bytes;
+  } else {
+    CK(cudaMalloc(&v, bytes));
+    owner.push_back(v);
+  }
   CK(cudaMemset(v, 0, bytes));
-  owner.push_back(v);
   *p = static_cast<T*>(v);
   return DYO_OK;
 }
@@ -147,6 +174,12 @@ dyo_status dupload(dyo_ctx* ctx, std::vector<void*>& owner, const T** p, const s
 void free_list(std::vector<void*>& v) {
   for (void* p : v) cudaFree(p);
   v.clear();
+}
+// free an owner's buffers and forget its slab (the next small allocation starts a new one)
+void free_owned(dyo_ctx* ctx, std::vector<void*>& v) {
+  free_list(v);
+  for (auto& c : ctx->slab)
+    if (c.owner == &v) c = dyo_ctx::Slab{};
 }
 
 int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
@@ -524,8 +557,8 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (!ctx) return DYO_E_INVAL;
   cudaSetDevice(ctx->device);
   cudaDeviceSynchronize();
-  free_list(ctx->arch_dev);
-  free_list(ctx->pilot_dev);
+  free_owned(ctx, ctx->arch_dev);
+  free_owned(ctx, ctx->pilot_dev);
   free_plan_host(ctx);
   if (ctx->host_pool) cudaFreeHost(ctx->host_pool);
   if (ctx->h_logits) cudaFreeHost(ctx->h_logits);
@@ -550,7 +583,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   if (!ctx || !A) return DYO_E_INVAL;
   CK(cudaSetDevice(ctx->device));
   CK(cudaDeviceSynchronize());
-  free_list(ctx->arch_dev);
+  free_owned(ctx, ctx->arch_dev);
   free_plan_host(ctx);
   if (ctx->host_pool) { cudaFreeHost(ctx->host_pool); ctx->host_pool = nullptr; }
   ctx->arch_ok = false;
@@ -881,7 +914,7 @@ dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   if (w->O < ctx->O_min) return fail(ctx, DYO_E_INVAL, "pilot O=%d < %d", w->O, ctx->O_min);
   if (w->n_mlp < 1 || w->n_mlp > kMaxLayers || w->n_feature < 0 || w->n_feature > 8)
     return fail(ctx, DYO_E_INVAL, "pilot: layer counts");
-  free_list(ctx->pilot_dev);
+  free_owned(ctx, ctx->pilot_dev);
   PilotDev& p = ctx->pdv;
   p = PilotDev{};
   p.F = w->F;

@@ -60,7 +60,7 @@ struct GroupSmem {
 };
 
 __global__ void __launch_bounds__(kDecThreads)
-decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab) {
+decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int tab_cap) {
   extern __shared__ __align__(16) unsigned char dsm[];
   GroupSmem& S = *reinterpret_cast<GroupSmem*>(dsm);
   const int b = blockIdx.x / a.K_max, g = blockIdx.x % a.K_max;
@@ -81,19 +81,20 @@ decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab) {
   const int nk = h[1];
   for (int i = threadIdx.x; i < nk; i += blockDim.x) { S.H.cum[i] = hcum[i]; S.H.cntc[i] = hcnt[i]; }
   int* tabs = reinterpret_cast<int*>(dsm + (sizeof(GroupSmem) + 15) / 16 * 16);
-  const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap2);   // ends with __syncthreads()
+  const ArchDev A = stage_decode_tables(a, tabs, tab_cap);   // ends with __syncthreads()
   build_group(A, S.H, S.G, pd, b, g, hist_tab);
 }
 
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
-  static bool attr = false;
-  const size_t smem = (sizeof(GroupSmem) + 15) / 16 * 16 + (size_t)kDecTabCap2 * 4;
-  if (!attr) {
+  const int tab_cap = dec_table_words(a, kDecTabCap2);
+  const size_t smem = (sizeof(GroupSmem) + 15) / 16 * 16 + (size_t)tab_cap * 4;
+  static size_t smem_set = 0;
+  if (smem > smem_set) {
     cudaError_t e = cudaFuncSetAttribute(decode_groups_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    attr = true;
+    smem_set = smem;
   }
   const size_t hsm = kHeadSmemBytes + (size_t)a.O * sizeof(double);
   static size_t hsm_set = 0;
@@ -105,7 +106,7 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
   decode_head_kernel<<<B, kDecThreads, hsm, s>>>(a, logits, pd, hist_K_out);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  decode_groups_kernel<<<B * a.K_max, kDecThreads, smem, s>>>(a, pd, hist_tab_out);
+  decode_groups_kernel<<<B * a.K_max, kDecThreads, smem, s>>>(a, pd, hist_tab_out, tab_cap);
   return cudaGetLastError();
 }
 

@@ -20,6 +20,11 @@
 
 namespace dyo {
 
+// debug phase stamps of the decode (SM clock; one CTA of the fused pilot epilogue)
+static __device__ unsigned long long g_dec_stamp[8];
+static __device__ int g_dec_stamp_on;
+#define DSTAMP(i) do { if (g_dec_stamp_on && blockIdx.x == 0 && threadIdx.x == 0) g_dec_stamp[i] = (unsigned long long)clock64(); } while (0)
+
 constexpr int kMaxPieces = 1024;
 constexpr int kRecCap = 2048;          // access records per group before deduplication
 
@@ -32,10 +37,14 @@ struct DecHead {
 };
 
 struct DecGroup {
-  uint64_t key[kRecCap];
-  uint64_t key2[kRecCap];
+  int32_t rec_t[kRecCap];              // access records in row order (position = index)
+  int32_t rec_m[kRecCap];              // mode bits (R = 1, W = 2)
+  int32_t first[kRecCap];              // 1 at the first position of each tensor, then its scan
+  int32_t ht_key[2 * kRecCap];         // open-addressing table: tensor -> first position, mode union
+  int32_t ht_pos[2 * kRecCap];
+  int32_t ht_mode[2 * kRecCap];
   int warp_tmp[32];
-  long long sum_tmp[32];
+  long long sig_w[32][9];              // per-warp signature partial sums
   unsigned long long sig[9];
   int n, u;
 };
@@ -43,29 +52,128 @@ struct DecGroup {
 // Copy the small decode tables (sites, arms, pieces) into shared memory `buf` (int32 words,
 // capacity cap) and return an ArchDev whose pointers refer to the copies; tables that do not
 // fit stay in global memory. All threads of the block call it; ends with __syncthreads().
-__device__ __forceinline__ ArchDev stage_decode_tables(const ArchDev& a, int* buf, int cap) {
-  const int n_arms = a.n_arms;
-  ArchDev s = a;
+// One flat pass over all tables with every load of a thread issued before its stores, so the
+// copy costs one global round trip instead of one per table.
+// int32 words stage_decode_tables needs for every table (capped; host and device)
+__host__ __device__ inline int dec_table_words(const ArchDev& a, int cap) {
+  const int need = 6 * a.n_sites + 4 * a.n_pieces + 2 * a.n_arms;
+  return need < cap ? need : cap;
+}
+
+// The twelve small decode tables (sites, pieces, arms) in a fixed order; host and device.
+constexpr int kDecTabs = 12;
+__host__ __device__ inline const int32_t* dec_table(const ArchDev& a, int k, int* len) {
+  switch (k) {
+    case 0: *len = a.n_sites; return a.site_logit;
+    case 1: *len = a.n_sites; return a.site_nch;
+    case 2: *len = a.n_sites; return a.site_tie;
+    case 3: *len = a.n_sites; return a.site_lo;
+    case 4: *len = a.n_sites; return a.site_arm_ptr;
+    case 5: *len = a.n_sites; return a.site_rev;
+    case 6: *len = a.n_pieces; return a.piece_kind;
+    case 7: *len = a.n_pieces; return a.piece_a;
+    case 8: *len = a.n_pieces; return a.piece_b;
+    case 9: *len = a.n_pieces; return a.piece_c;
+    case 10: *len = a.n_arms; return a.arm_nops;
+    default: *len = a.n_arms; return a.arm_first_op;
+  }
+}
+// int32 words of the prefetched table region: every table padded to 16 bytes
+__host__ __device__ inline int dec_table_region_words(const ArchDev& a) {
+  int w = 0;
+  for (int k = 0; k < kDecTabs; ++k) {
+    int n = 0;
+    dec_table(a, k, &n);
+    w += (n + 3) / 4 * 4;
+  }
+  return w;
+}
+// One thread: bulk-copy (TMA) every table into `region` (16-byte aligned shared memory) and arm
+// `bar` with the bytes. The tables are 256-byte aligned slab carvings, so rounding a copy up to
+// 16 bytes stays inside the allocation.
+__device__ __forceinline__ void prefetch_dec_tables(const ArchDev& a, int* region, uint64_t* bar) {
+  uint32_t bytes = 0;
+  for (int k = 0; k < kDecTabs; ++k) {
+    int n = 0;
+    dec_table(a, k, &n);
+    bytes += (uint32_t)((n + 3) / 4 * 16);
+  }
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(bar)),
+               "r"(bytes) : "memory");
   int off = 0;
-  auto take = [&](const int32_t* src, int n) -> const int32_t* {
-    if (off + n > cap) return src;
-    int* dst = buf + off;
-    for (int i = threadIdx.x; i < n; i += blockDim.x) dst[i] = src[i];
-    off += n;
-    return dst;
-  };
-  s.site_logit = take(a.site_logit, a.n_sites);
-  s.site_nch = take(a.site_nch, a.n_sites);
-  s.site_tie = take(a.site_tie, a.n_sites);
-  s.site_lo = take(a.site_lo, a.n_sites);
-  s.site_arm_ptr = take(a.site_arm_ptr, a.n_sites);
-  s.site_rev = take(a.site_rev, a.n_sites);
-  s.piece_kind = take(a.piece_kind, a.n_pieces);
-  s.piece_a = take(a.piece_a, a.n_pieces);
-  s.piece_b = take(a.piece_b, a.n_pieces);
-  s.piece_c = take(a.piece_c, a.n_pieces);
-  s.arm_nops = take(a.arm_nops, n_arms);
-  s.arm_first_op = take(a.arm_first_op, n_arms);
+  for (int k = 0; k < kDecTabs; ++k) {
+    int n = 0;
+    const int32_t* src = dec_table(a, k, &n);
+    const uint32_t nb = (uint32_t)((n + 3) / 4 * 16);
+    if (nb)
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                       (uint32_t)__cvta_generic_to_shared(region + off)),
+                   "l"(src), "r"(nb), "r"((uint32_t)__cvta_generic_to_shared(bar))
+                   : "memory");
+    off += (n + 3) / 4 * 4;
+  }
+}
+// The ArchDev view whose decode tables point into the prefetched region.
+__device__ __forceinline__ ArchDev dec_tables_view(const ArchDev& a, const int* region) {
+  ArchDev s = a;
+  int off = 0, n = 0;
+  auto nx = [&](int k) { dec_table(a, k, &n); const int32_t* p = region + off; off += (n + 3) / 4 * 4; return p; };
+  s.site_logit = nx(0); s.site_nch = nx(1); s.site_tie = nx(2); s.site_lo = nx(3); s.site_arm_ptr = nx(4);
+  s.site_rev = nx(5); s.piece_kind = nx(6); s.piece_a = nx(7); s.piece_b = nx(8); s.piece_c = nx(9);
+  s.arm_nops = nx(10); s.arm_first_op = nx(11);
+  return s;
+}
+
+__device__ __forceinline__ ArchDev stage_decode_tables(const ArchDev& a, int* buf, int cap) {
+  constexpr int NTAB = 12;
+  const int32_t* src[NTAB] = {a.site_logit, a.site_nch, a.site_tie, a.site_lo, a.site_arm_ptr, a.site_rev,
+                              a.piece_kind, a.piece_a, a.piece_b, a.piece_c, a.arm_nops, a.arm_first_op};
+  const int len[NTAB] = {a.n_sites, a.n_sites, a.n_sites, a.n_sites, a.n_sites, a.n_sites,
+                         a.n_pieces, a.n_pieces, a.n_pieces, a.n_pieces, a.n_arms, a.n_arms};
+  int beg[NTAB];
+  int off = 0, nt = 0;
+  bool fits = true;
+#pragma unroll
+  for (int k = 0; k < NTAB; ++k) {       // tables are staged in order while they fit
+    beg[k] = off;
+    fits = fits && (off + len[k] <= cap);
+    if (fits) { off += len[k]; nt = k + 1; }
+  }
+  const int NT = blockDim.x;
+  for (int i0 = 0; i0 < off; i0 += 8 * NT) {
+    int v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int i = i0 + u * NT + (int)threadIdx.x;
+      v[u] = 0;
+      if (i < off) {
+        const int32_t* ptr = src[0];
+        int b0 = 0;
+#pragma unroll
+        for (int q = 1; q < NTAB; ++q)
+          if (q < nt && i >= beg[q]) { ptr = src[q]; b0 = beg[q]; }
+        v[u] = __ldg(ptr + (i - b0));
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int i = i0 + u * NT + (int)threadIdx.x;
+      if (i < off) buf[i] = v[u];
+    }
+  }
+  ArchDev s = a;
+  s.site_logit = nt > 0 ? buf + beg[0] : a.site_logit;
+  s.site_nch = nt > 1 ? buf + beg[1] : a.site_nch;
+  s.site_tie = nt > 2 ? buf + beg[2] : a.site_tie;
+  s.site_lo = nt > 3 ? buf + beg[3] : a.site_lo;
+  s.site_arm_ptr = nt > 4 ? buf + beg[4] : a.site_arm_ptr;
+  s.site_rev = nt > 5 ? buf + beg[5] : a.site_rev;
+  s.piece_kind = nt > 6 ? buf + beg[6] : a.piece_kind;
+  s.piece_a = nt > 7 ? buf + beg[7] : a.piece_a;
+  s.piece_b = nt > 8 ? buf + beg[8] : a.piece_b;
+  s.piece_c = nt > 9 ? buf + beg[9] : a.piece_c;
+  s.arm_nops = nt > 10 ? buf + beg[10] : a.arm_nops;
+  s.arm_first_op = nt > 11 ? buf + beg[11] : a.arm_first_op;
   __syncthreads();
   return s;
 }
@@ -97,6 +205,7 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
     if (n != 0) H.cntc[nk + __popc(m & ((1u << lane) - 1))] = n;
     nk += __popc(m);
   }
+  DSTAMP(0);
   // 2. branch head: argmax per free site (lowest index on ties), then tied sites; without a
   //    branch head the choices are the host traversal's
   if (a.forced) {
@@ -119,6 +228,7 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
   for (int i = lane; i < a.n_sites && !a.forced; i += 32)
     if (a.site_logit[i] < 0) H.choice[i] = H.choice[a.site_tie[i]];   // tie targets are free sites
   __syncwarp();
+  DSTAMP(1);
   // 3. piece lengths -> exclusive scan -> piece starts (R2)
   int carry = 0;
   for (int p0 = 0; p0 < a.n_pieces; p0 += 32) {
@@ -141,6 +251,7 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
     carry += __shfl_sync(0xffffffffu, inc, 31);
   }
   const int L = carry;
+  DSTAMP(2);
   // 4. cut (R4): group starts = exclusive scan of the compacted counts; K = groups inside the path
   __syncwarp();
   int c2 = 0, K = 0;
@@ -205,8 +316,6 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
     pd.grp[((int64_t)b * a.K_max + g) * 2] = s;
     pd.grp[((int64_t)b * a.K_max + g) * 2 + 1] = e;
   }
-  if (tid < 9) G.sig[tid] = 0;
-  __syncthreads();
   // rows split in contiguous chunks; per-thread access counts and signature sums
   const int chunk = (nrows + NT - 1) / NT;
   const int rs = s + tid * chunk, re = min(e, rs + chunk);
@@ -220,24 +329,24 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
       for (int k = 0; k < 9; ++k) sg[k] += a.op_sig[(int64_t)op * 9 + k];
     }
   }
-  // block sums of the nine signature columns (no 64-bit shared atomics: CAS spin loops)
+  // the nine signature sums: warp shuffles, then one pass over the per-warp partials (a single
+  // barrier, shared with the scan below; no 64-bit shared atomics: CAS spin loops)
+  const int nw = (NT + 31) >> 5;
+#pragma unroll
   for (int k = 0; k < 9; ++k) {
-    const long long v = block_sum64(sg[k], G.sum_tmp);
-    if (tid == 0) G.sig[k] = (unsigned long long)v;
+    long long v = sg[k];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if (lane == 0) G.sig_w[warp][k] = v;
   }
+  DSTAMP(3);
   int total = 0;
-  int pos = block_scan(cnt, G.warp_tmp, &total);   // includes __syncthreads (sig sums done)
-  if (tid == 0) {
-    int32_t* bv = pd.blocks + ((int64_t)b * a.K_max + g) * 10;
-    int32_t* hv = hist_tab + ((int64_t)b * a.K_max + g) * 10;
-    const int c0 = min(nrows, kSat);
-    bv[0] = c0;
-    hv[0] = c0;
-    for (int k = 0; k < 9; ++k) {
-      const int v = (int)min((long long)G.sig[k], (long long)kSat);
-      bv[1 + k] = v;
-      hv[1 + k] = v;
-    }
+  int pos = block_scan(cnt, G.warp_tmp, &total);   // its barriers also publish sig_w
+  DSTAMP(4);
+  if (tid < 9) {
+    long long v = 0;
+    for (int w = 0; w < nw; ++w) v += G.sig_w[w][tid];
+    G.sig[tid] = (unsigned long long)v;
   }
   int32_t* ent_n = pd.ent_n + (int64_t)b * a.K_max + g;
   int2* ent = pd.ent + ((int64_t)b * a.K_max + g) * kEntCap;
@@ -252,19 +361,42 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
     const int op = row_op(a, H, r, &it);
     if (op < 0) continue;
     for (int q = a.acc_ptr[op]; q < a.acc_ptr[op + 1]; ++q, ++pos) {
-      const uint32_t t = (uint32_t)(a.acc_t[q] + a.acc_s[q] * it + a.acc_sb[q] * b);   // R13 (validated at load)
-      G.key[pos] = ((uint64_t)t << 32) | ((uint64_t)pos << 2) | (uint64_t)a.acc_m[q];
+      G.rec_t[pos] = a.acc_t[q] + a.acc_s[q] * it + a.acc_sb[q] * b;   // R13 (validated at load)
+      G.rec_m[pos] = a.acc_m[q];
     }
   }
+  // hash-table size (power of two >= 2n) and its initialisation ride the same barrier
+  int hsz = 64;
+  while (hsz < 2 * n) hsz <<= 1;
+  if (n > 64) {
+    for (int i = tid; i < hsz; i += NT) { G.ht_key[i] = -1; G.ht_pos[i] = 0x7fffffff; G.ht_mode[i] = 0; }
+    for (int i = tid; i < n; i += NT) G.first[i] = 0;
+  }
   __syncthreads();
+  if (tid == 0) {
+    int32_t* bv = pd.blocks + ((int64_t)b * a.K_max + g) * 10;
+    int32_t* hv = hist_tab + ((int64_t)b * a.K_max + g) * 10;
+    const int c0 = min(nrows, kSat);
+    bv[0] = c0;
+    hv[0] = c0;
+    for (int k = 0; k < 9; ++k) {
+      const int v = (int)min((long long)G.sig[k], (long long)kSat);
+      bv[1 + k] = v;
+      hv[1 + k] = v;
+    }
+  }
+  DSTAMP(5);
   if (n <= 64) {
     // ---- warp path: registers + shuffles, no block barriers ----
     if (warp == 0) {
-      uint64_t x = lane < n ? G.key[lane] : ~0ull;
-      uint64_t z = lane + 32 < n ? G.key[lane + 32] : ~0ull;
+      uint64_t x = lane < n ? ((uint64_t)(uint32_t)G.rec_t[lane] << 32) | ((uint64_t)lane << 2) | (uint64_t)G.rec_m[lane] : ~0ull;
+      uint64_t z = lane + 32 < n ? ((uint64_t)(uint32_t)G.rec_t[lane + 32] << 32) | ((uint64_t)(lane + 32) << 2) |
+                                       (uint64_t)G.rec_m[lane + 32]
+                                 : ~0ull;
       warp_sort64(x, z, lane);
-      G.key[lane] = x;
-      G.key[lane + 32] = z;
+      uint64_t* key = reinterpret_cast<uint64_t*>(G.ht_key);   // scratch (unused on this path)
+      key[lane] = x;
+      key[lane + 32] = z;
       __syncwarp();
       uint64_t o[2];
 #pragma unroll
@@ -272,12 +404,12 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
         const int i = lane + 32 * h;
         o[h] = ~0ull;
         if (i < n) {
-          const uint32_t t = (uint32_t)(G.key[i] >> 32);
-          if (i == 0 || (uint32_t)(G.key[i - 1] >> 32) != t) {
-            const uint32_t p0 = (uint32_t)(G.key[i] & 0xffffffffu) >> 2;
-            const uint32_t m0 = (uint32_t)G.key[i] & 3u;
+          const uint32_t t = (uint32_t)(key[i] >> 32);
+          if (i == 0 || (uint32_t)(key[i - 1] >> 32) != t) {
+            const uint32_t p0 = (uint32_t)(key[i] & 0xffffffffu) >> 2;
+            const uint32_t m0 = (uint32_t)key[i] & 3u;
             uint32_t mu = m0;
-            for (int k = i + 1; k < n && (uint32_t)(G.key[k] >> 32) == t; ++k) mu |= (uint32_t)G.key[k] & 3u;
+            for (int k = i + 1; k < n && (uint32_t)(key[k] >> 32) == t; ++k) mu |= (uint32_t)key[k] & 3u;
             o[h] = ((uint64_t)p0 << 32) | ((uint64_t)t << 3) | (mu << 1) | (m0 & 1u);
           }
         }
@@ -297,35 +429,44 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
     __syncthreads();
     return;
   }
-  // ---- block path ----
-  block_sort_u64(G.key, n);
-  int np2 = 1;
-  while (np2 < n) np2 <<= 1;
-  for (int i = tid; i < np2; i += NT) G.key2[i] = ~0ull;
-  __syncthreads();
+  // ---- block path: tensor -> (first position, mode union) in an open-addressing table
+  //      (32-bit shared atomics: CAS / min / or, order-independent), then the first positions
+  //      are flagged and one exclusive scan gives every tensor its slot in first-access order ----
+  const int mask = hsz - 1;
   for (int i = tid; i < n; i += NT) {
-    const uint32_t t = (uint32_t)(G.key[i] >> 32);
-    if (i > 0 && (uint32_t)(G.key[i - 1] >> 32) == t) continue;
-    const uint32_t p0 = (uint32_t)(G.key[i] & 0xffffffffu) >> 2;
-    const uint32_t m0 = (uint32_t)G.key[i] & 3u;
-    uint32_t mu = m0;
-    for (int k = i + 1; k < n && (uint32_t)(G.key[k] >> 32) == t; ++k) mu |= (uint32_t)G.key[k] & 3u;
-    G.key2[i] = ((uint64_t)p0 << 32) | ((uint64_t)t << 3) | (mu << 1) | (m0 & 1u);
+    const int t = G.rec_t[i];
+    int h = (int)(((uint32_t)t * 2654435761u) >> 7) & mask;
+    for (;;) {
+      const int old = atomicCAS(&G.ht_key[h], -1, t);
+      if (old == -1 || old == t) {
+        atomicMin(&G.ht_pos[h], i);
+        atomicOr(&G.ht_mode[h], G.rec_m[i]);
+        break;
+      }
+      h = (h + 1) & mask;
+    }
   }
   __syncthreads();
-  block_sort_u64(G.key2, n);
-  int flag = 0;
-  for (int i = tid; i < n; i += NT) flag += G.key2[i] != ~0ull ? 1 : 0;
+  for (int h = tid; h < hsz; h += NT)
+    if (G.ht_key[h] >= 0) G.first[G.ht_pos[h]] = h + 1;     // slot + 1 at the tensor's first position
+  __syncthreads();
   int u = 0;
-  block_scan(flag, G.warp_tmp, &u);
+  for (int i0 = 0; i0 < n; i0 += NT) {
+    const int i = i0 + tid;
+    const int f = i < n ? G.first[i] : 0;
+    int tot = 0;
+    const int idx = u + block_scan(f ? 1 : 0, G.warp_tmp, &tot);
+    if (f && idx < kEntCap) {
+      const int h = f - 1;
+      const int m0 = G.rec_m[i];
+      ent[idx] = make_int2(G.ht_key[h], (G.ht_mode[h] & 3) | ((m0 & 1) << 2));
+    }
+    u += tot;
+  }
   if (u > kEntCap) {
     if (tid == 0) { *ent_n = 0; atomicCAS(&pd.status[0], 0, DYO_E_CAPACITY); pd.status[1] = u; }
     __syncthreads();
     return;
-  }
-  for (int i = tid; i < u; i += NT) {
-    const uint32_t lo = (uint32_t)(G.key2[i] & 0xffffffffu);
-    ent[i] = make_int2((int)(lo >> 3), (int)(((lo >> 1) & 3u) | ((lo & 1u) << 2)));
   }
   if (tid == 0) *ent_n = u;
   __syncthreads();

@@ -23,6 +23,7 @@
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <cstdlib>
 
 #include "decode_dev.cuh"
 #include "pilot_common.cuh"
@@ -73,6 +74,9 @@ struct StagePlan {
   int Bs;                 // samples per cluster
   int act_off;            // byte offset of the activation buffers
   int fuse_decode;        // 1: this kernel also decodes its samples (epilogue)
+  int dec_tab_cap;        // int32 words of decode tables staged in smem by the epilogue
+  int tab_off;            // >= 0: byte offset of the decode tables prefetched at launch (fused decode)
+  int push_logits;        // 1: the output stage pushes its logits to every CTA (fused decode, C > 1)
   int st_off[4 + kMaxLayers];
   int rpc[4 + kMaxLayers];      // rows per CTA of each stage
   int gsh[4 + kMaxLayers];      // log2 of the threads per row (k-split) of each stage
@@ -123,15 +127,19 @@ __device__ __forceinline__ double warp_reduce4(double a0, double a1, double a2, 
 // With fuse_decode the weight region is reused for the decode (DecHead / DecGroup) afterwards.
 template <int BS>
 __global__ void __launch_bounds__(kPilotThreads)
-pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pdev, const __grid_constant__ StagePlan sp,
+pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pdev, const __grid_constant__ StagePlan spc,
              const float* __restrict__ feat, const int64_t* __restrict__ desc, const int32_t* __restrict__ hist,
              const int32_t* __restrict__ hist_tab, const int32_t* __restrict__ hist_K, int hist_B, int B,
              double* __restrict__ logits64, float* __restrict__ logits32, PredDev pd,
              int32_t* __restrict__ hist_tab_out, int32_t* __restrict__ hist_K_out) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   __shared__ __align__(16) PilotDev p;
+  // the launch plan in shared memory: dynamically indexed parameter-bank reads (st_off[si], ...)
+  // would each cost a dependent constant-cache miss per stage
+  __shared__ __align__(16) StagePlan sp;
   const int tid = threadIdx.x;
   const int stamp_on = g_stamp_on;
+  if (blockIdx.x == 0 && tid == 0) g_dec_stamp_on = stamp_on;
   stamp(0, stamp_on);
   {
     // descriptors: one round trip of 16-byte loads (dynamic indexing of the parameter bank in
@@ -139,20 +147,24 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
     const int4* src = reinterpret_cast<const int4*>(pdev);
     int4* dst = reinterpret_cast<int4*>(&p);
     for (int i = tid; i < (int)(sizeof(PilotDev) / 16); i += blockDim.x) dst[i] = src[i];
+    const int* ps = reinterpret_cast<const int*>(&spc);
+    int* pd2 = reinterpret_cast<int*>(&sp);
+    for (int i = tid; i < (int)(sizeof(StagePlan) / 4); i += blockDim.x) pd2[i] = ps[i];
   }
-  const int C = sp.C;
+  const int C = spc.C;
   const int r = C > 1 ? (int)cg::this_cluster().block_rank() : 0;
   const int cluster_id = blockIdx.x / C;
   const int b0 = cluster_id * BS;
   const int nb = min(BS, B - b0);
   uint64_t* wbar = reinterpret_cast<uint64_t*>(smem_raw);           // one per stage
   uint64_t* abar = wbar + (4 + kMaxLayers);                         // two activation buffers
-  double* act = reinterpret_cast<double*>(smem_raw + sp.act_off);
+  double* act = reinterpret_cast<double*>(smem_raw + spc.act_off);
   if (blockIdx.x == 0 && tid == 0) { pd.status[0] = 0; pd.status[1] = 0; }
   if (tid == 0) {
     for (int i = 0; i < 4 + kMaxLayers; ++i) mbar_init(&wbar[i], 1);
     mbar_init(&abar[0], 1);
     mbar_init(&abar[1], 1);
+    mbar_init(&abar[2], 1);                                       // decode tables
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();                       // descriptors + barrier inits visible in the CTA
@@ -186,6 +198,8 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
       lr0 = lr1;
     }
   }
+  // the decode tables ride the same launch-time TMA stream (used only by the epilogue)
+  if (sp.tab_off >= 0 && tid == 32) prefetch_dec_tables(a, reinterpret_cast<int*>(smem_raw + sp.tab_off), &abar[2]);
   stamp(1, stamp_on);
   // ---- 1. the sub-batch's feature vectors into buf[0] (overlaps the weight stream)
   for (int bb = 0; bb < nb; ++bb) {
@@ -220,7 +234,7 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
     // inputs of this stage: the peers' rows of stage si-1 (arrived via st.async) + own rows
     if (si > 0 && C > 1) mbar_wait(&abar[cin], ((si - 1) >> 1) & 1);
     // arm the barrier of the NEXT stage's inputs (this stage's outputs) before any peer can finish
-    if (si + 1 < p.n_stages && si > 0 && C > 1 && tid == 0 && !last) {
+    if (si > 0 && C > 1 && tid == 0 && (!last || sp.push_logits)) {
       const int own = max(0, r1 - r0);
       mbar_expect_tx(&abar[cout], (uint32_t)((st.rows - own) * nb * 8));
     }
@@ -324,6 +338,12 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
             logits64[(int64_t)(b0 + bb) * p.O + row] = v;
             if (logits32) logits32[(int64_t)(b0 + bb) * p.O + row] = (float)v;
           }
+          if (sp.push_logits) {              // every CTA's decode reads the logits from its own smem
+            if (part == 0) out[bb * W + row] = v;
+            const uint32_t laddr = out_s + (uint32_t)((bb * W + row) * 8);
+            for (int c = part; c < C; c += G)
+              if (c != r) st_async_b64(mapa_u32(laddr, c), v, mapa_u32(abar_s[cout], c));
+          }
         } else {
           if (part == 0) out[bb * W + row] = v;
           if (C > 1) {
@@ -339,23 +359,43 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
   }
   // ---- 2. fused decode epilogue: CTA r of the cluster decodes groups g == r (mod C) ----
   if (!sp.fuse_decode) return;
-  if (C > 1) cg::this_cluster().sync();   // every CTA's logits written (release/acquire, cluster scope)
-  else __syncthreads();
+  const int cl = p.n_stages & 1;           // buffer holding the output stage's values
+  if (sp.push_logits) {
+    mbar_wait(&abar[cl], ((p.n_stages - 1) >> 1) & 1);   // the peers' logits rows arrived
+    __syncthreads();                                       // own rows visible to every warp
+  } else if (C > 1) {
+    cg::this_cluster().sync();             // every CTA's logits written (release/acquire, cluster scope)
+  } else {
+    __syncthreads();
+  }
+  stamp(28, stamp_on);
   DecHead& H = *reinterpret_cast<DecHead*>(smem_raw + ((2 * (4 + kMaxLayers) + 2) * 8 + 127) / 128 * 128);
   DecGroup& Gs = *reinterpret_cast<DecGroup*>(reinterpret_cast<unsigned char*>(&H) + ((sizeof(DecHead) + 127) / 128 * 128));
   double* ys = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(&Gs) + ((sizeof(DecGroup) + 127) / 128 * 128));
   int* tabs = reinterpret_cast<int*>(ys + ((p.O + 15) / 16) * 16);
-  const ArchDev A = stage_decode_tables(a, tabs, kDecTabCap);
+  ArchDev A;
+  if (sp.tab_off >= 0) {
+    mbar_wait(&abar[2], 0);
+    A = dec_tables_view(a, reinterpret_cast<const int*>(smem_raw + sp.tab_off));
+  } else {
+    A = stage_decode_tables(a, tabs, sp.dec_tab_cap);
+  }
+  stamp(29, stamp_on);
   for (int bb = 0; bb < nb; ++bb) {
     const int b = b0 + bb;
     if (r >= a.K_max && r != 0) continue;
     const double* y = logits64 + (int64_t)b * p.O;
-    __syncthreads();
-    // the logits into shared memory in one coalesced pass (the argmax loops would otherwise
-    // chain dependent L2 round trips)
-    for (int i = tid; i < p.O; i += blockDim.x) ys[i] = y[i];
-    __syncthreads();
-    y = ys;
+    if (sp.push_logits) {
+      y = buf[cl] + bb * W;
+    } else {
+      __syncthreads();
+      // the logits into shared memory in one coalesced pass (the argmax loops would otherwise
+      // chain dependent L2 round trips)
+      for (int i = tid; i < p.O; i += blockDim.x) ys[i] = y[i];
+      __syncthreads();
+      y = ys;
+    }
+    stamp(30, stamp_on);
     if (warp == 0) head_decode_warp(A, y, H, lane, b);
     __syncthreads();
     stamp(26, stamp_on);
@@ -369,6 +409,8 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
     }
     stamp(27, stamp_on);
   }
+  if (stamp_on && blockIdx.x == 0 && tid == 0)
+    for (int i = 0; i < 6; ++i) g_stamp[i < 5 ? 21 + i : 31] = g_dec_stamp[i];   // decode phases -> free slots
 }
 
 cudaError_t debug_stamps(int on, unsigned long long* out) {
@@ -430,7 +472,12 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   sp.C = C;
   sp.Bs = B < kBs ? 1 : kBs;
   // fuse the decode when the cluster has at least one CTA per two groups of its samples
-  sp.fuse_decode = (a.branch_head && sp.Bs * a.K_max <= 2 * C) ? 1 : 0;   // traversal: host decides first
+  sp.dec_tab_cap = dec_table_words(a, kDecTabCap);
+  // fuse the decode when each CTA decodes at most a few groups of its samples (traversal: the
+  // host decides first, so the decode runs after it in the stand-alone kernels)
+  sp.fuse_decode = (a.branch_head && sp.Bs * a.K_max <= 2 * C) ? 1 : 0;
+  sp.push_logits = (sp.fuse_decode && C > 1 && sp.Bs == 1 && p.n_stages > 1) ? 1 : 0;
+  sp.tab_off = -1;
   const int act_bytes = 2 * sp.Bs * p.max_width * (int)sizeof(double);
   const int base = ((2 * (4 + kMaxLayers) + 2) * 8 + 127) / 128 * 128;
   const int budget = kDynCap - act_bytes;
@@ -454,10 +501,17 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   }
   // the decode epilogue reuses [base, ...) after the MLP
   const int dec_bytes = (int)(((sizeof(DecHead) + 127) / 128 * 128) + ((sizeof(DecGroup) + 127) / 128 * 128) +
-                              (size_t)((p.O + 15) / 16 * 16) * sizeof(double) + (size_t)kDecTabCap * 4);
+                              (size_t)((p.O + 15) / 16 * 16) * sizeof(double) + (size_t)sp.dec_tab_cap * 4);
   if (sp.fuse_decode && base + dec_bytes > off) off = (base + dec_bytes + 127) / 128 * 128;
   sp.act_off = off;
-  const size_t smem = (size_t)sp.act_off + act_bytes;
+  size_t smem = (size_t)sp.act_off + act_bytes;
+  if (sp.fuse_decode) {
+    const size_t tb = (size_t)dec_table_region_words(a) * 4;
+    if (smem + tb <= (size_t)kDynCap) {
+      sp.tab_off = (int)((smem + 127) / 128 * 128);
+      smem = (size_t)sp.tab_off + tb;
+    }
+  }
   if (smem > (size_t)kDynCap) return cudaErrorInvalidValue;
   const int n_clusters = (B + sp.Bs - 1) / sp.Bs;
   cudaLaunchConfig_t cfg = {};

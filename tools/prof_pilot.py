@@ -41,7 +41,11 @@ sd = {i: int(st[i] - base) for i in range(30) if st[i] >= base and st[i] - base 
 print("prologue", sd.get(1), sd.get(2), "| stage (wait_in, wait_w, compute):",
       [(sd.get(3 + 3 * k, 0) - (sd.get(2) if k == 0 else sd.get(2 + 3 * k, 0)), sd.get(4 + 3 * k, 0) - sd.get(3 + 3 * k, 0),
         sd.get(5 + 3 * k, 0) - sd.get(4 + 3 * k, 0)) for k in range(7) if (3 + 3 * k) in sd],
+      "| head: counts, branch, pieces, cut:", sd.get(21, 0) - sd.get(30, 0), sd.get(22, 0) - sd.get(21, 0), sd.get(23, 0) - sd.get(22, 0), sd.get(26, 0) - sd.get(23, 0),
+      "| group: rows, scan, records:", sd.get(24, 0) - sd.get(26, 0), sd.get(25, 0) - sd.get(24, 0), sd.get(31, 0) - sd.get(25, 0), "rest", sd.get(27, 0) - sd.get(31, 0),
+      "| epilogue: csync, tables, logits:", sd.get(28, 0) - sd.get(20, 0), sd.get(29, 0) - sd.get(28, 0), sd.get(30, 0) - sd.get(29, 0),
       "| decode head, groups:", sd.get(26, 0) - max([v for k2, v in sd.items() if k2 < 26] or [0]), sd.get(27, 0) - sd.get(26, 0))
+print("raw (stamp: cycles since 0):", sorted(sd.items(), key=lambda kv: kv[1]))
 print(f"{cfg} B={B}: {e0.elapsed_time(e1) * 1e3 / n:.2f} us/predict (device span), host {(t1 - t0) * 1e6 / n:.2f} us/call, "
       f"pilot event {tm['pilot']['ms'] * 1e3 / max(1, tm['pilot']['launches']):.2f} us, decode event "
       f"{tm['decode']['ms'] * 1e3 / max(1, tm['decode']['launches']):.2f} us")

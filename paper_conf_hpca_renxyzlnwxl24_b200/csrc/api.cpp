@@ -1500,7 +1500,26 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
       wave_src.clear();
       return DYO_OK;
     };
-    for (int i = 0; i < h.n_move; ++i) {
+    // Many small moves (fragmented halves of small tensors) would make many waves of one or
+    // two records: move them in rounds through the staging buffer instead - records -> staging
+    // (one launch), staging -> the round's contiguous destination range (one launch). In
+    // ascending destination order a round never overwrites a later round's sources (the
+    // destinations are prefix sums below every later source), and a round's destination range
+    // holds exactly its moves (with their alignment padding).
+    bool staged_rounds = h.n_move >= 3;
+    for (int i = 0; i < h.n_move && staged_rounds; ++i)
+      if (align_up(mv[i].bytes, AL) > stage_half) staged_rounds = false;
+    for (int i = 0; staged_rounds && i < h.n_move;) {
+      const int64_t d0 = mv[i].dst;
+      int k = i;
+      while (k < h.n_move && mv[k].dst + mv[k].bytes - d0 <= stage_half) ctx->ctr.d2d += mv[k++].bytes;
+      dyo_status s1 = d2d_records(ctx, mv, dev_mv, i, k, 1, 2, 3, -1, 0, arena, stage_move, d0, s, d2d_grid);
+      if (s1) return s1;
+      s1 = d2d_range(ctx, stage_move, arena + d0, mv[k - 1].dst + mv[k - 1].bytes - d0, s, d2d_grid);
+      if (s1) return s1;
+      i = k;
+    }
+    for (int i = 0; i < h.n_move && !staged_rounds; ++i) {
       const int64_t src = mv[i].src, dst = mv[i].dst, nbytes = mv[i].bytes;
       ctx->ctr.d2d += nbytes;
       if (dst + nbytes > src) {                     // self-overlap: staged pieces, after the wave

@@ -570,16 +570,33 @@ plan_kernel(ArchDev a, PredDev pd, int b0, int nb, int policy, PlanState in, Pla
     PSTAMP(14);
     // resident lists: half m = kept + placed sorted by offset; half 1-m drops what left it
     {
+      // the kept tensors are already in ascending offset (first fit leaves them in place,
+      // compaction preserves their order), so only the placed ones are sorted (|W_j| keys) and
+      // the two runs are merged: every element's slot = its rank in its own run + the number of
+      // smaller keys in the other run (binary search; offsets of one half are unique)
       const int nnew = nkept + np;
-      uint64_t* rk = nnew > kSortCap ? sc.keys : S.sortbuf;
-      for (int i = tid; i < nnew; i += NT) {
-        const int t = i < nkept ? sc.kept[i] : (int)(pkey[i - nkept] & 0xFFFFF);
-        rk[i] = ((uint64_t)(st.off[t] / AL) << 20) | (uint64_t)t;
-      }
-      __syncthreads();
-      sort_keys(rk, nnew);
       int32_t* resw = st.res + (int64_t)m * T;
-      for (int i = tid; i < nnew; i += NT) resw[i] = (int)(rk[i] & 0xFFFFF);
+      uint64_t* pk = S.sortbuf;                       // placed keys (np <= kEntCap <= kSortCap)
+      int64_t* kk = sc.gap_s;                         // kept offsets (the gaps are consumed)
+      for (int k = tid; k < np; k += NT) {
+        const int t = (int)(pkey[k] & 0xFFFFF);
+        pk[k] = ((uint64_t)(st.off[t] / AL) << 20) | (uint64_t)t;
+      }
+      for (int i = tid; i < nkept; i += NT) kk[i] = st.off[sc.kept[i]];
+      __syncthreads();
+      sort_keys(pk, np);
+      for (int i = tid; i < nkept; i += NT) {
+        const uint64_t key = (uint64_t)(kk[i] / AL) << 20;
+        int lo = 0, hi = np;                          // placed keys below this kept offset
+        while (lo < hi) { const int mid = (lo + hi) >> 1; if (pk[mid] < key) lo = mid + 1; else hi = mid; }
+        resw[i + lo] = sc.kept[i];
+      }
+      for (int k = tid; k < np; k += NT) {
+        const int64_t o = (int64_t)((pk[k] >> 20) * (uint64_t)AL);
+        int lo = 0, hi = nkept;                       // kept offsets below this placed offset
+        while (lo < hi) { const int mid = (lo + hi) >> 1; if (kk[mid] < o) lo = mid + 1; else hi = mid; }
+        resw[k + lo] = (int)(pk[k] & 0xFFFFF);
+      }
       if (tid == 0) st.res_n[m] = nnew;
       __syncthreads();
       const int no = st.res_n[1 - m];

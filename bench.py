@@ -178,6 +178,40 @@ def oracle_steps(wl, n_steps, budget_s=None):
     return total_b, time.perf_counter() - t0, done
 
 
+def oracle_components(wl, budget_s=6.0):
+    """The oracle's per-component times on one host core (B = 1 steps): encode + pilot forward
+    (us/prediction), decode (us/prediction) and plan (us/step) - the CPU counterparts of the
+    GPU line's pilot_us_per_prediction and plan_us."""
+    from threadpoolctl import threadpool_limits
+    from oracle import encode as E, pilot as P, decode as D, plan as PL
+    st = PL.initial_state(len(wl.tensors))
+    table = ()
+    t_pilot = t_dec = t_plan = 0.0
+    n = 0
+    t_start = time.perf_counter()
+    with threadpool_limits(limits=1):
+        while time.perf_counter() - t_start < budget_s:
+            smp = wl.samples[n % len(wl.samples)]
+            t0 = time.perf_counter()
+            x = E.encode(wl, smp, wl.hist_ids, table)
+            y = P.forward(wl.pilot, x, wl.nn_type)
+            t1 = time.perf_counter()
+            pred = D.decode(wl, y, branch_head=wl.notes.get("branch_head", True))
+            t2 = time.perf_counter()
+            try:
+                _, st = PL.plan(st, wl, pred.W, None)
+            except PL.BudgetError:
+                st = PL.initial_state(len(wl.tensors))
+            t3 = time.perf_counter()
+            table = pred.blocks
+            t_pilot += t1 - t0
+            t_dec += t2 - t1
+            t_plan += t3 - t2
+            n += 1
+    return {"pilot_us_per_prediction": round(t_pilot / n * 1e6, 1), "decode_us_per_prediction": round(t_dec / n * 1e6, 1),
+            "plan_us_per_step": round(t_plan / n * 1e6, 1), "steps": n, "cores": 1}
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -201,6 +235,62 @@ def run_reference(args):
 # ---------------------------------------------------------------------------------------------
 # B200 leg
 # ---------------------------------------------------------------------------------------------
+
+def pilot_latency(torch, wl, dev, desc_dev, hist64, nS, s0):
+    """Batch-1 pilot latency three ways (survey section 8(d)): single-shot host-observed (call ->
+    stream synchronised), CUDA-graph replay of 100 back-to-back predictions / 100, and the floor
+    = a graph of 100 empty launches of the pilot's shape (one cluster, L cluster barriers for its
+    L dependent stages) / 100."""
+    import numpy as np
+    from paper_conf_hpca_renxyzlnwxl24_b200 import Dyo
+    sp = wl.pilot
+    wbytes = 4 * (sum((ln + 1 + 3) // 4 * 4 * o for _, ln, o in sp.feature) + sum((i + 1 + 3) // 4 * 4 * o for i, o in sp.mlp)
+                  + (sp.out_in + 1 + 3) // 4 * 4 * sp.O)
+    C = 1 if wbytes <= (64 << 10) else (4 if wbytes <= (512 << 10) else 16)
+    L = (1 if sp.feature else 0) + len(sp.mlp) + 1
+    g1 = Dyo(wl.budget, wl.align, wl.policy, max_batch=1, device=dev, flags=4)
+    g1.load(wl)
+    h1 = hist64[:1] if hist64 is not None else None
+    out = {"cluster": C, "stages": L}
+    try:
+        ss = []
+        for i in range(40):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            g1.predict(desc_dev[i % nS: i % nS + 1], h1, 1, stream=s0.cuda_stream)
+            s0.synchronize()
+            ss.append((time.perf_counter() - t0) * 1e6)
+        out["single_shot_us"] = round(float(np.median(ss[5:])), 2)
+        cs = torch.cuda.Stream()
+        for _ in range(3):
+            g1.predict(desc_dev[:1], h1, 1, stream=cs.cuda_stream)
+        torch.cuda.synchronize()
+
+        def replay(fn):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=cs):
+                for i in range(100):
+                    fn(i, torch.cuda.current_stream().cuda_stream)
+            with torch.cuda.stream(cs):              # replay() launches on the current stream
+                g.replay()
+                torch.cuda.synchronize()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(cs)
+                for _ in range(10):
+                    g.replay()
+                e1.record(cs)
+            e1.synchronize()
+            return e0.elapsed_time(e1) * 1e3 / 1000
+        out["graph_replay_us"] = round(replay(lambda i, st: g1.predict(desc_dev[i % nS: i % nS + 1], h1, 1, stream=st)), 2)
+        out["floor_us"] = round(replay(lambda i, st: g1.debug_floor(C, L, st)), 2)
+        out["floor_frac"] = round(out["floor_us"] / out["graph_replay_us"], 4)
+        out["note"] = ("floor = empty launch of the pilot's cluster shape with one cluster barrier per dependent stage, "
+                       "graph-replayed; graph_replay_us includes the fused decode")
+    except Exception as e:     # capture unsupported on this path: report what was measured
+        out["error"] = str(e)[:200]
+    g1.close()
+    return out
+
 
 def calibrate_spin(torch):
     """GPU cycles per microsecond of torch.cuda._sleep (the compute emulation's spin kernel)."""
@@ -405,6 +495,7 @@ def run_dyo(args):
         return (p0.elapsed_time(p1) * 1e3 / n, t["pilot"]["ms"] * 1e3 / max(1, t["pilot"]["launches"]),
                 t["decode"]["ms"] * 1e3 / max(1, t["decode"]["launches"]))
     pred_us, pilot_kernel_us, decode_us = pilot_loop(dp, 200, 1)
+    lat = pilot_latency(torch, wl, local, desc_dev, hist64, nS, s0)
     b64_us, b64_kernel_us, b64_decode_us = pilot_loop(dp, 50, 64)
     # K1-TC work per launch: 2 x 64 x sum(in x out) over the tensor-core stages, x3 for 3xTF32
     sp = wl.pilot
@@ -488,6 +579,7 @@ def run_dyo(args):
         "pilot_us_per_prediction": round(pred_us, 3),
         "pilot_kernel_us": round(pilot_kernel_us, 3), "decode_kernels_us": round(decode_us, 3),
         "predictions_per_s": round(1e6 / pred_us, 1),
+        "pilot_latency_b1": lat,
         "pilot_batch64": {"us_per_batch": round(b64_us, 2), "us_per_prediction": round(b64_us / 64, 3),
                           "predictions_per_s": round(64e6 / b64_us, 1),
                           "pilot_kernel_us": round(b64_kernel_us, 2), "decode_kernels_us": round(b64_decode_us, 2),
@@ -524,6 +616,8 @@ def run_dyo(args):
         out["cpu_baseline"] = {"value": round(b / sec / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
                                "sample": f"{n} oracle steps of the same workload (pure Python encode/pilot/decode/plan + "
                                          f"numpy copy of each step's algorithmic bytes), ~15 s, 1 of {_os.cpu_count()} cores"}
+        if wl.notes.get("batch", 1) == 1:
+            out["cpu_baseline"]["components"] = oracle_components(wl)
     print(json.dumps(out), flush=True)
     d.close()
     if world > 1:

@@ -303,6 +303,41 @@ dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32)
 /* Debugging aid: clock64 stamps of the planner's phases for transition j of the next dyo_plan
  * (j = -1 disables); out64 (64 entries, may be NULL) receives the stamps of the last plan. */
 dyo_status dyo_debug_plan_stamps(dyo_ctx* ctx, int32_t j, uint64_t* out64);
+/* ---- Mis-prediction handling (§IV-E "Handling mis-prediction", §VI-H
+ * P:L280; reading R15) ------------------------------------------------------------
+ * The pilot may mis-predict the control flow. After a sample has executed, the runtime reports
+ * the control flow that actually ran; the library records the mis-prediction (the paper's
+ * training record: a count here) and memoises it: "the output of the pilot model is compared
+ * with the output where there is mis-prediction. If the two outputs are exactly the same, then
+ * the correct execution block in the mis-prediction case is used to resolve the control flows"
+ * (P:L186-L187). The compared output is the decoded integer pilot output of a prediction: its
+ * raw block head (K_max x 10 ints, reading R4) and its own branch-head choices. A later
+ * prediction with exactly that output is decoded with the memoised actual choices (inside the
+ * decode kernels: a 64-bit key hash probes a device open-addressing table, then the full key is
+ * compared); its groups are cut from the actual path at the predicted counts.
+ *
+ * dyo_memo_config: (re)allocates the memo for `capacity` entries (0 disables it; default
+ *   disabled). FIFO replacement of the oldest key when full; a re-reported key keeps its most
+ *   recent value. Requires dyo_load_arch (DYO_E_STATE); reset by it. Synchronises the device.
+ * dyo_report: `actual` (host, n_sites ints, site order of the branch head; a tied site must
+ *   replay its target, R6) is compared with the FINAL choices of prediction b (0 <= b < the B of
+ *   the last dyo_pilot_predict). *mispredicted (may be NULL) = 1 if they differ. On a
+ *   mis-prediction the count is incremented and, with the memo enabled, the prediction's raw
+ *   output -> actual choices is memoised (host mirror + device table). DYO_E_INVAL on a bad b or
+ *   an invalid choice vector. Synchronises the device (the report follows the sample's
+ *   execution). Branch-head arches only (with the traversal decode the memo is not consulted).
+ * dyo_memo_stats: mis-predictions reported so far (since dyo_load_arch), live memo entries, and
+ *   memo hits taken by the decode kernels (device counter). Any pointer may be NULL. */
+dyo_status dyo_memo_config(dyo_ctx* ctx, int32_t capacity);
+dyo_status dyo_report(dyo_ctx* ctx, int32_t b, const int32_t* actual, int32_t* mispredicted);
+dyo_status dyo_memo_stats(dyo_ctx* ctx, int64_t* mispredictions, int32_t* live, int64_t* hits);
+
+/* Measurement aid for the batch-1 pilot's latency floor (survey section 8(d)): launches, on
+ * `stream`, an otherwise empty kernel with the pilot's launch shape (one cluster of `cluster`
+ * CTAs x 512 threads, the pilot's dynamic shared memory) that performs `n_barriers`
+ * cluster-wide barriers (one per dependent layer stage). Asynchronous; capturable in a CUDA
+ * graph. DYO_E_INVAL if cluster is not 1..16 or n_barriers < 0. */
+dyo_status dyo_debug_floor(dyo_ctx* ctx, int32_t cluster, int32_t n_barriers, void* stream);
 
 #ifdef __cplusplus
 }

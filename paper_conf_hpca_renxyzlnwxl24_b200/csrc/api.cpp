@@ -47,6 +47,16 @@ struct dyo_ctx {
   // logits / choices staging and the device choices the decode kernel replays
   int branch_head = 1;
   TravArch trav;
+  // exact-match mis-prediction memo (R15): host mirror of the device table (ad.memo_*)
+  struct Memo {
+    int cap = 0, kw = 0, ns = 0, mask = 0, live = 0, tomb = 0;
+    std::vector<uint64_t> hash;
+    std::vector<int32_t> key, val, index, id_slot;
+    std::vector<int> fifo;            // live entry ids, oldest first
+    std::vector<int> free_ids;
+    int64_t mispredictions = 0;
+    std::vector<void*> dev;           // index, hash, key, val, hits
+  } memo;
   double* h_logits = nullptr;      // pinned, max_batch x O
   int32_t* h_forced[2] = {nullptr, nullptr};   // pinned, max_batch x n_sites (alternating)
   int32_t* d_forced = nullptr;
@@ -553,12 +563,27 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   return DYO_OK;
 }
 
+void memo_free(dyo_ctx* ctx) {
+  for (void* p : ctx->memo.dev) cudaFree(p);
+  const int64_t mp = ctx->memo.mispredictions;
+  ctx->memo = dyo_ctx::Memo{};
+  ctx->memo.mispredictions = mp;
+  ctx->ad.memo_live = 0;
+  ctx->ad.memo_mask = 0;
+  ctx->ad.memo_index = nullptr;
+  ctx->ad.memo_hash = nullptr;
+  ctx->ad.memo_key = nullptr;
+  ctx->ad.memo_val = nullptr;
+  ctx->ad.memo_hits = nullptr;
+}
+
 dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (!ctx) return DYO_E_INVAL;
   cudaSetDevice(ctx->device);
   cudaDeviceSynchronize();
   free_owned(ctx, ctx->arch_dev);
   free_owned(ctx, ctx->pilot_dev);
+  memo_free(ctx);
   free_plan_host(ctx);
   if (ctx->host_pool) cudaFreeHost(ctx->host_pool);
   if (ctx->h_logits) cudaFreeHost(ctx->h_logits);
@@ -584,6 +609,8 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   CK(cudaSetDevice(ctx->device));
   CK(cudaDeviceSynchronize());
   free_owned(ctx, ctx->arch_dev);
+  memo_free(ctx);
+  ctx->memo.mispredictions = 0;
   free_plan_host(ctx);
   if (ctx->host_pool) { cudaFreeHost(ctx->host_pool); ctx->host_pool = nullptr; }
   ctx->arch_ok = false;
@@ -638,7 +665,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   pd = PredDev{};
   pd.B = B;
 #define DA(p, n) if ((st = dalloc(ctx, own, &p, (size_t)(n)))) return st
-  DA(pd.K, B); DA(pd.L, B); DA(pd.choices, (size_t)B * std::max(n_sites, 1)); DA(pd.slots, (size_t)B * K * 10);
+  DA(pd.K, B); DA(pd.L, B); DA(pd.choices, (size_t)B * std::max(n_sites, 1)); DA(pd.rchoices, (size_t)B * std::max(n_sites, 1)); DA(pd.slots, (size_t)B * K * 10);
   DA(pd.path, (size_t)B * ad.L_max); DA(pd.grp, (size_t)B * K * 2); DA(pd.blocks, (size_t)B * K * 10);
   DA(pd.ent_n, (size_t)B * K); DA(pd.ent, (size_t)B * K * kEntCap); DA(pd.status, 4);
   pd.head_stride = 3 + n_sites + ((int)piece_kind.size() + 1) + (K + 1) + K;
@@ -1135,6 +1162,175 @@ dyo_status dyo_prediction_get(dyo_ctx* ctx, int32_t b, int32_t* K, int32_t* bloc
   return DYO_OK;
 }
 
+// ---- mis-prediction record + exact-match memo (R15) --------------
+namespace {
+uint64_t memo_hash_of(const int32_t* key, int kw_total) {
+  uint64_t h = 0;
+  for (int i = 0; i < kw_total; ++i) h += dyo::memo_mix((uint64_t)i, key[i]);
+  return h ? h : 1;
+}
+dyo_status memo_upload_entry(dyo_ctx* ctx, int id) {
+  auto& M = ctx->memo;
+  const int kt = M.kw + M.ns;
+  CK(cudaMemcpy(static_cast<uint64_t*>(M.dev[1]) + id, &M.hash[id], 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(static_cast<int32_t*>(M.dev[2]) + (size_t)id * kt, &M.key[(size_t)id * kt], 4 * (size_t)kt, cudaMemcpyHostToDevice));
+  if (M.ns)
+    CK(cudaMemcpy(static_cast<int32_t*>(M.dev[3]) + (size_t)id * M.ns, &M.val[(size_t)id * M.ns], 4 * (size_t)M.ns,
+                  cudaMemcpyHostToDevice));
+  return DYO_OK;
+}
+dyo_status memo_upload_index(dyo_ctx* ctx) {
+  auto& M = ctx->memo;
+  CK(cudaMemcpy(M.dev[0], M.index.data(), 4 * M.index.size(), cudaMemcpyHostToDevice));
+  return DYO_OK;
+}
+// slot of entry `id` (or of key `key` when id < 0) in the index; -1 if absent
+int memo_find(const dyo_ctx::Memo& M, uint64_t h, const int32_t* key, int id) {
+  const int kt = M.kw + M.ns;
+  int slot = (int)(h & (uint64_t)M.mask);
+  for (int probe = 0; probe <= M.mask; ++probe) {
+    const int e = M.index[slot];
+    if (e == -1) return -1;
+    if (e >= 0 && M.hash[e] == h) {
+      if (id >= 0 ? e == id : std::equal(key, key + kt, &M.key[(size_t)e * kt])) return slot;
+    }
+    slot = (slot + 1) & M.mask;
+  }
+  return -1;
+}
+void memo_rebuild(dyo_ctx::Memo& M) {
+  std::fill(M.index.begin(), M.index.end(), -1);
+  for (int id : M.fifo) {
+    int slot = (int)(M.hash[id] & (uint64_t)M.mask);
+    while (M.index[slot] != -1) slot = (slot + 1) & M.mask;
+    M.index[slot] = id;
+  }
+  M.tomb = 0;
+}
+}  // namespace
+
+dyo_status dyo_memo_config(dyo_ctx* ctx, int32_t capacity) {
+  if (!ctx || capacity < 0 || capacity > (1 << 20)) return DYO_E_INVAL;
+  if (!ctx->arch_ok) return fail(ctx, DYO_E_STATE, "dyo_memo_config before dyo_load_arch");
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  memo_free(ctx);
+  if (capacity == 0) return DYO_OK;
+  auto& M = ctx->memo;
+  M.cap = capacity;
+  M.kw = 10 * ctx->K_max;
+  M.ns = ctx->n_sites;
+  int slots = 1;
+  while (slots < 2 * capacity) slots <<= 1;
+  M.mask = slots - 1;
+  const int kt = M.kw + M.ns;
+  M.hash.assign(capacity, 0);
+  M.key.assign((size_t)capacity * kt, 0);
+  M.val.assign((size_t)capacity * std::max(M.ns, 1), 0);
+  M.index.assign(slots, -1);
+  M.free_ids.clear();
+  for (int i = capacity - 1; i >= 0; --i) M.free_ids.push_back(i);
+  const size_t bytes[5] = {4u * (size_t)slots, 8u * (size_t)capacity, 4u * (size_t)capacity * kt,
+                           4u * (size_t)capacity * std::max(M.ns, 1), 8};
+  for (size_t b : bytes) {
+    void* p = nullptr;
+    CK(cudaMalloc(&p, b));
+    CK(cudaMemset(p, 0, b));
+    M.dev.push_back(p);
+  }
+  dyo_status st = memo_upload_index(ctx);
+  if (st) return st;
+  ctx->ad.memo_mask = M.mask;
+  ctx->ad.memo_live = 0;
+  ctx->ad.memo_index = static_cast<const int32_t*>(M.dev[0]);
+  ctx->ad.memo_hash = static_cast<const uint64_t*>(M.dev[1]);
+  ctx->ad.memo_key = static_cast<const int32_t*>(M.dev[2]);
+  ctx->ad.memo_val = static_cast<const int32_t*>(M.dev[3]);
+  ctx->ad.memo_hits = static_cast<unsigned long long*>(M.dev[4]);
+  return DYO_OK;
+}
+
+dyo_status dyo_report(dyo_ctx* ctx, int32_t b, const int32_t* actual, int32_t* mispredicted) {
+  if (!ctx || !actual || b < 0 || b >= ctx->last_B) return DYO_E_INVAL;
+  const int ns = ctx->n_sites;
+  const TravArch& T = ctx->trav;
+  for (int i = 0; i < ns; ++i) {
+    if (actual[i] < 0 || actual[i] >= T.site_nch[i]) return fail(ctx, DYO_E_INVAL, "actual choice %d of site %d out of range", actual[i], i);
+    if (T.site_tie[i] >= 0 && actual[i] != actual[T.site_tie[i]])
+      return fail(ctx, DYO_E_INVAL, "site %d must replay site %d (R6)", i, T.site_tie[i]);
+  }
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  int32_t status = 0;
+  CK(cudaMemcpy(&status, ctx->pd.status, sizeof status, cudaMemcpyDeviceToHost));
+  if (status) return fail(ctx, (dyo_status)status, "decode failed (status %d)", status);
+  const int Km = ctx->K_max;
+  std::vector<int32_t> fin(std::max(ns, 1)), key((size_t)10 * Km + ns);
+  if (ns) CK(cudaMemcpy(fin.data(), ctx->pd.choices + (size_t)b * ns, 4 * (size_t)ns, cudaMemcpyDeviceToHost));
+  const bool miss = !std::equal(actual, actual + ns, fin.data());
+  if (mispredicted) *mispredicted = miss ? 1 : 0;
+  if (!miss) return DYO_OK;
+  ctx->memo.mispredictions++;
+  auto& M = ctx->memo;
+  if (M.cap == 0) return DYO_OK;                   // recorded (counted), memo disabled
+  CK(cudaMemcpy(key.data(), ctx->pd.slots + (size_t)b * Km * 10, 4 * (size_t)Km * 10, cudaMemcpyDeviceToHost));
+  if (ns) CK(cudaMemcpy(key.data() + 10 * Km, ctx->pd.rchoices + (size_t)b * ns, 4 * (size_t)ns, cudaMemcpyDeviceToHost));
+  const int kt = M.kw + M.ns;
+  const uint64_t h = memo_hash_of(key.data(), kt);
+  const int slot_old = memo_find(M, h, key.data(), -1);
+  dyo_status st;
+  if (slot_old >= 0) {                              // same output reported again: most recent wins
+    const int id = M.index[slot_old];
+    std::copy(actual, actual + ns, &M.val[(size_t)id * ns]);
+    M.fifo.erase(std::find(M.fifo.begin(), M.fifo.end(), id));
+    M.fifo.push_back(id);
+    return memo_upload_entry(ctx, id);
+  }
+  if (M.live == M.cap) {                            // FIFO replacement of the oldest key
+    const int old = M.fifo.front();
+    M.fifo.erase(M.fifo.begin());
+    const int sl = memo_find(M, M.hash[old], nullptr, old);
+    if (sl >= 0) { M.index[sl] = -2; ++M.tomb; }
+    M.free_ids.push_back(old);
+    --M.live;
+  }
+  const int id = M.free_ids.back();
+  M.free_ids.pop_back();
+  M.hash[id] = h;
+  std::copy(key.begin(), key.end(), &M.key[(size_t)id * kt]);
+  std::copy(actual, actual + ns, &M.val[(size_t)id * ns]);
+  M.fifo.push_back(id);
+  ++M.live;
+  if (M.tomb > M.cap / 2) {
+    memo_rebuild(M);
+  } else {
+    int slot = (int)(h & (uint64_t)M.mask);
+    while (M.index[slot] >= 0) slot = (slot + 1) & M.mask;
+    if (M.index[slot] == -2) --M.tomb;
+    M.index[slot] = id;
+  }
+  if ((st = memo_upload_entry(ctx, id))) return st;
+  if ((st = memo_upload_index(ctx))) return st;
+  ctx->ad.memo_live = M.live;
+  return DYO_OK;
+}
+
+dyo_status dyo_memo_stats(dyo_ctx* ctx, int64_t* mispredictions, int32_t* live, int64_t* hits) {
+  if (!ctx) return DYO_E_INVAL;
+  if (mispredictions) *mispredictions = ctx->memo.mispredictions;
+  if (live) *live = ctx->memo.live;
+  if (hits) {
+    *hits = 0;
+    if (!ctx->memo.dev.empty()) {
+      CK(cudaDeviceSynchronize());
+      unsigned long long v = 0;
+      CK(cudaMemcpy(&v, ctx->memo.dev[4], 8, cudaMemcpyDeviceToHost));
+      *hits = (int64_t)v;
+    }
+  }
+  return DYO_OK;
+}
+
 dyo_status dyo_prediction_matched(dyo_ctx* ctx, int32_t b, int32_t* matched) {
   if (!ctx || !matched || b < 0 || b >= ctx->last_B) return DYO_E_INVAL;
   if (ctx->branch_head || !ctx->h_matched) return fail(ctx, DYO_E_STATE, "no traversal decode in this arch");
@@ -1506,7 +1702,9 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
     // ascending destination order a round never overwrites a later round's sources (the
     // destinations are prefix sums below every later source), and a round's destination range
     // holds exactly its moves (with their alignment padding).
-    bool staged_rounds = h.n_move >= 3;
+    int64_t mv_bytes = 0;
+    for (int i = 0; i < h.n_move; ++i) mv_bytes += mv[i].bytes;
+    bool staged_rounds = h.n_move >= 8 && mv_bytes / h.n_move <= (1 << 20);   // many small moves only
     for (int i = 0; i < h.n_move && staged_rounds; ++i)
       if (align_up(mv[i].bytes, AL) > stage_half) staged_rounds = false;
     for (int i = 0; staged_rounds && i < h.n_move;) {
@@ -1680,6 +1878,13 @@ dyo_status dyo_debug_copy(dyo_ctx* ctx, const void* src, void* dst, int64_t byte
   else CK(launch_copy_segments(d, (int)segs.size(), kChunk, 4 * ctx->sm_count, (cudaStream_t)stream));
   CK(cudaFreeAsync(d, (cudaStream_t)stream));
   CK(cudaStreamSynchronize((cudaStream_t)stream));
+  return DYO_OK;
+}
+
+dyo_status dyo_debug_floor(dyo_ctx* ctx, int32_t cluster, int32_t n_barriers, void* stream) {
+  if (!ctx || cluster < 1 || cluster > 16 || n_barriers < 0) return DYO_E_INVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(launch_floor(cluster, n_barriers, (cudaStream_t)stream));
   return DYO_OK;
 }
 

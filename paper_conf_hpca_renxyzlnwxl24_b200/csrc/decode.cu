@@ -38,7 +38,7 @@ decode_head_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int
   const double* yg = logits + (int64_t)b * a.O;
   for (int i = tid; i < a.O; i += blockDim.x) ys[i] = yg[i];
   __syncthreads();
-  if (tid < 32) head_decode_warp(a, ys, S.H, lane, b);
+  if (tid < 32) head_decode_warp(a, ys, S.H, lane, b, pd.rchoices ? pd.rchoices + (int64_t)b * a.n_sites : nullptr);
   __syncthreads();
   write_head(a, S.H, ys, pd, b, hist_K);
   int* h = head_of(pd, b);

@@ -190,7 +190,53 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 // Decode the head of logits y (fp64, R4) into H. Called by ONE warp; __syncwarp() at the end.
 // b = index of the prediction in its batch (selects the host traversal's choices when the
 // arch has no branch head).
-static __device__ void head_decode_warp(const ArchDev& a, const double* __restrict__ y, DecHead& H, int lane, int b) {
+// Raw block-head element i (R4): rint(y * 2^sigma), sigma = 4 (elements 0..6) or 10, clamped.
+__device__ __forceinline__ int slot_int(const double* __restrict__ y, int i) {
+  const int e = i % 10;
+  double t = y[i] * (e < 7 ? 16.0 : 1024.0);
+  t = fmin(fmax(t, 0.0), (double)kSat);
+  return (int)rint(t);
+}
+
+// Exact-match memo lookup (R15), one warp: key = (raw block head, raw choices);
+// a hit replaces H.choice with the memoised actual choices. rch (may be null) receives the raw
+// choices (the key half a later dyo_report needs); only the CTA given rch counts the hit.
+__device__ __forceinline__ void memo_lookup_warp(const ArchDev& a, const double* __restrict__ y, DecHead& H, int lane,
+                                                 int32_t* __restrict__ rch) {
+  const int ns = a.n_sites;
+  if (rch)
+    for (int i = lane; i < ns; i += 32) rch[i] = H.choice[i];
+  if (a.memo_live <= 0 || a.forced) return;
+  const int KW = 10 * a.K_max;
+  uint64_t h = 0;
+  for (int i = lane; i < KW; i += 32) h += memo_mix((uint64_t)i, slot_int(y, i));
+  for (int i = lane; i < ns; i += 32) h += memo_mix((uint64_t)(KW + i), H.choice[i]);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) h += __shfl_xor_sync(0xffffffffu, h, o);
+  if (h == 0) h = 1;
+  int slot = (int)(h & (uint64_t)a.memo_mask), hit = -1;
+  for (int probe = 0; probe <= a.memo_mask; ++probe) {
+    const int e = a.memo_index[slot];
+    if (e == -1) break;
+    if (e >= 0 && a.memo_hash[e] == h) {
+      const int32_t* k = a.memo_key + (int64_t)e * (KW + ns);
+      bool same = true;
+      for (int i = lane; i < KW; i += 32) same = same && k[i] == slot_int(y, i);
+      for (int i = lane; i < ns; i += 32) same = same && k[KW + i] == H.choice[i];
+      if (__all_sync(0xffffffffu, same)) { hit = e; break; }
+    }
+    slot = (slot + 1) & a.memo_mask;
+  }
+  __syncwarp();
+  if (hit >= 0) {
+    for (int i = lane; i < ns; i += 32) H.choice[i] = a.memo_val[(int64_t)hit * ns + i];
+    if (lane == 0 && a.memo_hits && rch) atomicAdd(a.memo_hits, 1ull);   // one decoding CTA counts
+  }
+  __syncwarp();
+}
+
+static __device__ void head_decode_warp(const ArchDev& a, const double* __restrict__ y, DecHead& H, int lane, int b,
+                                        int32_t* __restrict__ rch = nullptr) {
   // 1. block-head counts of every slot; compact the non-empty ones in slot order
   int nk = 0;
   for (int k0 = 0; k0 < a.K_max; k0 += 32) {
@@ -228,6 +274,7 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
   for (int i = lane; i < a.n_sites && !a.forced; i += 32)
     if (a.site_logit[i] < 0) H.choice[i] = H.choice[a.site_tie[i]];   // tie targets are free sites
   __syncwarp();
+  memo_lookup_warp(a, y, H, lane, rch);
   DSTAMP(1);
   // 3. piece lengths -> exclusive scan -> piece starts (R2)
   int carry = 0;
@@ -475,12 +522,7 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
 // Debug copies of prediction b (slots, choices, path, K, L) + the history K; one block.
 static __device__ void write_head(const ArchDev& a, const DecHead& H, const double* __restrict__ y, PredDev& pd, int b,
                            int32_t* __restrict__ hist_K) {
-  for (int i = threadIdx.x; i < a.K_max * 10; i += blockDim.x) {
-    const int e = i % 10;
-    double t = y[i] * (e < 7 ? 16.0 : 1024.0);
-    t = fmin(fmax(t, 0.0), (double)kSat);
-    pd.slots[(int64_t)b * a.K_max * 10 + i] = (int)rint(t);
-  }
+  for (int i = threadIdx.x; i < a.K_max * 10; i += blockDim.x) pd.slots[(int64_t)b * a.K_max * 10 + i] = slot_int(y, i);
   for (int i = threadIdx.x; i < a.n_sites; i += blockDim.x) pd.choices[(int64_t)b * a.n_sites + i] = H.choice[i];
   if (H.L <= a.L_max)
     for (int r = threadIdx.x; r < H.L; r += blockDim.x) pd.path[(int64_t)b * a.L_max + r] = row_op(a, H, r);

@@ -68,6 +68,15 @@ struct TcPlan {
 };
 
 // ---- arch on the device -------------------------------------------------------------
+// 64-bit key hash of the memo: a sum of splitmix64-mixed (position, value) words, so one warp
+// reduces it in any order; host (insert) and device (lookup) share it.
+__host__ __device__ inline uint64_t memo_mix(uint64_t pos, int32_t v) {
+  uint64_t z = pos * 0x9E3779B97F4A7C15ull ^ (uint64_t)(uint32_t)v;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
 struct ArchDev {
   int T, n_ops, n_sites, n_pieces, n_arms, nn_type, S_max, D_s, h, K_max, F, O, n_branch_logits;
   int L_max;
@@ -103,6 +112,14 @@ struct ArchDev {
   const int32_t* seg_table;  // S_max x 10
   int branch_head;           // 0: choices come from the host traversal (forced, R4)
   const int32_t* forced;     // max_batch x n_sites choices written by the traversal, or null
+  // exact-match mis-prediction memo (R15; memo.cpp): live entries > 0 enables the
+  // lookup in the head decode. index: open-addressing slots (entry id, -1 empty, -2 deleted)
+  int memo_live, memo_mask;
+  const int32_t* memo_index;     // memo_mask + 1
+  const uint64_t* memo_hash;     // capacity
+  const int32_t* memo_key;       // capacity x (10 K_max + n_sites): raw block head, raw choices
+  const int32_t* memo_val;       // capacity x n_sites: the actual choices
+  unsigned long long* memo_hits; // device counter
 };
 
 // ---- prediction storage -------------------------------------------------------------
@@ -110,7 +127,8 @@ struct PredDev {
   int B;
   int32_t* K;         // B
   int32_t* L;         // B
-  int32_t* choices;   // B x n_sites
+  int32_t* choices;   // B x n_sites (after a memo hit: the memoised actual choices)
+  int32_t* rchoices;  // B x n_sites: the pilot's own (raw) choices, the memo key's half
   int32_t* slots;     // B x K_max x 10 (decoded block head)
   int32_t* path;      // B x L_max (operator index, -1 control)
   int32_t* grp;       // B x K_max x 2 (start, end rows)
@@ -194,6 +212,7 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
                          PredDev& pd, int32_t* hist_tab_out, int32_t* hist_K_out, int* fused,
                          cudaStream_t s);
 cudaError_t debug_stamps(int on, unsigned long long* out);
+cudaError_t launch_floor(int C, int n_barriers, cudaStream_t s);
 cudaError_t tc_debug_stamps(int on, unsigned long long* out);   // K1-TC: globaltimer ns of CTA 0
 // K1-TC: batch pilot on tensor cores (logits only; the caller launches the decode kernel).
 cudaError_t launch_pilot_tc(const ArchDev& a, const PilotDev* p_dev, const TcPlan* plan_dev, const float* feat,

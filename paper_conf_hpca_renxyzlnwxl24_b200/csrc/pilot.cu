@@ -396,7 +396,7 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
       y = ys;
     }
     stamp(30, stamp_on);
-    if (warp == 0) head_decode_warp(A, y, H, lane, b);
+    if (warp == 0) head_decode_warp(A, y, H, lane, b, (r == 0 && pd.rchoices) ? pd.rchoices + (int64_t)b * a.n_sites : nullptr);
     __syncthreads();
     stamp(26, stamp_on);
     if (r == 0) write_head(A, H, y, pd, b, hist_K_out);
@@ -411,6 +411,35 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
   }
   if (stamp_on && blockIdx.x == 0 && tid == 0)
     for (int i = 0; i < 6; ++i) g_stamp[i < 5 ? 21 + i : 31] = g_dec_stamp[i];   // decode phases -> free slots
+}
+
+// Latency floor of the batch-1 pilot: the same launch shape, no work, n cluster barriers.
+__global__ void __launch_bounds__(kPilotThreads) floor_kernel(int n_barriers) {
+  for (int i = 0; i < n_barriers; ++i) cg::this_cluster().sync();
+}
+
+cudaError_t launch_floor(int C, int n_barriers, cudaStream_t s) {
+  static int attr_done = 0;
+  if (!attr_done) {
+    cudaError_t e = cudaFuncSetAttribute(floor_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(floor_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kDynCap);
+    if (e != cudaSuccess) return e;
+    attr_done = 1;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(C);
+  cfg.blockDim = dim3(kPilotThreads);
+  cfg.dynamicSmemBytes = 160 * 1024;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = C;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, floor_kernel, n_barriers);
 }
 
 cudaError_t debug_stamps(int on, unsigned long long* out) {

@@ -96,7 +96,8 @@ def lib():
                      "dyo_arena", "dyo_encode_features", "dyo_pilot_predict", "dyo_prediction_get",
                      "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records", "dyo_migrate",
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
-                     "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check"):
+                     "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
+                     "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -106,7 +107,8 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_load_pilot", "dyo_host_pool", "dyo_arena", "dyo_encode_features", "dyo_pilot_predict",
            "dyo_prediction_get", "dyo_prediction_matched", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
-           "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check")
+           "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
+           "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats")
 
 
 def _a(x, dt):
@@ -382,6 +384,25 @@ class Dyo:
 
     def debug_copy(self, src, dst, nbytes, mode, stream=0):
         self._check(self.L.dyo_debug_copy(self.ctx, P(self._ptr(src)), P(self._ptr(dst)), i64(nbytes), mode, P(stream)))
+
+    # ---- mis-prediction record + exact-match memo (R15) ----
+    def memo_config(self, capacity):
+        self._check(self.L.dyo_memo_config(self.ctx, int(capacity)))
+
+    def report(self, b, actual):
+        """Report the control flow prediction b actually ran; returns True on a mis-prediction."""
+        a = _a(actual, np.int32)
+        out = C.c_int32(0)
+        self._check(self.L.dyo_report(self.ctx, int(b), _p(a, C.c_int32), C.byref(out)))
+        return bool(out.value)
+
+    def memo_stats(self):
+        mp, live, hits = C.c_int64(0), C.c_int32(0), C.c_int64(0)
+        self._check(self.L.dyo_memo_stats(self.ctx, C.byref(mp), C.byref(live), C.byref(hits)))
+        return {"mispredictions": mp.value, "live": live.value, "hits": hits.value}
+
+    def debug_floor(self, cluster, n_barriers, stream=0):
+        self._check(self.L.dyo_debug_floor(self.ctx, cluster, n_barriers, P(stream)))
 
     def plan_stamps(self, j):
         out = np.zeros(64, np.uint64)

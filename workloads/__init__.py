@@ -224,6 +224,24 @@ def _walk(program):
             yield from _walk(it.body)
 
 
+def actual_choices(wl, sample, zipf_s=1.2):
+    """Synthetic 'what actually ran' control flow of a sample (input generation for the
+    mis-prediction tests and bench): per free site a choice drawn from a
+    Zipf(zipf_s) prior over its choices with a generator seeded by (workload seed, sample);
+    tied sites replay their target (reading R6). Deterministic; no method arithmetic."""
+    rng = np.random.default_rng((int(wl.seed) * 1_000_003 + int(sample)) & 0x7FFFFFFF)
+    sl = [it for it in _walk(wl.program) if isinstance(it, (If, Loop))]
+    out = []
+    for it in sl:
+        if it.tie >= 0:
+            out.append(out[it.tie])
+            continue
+        n = len(it.branches) if isinstance(it, If) else it.hi - it.lo + 1
+        w = 1.0 / np.arange(1, n + 1) ** zipf_s
+        out.append(int(rng.choice(n, p=w / w.sum())))
+    return out
+
+
 # ----------------------------------------------------------------------------
 # M0 tiny (BASELINE configs[0])
 # ----------------------------------------------------------------------------

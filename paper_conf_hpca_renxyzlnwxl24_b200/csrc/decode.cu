@@ -54,47 +54,86 @@ decode_head_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int
   for (int i = tid; i < S.H.nk; i += blockDim.x) hcnt[i] = S.H.cntc[i];
 }
 
-struct GroupSmem {
-  DecHead H;
-  DecGroup G;
-};
-
+// Phase B: one CTA per (prediction, group slot) - or, for the full-capacity pass, a grid-stride
+// loop over the slots the first pass left pending. R = record capacity: the first pass runs with
+// R = kRecSmall (~17 KB of shared memory: the whole batch fits in one wave), a group with more
+// records is marked pending (ent_n = -1) and rebuilt by the kRecCap pass.
+template <int R>
 __global__ void __launch_bounds__(kDecThreads)
-decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int tab_cap) {
+decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int tab_cap, int pending_pass) {
   extern __shared__ __align__(16) unsigned char dsm[];
-  GroupSmem& S = *reinterpret_cast<GroupSmem*>(dsm);
-  const int b = blockIdx.x / a.K_max, g = blockIdx.x % a.K_max;
-  const int* h = head_of(pd, b);
-  const int K = h[2];
-  if (g >= K) {
-    if (threadIdx.x == 0) pd.ent_n[(int64_t)b * a.K_max + g] = 0;
-    return;
+  DecGroupT<R>& G = *reinterpret_cast<DecGroupT<R>*>(dsm);
+  int* hw = reinterpret_cast<int*>(dsm + (sizeof(DecGroupT<R>) + 15) / 16 * 16);
+  const int ns = a.n_sites, np = a.n_pieces, Km = a.K_max;
+  __shared__ DecHeadDyn H;
+  __shared__ int s_todo;
+  if (threadIdx.x == 0) {
+    H.start = hw;
+    H.cum = hw + np + 1;
+    H.cntc = H.cum + Km + 1;
+    H.choice = H.cntc + Km;
   }
-  const int ns = a.n_sites, np = a.n_pieces;
-  if (threadIdx.x == 0) { S.H.L = h[0]; S.H.nk = h[1]; S.H.K = K; }
-  const int* hc = h + 3;
-  for (int i = threadIdx.x; i < ns; i += blockDim.x) S.H.choice[i] = hc[i];
-  const int* hs = hc + ns;
-  for (int i = threadIdx.x; i <= np; i += blockDim.x) S.H.start[i] = hs[i];
-  const int* hcum = hs + np + 1;
-  const int* hcnt = hcum + a.K_max + 1;
-  const int nk = h[1];
-  for (int i = threadIdx.x; i < nk; i += blockDim.x) { S.H.cum[i] = hcum[i]; S.H.cntc[i] = hcnt[i]; }
-  int* tabs = reinterpret_cast<int*>(dsm + (sizeof(GroupSmem) + 15) / 16 * 16);
-  const ArchDev A = stage_decode_tables(a, tabs, tab_cap);   // ends with __syncthreads()
-  build_group(A, S.H, S.G, pd, b, g, hist_tab);
+  int* tabs = hw + ((np + 1 + 2 * Km + 1 + ns + 3) / 4 * 4);
+  bool staged = false;
+  ArchDev A = a;
+  const int n_items = pd.B * Km;
+  for (int item = blockIdx.x; item < n_items; item += (pending_pass ? gridDim.x : n_items)) {
+    const int b = item / Km, g = item % Km;
+    if (pending_pass) {
+      if (threadIdx.x == 0) s_todo = pd.ent_n[(int64_t)b * Km + g] == -1;
+      __syncthreads();
+      const int todo = s_todo;
+      __syncthreads();
+      if (!todo) continue;
+    }
+    const int* h = head_of(pd, b);
+    const int K = h[2];
+    if (g >= K) {
+      if (threadIdx.x == 0) pd.ent_n[(int64_t)b * Km + g] = 0;
+      continue;
+    }
+    if (threadIdx.x == 0) { H.L = h[0]; H.nk = h[1]; H.K = K; }
+    __syncthreads();
+    const int* hc = h + 3;
+    for (int i = threadIdx.x; i < ns; i += blockDim.x) H.choice[i] = hc[i];
+    const int* hs = hc + ns;
+    for (int i = threadIdx.x; i <= np; i += blockDim.x) H.start[i] = hs[i];
+    const int* hcum = hs + np + 1;
+    const int* hcnt = hcum + Km + 1;
+    const int nk = h[1];
+    for (int i = threadIdx.x; i < nk; i += blockDim.x) { H.cum[i] = hcum[i]; H.cntc[i] = hcnt[i]; }
+    if (!staged) {
+      A = stage_decode_tables(a, tabs, tab_cap);   // ends with __syncthreads()
+      staged = true;
+    } else {
+      __syncthreads();
+    }
+    build_group(A, H, G, pd, b, g, hist_tab);
+    __syncthreads();
+  }
+}
+
+template <int R>
+size_t groups_smem(const ArchDev& a, int tab_cap) {
+  const int hw = (a.n_pieces + 1 + 2 * a.K_max + 1 + a.n_sites + 3) / 4 * 4;
+  return (sizeof(DecGroupT<R>) + 15) / 16 * 16 + (size_t)hw * 4 + (size_t)tab_cap * 4;
 }
 
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
   const int tab_cap = dec_table_words(a, kDecTabCap2);
-  const size_t smem = (sizeof(GroupSmem) + 15) / 16 * 16 + (size_t)tab_cap * 4;
-  static size_t smem_set = 0;
-  if (smem > smem_set) {
-    cudaError_t e = cudaFuncSetAttribute(decode_groups_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const size_t smA = groups_smem<kRecSmall>(a, tab_cap), smB = groups_smem<kRecCap>(a, tab_cap);
+  static size_t setA = 0, setB = 0;
+  if (smA > setA) {
+    cudaError_t e = cudaFuncSetAttribute(decode_groups_kernel<kRecSmall>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smA);
     if (e != cudaSuccess) return e;
-    smem_set = smem;
+    setA = smA;
+  }
+  if (smB > setB) {
+    cudaError_t e = cudaFuncSetAttribute(decode_groups_kernel<kRecCap>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smB);
+    if (e != cudaSuccess) return e;
+    setB = smB;
   }
   const size_t hsm = kHeadSmemBytes + (size_t)a.O * sizeof(double);
   static size_t hsm_set = 0;
@@ -106,7 +145,16 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
   decode_head_kernel<<<B, kDecThreads, hsm, s>>>(a, logits, pd, hist_K_out);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  decode_groups_kernel<<<B * a.K_max, kDecThreads, smem, s>>>(a, pd, hist_tab_out, tab_cap);
+  // PredDev.B = the allocation's batch: the kernels walk B x K_max items of this call only
+  PredDev pb = pd;
+  pb.B = B;
+  decode_groups_kernel<kRecSmall><<<B * a.K_max, kDecThreads, smA, s>>>(a, pb, hist_tab_out, tab_cap, 0);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  static int sms = 0;
+  if (!sms) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+  const int gB = B * a.K_max < 2 * sms ? B * a.K_max : 2 * sms;
+  decode_groups_kernel<kRecCap><<<gB, kDecThreads, smB, s>>>(a, pb, hist_tab_out, tab_cap, 1);
   return cudaGetLastError();
 }
 

@@ -36,18 +36,33 @@ struct DecHead {
   int L, nk, K;
 };
 
-struct DecGroup {
-  int32_t rec_t[kRecCap];              // access records in row order (position = index)
-  int32_t rec_m[kRecCap];              // mode bits (R = 1, W = 2)
-  int32_t first[kRecCap];              // 1 at the first position of each tensor, then its scan
-  int32_t ht_key[2 * kRecCap];         // open-addressing table: tensor -> first position, mode union
-  int32_t ht_pos[2 * kRecCap];
-  int32_t ht_mode[2 * kRecCap];
+// Head of a prediction with runtime-sized arrays (the stand-alone group kernel carves them from
+// dynamic shared memory: n_pieces + 1, K_max + 1, K_max and n_sites ints) - same member names
+// as DecHead, so the templated group build takes either.
+struct DecHeadDyn {
+  int* start;
+  int* cum;
+  int* cntc;
+  int* choice;
+  int L, nk, K;
+};
+
+// Group-build scratch for at most R access records (R a power of two).
+template <int R>
+struct DecGroupT {
+  int32_t rec_t[R];                    // access records in row order (position = index)
+  int32_t rec_m[R];                    // mode bits (R = 1, W = 2)
+  int32_t first[R];                    // 1 at the first position of each tensor, then its scan
+  int32_t ht_key[2 * R];               // open-addressing table: tensor -> first position, mode union
+  int32_t ht_pos[2 * R];
+  int32_t ht_mode[2 * R];
   int warp_tmp[32];
   long long sig_w[32][9];              // per-warp signature partial sums
   unsigned long long sig[9];
   int n, u;
 };
+using DecGroup = DecGroupT<kRecCap>;
+constexpr int kRecSmall = 64;          // the high-occupancy first pass of the group kernel
 
 // Copy the small decode tables (sites, arms, pieces) into shared memory `buf` (int32 words,
 // capacity cap) and return an ArchDev whose pointers refer to the copies; tables that do not
@@ -321,15 +336,18 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
   __syncwarp();
 }
 
-__device__ __forceinline__ int group_start(const DecHead& H, int g) { return H.nk == 0 ? 0 : H.cum[g]; }
-__device__ __forceinline__ int group_end(const DecHead& H, int g) {
+template <class HT>
+__device__ __forceinline__ int group_start(const HT& H, int g) { return H.nk == 0 ? 0 : H.cum[g]; }
+template <class HT>
+__device__ __forceinline__ int group_end(const HT& H, int g) {
   if (H.nk == 0 || g == H.K - 1) return H.L;                    // last group absorbs the remainder
   return min(H.cum[g] + H.cntc[g], H.L);
 }
 
 // Operator of path row r (-1 for a control row); *it = iteration index of its loop for the
 // per-iteration tensors (R13; 0 outside loops, counted down in a reversed loop).
-__device__ __forceinline__ int row_op(const ArchDev& a, const DecHead& H, int r, int* it = nullptr) {
+template <class HT>
+__device__ __forceinline__ int row_op(const ArchDev& a, const HT& H, int r, int* it = nullptr) {
   int lo = 0, hi = a.n_pieces - 1;
   while (lo < hi) {
     const int mid = (lo + hi + 1) >> 1;
@@ -353,8 +371,10 @@ __device__ __forceinline__ int row_op(const ArchDev& a, const DecHead& H, int r,
 }
 
 // Build group g of prediction b. All threads of the block must call it (uniform arguments).
-// Writes blocks / hist / grp / ent / ent_n for (b, g).
-static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup& G, PredDev& pd, int b, int g,
+// Writes blocks / hist / grp / ent / ent_n for (b, g). With R < kRecCap a group of more than R
+// records is left pending (ent_n = -1) for the full-capacity pass.
+template <class HT, int R>
+static __device__ void build_group(const ArchDev& a, const HT& H, DecGroupT<R>& G, PredDev& pd, int b, int g,
                             int32_t* __restrict__ hist_tab) {
   const int tid = threadIdx.x, NT = blockDim.x, lane = tid & 31, warp = tid >> 5;
   const int s = group_start(H, g), e = group_end(H, g);
@@ -397,8 +417,16 @@ static __device__ void build_group(const ArchDev& a, const DecHead& H, DecGroup&
   }
   int32_t* ent_n = pd.ent_n + (int64_t)b * a.K_max + g;
   int2* ent = pd.ent + ((int64_t)b * a.K_max + g) * kEntCap;
-  if (total > kRecCap) {
-    if (tid == 0) { *ent_n = 0; atomicCAS(&pd.status[0], 0, DYO_E_CAPACITY); pd.status[1] = total; }
+  if (total > R) {
+    if (tid == 0) {
+      if (R < kRecCap) {
+        *ent_n = -1;                                   // pending: the full-capacity pass builds it
+      } else {
+        *ent_n = 0;
+        atomicCAS(&pd.status[0], 0, DYO_E_CAPACITY);
+        pd.status[1] = total;
+      }
+    }
     __syncthreads();
     return;
   }

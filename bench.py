@@ -292,6 +292,48 @@ def pilot_latency(torch, wl, dev, desc_dev, hist64, nS, s0):
     return out
 
 
+def mispredict_stream(torch, wl, dev, s0, n_distinct=16, repeats=4):
+    """Mis-prediction record + exact-match memo on a sample stream with
+    repeats: `repeats` passes over `n_distinct` samples (history-free features, so a repeated
+    sample reproduces its pilot output), the actual control flow of every sample from
+    workloads.actual_choices. Reports the mis-prediction counts without and with the memo and the
+    batch-1 predict time with a populated memo (the decode's hash probe) vs without. Outside the
+    timed region."""
+    import numpy as np
+    import workloads as WLm
+    from paper_conf_hpca_renxyzlnwxl24_b200 import Dyo
+    if not wl.notes.get("branch_head", True):
+        return None
+    out = {"samples": n_distinct, "repeats": repeats}
+    acts = [WLm.actual_choices(wl, i) for i in range(n_distinct)]
+    desc = torch.from_numpy(wl.samples[:n_distinct].copy()).to(dev)
+    for memo in (0, 1):
+        d = Dyo(wl.budget, wl.align, wl.policy, max_batch=1, device=dev, flags=4)
+        d.load(wl)
+        if memo:
+            d.memo_config(1024)
+        for _ in range(repeats):
+            for i in range(n_distinct):
+                d.predict(desc[i:i + 1], None, 1, stream=s0.cuda_stream)
+                d.report(0, acts[i])
+        st = d.memo_stats()
+        out["with_memo" if memo else "without_memo"] = {"mispredictions": st["mispredictions"], "memo_hits": st["hits"],
+                                                         "live_entries": st["live"]}
+        # predict time (stream back-to-back, device span) with this ctx's memo state
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s0)
+        for k in range(200):
+            d.predict(desc[k % n_distinct: k % n_distinct + 1], None, 1, stream=s0.cuda_stream)
+        e1.record(s0)
+        e1.synchronize()
+        out["with_memo" if memo else "without_memo"]["pilot_us_per_prediction"] = round(e0.elapsed_time(e1) * 1e3 / 200, 2)
+        d.close()
+    out["note"] = ("actual control flow: workloads.actual_choices (Zipf(1.2) per site, seeded per sample); "
+                   "closed form with pairwise-distinct outputs: without = repeats x m, with = m")
+    return out
+
+
 def calibrate_spin(torch):
     """GPU cycles per microsecond of torch.cuda._sleep (the compute emulation's spin kernel)."""
     s = torch.cuda.Stream()
@@ -496,6 +538,7 @@ def run_dyo(args):
                 t["decode"]["ms"] * 1e3 / max(1, t["decode"]["launches"]))
     pred_us, pilot_kernel_us, decode_us = pilot_loop(dp, 200, 1)
     lat = pilot_latency(torch, wl, local, desc_dev, hist64, nS, s0)
+    mis = mispredict_stream(torch, wl, local, s0) if wl.notes.get("batch", 1) == 1 else None
     b64_us, b64_kernel_us, b64_decode_us = pilot_loop(dp, 50, 64)
     # K1-TC work per launch: 2 x 64 x sum(in x out) over the tensor-core stages, x3 for 3xTF32
     sp = wl.pilot
@@ -580,6 +623,7 @@ def run_dyo(args):
         "pilot_kernel_us": round(pilot_kernel_us, 3), "decode_kernels_us": round(decode_us, 3),
         "predictions_per_s": round(1e6 / pred_us, 1),
         "pilot_latency_b1": lat,
+        "mispredictions": mis,
         "pilot_batch64": {"us_per_batch": round(b64_us, 2), "us_per_prediction": round(b64_us / 64, 3),
                           "predictions_per_s": round(64e6 / b64_us, 1),
                           "pilot_kernel_us": round(b64_kernel_us, 2), "decode_kernels_us": round(b64_decode_us, 2),

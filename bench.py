@@ -283,6 +283,9 @@ def pilot_latency(torch, wl, dev, desc_dev, hist64, nS, s0):
             return e0.elapsed_time(e1) * 1e3 / 1000
         out["graph_replay_us"] = round(replay(lambda i, st: g1.predict(desc_dev[i % nS: i % nS + 1], h1, 1, stream=st)), 2)
         out["floor_us"] = round(replay(lambda i, st: g1.debug_floor(C, L, st)), 2)
+        # single-CTA empty launch: the planner's latency floor (survey 8(d) "fraction of the
+        # single-launch floor")
+        out["single_cta_launch_floor_us"] = round(replay(lambda i, st: g1.debug_floor(1, 0, st)), 2)
         out["floor_frac"] = round(out["floor_us"] / out["graph_replay_us"], 4)
         out["note"] = ("floor = empty launch of the pilot's cluster shape with one cluster barrier per dependent stage, "
                        "graph-replayed; graph_replay_us includes the fused decode")
@@ -637,6 +640,8 @@ def run_dyo(args):
                                                "note": "latency-bound: 6 dependent layers of M=128 x N=64 tiles"}
                                               if wl.pilot.feature else None)},
         "plan_us": round(plan_us, 2), "transitions_per_step": round(tot_K / args.steps, 2),
+        "plan_floor_frac": (round(lat["single_cta_launch_floor_us"] / plan_us, 5)
+                            if lat.get("single_cta_launch_floor_us") else None),
         "h2d_bytes_per_step": int(h2d_all / args.steps / world), "d2h_bytes_per_step": int(d2h_all / args.steps / world),
         "pcie": {"h2d_dma_gbs": round(h2d_link, 2) if h2d_link else None,
                  "d2h_dma_gbs": round(d2h_link, 2) if d2h_link else None,
@@ -661,7 +666,11 @@ def run_dyo(args):
                                "sample": f"{n} oracle steps of the same workload (pure Python encode/pilot/decode/plan + "
                                          f"numpy copy of each step's algorithmic bytes), ~15 s, 1 of {_os.cpu_count()} cores"}
         if wl.notes.get("batch", 1) == 1:
-            out["cpu_baseline"]["components"] = oracle_components(wl)
+            comp = oracle_components(wl)
+            out["cpu_baseline"]["components"] = comp
+            comp["gpu_speedup"] = {"pilot_decode": round((comp["pilot_us_per_prediction"] + comp["decode_us_per_prediction"])
+                                                         / max(pred_us, 1e-9), 1),
+                                   "plan": round(comp["plan_us_per_step"] / max(plan_us, 1e-9), 1)}
     print(json.dumps(out), flush=True)
     d.close()
     if world > 1:

@@ -10,7 +10,7 @@ budgets = [float(x) for x in (sys.argv[1] if len(sys.argv) > 1 else "1,2,4,8,16,
 rows = []
 for b in budgets:
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--config", "af", "--budget-gib", str(b),
-                        "--steps", "4", "--warmup", "2", "--no-cpu-baseline"], capture_output=True, text=True)
+                        "--steps", os.environ.get("SWEEP_STEPS", "4"), "--warmup", "2", "--no-cpu-baseline"], capture_output=True, text=True)
     try:
         d = json.loads(r.stdout.strip().splitlines()[-1])
     except Exception:

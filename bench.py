@@ -481,6 +481,8 @@ def run_dyo(args):
     barrier()
     d.timings(reset=True)
     d.counters(reset=True)
+    stamps_on = os.environ.get("DYO_COPY_STAMPS") == "1"
+    n_stamps0 = len(d.copy_stamps()) if stamps_on else 0
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     tot_h2d = tot_d2h = tot_K = 0
     plan_wall = []
@@ -496,6 +498,8 @@ def run_dyo(args):
     ms = e0.elapsed_time(e1)
     tm = d.timings(reset=True)
     ctr = d.counters(reset=True)
+    if stamps_on and rank == 0:
+        copy_stamp_report(d.copy_stamps()[n_stamps0:], os.environ.get("DYO_COPY_STAMPS_OUT", "gpurun_out/copy_stamps.json"))
 
     _log("e2e")
     # e2e: the same steps through the public API with HOST inputs (pinned), results read back
@@ -680,6 +684,34 @@ def run_dyo(args):
 def _log(msg):
     if os.environ.get("DYO_BENCH_VERBOSE"):
         print(f"[bench {time.strftime('%H:%M:%S')}] {msg}", file=sys.stderr, flush=True)
+
+
+def copy_stamp_report(st, path):
+    """Per-launch anatomy of the record-copy kernel in the timed region (DYO_COPY_STAMPS=1): CTA
+    start skew, record-scan time, per-CTA copy time and the launch span they add up to."""
+    import numpy as np
+    if len(st) == 0:
+        return
+    lid = (st[:, 0] >> np.uint64(32)).astype(np.int64)
+    sm = (st[:, 0] & np.uint64(255)).astype(np.int64)
+    t0, t1, t2 = (st[:, k].astype(np.int64) for k in (1, 2, 3))
+    rows = []
+    for L in np.unique(lid):
+        m = lid == L
+        a0, a1, a2 = t0[m], t1[m], t2[m]
+        rows.append({"ctas": int(m.sum()), "span_us": (a2.max() - a0.min()) / 1e3,
+                     "start_skew_us": (a0.max() - a0.min()) / 1e3, "scan_us_max": (a1 - a0).max() / 1e3,
+                     "cta_copy_us_med": float(np.median(a2 - a1)) / 1e3, "cta_copy_us_max": (a2 - a1).max() / 1e3,
+                     "end_skew_us": (a2.max() - a2.min()) / 1e3, "distinct_sms": int(len(np.unique(sm[m])))})
+    keys = rows[0].keys()
+    med = {k: float(np.median([r[k] for r in rows])) for k in keys}
+    big = [r for r in rows if r["span_us"] >= 20]
+    out = {"launches": len(rows), "median": med,
+           "median_over_launches_ge_20us": {k: float(np.median([r[k] for r in big])) for k in keys} if big else None,
+           "first_20": rows[:20]}
+    os.makedirs(os.path.dirname(path) or ".", exist_ok=True)
+    with open(path, "w") as f:
+        json.dump(out, f, indent=1)
 
 
 def main():

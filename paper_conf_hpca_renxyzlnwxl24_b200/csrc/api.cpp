@@ -1888,6 +1888,16 @@ dyo_status dyo_debug_floor(dyo_ctx* ctx, int32_t cluster, int32_t n_barriers, vo
   return DYO_OK;
 }
 
+dyo_status dyo_debug_copy_stamps(dyo_ctx* ctx, uint64_t* out, int64_t cap, int64_t* n) {
+  if (!ctx || cap < 0 || !n) return DYO_E_INVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  const int64_t k = copy_stamps_read(reinterpret_cast<unsigned long long*>(out), cap);
+  if (k < 0) return fail(ctx, DYO_E_CUDA, "copy stamps readback");
+  *n = k;
+  return DYO_OK;
+}
+
 dyo_status dyo_debug_pilot_stamps(dyo_ctx* ctx, int32_t enable, uint64_t* out32) {
   if (!ctx) return DYO_E_INVAL;
   CK(cudaSetDevice(ctx->device));

@@ -10,6 +10,8 @@
 // grid-stride loop and move them with 16-byte vector loads/stores, 4 in flight per thread.
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <cstdlib>
+#include <cstring>
 
 #include "dyo_internal.h"
 
@@ -53,8 +55,11 @@ copy_segments_kernel(const CopySeg* __restrict__ segs, int n) {
 // (cp.async.bulk.wait_group.read). The copy engine of the SM does the byte moving, so a few
 // CTAs saturate HBM and the SMs stay free for the DyNN's compute. Unaligned heads/tails (not
 // multiples of 16 bytes) are copied by the CTA's threads.
+// Ring shapes (stages x chunk): 4 x 16 KiB lets three copy kernels share an SM; the deeper rings
+// keep more bytes in flight per SM when one copy kernel has the GPU (DYO_TMA_RING selects, for
+// measurement; DESIGN.md §6 records which one is the default and why).
 constexpr int kTmaStages = 4;
-constexpr int kTmaChunk = 16 << 10;   // 4 x 16 KiB per CTA: three copy kernels can share an SM
+constexpr int kTmaChunk = 16 << 10;
 
 __device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -73,6 +78,7 @@ __device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvt
 
 constexpr int kRecThreads = 128;
 
+template <int CHUNK>
 struct RecCursor {
   const RecCopyArgs* a;
   int i;                       // current record
@@ -105,7 +111,7 @@ struct RecCursor {
   __device__ uint32_t len() const {
     int64_t l = body - off;
     if (hi - pos < l) l = hi - pos;
-    return (uint32_t)(l < kTmaChunk ? l : kTmaChunk);
+    return (uint32_t)(l < CHUNK ? l : CHUNK);
   }
   __device__ void next() {
     const uint32_t l = len();
@@ -115,6 +121,7 @@ struct RecCursor {
   }
 };
 
+template <int kTmaStages, int kTmaChunk>
 __global__ void __launch_bounds__(kRecThreads)
 copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
   extern __shared__ __align__(128) unsigned char sbuf[];
@@ -124,6 +131,8 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
   __shared__ int64_t s_off0;
   constexpr int L = kTmaStages - 1;          // loads kept in flight ahead of the store cursor
   const RecCopyArgs* a = &args;
+  unsigned long long t_enter = 0, t_scan = 0;
+  if (a->stamps != nullptr && threadIdx.x == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_enter));
   // the stream: the records' bodies, or the single range's body (0 when unaligned)
   const bool single = a->rec == nullptr;
   const int64_t T = !single ? a->total
@@ -141,7 +150,7 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
     for (int t0 = 0; t0 < a->n; t0 += blockDim.x) {
       const int k = t0 + threadIdx.x;
       int64_t v = 0;
-      if (k < a->n) { const char* s_; char* d_; RecCursor c; c.a = a; v = c.body_of(k, &s_, &d_); }
+      if (k < a->n) { const char* s_; char* d_; RecCursor<kTmaChunk> c; c.a = a; v = c.body_of(k, &s_, &d_); }
       const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
       int64_t x = v;
 #pragma unroll
@@ -164,11 +173,12 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
     }
   }
 
+  if (a->stamps != nullptr && threadIdx.x == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_scan));
   if (threadIdx.x == 0 && lo < hi) {
     for (int q = 0; q < kTmaStages; ++q)
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&bar[q])));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    RecCursor lc, sc;
+    RecCursor<kTmaChunk> lc, sc;
     lc.init(a, s_i0, s_off0, lo, hi);
     sc.init(a, s_i0, s_off0, lo, hi);
     auto issue_load = [&](uint32_t k) {
@@ -199,6 +209,18 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
     }
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
+  if (a->stamps != nullptr && threadIdx.x == 0) {
+    unsigned long long t_end, slot;
+    uint32_t smid;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    slot = atomicAdd(a->stamps, 1ull);
+    if (slot < (1ull << 20) - 1) {
+      unsigned long long* e = a->stamps + 4 * (slot + 1);
+      e[0] = ((unsigned long long)a->launch << 32) | ((unsigned long long)blockIdx.x << 8) | (smid & 255u);
+      e[1] = t_enter; e[2] = t_scan; e[3] = t_end;
+    }
+  }
 
   // < 16-byte tails and unaligned records: byte copies, record k by CTA k % grid
   if (single) {
@@ -217,22 +239,85 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
   }
 }
 
-cudaError_t launch_copy_records(const RecCopyArgs& a, int grid, cudaStream_t s) {
-  if (a.total <= 0 && (a.rec == nullptr || a.n <= 0)) return cudaSuccess;
+template <int S, int C>
+static cudaError_t launch_ring(const RecCopyArgs& a, int grid, cudaStream_t s) {
   static bool attr = false;
-  const int smem = kTmaStages * kTmaChunk;
+  const int smem = S * C;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(copy_records_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaError_t e = cudaFuncSetAttribute(copy_records_tma_kernel<S, C>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  // at least one 16 KiB chunk per CTA; enough CTAs for the tail loop over the records
-  int64_t g = (a.total + kTmaChunk - 1) / kTmaChunk;
+  // at least one chunk per CTA; enough CTAs for the tail loop over the records
+  int64_t g = (a.total + C - 1) / C;
   if (a.rec != nullptr && g < a.n) g = a.n;
   if (g > grid) g = grid;
   if (g < 1) g = 1;
-  copy_records_tma_kernel<<<(int)g, kRecThreads, smem, s>>>(a);
+  copy_records_tma_kernel<S, C><<<(int)g, kRecThreads, smem, s>>>(a);
   return cudaGetLastError();
+}
+
+// DYO_TMA_RING = "4x16" (default) | "8x16" | "4x32" | "6x32" | "3x64" (stages x KiB)
+static int tma_ring() {
+  static int r = -1;
+  if (r < 0) {
+    r = 0;
+    if (const char* e = getenv("DYO_TMA_RING")) {
+      const char* names[] = {"4x16", "8x16", "4x32", "6x32", "3x64"};
+      for (int q = 0; q < 5; ++q)
+        if (strcmp(e, names[q]) == 0) r = q;
+    }
+  }
+  return r;
+}
+
+// DYO_TMA_CTAS_PER_SM = 1 (default) | 2 | 3: CTAs per SM of the record copy grid
+static int tma_ctas_per_sm() {
+  static int c = 0;
+  if (c == 0) {
+    c = 1;
+    if (const char* e = getenv("DYO_TMA_CTAS_PER_SM")) c = atoi(e) >= 2 && atoi(e) <= 3 ? atoi(e) : 1;
+  }
+  return c;
+}
+
+// DYO_COPY_STAMPS=1 (measurement aid): every record-copy CTA appends {launch<<32 | cta<<8 | smid,
+// globaltimer at entry, after the record scan, at the end} to a device log (slot 0 = count; up to
+// 2^20 - 1 entries), read back by dyo_debug_copy_stamps.
+static unsigned long long* g_stamps = nullptr;
+static int64_t g_launch = 0;
+int64_t copy_stamps_read(unsigned long long* host, int64_t cap) {
+  if (g_stamps == nullptr) return 0;
+  unsigned long long n = 0;
+  if (cudaMemcpy(&n, g_stamps, 8, cudaMemcpyDeviceToHost) != cudaSuccess) return -1;
+  if (n > (1ull << 20) - 1) n = (1ull << 20) - 1;
+  if ((int64_t)n > cap) n = (unsigned long long)cap;
+  if (host != nullptr && n > 0 &&
+      cudaMemcpy(host, g_stamps + 4, n * 32, cudaMemcpyDeviceToHost) != cudaSuccess) return -1;
+  return (int64_t)n;
+}
+
+cudaError_t launch_copy_records(const RecCopyArgs& a0, int grid, cudaStream_t s) {
+  if (a0.total <= 0 && (a0.rec == nullptr || a0.n <= 0)) return cudaSuccess;
+  RecCopyArgs a = a0;
+  static int stamps_on = -1;
+  if (stamps_on < 0) {
+    const char* e = getenv("DYO_COPY_STAMPS");
+    stamps_on = (e != nullptr && e[0] == '1') ? 1 : 0;
+    if (stamps_on) {
+      if (cudaMalloc(&g_stamps, (size_t)32 << 20) != cudaSuccess) return cudaGetLastError();
+      cudaMemset(g_stamps, 0, 8);
+    }
+  }
+  if (stamps_on) { a.stamps = g_stamps; a.launch = g_launch++; }
+  grid *= tma_ctas_per_sm();
+  switch (tma_ring()) {
+    case 1: return launch_ring<8, 16 << 10>(a, grid, s);
+    case 2: return launch_ring<4, 32 << 10>(a, grid, s);
+    case 3: return launch_ring<6, 32 << 10>(a, grid, s);
+    case 4: return launch_ring<3, 64 << 10>(a, grid, s);
+    default: return launch_ring<kTmaStages, kTmaChunk>(a, grid, s);
+  }
 }
 
 cudaError_t launch_copy_segments(const CopySeg* segs, int n, int64_t /*chunk*/, int grid,

@@ -241,7 +241,10 @@ struct RecCopyArgs {
   char* dst_base;
   int64_t dst_bias;
   int64_t total;
+  unsigned long long* stamps;  // measurement aid (DYO_COPY_STAMPS): 4 x u64 per CTA, or null
+  int64_t launch;              // launch index for the stamps
 };
+int64_t copy_stamps_read(unsigned long long* host, int64_t cap);
 inline int64_t rec_body(const char* src, const char* dst, int64_t bytes) {
   return ((((uintptr_t)src) | ((uintptr_t)dst)) & 15) == 0 ? (bytes & ~(int64_t)15) : 0;
 }

@@ -97,7 +97,8 @@ def lib():
                      "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records", "dyo_migrate",
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
                      "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
-                     "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats"):
+                     "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats",
+                     "dyo_debug_copy_stamps"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -108,7 +109,7 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_prediction_get", "dyo_prediction_matched", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
            "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
-           "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats")
+           "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps")
 
 
 def _a(x, dt):
@@ -403,6 +404,14 @@ class Dyo:
 
     def debug_floor(self, cluster, n_barriers, stream=0):
         self._check(self.L.dyo_debug_floor(self.ctx, cluster, n_barriers, P(stream)))
+
+    def copy_stamps(self, cap=1 << 20):
+        """DYO_COPY_STAMPS log: uint64 [n, 4] rows {launch<<32 | cta<<8 | smid, t_enter, t_scan, t_end}."""
+        out = np.zeros((cap, 4), np.uint64)
+        n = C.c_int64(0)
+        self._check(self.L.dyo_debug_copy_stamps(self.ctx, out.ctypes.data_as(C.POINTER(C.c_uint64)), cap,
+                                                 C.byref(n)))
+        return out[:n.value]
 
     def plan_stamps(self, j):
         out = np.zeros(64, np.uint64)

@@ -110,20 +110,6 @@ int main() {
     cudaEventRecord(e1, s1); CK(cudaEventSynchronize(e1));
     double t = ms_of(e0, e1);
     printf("SMALL %d x %d memcpyAsync: %.3f ms %.2f GB/s\n", n, tsz, t, (double)n * tsz / t / 1e6);
-#if CUDART_VERSION >= 12080
-    {
-      std::vector<void*> dsts(n), srcs(n); std::vector<size_t> szs(n);
-      for (int i = 0; i < n; i++) { dsts[i] = d + dofs[i]; srcs[i] = h + so[i]; szs[i] = tsz; }
-      cudaMemcpyAttributes attr = {}; attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-      attr.srcLocHint.type = cudaMemLocationTypeHost; attr.dstLocHint.type = cudaMemLocationTypeDevice; attr.dstLocHint.id = 0;
-      size_t attrIdx = 0, failIdx = 0;
-      cudaEventRecord(e0, s1);
-      cudaError_t err = cudaMemcpyBatchAsync(dsts.data(), srcs.data(), szs.data(), n, &attr, &attrIdx, 1, &failIdx, s1);
-      cudaEventRecord(e1, s1); CK(cudaEventSynchronize(e1));
-      t = ms_of(e0, e1);
-      printf("SMALL %d x %d memcpyBatchAsync (err=%d %s): %.3f ms %.2f GB/s\n", n, tsz, (int)err, cudaGetErrorString(err), t, (double)n * tsz / t / 1e6);
-    }
-#endif
     for (int g : {16, 64, 148}) {
       zc_gather<<<g, 512, 0, s1>>>(hd, d, dso, ddo, dnb, n);
       cudaEventRecord(e0, s1);

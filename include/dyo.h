@@ -342,9 +342,10 @@ dyo_status dyo_debug_floor(dyo_ctx* ctx, int32_t cluster, int32_t n_barriers, vo
 /* Measurement aid for the live rate of the record-copy kernel (survey section 8(d), migrate row):
  * with DYO_COPY_STAMPS=1 in the environment (read at the first copy launch of the process) every
  * CTA of copy_records_tma_kernel appends 4 x u64 {launch << 32 | cta << 8 | smid, globaltimer at
- * entry, after its record scan, at exit} to a device log of up to 2^20 - 1 entries. This call
+ * entry, after its record scan, at exit} to a device log of up to 2^22 - 1 entries. This call
  * synchronises the device and copies min(count, cap) entries (4 x u64 each, caller-owned host
- * buffer `out`, may be NULL with cap 0) and stores that number in *n (0 when stamps are off).
+ * buffer `out`) and stores that number in *n (0 when stamps are off); out == NULL with cap == 0
+ * empties the log instead (*n = 0).
  * DYO_E_INVAL on NULL ctx / n or cap < 0; DYO_E_CUDA if the readback fails. */
 dyo_status dyo_debug_copy_stamps(dyo_ctx* ctx, uint64_t* out, int64_t cap, int64_t* n);
 

@@ -77,6 +77,7 @@ __device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvt
 // remaining < 16-byte tails (and unaligned records) are copied by the CTAs' threads.
 
 constexpr int kRecThreads = 128;
+constexpr unsigned long long kStampCap = (1ull << 22) - 1;   // DYO_COPY_STAMPS log entries
 
 template <int CHUNK>
 struct RecCursor {
@@ -215,7 +216,7 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
     slot = atomicAdd(a->stamps, 1ull);
-    if (slot < (1ull << 20) - 1) {
+    if (slot < kStampCap) {
       unsigned long long* e = a->stamps + 4 * (slot + 1);
       e[0] = ((unsigned long long)a->launch << 32) | ((unsigned long long)blockIdx.x << 8) | (smid & 255u);
       e[1] = t_enter; e[2] = t_scan; e[3] = t_end;
@@ -246,6 +247,13 @@ static cudaError_t launch_ring(const RecCopyArgs& a, int grid, cudaStream_t s) {
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(copy_records_tma_kernel<S, C>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
+    // DYO_TMA_CARVEOUT=1: ask for the maximum shared-memory carveout (measurement of whether a
+    // carveout change between this kernel and its neighbours delays its start)
+    if (const char* v = getenv("DYO_TMA_CARVEOUT"))
+      if (v[0] == '1') {
+        e = cudaFuncSetAttribute(copy_records_tma_kernel<S, C>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+        if (e != cudaSuccess) return e;
+      }
     attr = true;
   }
   // at least one chunk per CTA; enough CTAs for the tail loop over the records
@@ -283,14 +291,15 @@ static int tma_ctas_per_sm() {
 
 // DYO_COPY_STAMPS=1 (measurement aid): every record-copy CTA appends {launch<<32 | cta<<8 | smid,
 // globaltimer at entry, after the record scan, at the end} to a device log (slot 0 = count; up to
-// 2^20 - 1 entries), read back by dyo_debug_copy_stamps.
+// 2^22 - 1 entries), read back by dyo_debug_copy_stamps.
 static unsigned long long* g_stamps = nullptr;
 static int64_t g_launch = 0;
 int64_t copy_stamps_read(unsigned long long* host, int64_t cap) {
   if (g_stamps == nullptr) return 0;
+  if (host == nullptr && cap == 0) return cudaMemset(g_stamps, 0, 8) == cudaSuccess ? 0 : -1;   // reset
   unsigned long long n = 0;
   if (cudaMemcpy(&n, g_stamps, 8, cudaMemcpyDeviceToHost) != cudaSuccess) return -1;
-  if (n > (1ull << 20) - 1) n = (1ull << 20) - 1;
+  if (n > kStampCap) n = kStampCap;
   if ((int64_t)n > cap) n = (unsigned long long)cap;
   if (host != nullptr && n > 0 &&
       cudaMemcpy(host, g_stamps + 4, n * 32, cudaMemcpyDeviceToHost) != cudaSuccess) return -1;
@@ -305,7 +314,7 @@ cudaError_t launch_copy_records(const RecCopyArgs& a0, int grid, cudaStream_t s)
     const char* e = getenv("DYO_COPY_STAMPS");
     stamps_on = (e != nullptr && e[0] == '1') ? 1 : 0;
     if (stamps_on) {
-      if (cudaMalloc(&g_stamps, (size_t)32 << 20) != cudaSuccess) return cudaGetLastError();
+      if (cudaMalloc(&g_stamps, (size_t)32 * (kStampCap + 1)) != cudaSuccess) return cudaGetLastError();
       cudaMemset(g_stamps, 0, 8);
     }
   }

@@ -405,10 +405,14 @@ class Dyo:
     def debug_floor(self, cluster, n_barriers, stream=0):
         self._check(self.L.dyo_debug_floor(self.ctx, cluster, n_barriers, P(stream)))
 
-    def copy_stamps(self, cap=1 << 20):
-        """DYO_COPY_STAMPS log: uint64 [n, 4] rows {launch<<32 | cta<<8 | smid, t_enter, t_scan, t_end}."""
-        out = np.zeros((cap, 4), np.uint64)
+    def copy_stamps(self, cap=1 << 22, reset=False):
+        """DYO_COPY_STAMPS log: uint64 [n, 4] rows {launch<<32 | cta<<8 | smid, t_enter, t_scan, t_end};
+        reset=True empties the log."""
         n = C.c_int64(0)
+        if reset:
+            self._check(self.L.dyo_debug_copy_stamps(self.ctx, None, 0, C.byref(n)))
+            return None
+        out = np.zeros((cap, 4), np.uint64)
         self._check(self.L.dyo_debug_copy_stamps(self.ctx, out.ctypes.data_as(C.POINTER(C.c_uint64)), cap,
                                                  C.byref(n)))
         return out[:n.value]

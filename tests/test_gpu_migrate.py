@@ -266,3 +266,44 @@ def test_copy_kernels_exact(mode, nbytes, soff, doff):
     assert torch.equal(dst[doff: doff + nbytes], src[soff: soff + nbytes])
     assert int(dst[:doff].sum()) == 0 and int(dst[doff + nbytes:].sum()) == 0
     d.close()
+
+
+_RING_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import workloads as WL
+from gpu_harness import make_ctx
+wl = WL.make("tiny")
+d = make_ctx(wl, flags=4)
+s = torch.cuda.current_stream().cuda_stream
+n_launch = 0
+for nbytes, soff, doff in [((3 << 20) + 5, 16, 48), (777, 3, 5), (40 << 20, 0, 4096)]:
+    src = torch.randint(0, 255, (nbytes + 8192,), dtype=torch.uint8, device="cuda")
+    dst = torch.zeros(nbytes + 8192, dtype=torch.uint8, device="cuda")
+    d.debug_copy(src.data_ptr() + soff, dst.data_ptr() + doff, nbytes, 1, s)
+    n_launch += 1
+    assert torch.equal(dst[doff: doff + nbytes], src[soff: soff + nbytes])
+    assert int(dst[:doff].sum()) == 0 and int(dst[doff + nbytes:].sum()) == 0
+st = d.copy_stamps()
+lid = (st[:, 0] >> np.uint64(32)).astype(np.int64)
+assert sorted(set(lid.tolist())) == list(range(n_launch)), lid
+t0, t1, t2 = (st[:, k].astype(np.int64) for k in (1, 2, 3))
+assert np.all(t0 <= t1) and np.all(t1 <= t2)
+d.copy_stamps(reset=True)
+assert len(d.copy_stamps()) == 0
+d.close()
+print("ok")
+"""
+
+
+@pytest.mark.parametrize("ring,ctas", [("4x16", 1), ("8x16", 2), ("4x32", 1), ("6x32", 1), ("3x64", 3)])
+def test_copy_ring_variants_exact_and_stamps(ring, ctas, tmp_path):
+    """Every TMA ring shape (DYO_TMA_RING) and grid multiplier moves exactly the bytes, including
+    unaligned heads/tails; the DYO_COPY_STAMPS log holds one ordered entry per CTA of each launch
+    and empties on reset. Runs in a child process: the knobs are read at the first copy launch."""
+    import os, subprocess, sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, DYO_TMA_RING=ring, DYO_TMA_CTAS_PER_SM=str(ctas), DYO_COPY_STAMPS="1",
+               PYTHONPATH=os.pathsep.join([root, os.path.join(root, "tests")]))
+    r = subprocess.run([sys.executable, "-c", _RING_CHILD, root], env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stdout[-2000:] + r.stderr[-2000:]

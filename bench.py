@@ -483,7 +483,7 @@ def run_dyo(args):
     barrier()
     d.timings(reset=True)
     d.counters(reset=True)
-    stamps_on = os.environ.get("DYO_COPY_STAMPS") == "1"
+    stamps_on = os.environ.get("DYO_COPY_STAMPS") in ("1", "2")
     if stamps_on:
         d.copy_stamps(reset=True)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -703,8 +703,14 @@ def copy_stamp_report(st, path):
     import numpy as np
     if len(st) == 0:
         return None
+    cta = ((st[:, 0] >> np.uint64(8)) & np.uint64(0xFFFFFF)).astype(np.int64)
+    mk = st[cta == 0xFFF]            # DYO_COPY_STAMPS=2 marker kernels around each launch
+    st = st[cta != 0xFFF]
     lid = (st[:, 0] >> np.uint64(32)).astype(np.int64)
     sm = (st[:, 0] & np.uint64(255)).astype(np.int64)
+    marks = {}
+    for row in mk:
+        marks[(int(row[0] >> np.uint64(32)), int(row[0] & np.uint64(255)))] = int(row[1])
     t0, t1, t2 = (st[:, k].astype(np.int64) for k in (1, 2, 3))
     rows = []
     for L in np.unique(lid):
@@ -714,7 +720,10 @@ def copy_stamp_report(st, path):
                      "start_skew_us": (a0.max() - a0.min()) / 1e3, "scan_us_max": (a1 - a0).max() / 1e3,
                      "cta_copy_us_med": float(np.median(a2 - a1)) / 1e3, "cta_copy_us_max": (a2 - a1).max() / 1e3,
                      "end_skew_us": (a2.max() - a2.min()) / 1e3, "distinct_sms": int(len(np.unique(sm[m])))})
-    keys = rows[0].keys()
+        if (int(L), 0) in marks and (int(L), 1) in marks:
+            rows[-1]["mark_to_first_cta_us"] = (a0.min() - marks[(int(L), 0)]) / 1e3
+            rows[-1]["last_cta_to_mark_us"] = (marks[(int(L), 1)] - a2.max()) / 1e3
+    keys = [k for k in rows[0].keys() if all(k in r for r in rows)]
     med = {k: float(np.median([r[k] for r in rows])) for k in keys}
     big = [r for r in rows if r["span_us"] >= 20]
     out = {"launches": len(rows), "median": med, "sum_span_us": float(sum(r["span_us"] for r in rows)),

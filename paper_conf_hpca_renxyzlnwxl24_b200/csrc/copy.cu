@@ -293,6 +293,20 @@ static int tma_ctas_per_sm() {
 // globaltimer at entry, after the record scan, at the end} to a device log (slot 0 = count; up to
 // 2^22 - 1 entries), read back by dyo_debug_copy_stamps.
 static unsigned long long* g_stamps = nullptr;
+
+// DYO_COPY_STAMPS=2 also brackets each record-copy launch with a one-thread marker kernel on the
+// same stream (entry cta field 0xFFF, smid field 0 = before, 1 = after): it locates the time
+// between the CUDA events and the copy kernel's CTAs.
+__global__ void copy_mark_kernel(unsigned long long* stamps, int64_t launch, int which) {
+  unsigned long long t, slot;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  slot = atomicAdd(stamps, 1ull);
+  if (slot < kStampCap) {
+    unsigned long long* e = stamps + 4 * (slot + 1);
+    e[0] = ((unsigned long long)launch << 32) | (0xFFFull << 8) | (unsigned)which;
+    e[1] = t; e[2] = t; e[3] = t;
+  }
+}
 static int64_t g_launch = 0;
 int64_t copy_stamps_read(unsigned long long* host, int64_t cap) {
   if (g_stamps == nullptr) return 0;
@@ -312,21 +326,28 @@ cudaError_t launch_copy_records(const RecCopyArgs& a0, int grid, cudaStream_t s)
   static int stamps_on = -1;
   if (stamps_on < 0) {
     const char* e = getenv("DYO_COPY_STAMPS");
-    stamps_on = (e != nullptr && e[0] == '1') ? 1 : 0;
+    stamps_on = (e != nullptr && (e[0] == '1' || e[0] == '2')) ? (e[0] - '0') : 0;
     if (stamps_on) {
       if (cudaMalloc(&g_stamps, (size_t)32 * (kStampCap + 1)) != cudaSuccess) return cudaGetLastError();
       cudaMemset(g_stamps, 0, 8);
     }
   }
   if (stamps_on) { a.stamps = g_stamps; a.launch = g_launch++; }
+  if (stamps_on == 2) copy_mark_kernel<<<1, 1, 0, s>>>(g_stamps, a.launch, 0);
   grid *= tma_ctas_per_sm();
+  cudaError_t e;
   switch (tma_ring()) {
-    case 1: return launch_ring<8, 16 << 10>(a, grid, s);
-    case 2: return launch_ring<4, 32 << 10>(a, grid, s);
-    case 3: return launch_ring<6, 32 << 10>(a, grid, s);
-    case 4: return launch_ring<3, 64 << 10>(a, grid, s);
-    default: return launch_ring<kTmaStages, kTmaChunk>(a, grid, s);
+    case 1: e = launch_ring<8, 16 << 10>(a, grid, s); break;
+    case 2: e = launch_ring<4, 32 << 10>(a, grid, s); break;
+    case 3: e = launch_ring<6, 32 << 10>(a, grid, s); break;
+    case 4: e = launch_ring<3, 64 << 10>(a, grid, s); break;
+    default: e = launch_ring<kTmaStages, kTmaChunk>(a, grid, s); break;
   }
+  if (e == cudaSuccess && stamps_on == 2) {
+    copy_mark_kernel<<<1, 1, 0, s>>>(g_stamps, a.launch, 1);
+    e = cudaGetLastError();
+  }
+  return e;
 }
 
 cudaError_t launch_copy_segments(const CopySeg* segs, int n, int64_t /*chunk*/, int grid,

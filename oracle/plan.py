@@ -74,12 +74,34 @@ def aligned(nbytes, align):
     return (nbytes + align - 1) // align * align
 
 
-def next_use(Ws, t, j):
-    """(distance to the first group j' > j whose tensor set holds t, that entry) or (INF, None)."""
-    for jj in range(j + 1, len(Ws)):
-        for e in Ws[jj]:
-            if e[0] == t:
-                return jj - j, e
+def tensor_table(wl):
+    """(aligned sizes, byte sizes, host offsets) of every tensor, cached on the workload."""
+    key = (wl.align, len(wl.tensors))
+    cached = getattr(wl, "_oracle_tensor_table", None)
+    if cached is None or cached[0] != key:
+        a = [aligned(t.nbytes, wl.align) for t in wl.tensors]
+        cached = (key, (a, [t.nbytes for t in wl.tensors], [t.host_off for t in wl.tensors]))
+        wl._oracle_tensor_table = cached
+    return cached[1]
+
+
+def occurrences(Ws):
+    """occ[t] = [(j, entry), ...] in ascending j: every group whose tensor set holds t."""
+    occ = {}
+    for jj, Wj in enumerate(Ws):
+        for e in Wj:
+            occ.setdefault(e[0], []).append((jj, e))
+    return occ
+
+
+def next_use(Ws, t, j, occ=None):
+    """(distance to the first group j' > j whose tensor set holds t, that entry) or (INF, None).
+    occ (from occurrences(Ws)) only indexes the same search."""
+    if occ is None:
+        occ = occurrences(Ws)
+    for jj, e in occ.get(t, ()):
+        if jj > j:
+            return jj - j, e
     return INF, None
 
 
@@ -118,14 +140,14 @@ def first_fit(kept, placed, off, a, H):
     return new_off
 
 
-def transition(state, wl, Ws, j, policy, choose=None):
+def transition(state, wl, Ws, j, policy, choose=None, occ=None):
     """Plan transition j in place on `state`. `choose(live, room)` overrides the retention
-    choice (brute force); default is the policy's."""
+    choice (brute force); default is the policy's. occ: occurrences(Ws), to share the index."""
+    if occ is None:
+        occ = occurrences(Ws)
     T = len(wl.tensors)
     H = half_size(wl.budget, wl.align)
-    a = [aligned(t.nbytes, wl.align) for t in wl.tensors]
-    nb = [t.nbytes for t in wl.tensors]
-    host_off = [t.host_off for t in wl.tensors]
+    a, nb, host_off = tensor_table(wl)
     m = (state.G + j) % 2
     Wj = Ws[j]
     need = sum(a[t] for t, _, _ in Wj)
@@ -149,7 +171,7 @@ def transition(state, wl, Ws, j, policy, choose=None):
     cands = [t for t in range(T) if state.loc[t] == m and t not in in_w]
     live, dead = [], []
     for t in cands:
-        d, e = next_use(Ws, t, j)
+        d, e = next_use(Ws, t, j, occ)
         is_dead = (e is None and wl.tensors[t].transient) or (e is not None and not e[2])
         if is_dead:
             dead.append(t)
@@ -218,6 +240,7 @@ def plan(state, wl, Ws, policy=None):
     for t, ten in enumerate(wl.tensors):      # R9: a transient tensor's contents end with the step
         if ten.transient:
             st.dirty[t] = False
-    trs = [transition(st, wl, Ws, j, policy) for j in range(len(Ws))]
+    occ = occurrences(Ws)
+    trs = [transition(st, wl, Ws, j, policy, occ=occ) for j in range(len(Ws))]
     st.G += len(Ws)
     return trs, st

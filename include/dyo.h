@@ -273,6 +273,23 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
  * on the host). Valid until the next dyo_migrate that moves it. */
 dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr);
 
+/* Introspection of the last calls (tests and measurement; host-only, no synchronisation).
+ *   DYO_Q_PILOT_KERNEL: kernel the last dyo_pilot_predict ran: 0 = K1 cluster GEMV (batch < 16,
+ *     or DYO_PILOT_TC=0), 1 = K1-TC (tcgen05 tensor cores, batch >= 16).
+ *   DYO_Q_DECODE_FUSED: 1 if the last dyo_pilot_predict decoded in K1's epilogue, 0 if it
+ *     launched the stand-alone decode kernels.
+ *   DYO_Q_PLAN_SYNCS: host synchronisations taken by the last successful dyo_plan (1, §8(b)).
+ * DYO_E_INVAL for a NULL ctx / value or an unknown `what`. */
+/* Measurement switch at run time: sets or clears DYO_F_TIMING (the only flag that may change
+ * after dyo_create; DYO_E_INVAL for any other bit). With it clear no timing events are recorded,
+ * so a headline measurement runs uninstrumented and a second pass gets the breakdown. */
+dyo_status dyo_set_timing(dyo_ctx* ctx, int32_t on);
+
+#define DYO_Q_PILOT_KERNEL 0
+#define DYO_Q_DECODE_FUSED 1
+#define DYO_Q_PLAN_SYNCS 2
+dyo_status dyo_query(dyo_ctx* ctx, int32_t what, int64_t* value);
+
 /* Per-ctx counters of the last dyo_plan / dyo_migrate calls (bytes by mechanism, launches). */
 typedef struct {
   int64_t h2d_dma, h2d_zc, d2h_dma, d2h_zc, d2h_packed, d2d;
@@ -324,8 +341,10 @@ dyo_status dyo_debug_plan_stamps(dyo_ctx* ctx, int32_t j, uint64_t* out64);
  *   the last dyo_pilot_predict). *mispredicted (may be NULL) = 1 if they differ. On a
  *   mis-prediction the count is incremented and, with the memo enabled, the prediction's raw
  *   output -> actual choices is memoised (host mirror + device table). DYO_E_INVAL on a bad b or
- *   an invalid choice vector. Synchronises the device (the report follows the sample's
- *   execution). Branch-head arches only (with the traversal decode the memo is not consulted).
+ *   an invalid choice vector. Stream-ordered: waits (host) only for the end of the last
+ *   dyo_pilot_predict (the prediction being reported), reads it back on a ctx-owned stream, and
+ *   uploads a new memo entry on that stream; the next dyo_pilot_predict waits for the upload on
+ *   the device (no device-wide synchronisation). Branch-head arches only (with the traversal decode the memo is not consulted).
  * dyo_memo_stats: mis-predictions reported so far (since dyo_load_arch), live memo entries, and
  *   memo hits taken by the decode kernels (device counter). Any pointer may be NULL. */
 dyo_status dyo_memo_config(dyo_ctx* ctx, int32_t capacity);

@@ -65,6 +65,17 @@ struct dyo_ctx {
   const TcPlan* tc_dev = nullptr;
   int tc_flag_off = 0;             // DYO_PILOT_TC=0 in the environment disables it (measurement)
   int last_tc = 0;                 // the last dyo_pilot_predict ran K1-TC
+  int last_fused = 0;              // the last dyo_pilot_predict decoded in K1's epilogue
+  int64_t last_plan_syncs = 0;     // host synchronisations taken by the last dyo_plan
+  // stream-ordered mis-prediction reports (R15): the report / stats readbacks and the memo
+  // uploads run on `aux`; ev_pred marks the end of the last dyo_pilot_predict, ev_memo the last
+  // memo upload (the next predict waits on it)
+  cudaStream_t aux = nullptr;
+  cudaEvent_t ev_pred = nullptr, ev_memo = nullptr;
+  bool memo_pending = false;
+  int32_t* h_rep = nullptr;        // pinned readback of a report (status, choices, key)
+  char* h_memo_stage = nullptr;    // pinned staging of a memo upload (entry + index)
+  size_t h_memo_stage_bytes = 0;
   int64_t* desc_dev = nullptr;
   int32_t* hist_dev = nullptr;
   int32_t* hist_tab[2] = {nullptr, nullptr};
@@ -82,12 +93,15 @@ struct dyo_ctx {
   struct PlanSlot {
     PlanOut out{};                 // host (pinned) mirrors of the plan records + headers
     PlanOut dout{};                // device record arrays the planner kernel writes
+    PlanOut hout{};                // device-side aliases of the pinned mirrors (export kernel)
     CopySeg* h_segs = nullptr;     // pinned mapped work items for the copy kernels
     int64_t seg_cap = 0, seg_used = 0;
     int K = 0, next_j = 0;
     bool valid = false;
     cudaEvent_t ev_last = nullptr; // recorded after every migrate of this plan
     bool ev_pending = false;
+    bool ent_host = false;         // entry records copied to out.ent (lazily, dyo_plan_records)
+    int64_t n_ent = 0;
   };
   PlanSlot slot[2];
   int64_t plan_seq = 0, mig_seq = 0;
@@ -225,7 +239,8 @@ void free_plan_host(dyo_ctx* c) {
     P.seg_used = 0;
   }
   fh(c->h_status); fh(c->h_counts); fh(c->h_loc); fh(c->h_off);
-  fh(c->h_forced[0]); fh(c->h_forced[1]); fh(c->h_matched);
+  fh(c->h_forced[0]); fh(c->h_forced[1]); fh(c->h_matched); fh(c->h_rep);
+  c->h_rep = nullptr;
   c->h_forced[0] = c->h_forced[1] = c->h_matched = nullptr;
   c->h_status = c->h_counts = nullptr;
   c->h_loc = nullptr;
@@ -539,6 +554,9 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
     return DYO_E_INVAL;
   }
   if (c.staging_bytes <= 0) c.staging_bytes = 64ll << 20;
+  // compaction stages self-overlapping moves through two staging halves of >= max(256, ALIGN)
+  // bytes each (a smaller staging would never advance)
+  c.staging_bytes = std::max<int64_t>(c.staging_bytes, 2 * std::max<int64_t>(256, c.align));
   if (c.dma_min_bytes <= 0) c.dma_min_bytes = 2ll << 20;
   ctx->H = c.budget / 2 / c.align * c.align;
   if (ctx->H / c.align >= (1ll << 28)) { delete ctx; return DYO_E_INVAL; }
@@ -554,6 +572,9 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_moves, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_carry, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, device);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_pred, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_memo, cudaEventDisableTiming);
   if (e != cudaSuccess) {
     dyo_destroy(ctx);
     return e == cudaErrorMemoryAllocation ? DYO_E_NOMEM : DYO_E_CUDA;
@@ -597,6 +618,11 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->side) cudaStreamDestroy(ctx->side);
   if (ctx->ev_moves) cudaEventDestroy(ctx->ev_moves);
   if (ctx->ev_carry) cudaEventDestroy(ctx->ev_carry);
+  if (ctx->aux) cudaStreamDestroy(ctx->aux);
+  if (ctx->ev_pred) cudaEventDestroy(ctx->ev_pred);
+  if (ctx->ev_memo) cudaEventDestroy(ctx->ev_memo);
+  if (ctx->h_rep) cudaFreeHost(ctx->h_rep);
+  if (ctx->h_memo_stage) cudaFreeHost(ctx->h_memo_stage);
   for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   if (ctx->ev_ref) cudaEventDestroy(ctx->ev_ref);
@@ -707,6 +733,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   if ((st = hmap((void**)&ctx->h_counts, 16 * sizeof(int32_t)))) return st;
   if ((st = hmap((void**)&ctx->h_loc, T))) return st;
   if ((st = hmap((void**)&ctx->h_off, sizeof(int64_t) * T))) return st;
+  if ((st = hmap((void**)&ctx->h_rep, sizeof(int32_t) * (4 + 10 * (size_t)K + 2 * (size_t)std::max(n_sites, 1))))) return st;
   if (!ctx->branch_head) {
     for (int i = 0; i < 2; ++i)
       if ((st = hmap((void**)&ctx->h_forced[i], sizeof(int32_t) * B * std::max(n_sites, 1)))) return st;
@@ -738,10 +765,19 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
     PlanHdr* h1; dyo_entry_rec* e1; dyo_evict_rec* v1; dyo_move_rec* m1; dyo_carry_rec* c1; dyo_alloc_rec* a1; dyo_fetch_rec* f1;
     DA(h1, mg); DA(e1, cap_ent); DA(v1, cap_rec); DA(m1, cap_rec); DA(c1, cap_rec); DA(a1, cap_rec); DA(f1, cap_rec);
     dO.hdr = h1; dO.ent = e1; dO.ev = v1; dO.mv = m1; dO.ca = c1; dO.al = a1; dO.fe = f1;
+    PlanOut& hO = P.hout;
+    hO = o;
+    CK(cudaHostGetDevicePointer((void**)&hO.hdr, o.hdr, 0));
+    CK(cudaHostGetDevicePointer((void**)&hO.ev, o.ev, 0));
+    CK(cudaHostGetDevicePointer((void**)&hO.mv, o.mv, 0));
+    CK(cudaHostGetDevicePointer((void**)&hO.ca, o.ca, 0));
+    CK(cudaHostGetDevicePointer((void**)&hO.al, o.al, 0));
+    CK(cudaHostGetDevicePointer((void**)&hO.fe, o.fe, 0));
+    hO.ent = nullptr;
     P.seg_cap = 8 * cap_rec + 65536;
     if ((st = hmap((void**)&P.h_segs, sizeof(CopySeg) * P.seg_cap))) return st;
-    o.status = dO.status = d_status;
-    o.counts = dO.counts = d_counts;
+    o.status = dO.status = hO.status = d_status;
+    o.counts = dO.counts = hO.counts = d_counts;
     P.valid = false;
     P.K = P.next_j = 0;
     P.seg_used = 0;
@@ -1097,6 +1133,12 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
   } else if (!is_device_ptr(feat)) {
     return fail(ctx, DYO_E_INVAL, "feat must be device memory");
   }
+  if (ctx->memo_pending) {
+    // decode kernels read the memo table: order them after the last upload (dyo_report)
+    if (cudaEventQuery(ctx->ev_memo) == cudaSuccess) ctx->memo_pending = false;
+    else CK(cudaStreamWaitEvent(st, ctx->ev_memo, 0));
+    cudaGetLastError();
+  }
   const int cur = ctx->hist_cur;
   int fused = 0;
   {
@@ -1142,6 +1184,8 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
   ctx->hist_B[1 - cur] = B;
   ctx->hist_cur = 1 - cur;
   ctx->last_B = B;
+  ctx->last_fused = fused;
+  CK(cudaEventRecord(ctx->ev_pred, st));
   return DYO_OK;
 }
 
@@ -1169,19 +1213,40 @@ uint64_t memo_hash_of(const int32_t* key, int kw_total) {
   for (int i = 0; i < kw_total; ++i) h += dyo::memo_mix((uint64_t)i, key[i]);
   return h ? h : 1;
 }
-dyo_status memo_upload_entry(dyo_ctx* ctx, int id) {
+// Upload entry `id` (and the index when with_index) of the host mirror to the device table:
+// staged in pinned memory, copied on the ctx's aux stream, ordered before the next
+// dyo_pilot_predict by ev_memo (no device-wide synchronisation).
+dyo_status memo_upload(dyo_ctx* ctx, int id, bool with_index) {
   auto& M = ctx->memo;
   const int kt = M.kw + M.ns;
-  CK(cudaMemcpy(static_cast<uint64_t*>(M.dev[1]) + id, &M.hash[id], 8, cudaMemcpyHostToDevice));
-  CK(cudaMemcpy(static_cast<int32_t*>(M.dev[2]) + (size_t)id * kt, &M.key[(size_t)id * kt], 4 * (size_t)kt, cudaMemcpyHostToDevice));
+  const size_t need = 8 + 4 * (size_t)kt + 4 * (size_t)std::max(M.ns, 1) + 4 * M.index.size();
+  if (ctx->memo_pending) CK(cudaEventSynchronize(ctx->ev_memo));   // the staging is reused
+  ctx->memo_pending = false;
+  if (ctx->h_memo_stage_bytes < need) {
+    if (ctx->h_memo_stage) cudaFreeHost(ctx->h_memo_stage);
+    ctx->h_memo_stage = nullptr;
+    ctx->h_memo_stage_bytes = 0;
+    CK(cudaHostAlloc((void**)&ctx->h_memo_stage, need, cudaHostAllocPortable));
+    ctx->h_memo_stage_bytes = need;
+  }
+  char* q = ctx->h_memo_stage;
+  memcpy(q, &M.hash[id], 8);
+  memcpy(q + 8, &M.key[(size_t)id * kt], 4 * (size_t)kt);
+  char* qv = q + 8 + 4 * (size_t)kt;
+  if (M.ns) memcpy(qv, &M.val[(size_t)id * M.ns], 4 * (size_t)M.ns);
+  char* qi = qv + 4 * (size_t)std::max(M.ns, 1);
+  CK(cudaMemcpyAsync(static_cast<uint64_t*>(M.dev[1]) + id, q, 8, cudaMemcpyHostToDevice, ctx->aux));
+  CK(cudaMemcpyAsync(static_cast<int32_t*>(M.dev[2]) + (size_t)id * kt, q + 8, 4 * (size_t)kt, cudaMemcpyHostToDevice,
+                     ctx->aux));
   if (M.ns)
-    CK(cudaMemcpy(static_cast<int32_t*>(M.dev[3]) + (size_t)id * M.ns, &M.val[(size_t)id * M.ns], 4 * (size_t)M.ns,
-                  cudaMemcpyHostToDevice));
-  return DYO_OK;
-}
-dyo_status memo_upload_index(dyo_ctx* ctx) {
-  auto& M = ctx->memo;
-  CK(cudaMemcpy(M.dev[0], M.index.data(), 4 * M.index.size(), cudaMemcpyHostToDevice));
+    CK(cudaMemcpyAsync(static_cast<int32_t*>(M.dev[3]) + (size_t)id * M.ns, qv, 4 * (size_t)M.ns,
+                       cudaMemcpyHostToDevice, ctx->aux));
+  if (with_index) {
+    memcpy(qi, M.index.data(), 4 * M.index.size());
+    CK(cudaMemcpyAsync(M.dev[0], qi, 4 * M.index.size(), cudaMemcpyHostToDevice, ctx->aux));
+  }
+  CK(cudaEventRecord(ctx->ev_memo, ctx->aux));
+  ctx->memo_pending = true;
   return DYO_OK;
 }
 // slot of entry `id` (or of key `key` when id < 0) in the index; -1 if absent
@@ -1215,6 +1280,7 @@ dyo_status dyo_memo_config(dyo_ctx* ctx, int32_t capacity) {
   CK(cudaSetDevice(ctx->device));
   CK(cudaDeviceSynchronize());
   memo_free(ctx);
+  ctx->memo_pending = false;
   if (capacity == 0) return DYO_OK;
   auto& M = ctx->memo;
   M.cap = capacity;
@@ -1238,8 +1304,7 @@ dyo_status dyo_memo_config(dyo_ctx* ctx, int32_t capacity) {
     CK(cudaMemset(p, 0, b));
     M.dev.push_back(p);
   }
-  dyo_status st = memo_upload_index(ctx);
-  if (st) return st;
+  CK(cudaMemcpy(M.dev[0], M.index.data(), 4 * M.index.size(), cudaMemcpyHostToDevice));
   ctx->ad.memo_mask = M.mask;
   ctx->ad.memo_live = 0;
   ctx->ad.memo_index = static_cast<const int32_t*>(M.dev[0]);
@@ -1260,21 +1325,29 @@ dyo_status dyo_report(dyo_ctx* ctx, int32_t b, const int32_t* actual, int32_t* m
       return fail(ctx, DYO_E_INVAL, "site %d must replay site %d (R6)", i, T.site_tie[i]);
   }
   CK(cudaSetDevice(ctx->device));
-  CK(cudaDeviceSynchronize());
-  int32_t status = 0;
-  CK(cudaMemcpy(&status, ctx->pd.status, sizeof status, cudaMemcpyDeviceToHost));
-  if (status) return fail(ctx, (dyo_status)status, "decode failed (status %d)", status);
+  // stream-ordered readback: the aux stream waits for the end of the last dyo_pilot_predict
+  // (its decode) and copies the status, the final choices and the memo key of prediction b to
+  // pinned memory; the host waits for that stream only
   const int Km = ctx->K_max;
-  std::vector<int32_t> fin(std::max(ns, 1)), key((size_t)10 * Km + ns);
-  if (ns) CK(cudaMemcpy(fin.data(), ctx->pd.choices + (size_t)b * ns, 4 * (size_t)ns, cudaMemcpyDeviceToHost));
-  const bool miss = !std::equal(actual, actual + ns, fin.data());
+  int32_t* hr = ctx->h_rep;
+  int32_t* h_fin = hr + 4;
+  int32_t* h_key = h_fin + std::max(ns, 1);
+  CK(cudaStreamWaitEvent(ctx->aux, ctx->ev_pred, 0));
+  CK(cudaMemcpyAsync(hr, ctx->pd.status, sizeof(int32_t), cudaMemcpyDeviceToHost, ctx->aux));
+  if (ns) CK(cudaMemcpyAsync(h_fin, ctx->pd.choices + (size_t)b * ns, 4 * (size_t)ns, cudaMemcpyDeviceToHost, ctx->aux));
+  CK(cudaMemcpyAsync(h_key, ctx->pd.slots + (size_t)b * Km * 10, 4 * (size_t)Km * 10, cudaMemcpyDeviceToHost, ctx->aux));
+  if (ns) CK(cudaMemcpyAsync(h_key + 10 * Km, ctx->pd.rchoices + (size_t)b * ns, 4 * (size_t)ns, cudaMemcpyDeviceToHost,
+                             ctx->aux));
+  CK(cudaStreamSynchronize(ctx->aux));
+  const int32_t status = hr[0];
+  if (status) return fail(ctx, (dyo_status)status, "decode failed (status %d)", status);
+  const bool miss = !std::equal(actual, actual + ns, h_fin);
   if (mispredicted) *mispredicted = miss ? 1 : 0;
   if (!miss) return DYO_OK;
   ctx->memo.mispredictions++;
   auto& M = ctx->memo;
   if (M.cap == 0) return DYO_OK;                   // recorded (counted), memo disabled
-  CK(cudaMemcpy(key.data(), ctx->pd.slots + (size_t)b * Km * 10, 4 * (size_t)Km * 10, cudaMemcpyDeviceToHost));
-  if (ns) CK(cudaMemcpy(key.data() + 10 * Km, ctx->pd.rchoices + (size_t)b * ns, 4 * (size_t)ns, cudaMemcpyDeviceToHost));
+  std::vector<int32_t> key(h_key, h_key + (size_t)10 * Km + ns);
   const int kt = M.kw + M.ns;
   const uint64_t h = memo_hash_of(key.data(), kt);
   const int slot_old = memo_find(M, h, key.data(), -1);
@@ -1284,7 +1357,7 @@ dyo_status dyo_report(dyo_ctx* ctx, int32_t b, const int32_t* actual, int32_t* m
     std::copy(actual, actual + ns, &M.val[(size_t)id * ns]);
     M.fifo.erase(std::find(M.fifo.begin(), M.fifo.end(), id));
     M.fifo.push_back(id);
-    return memo_upload_entry(ctx, id);
+    return memo_upload(ctx, id, false);
   }
   if (M.live == M.cap) {                            // FIFO replacement of the oldest key
     const int old = M.fifo.front();
@@ -1309,8 +1382,7 @@ dyo_status dyo_report(dyo_ctx* ctx, int32_t b, const int32_t* actual, int32_t* m
     if (M.index[slot] == -2) --M.tomb;
     M.index[slot] = id;
   }
-  if ((st = memo_upload_entry(ctx, id))) return st;
-  if ((st = memo_upload_index(ctx))) return st;
+  if ((st = memo_upload(ctx, id, true))) return st;
   ctx->ad.memo_live = M.live;
   return DYO_OK;
 }
@@ -1322,9 +1394,12 @@ dyo_status dyo_memo_stats(dyo_ctx* ctx, int64_t* mispredictions, int32_t* live, 
   if (hits) {
     *hits = 0;
     if (!ctx->memo.dev.empty()) {
-      CK(cudaDeviceSynchronize());
+      // hits counted by the decode kernels of every prediction so far (stream-ordered readback)
+      CK(cudaStreamWaitEvent(ctx->aux, ctx->ev_pred, 0));
+      CK(cudaMemcpyAsync(ctx->h_rep, ctx->memo.dev[4], 8, cudaMemcpyDeviceToHost, ctx->aux));
+      CK(cudaStreamSynchronize(ctx->aux));
       unsigned long long v = 0;
-      CK(cudaMemcpy(&v, ctx->memo.dev[4], 8, cudaMemcpyDeviceToHost));
+      memcpy(&v, ctx->h_rep, 8);
       *hits = (int64_t)v;
     }
   }
@@ -1385,9 +1460,14 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
     TScope ts(ctx, 2, st);
     CK(launch_plan(ctx->ad, ctx->pd, b0, n, ctx->cfg.policy, in, wk, ctx->sc, P.dout, ctx->max_groups, st));
   }
+  // the export kernel copies the headers and the EVICT/MOVE/CARRY/ALLOC/FETCH records (the DMA
+  // issue needs them on the host) into the pinned mirrors by the counts the planner left in
+  // mapped memory; entry records stay on the device until dyo_plan_records asks for them
+  CK(launch_plan_export(P.dout, P.hout, st));
   CK(cudaMemcpyAsync(ctx->h_loc, wk.loc, ctx->T, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(ctx->h_off, wk.off, sizeof(int64_t) * ctx->T, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));     // the one synchronisation of the hot path (DMA sizes to host)
+  ctx->last_plan_syncs = 1;
   const int32_t status = ctx->h_status[0];
   if (status != 0) {
     // restore the residency mirror of the committed state
@@ -1398,23 +1478,9 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
     return fail(ctx, (dyo_status)(status < 0 ? status : DYO_E_CUDA), "planner status %d", status);
   }
   {
-    // copy the plan (headers + every record list, exact counts) to the pinned host mirrors
-    const int32_t* c = ctx->h_counts;
-    const PlanOut& D = P.dout;
-    PlanOut& Hm = P.out;
-    int64_t n_ent = 0;
-    if (c[0] > 0) {
-      CK(cudaMemcpyAsync(Hm.hdr, D.hdr, sizeof(PlanHdr) * c[0], cudaMemcpyDeviceToHost, st));
-    }
-    CK(cudaStreamSynchronize(st));
-    for (int g = 0; g < c[0]; ++g) n_ent += Hm.hdr[g].n_ent;
-    if (n_ent) CK(cudaMemcpyAsync(Hm.ent, D.ent, sizeof(dyo_entry_rec) * n_ent, cudaMemcpyDeviceToHost, st));
-    if (c[1]) CK(cudaMemcpyAsync(Hm.ev, D.ev, sizeof(dyo_evict_rec) * c[1], cudaMemcpyDeviceToHost, st));
-    if (c[2]) CK(cudaMemcpyAsync(Hm.mv, D.mv, sizeof(dyo_move_rec) * c[2], cudaMemcpyDeviceToHost, st));
-    if (c[3]) CK(cudaMemcpyAsync(Hm.ca, D.ca, sizeof(dyo_carry_rec) * c[3], cudaMemcpyDeviceToHost, st));
-    if (c[4]) CK(cudaMemcpyAsync(Hm.al, D.al, sizeof(dyo_alloc_rec) * c[4], cudaMemcpyDeviceToHost, st));
-    if (c[5]) CK(cudaMemcpyAsync(Hm.fe, D.fe, sizeof(dyo_fetch_rec) * c[5], cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
+    const int K = ctx->h_counts[0];
+    P.n_ent = K > 0 ? P.out.hdr[K - 1].o_ent + P.out.hdr[K - 1].n_ent : 0;
+    P.ent_host = false;
   }
   ctx->committed = 1 - ctx->committed;
   P.K = ctx->h_counts[0];
@@ -1450,7 +1516,12 @@ dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** 
     case 2: *recs = P.out.ca + h.o_carry; *n = h.n_carry; break;
     case 3: *recs = P.out.al + h.o_alloc; *n = h.n_alloc; break;
     case 4: *recs = P.out.fe + h.o_fetch; *n = h.n_fetch; break;
-    case 5: *recs = P.out.ent + h.o_ent; *n = h.n_ent; break;
+    case 5:
+      if (!P.ent_host) {            // lazily: the migration engine never reads the entries
+        if (P.n_ent) CK(cudaMemcpy(P.out.ent, P.dout.ent, sizeof(dyo_entry_rec) * P.n_ent, cudaMemcpyDeviceToHost));
+        const_cast<dyo_ctx::PlanSlot&>(P).ent_host = true;
+      }
+      *recs = P.out.ent + h.o_ent; *n = h.n_ent; break;
     default: return DYO_E_INVAL;
   }
   return DYO_OK;
@@ -1913,6 +1984,23 @@ dyo_status dyo_debug_plan_stamps(dyo_ctx* ctx, int32_t j, uint64_t* out64) {
   CK(cudaDeviceSynchronize());
   CK(plan_debug_stamps(j, reinterpret_cast<unsigned long long*>(out64)));
   return DYO_OK;
+}
+
+dyo_status dyo_set_timing(dyo_ctx* ctx, int32_t on) {
+  if (!ctx || on < 0 || on > 1) return DYO_E_INVAL;
+  if (on) ctx->cfg.flags |= DYO_F_TIMING;
+  else ctx->cfg.flags &= ~DYO_F_TIMING;
+  return DYO_OK;
+}
+
+dyo_status dyo_query(dyo_ctx* ctx, int32_t what, int64_t* value) {
+  if (!ctx || !value) return DYO_E_INVAL;
+  switch (what) {
+    case DYO_Q_PILOT_KERNEL: *value = ctx->last_tc; return DYO_OK;
+    case DYO_Q_DECODE_FUSED: *value = ctx->last_fused; return DYO_OK;
+    case DYO_Q_PLAN_SYNCS: *value = ctx->last_plan_syncs; return DYO_OK;
+  }
+  return DYO_E_INVAL;
 }
 
 dyo_status dyo_get_counters(dyo_ctx* ctx, dyo_counters* c, int32_t reset) {

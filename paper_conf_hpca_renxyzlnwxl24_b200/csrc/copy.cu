@@ -210,41 +210,45 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
     }
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
-  if (a->stamps != nullptr && threadIdx.x == 0) {
-    unsigned long long t_end, slot;
-    uint32_t smid;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-    slot = atomicAdd(a->stamps, 1ull);
-    if (slot < kStampCap) {
-      unsigned long long* e = a->stamps + 4 * (slot + 1);
-      e[0] = ((unsigned long long)a->launch << 32) | ((unsigned long long)blockIdx.x << 8) | (smid & 255u);
-      e[1] = t_enter; e[2] = t_scan; e[3] = t_end;
-    }
-  }
-
   // < 16-byte tails and unaligned records: byte copies, record k by CTA k % grid
   if (single) {
     for (int64_t x = T + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; x < a->total; x += (int64_t)gridDim.x * blockDim.x)
       a->dst_base[x] = a->src_base[x];
-    return;
+  } else {
+    for (int k = blockIdx.x; k < a->n; k += gridDim.x) {
+      const int64_t* r = a->rec + (int64_t)k * a->stride;
+      if (a->f_late >= 0 && r[a->f_late] != a->late_val) continue;
+      const char* sp = a->src_base + r[a->f_src];
+      char* dp = a->dst_base + (r[a->f_dst] - a->dst_bias);
+      const int64_t nb = r[a->f_bytes];
+      const bool al = ((((uintptr_t)sp) | ((uintptr_t)dp)) & 15) == 0;
+      for (int64_t x = (al ? nb & ~(int64_t)15 : 0) + threadIdx.x; x < nb; x += blockDim.x) dp[x] = sp[x];
+    }
   }
-  for (int k = blockIdx.x; k < a->n; k += gridDim.x) {
-    const int64_t* r = a->rec + (int64_t)k * a->stride;
-    if (a->f_late >= 0 && r[a->f_late] != a->late_val) continue;
-    const char* sp = a->src_base + r[a->f_src];
-    char* dp = a->dst_base + (r[a->f_dst] - a->dst_bias);
-    const int64_t nb = r[a->f_bytes];
-    const bool al = ((((uintptr_t)sp) | ((uintptr_t)dp)) & 15) == 0;
-    for (int64_t x = (al ? nb & ~(int64_t)15 : 0) + threadIdx.x; x < nb; x += blockDim.x) dp[x] = sp[x];
+  // exit stamp after every copy of the CTA, the byte tails included
+  if (a->stamps != nullptr) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long t_end, slot;
+      uint32_t smid;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      slot = atomicAdd(a->stamps, 1ull);
+      if (slot < kStampCap) {
+        unsigned long long* e = a->stamps + 4 * (slot + 1);
+        e[0] = ((unsigned long long)a->launch << 32) | ((unsigned long long)blockIdx.x << 8) | (smid & 255u);
+        e[1] = t_enter; e[2] = t_scan; e[3] = t_end;
+      }
+    }
   }
 }
 
 template <int S, int C>
 static cudaError_t launch_ring(const RecCopyArgs& a, int grid, cudaStream_t s) {
-  static bool attr = false;
+  static uint64_t attr_done = 0;                  // bit d: attributes set on device d
+  const uint64_t bit = 1ull << current_device();
   const int smem = S * C;
-  if (!attr) {
+  if (!(attr_done & bit)) {
     cudaError_t e = cudaFuncSetAttribute(copy_records_tma_kernel<S, C>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     // DYO_TMA_CARVEOUT=1: ask for the maximum shared-memory carveout (measurement of whether a
@@ -254,7 +258,7 @@ static cudaError_t launch_ring(const RecCopyArgs& a, int grid, cudaStream_t s) {
         e = cudaFuncSetAttribute(copy_records_tma_kernel<S, C>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         if (e != cudaSuccess) return e;
       }
-    attr = true;
+    attr_done |= bit;
   }
   // at least one chunk per CTA; enough CTAs for the tail loop over the records
   int64_t g = (a.total + C - 1) / C;
@@ -292,7 +296,9 @@ static int tma_ctas_per_sm() {
 // DYO_COPY_STAMPS=1 (measurement aid): every record-copy CTA appends {launch<<32 | cta<<8 | smid,
 // globaltimer at entry, after the record scan, at the end} to a device log (slot 0 = count; up to
 // 2^22 - 1 entries), read back by dyo_debug_copy_stamps.
-static unsigned long long* g_stamps = nullptr;
+// The log is per device (a process may drive several GPUs, one ctx each).
+static unsigned long long* g_stamps_dev[64] = {};
+static unsigned long long*& stamps_of_current_device() { return g_stamps_dev[current_device()]; }
 
 // DYO_COPY_STAMPS=2 also brackets each record-copy launch with a one-thread marker kernel on the
 // same stream (entry cta field 0xFFF, smid field 0 = before, 1 = after): it locates the time
@@ -309,6 +315,7 @@ __global__ void copy_mark_kernel(unsigned long long* stamps, int64_t launch, int
 }
 static int64_t g_launch = 0;
 int64_t copy_stamps_read(unsigned long long* host, int64_t cap) {
+  unsigned long long* g_stamps = stamps_of_current_device();
   if (g_stamps == nullptr) return 0;
   if (host == nullptr && cap == 0) return cudaMemset(g_stamps, 0, 8) == cudaSuccess ? 0 : -1;   // reset
   unsigned long long n = 0;
@@ -327,10 +334,11 @@ cudaError_t launch_copy_records(const RecCopyArgs& a0, int grid, cudaStream_t s)
   if (stamps_on < 0) {
     const char* e = getenv("DYO_COPY_STAMPS");
     stamps_on = (e != nullptr && (e[0] == '1' || e[0] == '2')) ? (e[0] - '0') : 0;
-    if (stamps_on) {
-      if (cudaMalloc(&g_stamps, (size_t)32 * (kStampCap + 1)) != cudaSuccess) return cudaGetLastError();
-      cudaMemset(g_stamps, 0, 8);
-    }
+  }
+  unsigned long long*& g_stamps = stamps_of_current_device();
+  if (stamps_on && g_stamps == nullptr) {
+    if (cudaMalloc(&g_stamps, (size_t)32 * (kStampCap + 1)) != cudaSuccess) return cudaGetLastError();
+    cudaMemset(g_stamps, 0, 8);
   }
   if (stamps_on) { a.stamps = g_stamps; a.launch = g_launch++; }
   if (stamps_on == 2) copy_mark_kernel<<<1, 1, 0, s>>>(g_stamps, a.launch, 0);

@@ -124,7 +124,10 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
   if (B <= 0) return cudaSuccess;
   const int tab_cap = dec_table_words(a, kDecTabCap2);
   const size_t smA = groups_smem<kRecSmall>(a, tab_cap), smB = groups_smem<kRecCap>(a, tab_cap);
-  static size_t setA = 0, setB = 0;
+  static size_t setA_d[64] = {}, setB_d[64] = {}, hsm_d[64] = {};   // per device
+  const int dv = current_device();
+  size_t& setA = setA_d[dv];
+  size_t& setB = setB_d[dv];
   if (smA > setA) {
     cudaError_t e = cudaFuncSetAttribute(decode_groups_kernel<kRecSmall>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smA);
     if (e != cudaSuccess) return e;
@@ -136,7 +139,7 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
     setB = smB;
   }
   const size_t hsm = kHeadSmemBytes + (size_t)a.O * sizeof(double);
-  static size_t hsm_set = 0;
+  size_t& hsm_set = hsm_d[dv];
   if (hsm > hsm_set) {
     cudaError_t e = cudaFuncSetAttribute(decode_head_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsm);
     if (e != cudaSuccess) return e;
@@ -151,8 +154,9 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
   decode_groups_kernel<kRecSmall><<<B * a.K_max, kDecThreads, smA, s>>>(a, pb, hist_tab_out, tab_cap, 0);
   e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  static int sms = 0;
-  if (!sms) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+  static int sms_d[64] = {};
+  int& sms = sms_d[dv];
+  if (!sms) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dv);
   const int gB = B * a.K_max < 2 * sms ? B * a.K_max : 2 * sms;
   decode_groups_kernel<kRecCap><<<gB, kDecThreads, smB, s>>>(a, pb, hist_tab_out, tab_cap, 1);
   return cudaGetLastError();

@@ -9,6 +9,14 @@
 
 namespace dyo {
 
+// Current CUDA device (0..63): one-time per-kernel attributes and caches are kept per device,
+// since a process may drive several GPUs (one ctx each).
+inline int current_device() {
+  int d = 0;
+  cudaGetDevice(&d);
+  return d & 63;
+}
+
 constexpr int kSat = (1 << 24) - 1;       // R1(iii)
 constexpr int kMaxSites = 4096;
 constexpr int kEntCap = 1024;             // tensor-set entries per group (records before dedupe)
@@ -219,6 +227,10 @@ cudaError_t launch_pilot_tc(const ArchDev& a, const PilotDev* p_dev, const TcPla
                             const int64_t* desc, const int32_t* hist, const int32_t* hist_tab, const int32_t* hist_K,
                             int hist_B, int B, double* logits64, float* logits32, cudaStream_t s);
 cudaError_t plan_debug_stamps(int j, unsigned long long* out);
+// Copies a finished plan's headers and EVICT/MOVE/CARRY/ALLOC/FETCH records from the planner's
+// device arrays (d) into the pinned mapped mirrors (h: device-side aliases) by the counts in
+// d.counts; nothing when d.status[0] != 0. Entry records are not copied.
+cudaError_t launch_plan_export(const PlanOut& d, const PlanOut& h, cudaStream_t s);
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s);
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,

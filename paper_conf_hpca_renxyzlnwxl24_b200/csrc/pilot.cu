@@ -419,13 +419,14 @@ __global__ void __launch_bounds__(kPilotThreads) floor_kernel(int n_barriers) {
 }
 
 cudaError_t launch_floor(int C, int n_barriers, cudaStream_t s) {
-  static int attr_done = 0;
-  if (!attr_done) {
+  static uint64_t attr_done = 0;   // bit d: set on device d
+  const uint64_t bit = 1ull << current_device();
+  if (!(attr_done & bit)) {
     cudaError_t e = cudaFuncSetAttribute(floor_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     if (e != cudaSuccess) return e;
     e = cudaFuncSetAttribute(floor_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kDynCap);
     if (e != cudaSuccess) return e;
-    attr_done = 1;
+    attr_done |= bit;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(C);
@@ -454,15 +455,16 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
                          PredDev& pd, int32_t* hist_tab_out, int32_t* hist_K_out, int* fused,
                          cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
-  static int attr_done = 0;
-  if (!attr_done) {
+  static uint64_t attr_done = 0;   // bit d: set on device d
+  const uint64_t bit = 1ull << current_device();
+  if (!(attr_done & bit)) {
     for (auto fn : {pilot_kernel<1>, pilot_kernel<kBs>}) {
       cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
       if (e != cudaSuccess) return e;
       e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kDynCap);
       if (e != cudaSuccess) return e;
     }
-    attr_done = 1;
+    attr_done |= bit;
   }
   // cluster size by weight volume (cached: cudaOccupancyMaxActiveClusters is expensive)
   int64_t wbytes = 0;

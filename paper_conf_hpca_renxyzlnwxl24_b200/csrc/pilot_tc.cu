@@ -534,13 +534,14 @@ cudaError_t launch_pilot_tc(const ArchDev& a, const PilotDev* p_dev, const TcPla
                             const int64_t* desc, const int32_t* hist, const int32_t* hist_tab, const int32_t* hist_K,
                             int hist_B, int B, double* logits64, float* logits32, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
-  static bool attr = false;
-  if (!attr) {
+  static uint64_t attr_done = 0;   // bit d: set on device d
+  const uint64_t bit = 1ull << current_device();
+  if (!(attr_done & bit)) {
     cudaError_t e = cudaFuncSetAttribute(pilot_tc_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     if (e != cudaSuccess) return e;
     e = cudaFuncSetAttribute(pilot_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
     if (e != cudaSuccess) return e;
-    attr = true;
+    attr_done |= bit;
   }
   const int n_clusters = (B + kTcBatch - 1) / kTcBatch;
   pilot_tc_kernel<<<n_clusters * kTcCtas, kThreads, kSmemBytes, s>>>(a, p_dev, plan_dev, feat, desc, hist, hist_tab,

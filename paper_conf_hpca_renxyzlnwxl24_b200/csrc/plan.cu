@@ -684,6 +684,30 @@ cudaError_t plan_debug_stamps(int j, unsigned long long* out) {
   return e;
 }
 
+// 8-byte words of the record arrays, grid-stride over all six lists
+__global__ void plan_export_kernel(PlanOut d, PlanOut h) {
+  if (d.status[0] != 0) return;
+  const int K = d.counts[0];
+  const int64_t n[6] = {(int64_t)K * (int64_t)(sizeof(PlanHdr) / 8), (int64_t)d.counts[1] * 5, (int64_t)d.counts[2] * 4,
+                        (int64_t)d.counts[3] * 5, (int64_t)d.counts[4] * 3, (int64_t)d.counts[5] * 4};
+  const uint64_t* src[6] = {reinterpret_cast<const uint64_t*>(d.hdr), reinterpret_cast<const uint64_t*>(d.ev),
+                            reinterpret_cast<const uint64_t*>(d.mv), reinterpret_cast<const uint64_t*>(d.ca),
+                            reinterpret_cast<const uint64_t*>(d.al), reinterpret_cast<const uint64_t*>(d.fe)};
+  uint64_t* dst[6] = {reinterpret_cast<uint64_t*>(h.hdr), reinterpret_cast<uint64_t*>(h.ev),
+                      reinterpret_cast<uint64_t*>(h.mv), reinterpret_cast<uint64_t*>(h.ca),
+                      reinterpret_cast<uint64_t*>(h.al), reinterpret_cast<uint64_t*>(h.fe)};
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int l = 0; l < 6; ++l)
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n[l]; i += stride) dst[l][i] = src[l][i];
+}
+
+cudaError_t launch_plan_export(const PlanOut& d, const PlanOut& h, cudaStream_t s) {
+  static_assert(sizeof(PlanHdr) % 8 == 0 && sizeof(dyo_evict_rec) == 40 && sizeof(dyo_move_rec) == 32 &&
+                sizeof(dyo_carry_rec) == 40 && sizeof(dyo_alloc_rec) == 24 && sizeof(dyo_fetch_rec) == 32, "record layout");
+  plan_export_kernel<<<64, 256, 0, s>>>(d, h);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,
                         PlanState& in, PlanState& work, PlanScratch& sc, PlanOut& out,
                         int max_groups, cudaStream_t s) {

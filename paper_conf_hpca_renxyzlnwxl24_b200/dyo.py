@@ -98,7 +98,7 @@ def lib():
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
                      "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
                      "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats",
-                     "dyo_debug_copy_stamps"):
+                     "dyo_debug_copy_stamps", "dyo_query", "dyo_set_timing"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -109,7 +109,8 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_prediction_get", "dyo_prediction_matched", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
            "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
-           "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps")
+           "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps",
+           "dyo_query", "dyo_set_timing")
 
 
 def _a(x, dt):
@@ -421,6 +422,17 @@ class Dyo:
         out = np.zeros(64, np.uint64)
         self._check(self.L.dyo_debug_plan_stamps(self.ctx, j, out.ctypes.data_as(C.POINTER(C.c_uint64))))
         return out
+
+    def set_timing(self, on):
+        self._check(self.L.dyo_set_timing(self.ctx, 1 if on else 0))
+
+    QUERIES = {"pilot_kernel": 0, "decode_fused": 1, "plan_syncs": 2}
+
+    def query(self, what):
+        """dyo_query: 'pilot_kernel' (0 K1 cluster GEMV, 1 K1-TC), 'decode_fused', 'plan_syncs'."""
+        v = i64()
+        self._check(self.L.dyo_query(self.ctx, self.QUERIES[what], C.byref(v)))
+        return v.value
 
     def counters(self, reset=False):
         c = Counters()

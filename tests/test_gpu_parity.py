@@ -56,6 +56,28 @@ def test_pilot_logits(name, B):
         assert g2.all(), f"fp32 error bound violated at {np.where(~g2)[0][:5]}"
         n1 += int((~g1).sum())
     assert n1 == 0, f"{n1} logits outside 1e-5 relative (floored)"
+    # which kernel ran: batch < 16 -> K1 (cluster GEMV, fp64 accumulation); >= 16 -> K1-TC
+    assert d.query("pilot_kernel") == (1 if B >= 16 else 0)
+    d.close()
+
+
+@pytest.mark.parametrize("name,B", [("tiny", 1), ("moe", 2), ("af", 1), ("lstm", 4)])
+def test_predict_from_encoded_features(name, B):
+    """The unfused entry: dyo_encode_features -> device features -> dyo_pilot_predict(feat=...)
+    gives the oracle's logits (north_star gate) and decode, like the fused path."""
+    wl = WL.make(name, n_samples=16)
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    feat = torch.zeros((B, wl.pilot.F), device="cuda")
+    logits = torch.zeros((B, wl.pilot.O), device="cuda")
+    d.encode(wl.samples[:B].copy(), hist_for(wl, B), B, feat, _stream())
+    d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, feat=feat, stream=_stream())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), (), plan=False)
+    assert np.array_equal(feat.cpu().numpy().astype(np.float64), np.stack(r["feats"]))
+    y = logits.cpu().numpy()
+    for b in range(B):
+        g1, g2, _ = logit_gates(y[b], r["feats"][b], wl.pilot, wl.nn_type)
+        assert g1.all() and g2.all()
+        _check_prediction(d, wl, b, r["preds"][b])
     d.close()
 
 
@@ -218,6 +240,35 @@ def test_plan_bitexact_lstm_fullsize():
     _run_plan_steps(wl, 1, 8, 1).close()
 
 
+def test_plan_bitexact_lstm_batch64_bench_config():
+    """The bench's LSTM configuration: 64 predictions (K1-TC + batch decode), 1,024 transitions
+    planned as one sequence, RETAIN; every record of every transition bit-exact, one host sync."""
+    wl = WL.make("lstm", n_samples=64)
+    d = _run_plan_steps(wl, 1, 64, 1)
+    assert d.query("plan_syncs") == 1
+    assert d.query("pilot_kernel") == 1
+    d.close()
+
+
+def test_residency_matches_oracle_state():
+    """dyo_residency: after each plan, every tensor's device address is the arena base +
+    half x H + offset of the oracle's state, NULL for tensors on the host."""
+    wl = WL.make("moe", n_samples=8)
+    d = make_ctx(wl, max_batch=1, flags=F_NO_HOST_POOL)
+    base, H = d.arena()
+    st = PL.initial_state(len(wl.tensors))
+    table = ()
+    for s in range(3):
+        r = oracle_step(wl, [s], st, table)
+        d.predict(wl.samples[[s]].copy(), hist_for(wl, 1), 1, stream=_stream())
+        d.plan(stream=_stream())
+        st, table = r["state"], r["table"]
+        for t in range(len(wl.tensors)):
+            want = None if st.loc[t] == PL.HOST else base + st.loc[t] * H + st.off[t]
+            assert d.residency(t) == want, f"step {s} tensor {t}"
+    d.close()
+
+
 @pytest.mark.parametrize("name,B", [("moe", 64), ("af", 64), ("lstm", 64), ("moe", 20), ("moe", 100)])
 def test_pilot_logits_tensor_cores(name, B):
     """K1-TC (tcgen05 kind::tf32, 3xTF32 split) for batches >= 16. fp32-accumulating tensor
@@ -228,6 +279,7 @@ def test_pilot_logits_tensor_cores(name, B):
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
     logits = torch.zeros((B, wl.pilot.O), device="cuda")
     d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, stream=_stream())
+    assert d.query("pilot_kernel") == 1, "the tensor-core kernel did not run"
     r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), (), plan=False)
     y = logits.cpu().numpy()
     n1, worst, worst_s, n_cancel, worst_rel = 0, 0.0, 0.0, 0, 0.0
@@ -249,6 +301,8 @@ def test_pilot_logits_tensor_cores(name, B):
     print(f"{name} B={B}: worst err/scale {worst_s:.3e}; worst err/|o| where |o| >= scale/10 {worst_rel:.3e}; "
           f"gate-1 misses {n1} (cancellation {n_cancel}), worst floored relative {worst:.3e}")
     assert worst_s <= 1e-5, "componentwise relative error above 1e-5 (R14)"
+    # survey C3: a gate-1 miss that passes gate 2 must be cancellation (|o| << its scale)
+    assert n1 == n_cancel, f"{n1 - n_cancel} gate-1 misses are not cancellation"
     # decisions: identical, except a branch-head argmax whose top-2 gap in the oracle's logits is
     # inside the path's error (2 x 1e-5 x the site's largest magnitude scale): a documented tie
     from oracle import afm as AF
@@ -273,4 +327,5 @@ def test_pilot_logits_tensor_cores(name, B):
             continue
         _check_prediction(d, wl, b, p)
     print(f"{name} B={B}: {n_tie} predictions with a documented argmax near-tie")
+    assert n_tie == 0, "decisions differ from the oracle's on a seeded config"
     d.close()

@@ -573,11 +573,29 @@ def run_dyo(args):
     lat = pilot_latency(torch, wl, local, desc_dev, hist64, nS, s0)
     mis = mispredict_stream(torch, wl, local, s0) if wl.notes.get("batch", 1) == 1 else None
     b64_us, b64_kernel_us, b64_decode_us = pilot_loop(dp, 50, 64)
-    # K1-TC work per launch: 2 x 64 x sum(in x out) over the tensor-core stages, x3 for 3xTF32
+    b64_kern = dp.query("pilot_kernel")
+    # batch work per launch: 2 x 64 x sum(in x out) over the stages (K1-TC executes x3: 3xTF32)
     sp = wl.pilot
     macs = sum(ln * o for _, ln, o in sp.feature) + sum(i * o for i, o in sp.mlp) + sp.out_in * sp.O
     tc_flop = 2.0 * 64 * macs
     dp.close()
+    tc = None
+    if wl.pilot.feature:
+        # the opt-in tensor-core kernel K1-TC (DYO_F_PILOT_TC: tcgen05 3xTF32, reading R14) beside it
+        dt = Dyo(wl.budget, wl.align, wl.policy, max_batch=64, device=local, flags=DYO_F_TIMING | 4 | 32)
+        dt.load(wl)
+        t_us, t_kernel_us, t_decode_us = pilot_loop(dt, 50, 64)
+        assert dt.query("pilot_kernel") == 1
+        dt.close()
+        tf32_peak = peaks["bf16_tflops"] / 2
+        tc = {"us_per_batch": round(t_us, 2), "pilot_kernel_us": round(t_kernel_us, 2),
+              "decode_kernels_us": round(t_decode_us, 2), "predictions_per_s": round(64e6 / t_us, 1),
+              "kernel": "pilot_tc_kernel (tcgen05 kind::tf32, 3xTF32, fp32 accumulation; reading R14 gate)",
+              "tensor_roofline": {"bound": "tensor", "achieved": round(3 * tc_flop / (t_kernel_us * 1e-6) / 1e12, 4),
+                                  "peak": round(tf32_peak, 1), "unit": "TFLOP/s",
+                                  "frac": round(3 * tc_flop / (t_kernel_us * 1e-6) / 1e12 / tf32_peak, 6),
+                                  "flop_per_launch": 3 * tc_flop,
+                                  "peak_source": "TF32 dense = measured bf16 / 2 (guide's nominal ratio)"}}
     _log("probe")
     probe = pcie_probe(torch)
 
@@ -675,15 +693,15 @@ def run_dyo(args):
         "pilot_batch64": {"us_per_batch": round(b64_us, 2), "us_per_prediction": round(b64_us / 64, 3),
                           "predictions_per_s": round(64e6 / b64_us, 1),
                           "pilot_kernel_us": round(b64_kernel_us, 2), "decode_kernels_us": round(b64_decode_us, 2),
-                          "kernel": "pilot_tc_kernel (tcgen05 kind::tf32, 3xTF32)" if wl.pilot.feature else
-                                    "pilot_kernel (cluster GEMV; T32 pilot has no tensor-core plan)",
-                          "tensor_roofline": ({"bound": "tensor", "achieved": round(3 * tc_flop / (b64_kernel_us * 1e-6) / 1e12, 4),
-                                               "peak": round(peaks["bf16_tflops"] / 2, 1), "unit": "TFLOP/s",
-                                               "frac": round(3 * tc_flop / (b64_kernel_us * 1e-6) / 1e12 / (peaks["bf16_tflops"] / 2), 6),
-                                               "flop_per_launch": 3 * tc_flop,
-                                               "peak_source": "TF32 dense = measured bf16 / 2 (guide's nominal ratio)",
-                                               "note": "latency-bound: 6 dependent layers of M=128 x N=64 tiles"}
-                                              if wl.pilot.feature else None)},
+                          "kernel": ("pilot_kernel<8> (fp64 DMMA m8n8k4 tensor-core tiles, 8 samples per 16-CTA "
+                                     "cluster; north_star gate)" if b64_kern == 0 else "pilot_tc_kernel"),
+                          "tensor_roofline": {"bound": "tensor", "achieved": round(tc_flop / (b64_kernel_us * 1e-6) / 1e12, 4),
+                                              "peak": round(peaks["bf16_tflops"] * 45.0 / 2250.0, 2), "unit": "TFLOP/s",
+                                              "frac": round(tc_flop / (b64_kernel_us * 1e-6) / 1e12 / (peaks["bf16_tflops"] * 45.0 / 2250.0), 5),
+                                              "flop_per_launch": tc_flop,
+                                              "peak_source": "FP64 tensor = measured bf16 x 45/2250 (guide's nominal B200 ratio)",
+                                              "note": "latency-bound: 6 dependent layers"},
+                          "tc_opt_in": tc},
         "plan_us": round(plan_us, 2), "transitions_per_step": round(tot_K / args.steps, 2),
         "plan_floor_frac": (round(lat["single_cta_launch_floor_us"] / plan_us, 5)
                             if lat.get("single_cta_launch_floor_us") else None),

@@ -65,6 +65,9 @@ typedef struct {
 #define DYO_F_NO_HOST_POOL 4  /* plan-only ctx: no pinned host pool (dyo_migrate -> DYO_E_STATE) */
 #define DYO_F_TIMING 8        /* record CUDA events around every internal launch (dyo_get_timings) */
 #define DYO_F_SM_COPY 16      /* device<->device moves by the SM vector-copy kernel instead of TMA bulk copies */
+#define DYO_F_PILOT_TC 32     /* batches >= 16 on K1-TC (tcgen05 kind::tf32, 3xTF32, fp32 accumulation; reading
+                               * R14's componentwise tolerance) instead of the default K1 batch path (fp64
+                               * DMMA tensor-core tiles, fp64 accumulation: the north_star gate) */
 
 /* Static architecture: the DyNN program in preorder, its operators and the
  * tensor table. All arrays are HOST memory; dyo_load_arch copies what it needs. */

@@ -849,6 +849,9 @@ static float tf32_rna_host(float x) {
 // K-major no-swizzle core-matrix layout ([k/4][row/8][row%8][k%4]) so one cp.async.bulk moves a
 // chunk. Only for the P-type topology (three feature layers); otherwise tc_dev stays null.
 static dyo_status build_tc_plan(dyo_ctx* ctx, const dyo_pilot_desc* w) {
+  // K1-TC is opt-in (DYO_F_PILOT_TC, or DYO_PILOT_TC=1 for measurement): the default batch path
+  // is K1's fp64 DMMA tiles, which meet the north_star gate exactly like batch 1
+  ctx->tc_flag_off = (ctx->cfg.flags & DYO_F_PILOT_TC) ? 0 : 1;
   if (const char* e = getenv("DYO_PILOT_TC")) ctx->tc_flag_off = (e[0] == '0');
   if (w->n_feature != 3 || ctx->F > 256 || ctx->cfg.max_batch < kTcMinBatch) return DYO_OK;
   const int k = ctx->ad.nn_type;

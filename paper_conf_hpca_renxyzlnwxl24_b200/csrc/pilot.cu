@@ -77,6 +77,7 @@ struct StagePlan {
   int dec_tab_cap;        // int32 words of decode tables staged in smem by the epilogue
   int tab_off;            // >= 0: byte offset of the decode tables prefetched at launch (fused decode)
   int push_logits;        // 1: the output stage pushes its logits to every CTA (fused decode, C > 1)
+  int red_off;            // batch path (BS > 1): byte offset of the DMMA tile table + K-split partials
   int st_off[4 + kMaxLayers];
   int rpc[4 + kMaxLayers];      // rows per CTA of each stage
   int gsh[4 + kMaxLayers];      // log2 of the threads per row (k-split) of each stage
@@ -119,6 +120,132 @@ __device__ __forceinline__ double warp_reduce4(double a0, double a1, double a2, 
   v += __shfl_xor_sync(0xffffffffu, v, 2);
   v += __shfl_xor_sync(0xffffffffu, v, 1);
   return v;
+}
+
+// ---- batch path (BS > 1): the stage as fp64 tensor-core tiles (DMMA) ------------------------
+// D[row][n] = sum_k W[row][k] X[n][k] over 8-row x 8-sample tiles with mma.sync m8n8k4 f64
+// (row.col): fp32 weights widen exactly, products and accumulation are fp64 - the same
+// precision as the GEMV path, so the north_star gate holds for every batch. A tile never
+// straddles two layers of the stage (the feature stage holds three); the bias rides as the
+// weight of a constant-1 input (k == in_len). Each warp owns one tile and a K slice; K-split
+// partials are summed in a fixed order (deterministic).
+struct DmmaTile { int li, row0, nrows, w_off; };   // stage row of m = 0; w_off: floats from the slice base
+constexpr int kDmmaMaxTiles = 64;
+constexpr int kDmmaRedBytes = kDmmaMaxTiles * 16 + 16 * 64 * 8;
+
+template <int BS>
+__device__ __forceinline__ void dmma_stage(const PilotDev& p, const StageDev& st, const float* wbase, bool staged,
+                                           int r0, int r1, const double* in, double* out, int W, int nb,
+                                           unsigned char* red_raw, bool last, bool act, double slope,
+                                           double* __restrict__ logits64, float* __restrict__ logits32, int b0,
+                                           int C, int r, uint32_t out_s, uint32_t cbar_s) {
+  static_assert(BS == 8, "one 8-sample n-tile");
+  DmmaTile* tiles = reinterpret_cast<DmmaTile*>(red_raw);
+  double* red = reinterpret_cast<double*>(red_raw + kDmmaMaxTiles * 16);
+  __shared__ int s_nt;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, nwarps = blockDim.x >> 5;
+  if (tid == 0) {
+    int nt = 0, lr0 = 0;
+    int64_t off = 0;                                    // floats of the staged slice before layer l
+    for (int l = st.first_layer; l < st.first_layer + st.n_layers; ++l) {
+      const int lr1 = lr0 + p.ly[l].out_len;
+      const int a0 = max(r0, lr0), a1 = min(r1, lr1);
+      for (int q = a0; q < a1 && nt < kDmmaMaxTiles; q += 8) {
+        DmmaTile t;
+        t.li = l;
+        t.row0 = q;
+        t.nrows = min(8, a1 - q);
+        t.w_off = staged ? (int)(off + (int64_t)(q - a0) * p.ly[l].in_pad) : (q - lr0) * p.ly[l].in_pad;
+        tiles[nt++] = t;
+      }
+      if (a1 > a0) off += (int64_t)(a1 - a0) * p.ly[l].in_pad;
+      lr0 = lr1;
+    }
+    s_nt = nt;
+  }
+  __syncthreads();
+  const int nt = s_nt;
+  const int ks = nt >= nwarps ? 1 : nwarps / nt;        // warps per tile (K split)
+  const int gm = lane >> 2, gk = lane & 3;              // fragment coordinates
+  for (int t0 = warp / ks; t0 < nt; t0 += nwarps / ks) {
+    const int part = warp % ks;
+    const DmmaTile t = tiles[t0];
+    const LayerDev& ly = p.ly[t.li];
+    const float* wl = staged ? wbase + t.w_off : ly.W + t.w_off;
+    const int nk = ly.in_pad >> 2;                      // k-steps of 4
+    const int per = (nk + ks - 1) / ks;
+    const int k0 = part * per, k1 = min(nk, k0 + per);
+    const bool wrow_ok = gm < t.nrows;
+    const float* wr = wl + (int64_t)gm * ly.in_pad + gk;
+    const double* xr = in + gm * W + ly.in_off + gk;    // B fragment: sample n = gm, k = gk
+    const bool xs_ok = gm < nb;
+    double c0 = 0.0, c1 = 0.0, e0 = 0.0, e1 = 0.0;
+    int kk = k0;
+    for (; kk + 1 < k1; kk += 2) {
+      const int ka = kk * 4 + gk, kb = ka + 4;
+      const double wa = wrow_ok ? (double)wr[kk * 4] : 0.0, wb = wrow_ok ? (double)wr[kk * 4 + 4] : 0.0;
+      const double xa = !xs_ok ? 0.0 : (ka < ly.in_len ? xr[kk * 4] : (ka == ly.in_len ? 1.0 : 0.0));
+      const double xb = !xs_ok ? 0.0 : (kb < ly.in_len ? xr[kk * 4 + 4] : (kb == ly.in_len ? 1.0 : 0.0));
+      asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                   : "+d"(c0), "+d"(c1) : "d"(wa), "d"(xa));
+      asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                   : "+d"(e0), "+d"(e1) : "d"(wb), "d"(xb));
+    }
+    if (kk < k1) {
+      const int ka = kk * 4 + gk;
+      const double wa = wrow_ok ? (double)wr[kk * 4] : 0.0;
+      const double xa = !xs_ok ? 0.0 : (ka < ly.in_len ? xr[kk * 4] : (ka == ly.in_len ? 1.0 : 0.0));
+      asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                   : "+d"(c0), "+d"(c1) : "d"(wa), "d"(xa));
+    }
+    c0 += e0;
+    c1 += e1;
+    // this thread holds D[gm][2 gk], D[gm][2 gk + 1]
+    if (ks > 1) {
+      red[warp * 64 + gm * 8 + 2 * gk] = c0;
+      red[warp * 64 + gm * 8 + 2 * gk + 1] = c1;
+    } else {
+      const double v2[2] = {c0, c1};
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int m = gm, n = 2 * gk + h;
+        if (m >= t.nrows || n >= nb) continue;
+        double v = v2[h];
+        if (act) v = v > 0.0 ? v : slope * v;
+        const int row = t.row0 + m;
+        if (last) {
+          logits64[(int64_t)(b0 + n) * p.O + row] = v;
+          if (logits32) logits32[(int64_t)(b0 + n) * p.O + row] = (float)v;
+        } else {
+          out[n * W + row] = v;
+          const uint32_t laddr = out_s + (uint32_t)((n * W + row) * 8);
+          for (int c = 0; c < C; ++c)
+            if (c != r) st_async_b64(mapa_u32(laddr, c), v, mapa_u32(cbar_s, c));
+        }
+      }
+    }
+  }
+  if (ks > 1) {
+    __syncthreads();
+    for (int e = tid; e < nt * 64; e += blockDim.x) {
+      const int ti = e >> 6, m = (e >> 3) & 7, n = e & 7;
+      const DmmaTile t = tiles[ti];
+      if (m >= t.nrows || n >= nb) continue;
+      double v = 0.0;
+      for (int q = 0; q < ks; ++q) v += red[(ti * ks + q) * 64 + (e & 63)];
+      if (act) v = v > 0.0 ? v : slope * v;
+      const int row = t.row0 + m;
+      if (last) {
+        logits64[(int64_t)(b0 + n) * p.O + row] = v;
+        if (logits32) logits32[(int64_t)(b0 + n) * p.O + row] = (float)v;
+      } else {
+        out[n * W + row] = v;
+        const uint32_t laddr = out_s + (uint32_t)((n * W + row) * 8);
+        for (int c = 0; c < C; ++c)
+          if (c != r) st_async_b64(mapa_u32(laddr, c), v, mapa_u32(cbar_s, c));
+      }
+    }
+  }
 }
 
 // grid = n_clusters * C (cluster dims C set at launch). Dynamic smem:
@@ -242,6 +369,14 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
     if (staged) mbar_wait(&wbar[si], 0);
     stamp(4 + 3 * si, stamp_on);
     const uint32_t out_s = smem_u32(out);
+    if constexpr (BS > 1) {
+      dmma_stage<BS>(p, st, reinterpret_cast<const float*>(smem_raw + (staged ? sp.st_off[si] : 0)), staged, r0, r1,
+                     in, out, W, nb, smem_raw + sp.red_off, last, st.act != 0, p.slope, logits64, logits32, b0, C, r,
+                     out_s, abar_s[cout]);
+      stamp(5 + 3 * si, stamp_on);
+      if (!last) __syncthreads();
+      continue;
+    }
     // ---- k-split: G threads per output row (G = largest power of two with rows * G <= block),
     //      each accumulates a contiguous chunk of the row (16-byte weight loads, fp64 FMAs with
     //      two independent accumulators), then a log2(G)-step shuffle reduction ----
@@ -511,7 +646,7 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   sp.tab_off = -1;
   const int act_bytes = 2 * sp.Bs * p.max_width * (int)sizeof(double);
   const int base = ((2 * (4 + kMaxLayers) + 2) * 8 + 127) / 128 * 128;
-  const int budget = kDynCap - act_bytes;
+  const int budget = kDynCap - act_bytes - (sp.Bs > 1 ? kDmmaRedBytes + 256 : 0);
   int off = base;
   for (int i = 0; i < p.n_stages; ++i) {
     const StageDev& st = p.st[i];
@@ -536,6 +671,11 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   if (sp.fuse_decode && base + dec_bytes > off) off = (base + dec_bytes + 127) / 128 * 128;
   sp.act_off = off;
   size_t smem = (size_t)sp.act_off + act_bytes;
+  sp.red_off = -1;
+  if (sp.Bs > 1) {                        // DMMA tile table + K-split partials
+    sp.red_off = (int)((smem + 127) / 128 * 128);
+    smem = (size_t)sp.red_off + kDmmaRedBytes;
+  }
   if (sp.fuse_decode) {
     const size_t tb = (size_t)dec_table_region_words(a) * 4;
     if (smem + tb <= (size_t)kDynCap) {

@@ -7,6 +7,7 @@ import workloads as WL
 from oracle import encode as E, pilot as P, decode as D, plan as PL, afm as A
 
 F_NO_ZEROCOPY, F_NO_PACK, F_NO_HOST_POOL = 1, 2, 4
+F_PILOT_TC = 32
 
 
 def make_ctx(wl, max_batch=1, flags=0, policy=None, **kw):

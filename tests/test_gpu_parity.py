@@ -8,7 +8,7 @@ pytestmark = pytest.mark.gpu
 import workloads as WL
 from oracle import plan as PL, afm as A
 from gpu_harness import (make_ctx, oracle_step, hist_for, tr_lists, gpu_lists, logit_gates,
-                         F_NO_HOST_POOL)
+                         F_NO_HOST_POOL, F_PILOT_TC)
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -42,7 +42,8 @@ def test_encode_bitexact(name):
 
 
 @pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 16), ("moe", 1), ("moe", 8), ("af", 1), ("af", 3),
-                                    ("lstm", 8), ("lstm", 64)])
+                                    ("lstm", 8), ("lstm", 64), ("moe", 64), ("af", 64), ("moe", 20), ("moe", 100),
+                                    ("af", 17)])
 def test_pilot_logits(name, B):
     wl = WL.make(name, n_samples=max(16, B))
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
@@ -56,8 +57,8 @@ def test_pilot_logits(name, B):
         assert g2.all(), f"fp32 error bound violated at {np.where(~g2)[0][:5]}"
         n1 += int((~g1).sum())
     assert n1 == 0, f"{n1} logits outside 1e-5 relative (floored)"
-    # which kernel ran: batch < 16 -> K1 (cluster GEMV, fp64 accumulation); >= 16 -> K1-TC
-    assert d.query("pilot_kernel") == (1 if B >= 16 else 0)
+    # which kernel ran: K1 (fp64 accumulation: cluster GEMV at batch 1, DMMA tiles for batches)
+    assert d.query("pilot_kernel") == 0
     d.close()
 
 
@@ -246,7 +247,7 @@ def test_plan_bitexact_lstm_batch64_bench_config():
     wl = WL.make("lstm", n_samples=64)
     d = _run_plan_steps(wl, 1, 64, 1)
     assert d.query("plan_syncs") == 1
-    assert d.query("pilot_kernel") == 1
+    assert d.query("pilot_kernel") == 0
     d.close()
 
 
@@ -271,12 +272,15 @@ def test_residency_matches_oracle_state():
 
 @pytest.mark.parametrize("name,B", [("moe", 64), ("af", 64), ("lstm", 64), ("moe", 20), ("moe", 100)])
 def test_pilot_logits_tensor_cores(name, B):
-    """K1-TC (tcgen05 kind::tf32, 3xTF32 split) for batches >= 16. fp32-accumulating tensor
-    cores: every logit within 1e-5 of its magnitude scale max(|o|, sum |w z| + |b|) (reading R14)
-    and within the rigorous fp32 error bound; gate-1 (floored at 1e-3 max|o|) misses are counted
-    and must be cancellation (|o| < 1e-2 of the scale); decisions identical to the oracle's."""
+    """Opt-in K1-TC (DYO_F_PILOT_TC: tcgen05 kind::tf32, 3xTF32 split) for batches >= 16.
+    fp32-accumulating tensor cores: every logit within 1e-5 of its magnitude scale
+    max(|o|, sum |w z| + |b|) (reading R14) and within the rigorous fp32 error bound; gate-1
+    misses are counted and must be cancellation: |o| below a quarter of the logit's scale, i.e. a
+    condition number above 4, where fp32 accumulation (~2.4e-6 x scale measured) cannot reach
+    1e-5 x |o|; decisions identical to the oracle's. The default batch path (fp64 DMMA) meets
+    gate 1 outright (test_pilot_logits)."""
     wl = WL.make(name, n_samples=max(16, B))
-    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL | F_PILOT_TC)
     logits = torch.zeros((B, wl.pilot.O), device="cuda")
     d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, stream=_stream())
     assert d.query("pilot_kernel") == 1, "the tensor-core kernel did not run"
@@ -295,7 +299,7 @@ def test_pilot_logits_tensor_cores(name, B):
             worst_rel = max(worst_rel, float((err[wide] / np.abs(o[wide])).max()))
         miss = ~g1
         n1 += int(miss.sum())
-        n_cancel += int((miss & (np.abs(o) < 1e-2 * scale)).sum())
+        n_cancel += int((miss & (np.abs(o) < 0.25 * scale)).sum())
         den = np.maximum(np.abs(o), 1e-3 * np.abs(o).max())
         worst = max(worst, float((err / den).max()))
     print(f"{name} B={B}: worst err/scale {worst_s:.3e}; worst err/|o| where |o| >= scale/10 {worst_rel:.3e}; "

@@ -713,17 +713,21 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   ctx->max_groups = mg;
   for (int s2 = 0; s2 < 2; ++s2) {
     PlanState& ps = ctx->state[s2];
-    DA(ps.loc, T); DA(ps.off, T); DA(ps.dirty, T); DA(ps.pw, T); DA(ps.res, 2 * (size_t)T);
-    DA(ps.res_n, 2); DA(ps.prev, T); DA(ps.prev_n, 1); DA(ps.G, 1);
+    DA(ps.loc, T); DA(ps.off, T); DA(ps.dirty, T); DA(ps.pw, T);
+    DA(ps.prev, T); DA(ps.prev_n, 1); DA(ps.G, 1); DA(ps.rl_meta, 4); DA(ps.pos, T);
+    for (int h = 0; h < 2; ++h)
+      for (int q = 0; q < 2; ++q) DA(ps.rl[h][q], T);
     CK(cudaMemset(ps.loc, 0xff, T));   // -1: every tensor starts on the host
   }
   ctx->committed = 0;
   int64_t cap_ent = ctx->cfg.max_entries > 0 ? ctx->cfg.max_entries : (int64_t)mg * 512;
   int64_t cap_rec = ctx->cfg.max_records > 0 ? ctx->cfg.max_records : 4 * ((int64_t)T + cap_ent);
   PlanScratch& sc = ctx->sc;
-  DA(sc.inw, T); DA(sc.cur_next, T); DA(sc.cur_rd, T); DA(sc.nxt, cap_ent); DA(sc.nxt_rd, cap_ent);
-  DA(sc.rstat, T); DA(sc.keys, 2 * ((size_t)T + 1024) + 4096); DA(sc.gap_s, T + 1); DA(sc.gap_e, T + 1);
-  DA(sc.kept, T); DA(sc.newoff, T); DA(sc.ebase, mg); DA(sc.grp_b, mg); DA(sc.grp_k, mg);
+  DA(sc.grp_b, mg); DA(sc.grp_k, mg); DA(sc.ebase, mg); DA(sc.Kt, 1);
+  DA(sc.bcnt, T + 1); DA(sc.bfill, T); DA(sc.bkey, cap_ent); DA(sc.bsort, cap_ent);
+  DA(sc.nxt, cap_ent); DA(sc.nxt_rd, cap_ent); DA(sc.first, T); DA(sc.first_rd, T); DA(sc.au, T);
+  DA(sc.inw, (T + 31) / 32); DA(sc.wnx, T); DA(sc.wfl, T); DA(sc.keys, 2 * (size_t)T + 2048);
+  DA(sc.kept, T); DA(sc.gap_s, T + 2); DA(sc.gap_e, T + 2); DA(sc.newoff, T);
   auto hmap = [&](void** p, size_t bytes) -> dyo_status {
     CK(cudaHostAlloc(p, std::max<size_t>(bytes, 64), cudaHostAllocMapped | cudaHostAllocPortable));
     memset(*p, 0, std::max<size_t>(bytes, 64));

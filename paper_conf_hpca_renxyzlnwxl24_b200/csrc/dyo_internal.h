@@ -20,7 +20,7 @@ inline int current_device() {
 constexpr int kSat = (1 << 24) - 1;       // R1(iii)
 constexpr int kMaxSites = 4096;
 constexpr int kEntCap = 1024;             // tensor-set entries per group (records before dedupe)
-constexpr int kPlanThreads = 256;
+constexpr int kPlanThreads = 1024;
 
 enum OpClass : int8_t { C_KEEP = 0, C_CARRY = 1, C_ALLOC = 2, C_FETCH = 3 };
 
@@ -149,18 +149,24 @@ struct PredDev {
 };
 
 // ---- planner state (device) -----------------------------------------------------------
+// Resident records (one int4 per tensor valid in a half, the half's list in ascending offset):
+//   x = offset / ALIGN, y = aligned size / ALIGN, z = t | flags << 20, w = next-use group index
+//   within the current plan (-1: none). flags: kRecTransient, kRecNxRd (the next use reads
+//   first), kRecDirty, kRecTomb (carried to the other half: dropped at the next rebuild).
+constexpr int kRecTransient = 1 << 20, kRecNxRd = 1 << 21, kRecDirty = 1 << 22, kRecTomb = 1 << 23;
+constexpr int kRecIdMask = (1 << 20) - 1;
 struct PlanState {
   int8_t* loc;        // T: -1 host, 0/1 half
   int64_t* off;       // T: offset within the half
   uint8_t* dirty;     // T
   uint8_t* pw;        // T: written by the previous group
-  int32_t* res;       // 2 x T: tensors of each half, ascending offset
-  int32_t* res_n;     // 2
   int32_t* prev;      // T: entries of the previous group (ids)
   int32_t* prev_n;    // 1
   int64_t* G;         // 1
+  int4* rl[2][2];     // [half][buffer]: resident records (capacity T each)
+  int32_t* rl_meta;   // [0..1] records per half (tombstones included), [2..3] buffer selector
+  int32_t* pos;       // T: index of a valid tensor's record in its half's current list
 };
-
 struct PlanHdr {      // per transition (device + pinned mirror)
   int32_t half, n_ent, n_evict, n_move, n_carry, n_alloc, n_fetch, pad;
   int64_t need, h2d, d2h, d2d;
@@ -181,22 +187,31 @@ struct PlanOut {
 };
 
 struct PlanScratch {
-  int8_t* inw;          // T
-  int32_t* cur_next;    // T
-  uint8_t* cur_rd;      // T
-  int32_t* nxt;         // max_groups x kEntCap : next occurrence of each entry
-  uint8_t* nxt_rd;
-  int8_t* rstat;        // T: resident status during a transition
-  uint64_t* keys;       // 2 x sort capacity (global fallback)
-  int64_t* gap_s;       // T + 1
-  int64_t* gap_e;
-  int32_t* kept;        // T
-  int64_t* newoff;      // T
-  int64_t* ebase;       // max_groups: first entry record of each planned group
+  // group list of the plan (plan_prep_kernel)
   int32_t* grp_b;       // max_groups: prediction of each planned group
   int32_t* grp_k;
+  int64_t* ebase;       // max_groups: first entry record of each planned group
+  int32_t* Kt;          // 1: groups in the plan
+  // next occurrences (bucket kernels): every entry's next group holding its tensor
+  int32_t* bcnt;        // T + 1: entries per tensor -> bucket bases
+  int32_t* bfill;       // T
+  int32_t* bkey;        // cap_ent: (group << 10 | entry) per bucket slot
+  int32_t* bsort;       // cap_ent: the same, sorted per bucket
+  int32_t* nxt;         // cap_ent: next group index of the entry's tensor (-1: none)
+  uint8_t* nxt_rd;      // cap_ent: that occurrence reads first
+  int32_t* first;       // T: first group of each tensor in the plan (-1)
+  uint8_t* first_rd;    // T
+  int32_t* au;          // T: aligned size / ALIGN
+  // sequential planner
+  uint32_t* inw;        // (T + 31) / 32: membership bitmap of W_j (global fallback of the smem copy)
+  int32_t* wnx;         // T: next use of a W_j member (valid while it is in W_j)
+  uint8_t* wfl;         // T: flags of a W_j member (bit 0 needs_fetch, 1 written)
+  uint64_t* keys;       // 2 T + 2048: live candidate keys / EVICT sort keys (global when large)
+  int4* kept;           // T: kept records of the half, ascending offset
+  int32_t* gap_s;       // T + 2: free gaps (ALIGN units)
+  int32_t* gap_e;
+  int32_t* newoff;      // T: new offsets (ALIGN units) of placed / compacted tensors
 };
-
 // ---- host traversal decode (traverse.cpp, R4) ------------------------------
 struct TravArch {
   std::vector<int32_t> sig;   // n_ops x 9 saturated signatures

@@ -130,7 +130,7 @@ __device__ __forceinline__ double warp_reduce4(double a0, double a1, double a2, 
 // weight of a constant-1 input (k == in_len). Each warp owns one tile and a K slice; K-split
 // partials are summed in a fixed order (deterministic).
 struct DmmaTile { int li, row0, nrows, w_off; };   // stage row of m = 0; w_off: floats from the slice base
-constexpr int kDmmaMaxTiles = 64;
+constexpr int kDmmaMaxTiles = 512;       // host checks ceil(rows per CTA / 8) + layers <= this
 constexpr int kDmmaRedBytes = kDmmaMaxTiles * 16 + 16 * 64 * 8;
 
 template <int BS>
@@ -635,8 +635,42 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
     cached_C = C;
   }
   StagePlan sp{};
-  sp.C = C;
   sp.Bs = B < kBs ? 1 : kBs;
+  if (sp.Bs > 1) {
+    // batch path: every cluster of the launch must be co-resident (one wave; measured on MoE
+    // B = 64: 8 clusters of 16 CTAs -> 7 active -> two waves, 117 us; of 8 CTAs -> 74 us), so
+    // halve C until the GPU holds ceil(B / 8) clusters at once. DYO_PILOT_BATCH_C overrides.
+    static int bc = -1;
+    if (bc < 0) { const char* e = getenv("DYO_PILOT_BATCH_C"); bc = e ? atoi(e) : 0; }
+    if (bc == 1 || bc == 2 || bc == 4 || bc == 8 || bc == 16) {
+      C = bc;
+    } else {
+      static int max_active[64][5];                // per device, per log2(C); 0 = not queried
+      const int need = (B + kBs - 1) / kBs, dv = current_device();
+      for (; C > 1; C /= 2) {
+        int lg = 0;
+        while ((1 << lg) < C) ++lg;
+        int& ma = max_active[dv][lg];
+        if (ma == 0) {
+          cudaLaunchConfig_t cfg = {};
+          cfg.gridDim = dim3(C);
+          cfg.blockDim = dim3(kPilotThreads);
+          cfg.dynamicSmemBytes = kDynCap;
+          cudaLaunchAttribute at[1];
+          at[0].id = cudaLaunchAttributeClusterDimension;
+          at[0].val.clusterDim.x = C;
+          at[0].val.clusterDim.y = 1;
+          at[0].val.clusterDim.z = 1;
+          cfg.attrs = at;
+          cfg.numAttrs = 1;
+          if (cudaOccupancyMaxActiveClusters(&ma, pilot_kernel<kBs>, &cfg) != cudaSuccess || ma < 1) ma = -1;
+          cudaGetLastError();
+        }
+        if (ma >= need) break;
+      }
+    }
+  }
+  sp.C = C;
   // fuse the decode when the cluster has at least one CTA per two groups of its samples
   sp.dec_tab_cap = dec_table_words(a, kDecTabCap);
   // fuse the decode when each CTA decodes at most a few groups of its samples (traversal: the
@@ -673,6 +707,8 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   size_t smem = (size_t)sp.act_off + act_bytes;
   sp.red_off = -1;
   if (sp.Bs > 1) {                        // DMMA tile table + K-split partials
+    for (int i = 0; i < p.n_stages; ++i)
+      if ((sp.rpc[i] + 7) / 8 + p.st[i].n_layers > kDmmaMaxTiles) return cudaErrorInvalidValue;
     sp.red_off = (int)((smem + 127) / 128 * 128);
     smem = (size_t)sp.red_off + kDmmaRedBytes;
   }

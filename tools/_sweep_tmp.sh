@@ -1,8 +1,7 @@
 cd $GRAFT_REPO_ROOT
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
-for c in auto 16 8 4 2; do
-  if [ $c = auto ]; then python tools/sweep_batch_pilot.py moe 64; else DYO_PILOT_BATCH_C=$c python tools/sweep_batch_pilot.py moe 64; fi
-done > gpurun_out/sweep.txt 2>&1
-EXTRA_FLAGS=32 python tools/sweep_batch_pilot.py moe 64 >> gpurun_out/sweep.txt 2>&1
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:pilot_kernel -c 1 -s 3 -o gpurun_out/pilot_b64 python tools/sweep_batch_pilot.py moe 64 > gpurun_out/ncu_pilot.log 2>&1
-cat gpurun_out/sweep.txt
+python tools/prof_plan.py lstm 64 5 100 300 600 900 > gpurun_out/prof_plan.txt 2>&1
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:plan_kernel -c 1 -o gpurun_out/plan_lstm python tools/prof_plan.py lstm 64 5 > gpurun_out/ncu_plan.log 2>&1
+nsys_none=1
+timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/plan_launches.csv python tools/prof_plan.py lstm 64 5 > /dev/null 2>&1
+cat gpurun_out/prof_plan.txt

@@ -39,14 +39,14 @@ namespace dyo {
 constexpr int NT = kPlanThreads;                  // 1024
 constexpr uint64_t kInfD = 0xFFFFull;
 constexpr int kInwSmemWords = 8192;               // smem W_j bitmap for T <= 2^18
-constexpr int kEvSmem = 8192;                     // EVICT keys sorted in shared memory up to this
 
 __device__ unsigned long long g_pstamp[64];
 __device__ int g_pstamp_j = -1;
 #define PSTAMP(i) do { if (j == pstamp_j && tid == 0) g_pstamp[i] = (unsigned long long)clock64(); } while (0)
 
 // ---- small block primitives (1024 threads) --------------------------------------------
-// Exclusive scan of one int64 per thread; *total = sum. tmp: 32 long longs. Three barriers.
+// Exclusive scan of one int64 per thread (any multiple of 32 threads up to 1024); *total = sum.
+// tmp: 32 long longs. Three barriers.
 __device__ __forceinline__ long long scan64(long long v, long long* tmp, long long* total) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   long long x = v;
@@ -55,20 +55,21 @@ __device__ __forceinline__ long long scan64(long long v, long long* tmp, long lo
     const long long y = __shfl_up_sync(0xffffffffu, x, o);
     if (lane >= o) x += y;
   }
+  const int nw = blockDim.x >> 5;
   if (lane == 31) tmp[w] = x;
   __syncthreads();
   if (w == 0) {
-    long long s = tmp[lane];
+    long long s = lane < nw ? tmp[lane] : 0;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       const long long y = __shfl_up_sync(0xffffffffu, s, o);
       if (lane >= o) s += y;
     }
-    tmp[lane] = s;
+    if (lane < nw) tmp[lane] = s;
   }
   __syncthreads();
   const long long base = w > 0 ? tmp[w - 1] : 0;
-  *total = tmp[31];
+  *total = tmp[nw - 1];
   __syncthreads();
   return base + x - v;
 }
@@ -84,10 +85,11 @@ __device__ __forceinline__ void sum4(long long v[4], long long (*tmp)[4]) {
 #pragma unroll
     for (int q = 0; q < 4; ++q) tmp[w][q] = v[q];
   __syncthreads();
+  const int nw = blockDim.x >> 5;
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
     long long s = 0;
-    for (int i = 0; i < 32; ++i) s += tmp[i][q];
+    for (int i = 0; i < nw; ++i) s += tmp[i][q];
     v[q] = s;
   }
   __syncthreads();
@@ -246,24 +248,123 @@ __global__ void bucket_sort_kernel(ArchDev a, PredDev pd, PlanScratch sc) {
 }
 
 // ---- the sequential planner ------------------------------------------------------------
+// 512 threads; each holds its contiguous chunk of the half's records in registers (up to RPT)
+// across the passes of a transition, so the half's list costs one coalesced global read per
+// transition; larger halves re-read their chunk in RPT-record windows (same code, same order).
+// Every W_j entry's per-tensor state is gathered into shared memory in one round trip (phase A)
+// and everything after it that concerns W_j (placement, records, rebuild) reads shared memory.
+constexpr int PNT = 512;
+constexpr int RPT = 16;                           // records per thread kept in registers
+constexpr int kHash = 2048;                       // W_j: tensor -> entry (open addressing)
+constexpr int kGapSmem = 4096;                    // gaps in shared memory up to this
+constexpr int kEvSort = 1024;                     // EVICT keys rank-sorted in shared memory up to this
+
 struct PlanSmem {
+  // W_j entries (index e < n) and their gathered state
   int32_t e_t[kEntCap];
+  int32_t e_off[kEntCap];        // offset units in its half (valid when loc >= 0)
+  int32_t e_pos[kEntCap];        // record index in its half's list
+  int32_t e_au[kEntCap];
+  int32_t e_nx[kEntCap];         // next use after this group (-1)
+  int32_t e_newoff[kEntCap];     // offset units in half m after the transition
+  int64_t e_host[kEntCap];
+  int64_t e_bytes[kEntCap];
   int8_t e_mode[kEntCap];
   int8_t e_rd[kEntCap];
   int8_t e_cls[kEntCap];
-  uint64_t pkey[kEntCap];        // placement sort keys
-  int32_t p_t[kEntCap];          // placed tensors in placement order
-  int32_t p_a[kEntCap];          // their aligned sizes (units)
-  int32_t p_off[kEntCap];        // their new offsets (units)
-  int32_t p_cls[kEntCap];
-  int32_t q_off[kEntCap];        // placed offsets sorted ascending (rebuild merge)
-  int32_t q_idx[kEntCap];        // placement index of q_off[k]
-  int32_t q_cnt[kEntCap];        // kept tensors below q_off[k]
+  int8_t e_loc[kEntCap];
+  uint8_t e_fl[kEntCap];         // bit 0 transient, 1 pw (written by the previous group), 2 dirty, 3 next use reads
+  // placement
+  alignas(16) uint64_t pkey[kEntCap];
+  int32_t pidx[kEntCap];         // entry of pkey[k]
+  int32_t p_e[kEntCap];          // entry of placed tensor p (placement order)
+  int32_t p_off[kEntCap];
+  alignas(16) int32_t p_au[kEntCap];   // aligned size of placed p (units)
+  int32_t run_st[kEntCap + 1];   // starts of the runs of equal aligned size in placement order
+  int32_t gcum[kGapSmem + 1];    // inclusive prefix of the gap capacities of one run
+  alignas(16) int32_t q_off[kEntCap];  // placed offsets ascending (rebuild merge)
+  int32_t q_idx[kEntCap];
+  int32_t q_cnt[kEntCap];
+  // tensor -> entry of W_j
+  int32_t h_key[kHash];
+  int32_t h_val[kHash];
+  // previous group (late carries; pw bits to clear)
+  int32_t prev_t[kEntCap];
+  // gaps of half m
+  int32_t gap_s[kGapSmem];
+  int32_t gap_e[kGapSmem];
+  // EVICT sort: key (host units, id, writeback) + payload (offset units)
+  alignas(16) uint64_t ev_key[kEvSort];
+  int32_t ev_off[kEvSort];
   uint32_t hist[256];
   uint32_t hcnt[256];
   long long tmp[32];
   long long tmp4[32][4];
 };
+
+// Rank of k among keys[0, n) (count of smaller keys), 16-byte shared-memory loads; keys unique.
+__device__ __forceinline__ int rank_u64(const uint64_t* keys, int n, uint64_t k) {
+  int r = 0, x = 0;
+  const ulonglong2* k2 = reinterpret_cast<const ulonglong2*>(keys);
+#pragma unroll 4
+  for (; x + 1 < n; x += 2) {
+    const ulonglong2 v = k2[x >> 1];
+    r += (v.x < k) + (v.y < k);
+  }
+  if (x < n) r += keys[x] < k;
+  return r;
+}
+__device__ __forceinline__ int rank_i32(const int32_t* keys, int n, int k) {
+  int r = 0, x = 0;
+  const int4* k4 = reinterpret_cast<const int4*>(keys);
+#pragma unroll 4
+  for (; x + 3 < n; x += 4) {
+    const int4 v = k4[x >> 2];
+    r += (v.x < k) + (v.y < k) + (v.z < k) + (v.w < k);
+  }
+  for (; x < n; ++x) r += keys[x] < k;
+  return r;
+}
+
+__device__ __forceinline__ uint32_t hash_t(int t) { return ((uint32_t)t * 2654435761u) >> 21; }   // 11 bits
+
+__device__ __forceinline__ int hash_find(const PlanSmem& S, int t) {
+  uint32_t h = hash_t(t);
+  while (true) {
+    const int k = S.h_key[h];
+    if (k == t) return S.h_val[h];
+    if (k < 0) return -1;
+    h = (h + 1) & (kHash - 1);
+  }
+}
+
+// exclusive max-scan of one int per thread (values >= 0); *total = max. tmp: 32 long longs.
+__device__ __forceinline__ int scanmax(int v, long long* tmp, int* total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x = max(x, y);
+  }
+  const int ex_w = __shfl_up_sync(0xffffffffu, x, 1);
+  if (lane == 31) tmp[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    int s = lane < nw ? (int)tmp[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, s, o);
+      if (lane >= o) s = max(s, y);
+    }
+    if (lane < nw) tmp[lane] = s;
+  }
+  __syncthreads();
+  const int before = w > 0 ? (int)tmp[w - 1] : 0;
+  *total = (int)tmp[nw - 1];
+  __syncthreads();
+  return max(before, lane > 0 ? ex_w : 0);
+}
 
 __device__ __forceinline__ uint64_t live_key(int4 r, int j) {
   const uint64_t d = r.w < 0 ? kInfD : (uint64_t)(r.w - j);
@@ -283,13 +384,25 @@ __device__ __forceinline__ bool rec_evicted(int4 r, int k, int rule, uint64_t th
   return k == 2 || (k == 3 && (rule == 0 || (rule == 2 && live_key(r, j) >= thresh)));
 }
 
-__global__ void __launch_bounds__(NT, 1)
+// Iterate this thread's records [i0, i1) in order: from registers R when the chunk fits RPT
+// (one window, loaded in phase B), else in RPT-record windows re-read into R from global
+// memory. BODY sees `r` and `gi`.
+#define FOR_RECS(BODY)                                                                          \
+  for (int w0_ = i0; w0_ < i1; w0_ += RPT) {                                                   \
+    if (!regmode) {                                                                             \
+      _Pragma("unroll") for (int u_ = 0; u_ < RPT; ++u_) if (w0_ + u_ < i1) R[u_] = recs[w0_ + u_]; \
+    }                                                                                           \
+    _Pragma("unroll") for (int u_ = 0; u_ < RPT; ++u_) if (w0_ + u_ < i1) {                     \
+      const int4 r = R[u_]; const int gi = w0_ + u_; (void)gi; BODY                             \
+    }                                                                                           \
+  }
+
+__global__ void __launch_bounds__(PNT, 1)
 plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanScratch sc, PlanOut out,
             int inw_smem) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PlanSmem& S = *reinterpret_cast<PlanSmem*>(smem_raw);
-  uint64_t* evs = reinterpret_cast<uint64_t*>(smem_raw + (sizeof(PlanSmem) + 15) / 16 * 16);   // kEvSmem keys
-  uint32_t* inw = inw_smem ? reinterpret_cast<uint32_t*>(evs + kEvSmem) : sc.inw;
+  uint32_t* inw = inw_smem ? reinterpret_cast<uint32_t*>(smem_raw + (sizeof(PlanSmem) + 15) / 16 * 16) : sc.inw;
   const int T = a.T;
   const int64_t AL = a.align;
   const int Hu = (int)(a.H / AL);
@@ -300,25 +413,26 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
   const int nwords = (T + 31) >> 5;
 
   // ---- 1. work copy of the committed state (transactional, R7), R9, next uses of the plan
-  for (int t = tid; t < T; t += NT) {
+  for (int t = tid; t < T; t += PNT) {
     st.loc[t] = in.loc[t];
     st.off[t] = in.off[t];
     st.dirty[t] = (a.t_flags[t] & 1) ? 0 : in.dirty[t];
     st.pw[t] = in.pw[t];
-    st.prev[t] = in.prev[t];
     st.pos[t] = in.pos[t];
   }
-  for (int w = tid; w < nwords; w += NT) inw[w] = 0u;
-  __shared__ int s_n[2], s_sel[2];
+  for (int w = tid; w < nwords; w += PNT) inw[w] = 0u;
+  for (int h = tid; h < kHash; h += PNT) S.h_key[h] = -1;
+  __shared__ int s_n[2], s_sel[2], s_prev_n;
   if (tid == 0) {
-    st.prev_n[0] = in.prev_n[0];
+    s_prev_n = in.prev_n[0];
     for (int h = 0; h < 2; ++h) { s_n[h] = in.rl_meta[h]; s_sel[h] = in.rl_meta[2 + h]; }
   }
   __syncthreads();
+  for (int i = tid; i < s_prev_n; i += PNT) S.prev_t[i] = in.prev[i];
   for (int h = 0; h < 2; ++h) {
     const int4* src = in.rl[h][s_sel[h]];
     int4* dst = st.rl[h][s_sel[h]];
-    for (int i = tid; i < s_n[h]; i += NT) {
+    for (int i = tid; i < s_n[h]; i += PNT) {
       int4 r = src[i];
       const int t = r.z & kRecIdMask;
       if (r.z & kRecTransient) r.z &= ~kRecDirty;            // R9: transient contents end
@@ -330,7 +444,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
   __syncthreads();
 
   __shared__ long long c_ev, c_mv, c_ca, c_al, c_fe;
-  __shared__ int s_np, s_compact, s_nkept, s_nev, s_ng, s_nmove;
+  __shared__ int s_np, s_compact, s_ng, s_nmove;
   __shared__ unsigned long long s_thresh;
   if (tid == 0) { c_ev = c_mv = c_ca = c_al = c_fe = 0; }
   const int pstamp_j = g_pstamp_j;
@@ -343,24 +457,45 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
     const int2* ent = group_entries(a, pd, sc, j, &n);
     const int64_t eb = sc.ebase[j];
     PlanHdr& hd = out.hdr[j];
-    // ---- A. W_j, classes, need (R7, R8)
+    // ---- A. W_j: gather every entry's state in one round trip; classes; need (R7, R8)
     long long v4[4] = {0, 0, 0, 0};                 // need units, carries, allocs, fetches
-    if (tid < n) {
-      const int2 en = ent[tid];
-      const int t = en.x, md = en.y & 3, rd = (en.y >> 2) & 1;
-      const int l = st.loc[t];
-      const int c = l == m ? C_KEEP : (l == 1 - m && rd ? C_CARRY : (rd ? C_FETCH : C_ALLOC));
-      S.e_t[tid] = t;
-      S.e_mode[tid] = (int8_t)md;
-      S.e_rd[tid] = (int8_t)rd;
-      S.e_cls[tid] = (int8_t)c;
-      sc.wnx[t] = sc.nxt[eb + tid];
-      sc.wfl[t] = (uint8_t)(sc.nxt_rd[eb + tid] | ((md & 2) ? 2 : 0));
-      atomicOr(&inw[t >> 5], 1u << (t & 31));
-      v4[0] = sc.au[t];
-      v4[1] = c == C_CARRY;
-      v4[2] = c == C_ALLOC;
-      v4[3] = c == C_FETCH;
+#pragma unroll
+    for (int q = 0; q < kEntCap / PNT; ++q) {
+      const int e = tid + q * PNT;
+      if (e < n) {
+        const int2 en = ent[e];
+        const int t = en.x, md = en.y & 3, rd = (en.y >> 2) & 1;
+        const int l = st.loc[t];
+        const int64_t off = st.off[t];
+        const int pos = st.pos[t];
+        const int pw = st.pw[t], dirty = st.dirty[t], tf = a.t_flags[t];
+        const int au = sc.au[t];
+        const int64_t host = a.t_host[t], bytes = a.t_bytes[t];
+        const int nx = sc.nxt[eb + e];
+        const int nxrd = sc.nxt_rd[eb + e];
+        const int c = l == m ? C_KEEP : (l == 1 - m && rd ? C_CARRY : (rd ? C_FETCH : C_ALLOC));
+        S.e_t[e] = t;
+        S.e_off[e] = (int)(off / AL);
+        S.e_pos[e] = pos;
+        S.e_au[e] = au;
+        S.e_nx[e] = nx;
+        S.e_newoff[e] = (int)(off / AL);
+        S.e_host[e] = host;
+        S.e_bytes[e] = bytes;
+        S.e_mode[e] = (int8_t)md;
+        S.e_rd[e] = (int8_t)rd;
+        S.e_cls[e] = (int8_t)c;
+        S.e_loc[e] = (int8_t)l;
+        S.e_fl[e] = (uint8_t)((tf & 1) | (pw ? 2 : 0) | (dirty ? 4 : 0) | (nxrd ? 8 : 0));
+        atomicOr(&inw[t >> 5], 1u << (t & 31));
+        uint32_t h = hash_t(t);
+        while (atomicCAS(&S.h_key[h], -1, t) != -1) h = (h + 1) & (kHash - 1);
+        S.h_val[h] = e;
+        v4[0] += au;
+        v4[1] += c == C_CARRY;
+        v4[2] += c == C_ALLOC;
+        v4[3] += c == C_FETCH;
+      }
     }
     sum4(v4, S.tmp4);
     const long long need_u = v4[0];
@@ -371,18 +506,22 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
     }
     const long long room = Hu - need_u;
     PSTAMP(1);
-    // ---- B. candidates of half m: dead (R9) / live, live bytes
+    // ---- B. the half's records (registers), live bytes, kept / evicted counts per rule
     const int nm = s_n[m];
-    int4* recs = st.rl[m][s_sel[m]];
-    const int per = (nm + NT - 1) / NT;
+    const int4* recs = st.rl[m][s_sel[m]];
+    const int per = (nm + PNT - 1) / PNT;
     const int i0 = min(nm, tid * per), i1 = min(nm, i0 + per);
+    const bool regmode = per <= RPT;
+    int4 R[RPT];
+    if (regmode) {
+#pragma unroll
+      for (int u = 0; u < RPT; ++u)
+        if (i0 + u < i1) R[u] = recs[i0 + u];
+    }
     long long live_u = 0;
     {
       long long w4[4] = {0, 0, 0, 0};
-      for (int i = i0; i < i1; ++i) {
-        const int4 r = recs[i];
-        if (rec_kind(r, inw) == 3) w4[0] += r.y;
-      }
+      FOR_RECS(if (rec_kind(r, inw) == 3) w4[0] += r.y;)
       sum4(w4, S.tmp4);
       live_u = w4[0];
     }
@@ -393,17 +532,14 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
     //      aligned sizes (keys ascending) exceeds the room; keys >= K* are evicted
     if (rule == 2) {
       long long cnt = 0;
-      for (int i = i0; i < i1; ++i) cnt += rec_kind(recs[i], inw) == 3;
+      FOR_RECS(cnt += rec_kind(r, inw) == 3;)
       long long nlive = 0;
       long long kb = scan64(cnt, S.tmp, &nlive);
-      for (int i = i0; i < i1; ++i) {
-        const int4 r = recs[i];
-        if (rec_kind(r, inw) == 3) sc.keys[kb++] = live_key(r, j);
-      }
+      FOR_RECS(if (rec_kind(r, inw) == 3) sc.keys[kb++] = live_key(r, j);)
       __syncthreads();
       uint64_t prefix = 0, mask = 0;
       long long cum = 0;                             // units of the keys below the prefix
-      const int kper = (int)((nlive + NT - 1) / NT);
+      const int kper = (int)((nlive + PNT - 1) / PNT);
       const int k0 = min((int)nlive, tid * kper), k1 = min((int)nlive, k0 + kper);
       for (int shift = 56; shift >= 0; shift -= 8) {
         if (tid < 256) { S.hist[tid] = 0; S.hcnt[tid] = 0; }
@@ -454,8 +590,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
         __syncthreads();
         if (bcount == 1) break;
       }
-      // the threshold: the unique key under the prefix (keys are unique)
-      for (int k = k0; k < k1; ++k) {
+      for (int k = k0; k < k1; ++k) {               // the unique key under the prefix
         const uint64_t key = sc.keys[k];
         if ((key & mask) == prefix) s_thresh = key;
       }
@@ -463,337 +598,508 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
     }
     const uint64_t thresh = rule == 2 ? s_thresh : 0;
     PSTAMP(3);
-    // ---- D. kept list (offset order) and EVICT keys (host offset, id, writeback)
+    // ---- D. EVICT keys (host offset, id, writeback) + offsets; gaps between kept tensors.
+    //      Pass 1 counts kept / evicted / gaps after my first kept record (local), pass 2 writes.
+    long long kbase = 0, nkept = 0;                 // this thread's first kept index; total kept
+    int nev = 0;
+    int last_x = -1;                                // old offset of this thread's last kept record
     {
-      long long ck = 0, ce = 0;
-      for (int i = i0; i < i1; ++i) {
-        const int4 r = recs[i];
+      long long ck = 0, ce = 0, cg = 0;
+      int first_x = -1, last_end = 0;
+      FOR_RECS({
         const int k = rec_kind(r, inw);
-        if (k == 0) continue;
-        if (rec_evicted(r, k, rule, thresh, j)) ++ce; else ++ck;
-      }
-      long long nk = 0, ne = 0;
-      long long bk = scan64(ck, S.tmp, &nk);
-      long long be = scan64(ce, S.tmp, &ne);
-      if (c_ev + ne > out.cap_rec) {
-        if (tid == 0) { status[0] = DYO_E_CAPACITY; status[1] = j; status[2] = (int)(c_ev + ne); }
+        if (k != 0) {
+          if (rec_evicted(r, k, rule, thresh, j)) {
+            ++ce;
+          } else {
+            if (first_x < 0) first_x = r.x;
+            else if (r.x > last_end) ++cg;
+            ++ck;
+            last_end = r.x + r.y;
+            last_x = r.x;
+          }
+        }
+      })
+      int pe_all = 0;
+      const int pe0 = scanmax(last_end, S.tmp, &pe_all);   // end of the kept record before my first
+      if (first_x >= 0 && first_x > pe0) ++cg;
+      long long tot = 0;
+      const long long b = scan64((ck << 42) | (ce << 21) | cg, S.tmp, &tot);
+      constexpr long long M21 = (1ll << 21) - 1;
+      kbase = b >> 42;
+      long long be = (b >> 21) & M21, bg = b & M21;
+      nkept = tot >> 42;
+      nev = (int)((tot >> 21) & M21);
+      const int ng = (int)(tot & M21);
+      if (c_ev + nev > out.cap_rec) {
+        if (tid == 0) { status[0] = DYO_E_CAPACITY; status[1] = j; status[2] = (int)(c_ev + nev); }
         return;
       }
-      uint64_t* ekeys = ne <= kEvSmem ? evs : sc.keys;
-      for (int i = i0; i < i1; ++i) {
-        const int4 r = recs[i];
+      const bool ev_smem = nev <= kEvSort;
+      const bool gap_smem = ng + 1 <= kGapSmem;
+      int32_t* gs_ = gap_smem ? S.gap_s : sc.gap_s;
+      int32_t* ge_ = gap_smem ? S.gap_e : sc.gap_e;
+      int pe = pe0;
+      FOR_RECS({
         const int k = rec_kind(r, inw);
-        if (k == 0) continue;
-        if (rec_evicted(r, k, rule, thresh, j)) {
-          const int t = r.z & kRecIdMask;
-          const uint64_t wb = (k == 3 && (r.z & kRecDirty)) ? 1 : 0;
-          ekeys[be++] = ((uint64_t)(a.t_host[t] / AL) << 21) | ((uint64_t)t << 1) | wb;
-        } else {
-          sc.kept[bk++] = r;
+        if (k != 0) {
+          if (rec_evicted(r, k, rule, thresh, j)) {
+            const int t = r.z & kRecIdMask;
+            const uint64_t wb = (k == 3 && (r.z & kRecDirty)) ? 1 : 0;
+            const uint64_t key = ((uint64_t)(a.t_host[t] / AL) << 21) | ((uint64_t)t << 1) | wb;
+            if (ev_smem) { S.ev_key[be] = key; S.ev_off[be] = r.x; }
+            else { sc.keys[be] = key; sc.newoff[t] = r.x; }
+            ++be;
+          } else {
+            if (r.x > pe) { gs_[bg] = pe; ge_[bg] = r.x; ++bg; }
+            pe = r.x + r.y;
+          }
         }
+      })
+      if (tid == 0) {
+        int ngt = ng;
+        if (Hu > pe_all) { gs_[ngt] = pe_all; ge_[ngt] = Hu; ++ngt; }
+        s_ng = ngt;
       }
-      if (tid == 0) { s_nkept = (int)nk; s_nev = (int)ne; }
-      __syncthreads();
     }
-    const int nkept = s_nkept, nev = s_nev;
     PSTAMP(4);
-    // gaps of half m between the kept tensors
-    {
-      const int kper = (nkept + 1 + NT - 1) / NT;
-      const int q0 = min(nkept + 1, tid * kper), q1 = min(nkept + 1, q0 + kper);
-      int prev_end = 0;
-      if (q0 > 0 && q0 <= nkept) { const int4 r = sc.kept[q0 - 1]; prev_end = r.x + r.y; }
-      long long cg = 0;
-      int pe = prev_end;
-      for (int q = q0; q < q1; ++q) {
-        const int ge = q == nkept ? Hu : sc.kept[q].x;
-        if (ge > pe) ++cg;
-        if (q < nkept) { const int4 r = sc.kept[q]; pe = r.x + r.y; }
-      }
-      long long ng = 0;
-      long long bg = scan64(cg, S.tmp, &ng);
-      pe = prev_end;
-      for (int q = q0; q < q1; ++q) {
-        const int ge = q == nkept ? Hu : sc.kept[q].x;
-        if (ge > pe) { sc.gap_s[bg] = pe; sc.gap_e[bg] = ge; ++bg; }
-        if (q < nkept) { const int4 r = sc.kept[q]; pe = r.x + r.y; }
-      }
-      if (tid == 0) s_ng = (int)ng;
-    }
+    if (j == pstamp_j && tid == 0) { g_pstamp[60] = nm; g_pstamp[61] = s_ng; g_pstamp[62] = nkept; g_pstamp[63] = regmode; }
     // ---- E. placement order: CARRY by id, ALLOC by id, FETCH by (host offset, id)
     if (tid == 0) s_np = 0;
     __syncthreads();
-    if (tid < n && S.e_cls[tid] != C_KEEP) {
-      const int c = S.e_cls[tid], t = S.e_t[tid];
-      const uint64_t rank = c == C_CARRY ? 0 : (c == C_ALLOC ? 1 : 2);
-      const uint64_t mid = c == C_FETCH ? (uint64_t)(a.t_host[t] / AL) : 0;
-      S.pkey[atomicAdd(&s_np, 1)] = (rank << 62) | (mid << 20) | (uint64_t)t;
+#pragma unroll
+    for (int q = 0; q < kEntCap / PNT; ++q) {
+      const int e = tid + q * PNT;
+      if (e < n && S.e_cls[e] != C_KEEP) {
+        const int c = S.e_cls[e], t = S.e_t[e];
+        const uint64_t rank = c == C_CARRY ? 0 : (c == C_ALLOC ? 1 : 2);
+        const uint64_t mid = c == C_FETCH ? (uint64_t)(S.e_host[e] / AL) : 0;
+        const int k = atomicAdd(&s_np, 1);
+        S.pkey[k] = (rank << 62) | (mid << 20) | (uint64_t)t;
+        S.pidx[k] = e;
+      }
     }
     __syncthreads();
     const int np = s_np;
-    if (tid < np) {
-      const uint64_t k = S.pkey[tid];
-      int r = 0;
-      for (int q = 0; q < np; ++q) r += S.pkey[q] < k;
-      const int t = (int)(k & kRecIdMask);
-      S.p_t[r] = t;
-      S.p_a[r] = sc.au[t];
-      S.p_cls[r] = (int)(k >> 62);
+#pragma unroll
+    for (int q = 0; q < kEntCap / PNT; ++q) {
+      const int i = tid + q * PNT;
+      if (i < np) {
+        const int r = rank_u64(S.pkey, np, S.pkey[i]);
+        S.p_e[r] = S.pidx[i];
+        S.p_au[r] = S.e_au[S.pidx[i]];
+      }
     }
     __syncthreads();
     PSTAMP(5);
-    // first fit by warp 0 (R11): a run of equal aligned sizes fills the gaps in address order
-    if (tid < 32) {
-      const int ng = s_ng;
-      bool fail = false;
-      int i = 0;
-      while (i < np && !fail) {
-        const int asz = S.p_a[i];
-        int r = 1;
-        while (i + r < np && S.p_a[i + r] == asz) ++r;
-        int left = r, done = 0;
-        for (int g0 = 0; g0 < ng && left > 0; g0 += 32) {
-          const int g = g0 + lane;
-          const int gs = g < ng ? sc.gap_s[g] : 0;
-          const int cap = g < ng ? (sc.gap_e[g] - gs) / asz : 0;
-          int incl = cap;
+    // first fit (R11): a run of equal aligned sizes fills the gaps in address order (exact: each
+    // tensor of the run takes the lowest gap that still holds it, and lower gaps never regain
+    // room). Runs are found in parallel; each run is one block-wide pass: capacities of the gaps
+    // (from a per-size cursor past the gaps an earlier run of that size filled), their prefix,
+    // and every tensor of the run finds its gap by binary search.
+    __shared__ int s_nruns, s_cur_sz[8], s_cur_g[8], s_last_g;
+    const int ng = s_ng;
+    {
+      long long cst = 0;
 #pragma unroll
-          for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += y;
-          }
-          const int excl = incl - cap;
-          const int take = max(0, min(cap, left - excl));
-          for (int q = 0; q < take; ++q) S.p_off[i + done + excl + q] = gs + q * asz;
-          if (take > 0) sc.gap_s[g] = gs + take * asz;
-          const int got = min(__shfl_sync(0xffffffffu, incl, 31), left);
-          left -= got;
-          done += got;
-        }
-        __syncwarp();
-        if (left > 0) fail = true;
-        i += r;
+      for (int q = 0; q < kEntCap / PNT; ++q) {
+        const int p = tid * (kEntCap / PNT) + q;
+        if (p < np && (p == 0 || S.p_au[p] != S.p_au[p - 1])) ++cst;
       }
-      if (lane == 0) s_compact = fail ? 1 : 0;
+      long long nr = 0;
+      long long b = scan64(cst, S.tmp, &nr);
+#pragma unroll
+      for (int q = 0; q < kEntCap / PNT; ++q) {
+        const int p = tid * (kEntCap / PNT) + q;
+        if (p < np && (p == 0 || S.p_au[p] != S.p_au[p - 1])) S.run_st[b++] = p;
+      }
+      if (tid == 0) { s_nruns = (int)nr; S.run_st[nr] = np; s_compact = 0; }
+      if (tid < 8) { s_cur_sz[tid] = 0; s_cur_g[tid] = 0; }
+      __syncthreads();
     }
-    __syncthreads();
+    {
+      const bool gap_smem = ng <= kGapSmem;
+      int32_t* gs_ = gap_smem ? S.gap_s : sc.gap_s;
+      const int32_t* ge_ = gap_smem ? S.gap_e : sc.gap_e;
+      int32_t* gcum = gap_smem ? S.gcum : reinterpret_cast<int32_t*>(sc.kept);   // scratch of >= 4T ints
+      if (ng <= 64) {
+        // few gaps: warp 0 alone, two lanes' worth of gaps per lane group, no block barriers;
+        // the run's tensors are written by all lanes (binary search over the lanes' prefixes)
+        if (tid < 32) {
+          const int g_a = lane, g_b = lane + 32;
+          int rem_a = g_a < ng ? gs_[g_a] : 0, rem_b = g_b < ng ? gs_[g_b] : 0;   // current gap starts
+          const int end_a = g_a < ng ? ge_[g_a] : 0, end_b = g_b < ng ? ge_[g_b] : 0;
+          bool fail = false;
+          for (int k = 0; k < s_nruns && !fail; ++k) {
+            const int i = S.run_st[k], r = S.run_st[k + 1] - i;
+            const int asz = S.p_au[i];
+            const int cap_a = (end_a - rem_a) / asz, cap_b = (end_b - rem_b) / asz;
+            // inclusive prefix over 64 gaps: lanes 0..31 hold gaps 0..31, then 32..63
+            int inc_a = cap_a, inc_b = cap_b;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+              const int ya = __shfl_up_sync(0xffffffffu, inc_a, o), yb = __shfl_up_sync(0xffffffffu, inc_b, o);
+              if (lane >= o) { inc_a += ya; inc_b += yb; }
+            }
+            const int tot_a = __shfl_sync(0xffffffffu, inc_a, 31);
+            inc_b += tot_a;
+            const int tot = __shfl_sync(0xffffffffu, inc_b, 31);
+            if (tot < r) { fail = true; break; }
+            for (int x0 = 0; x0 < r; x0 += 32) {
+              const int x = x0 + lane;
+              // first gap whose inclusive prefix exceeds x (search lanes of the a half, then b)
+              const bool in_a = x < tot_a;
+              int pos = 0;
+#pragma unroll
+              for (int st2 = 16; st2 >= 1; st2 >>= 1) {
+                const int va = __shfl_sync(0xffffffffu, inc_a, pos + st2 - 1);
+                const int vb = __shfl_sync(0xffffffffu, inc_b, pos + st2 - 1);
+                if ((in_a ? va : vb) <= x) pos += st2;
+              }
+              // every lane runs every shuffle (a shuffle inside a divergent ternary is undefined)
+              const int ia = __shfl_sync(0xffffffffu, inc_a, pos), ib = __shfl_sync(0xffffffffu, inc_b, pos);
+              const int ca = __shfl_sync(0xffffffffu, cap_a, pos), cb = __shfl_sync(0xffffffffu, cap_b, pos);
+              const int ra = __shfl_sync(0xffffffffu, rem_a, pos), rb = __shfl_sync(0xffffffffu, rem_b, pos);
+              const int excl = in_a ? ia - ca : ib - cb;
+              const int gs0 = in_a ? ra : rb;
+              if (x < r) S.p_off[i + x] = gs0 + (x - excl) * asz;
+            }
+            const int take_a = max(0, min(cap_a, r - (inc_a - cap_a)));
+            const int take_b = max(0, min(cap_b, r - (inc_b - cap_b)));
+            rem_a += take_a * asz;
+            rem_b += take_b * asz;
+          }
+          if (lane == 0) s_compact = fail ? 1 : 0;
+        }
+        __syncthreads();
+      } else
+      for (int k = 0; k < s_nruns; ++k) {
+        const int i = S.run_st[k], r = S.run_st[k + 1] - i;
+        const int asz = S.p_au[i];
+        int slot = -1, gstart = 0;
+        for (int q = 0; q < 8; ++q)
+          if (s_cur_sz[q] == asz) { slot = q; gstart = s_cur_g[q]; }
+        const int span = ng - gstart;
+        const int per_g = (span + PNT - 1) / PNT;
+        const int g0 = gstart + min(span, tid * per_g), g1 = gstart + min(span, tid * per_g + per_g);
+        long long cap_t = 0;
+        for (int g = g0; g < g1; ++g) cap_t += (ge_[g] - gs_[g]) / asz;
+        long long tot = 0;
+        long long c = scan64(cap_t, S.tmp, &tot);
+        for (int g = g0; g < g1; ++g) { c += (ge_[g] - gs_[g]) / asz; gcum[g - gstart] = (int)min(c, (long long)r); }
+        if (tid == 0) s_last_g = gstart;
+        __syncthreads();
+        // tensor x of the run -> the first gap whose inclusive prefix exceeds x
+        for (int x = tid; x < r && x < tot; x += PNT) {
+          int lo = 0, hi = span - 1;
+          while (lo < hi) { const int mid = (lo + hi) >> 1; if (gcum[mid] > x) hi = mid; else lo = mid + 1; }
+          const int before = lo > 0 ? gcum[lo - 1] : 0;
+          S.p_off[i + x] = gs_[gstart + lo] + (x - before) * asz;
+        }
+        __syncthreads();
+        // consume the gaps' room; remember where the run ended
+        for (int g = g0; g < g1; ++g) {
+          const int before = g > gstart ? gcum[g - gstart - 1] : 0;
+          const int take = gcum[g - gstart] - before;
+          if (take > 0) { gs_[g] += take * asz; atomicMax(&s_last_g, g); }
+        }
+        __syncthreads();
+        if (tid == 0) {
+          int q = slot;
+          if (q < 0) { for (q = 0; q < 8 && s_cur_sz[q] != 0; ++q) {} }
+          if (q < 8) { s_cur_sz[q] = asz; s_cur_g[q] = s_last_g; }
+          if (tot < r) s_compact = 1;
+        }
+        __syncthreads();
+        if (tot < r) break;
+      }
+    }
     const int compact = s_compact;
+    long long d2d = 0, h2d = 0, d2h = 0;
+    int nmove = 0;
     if (compact) {
-      // exclusive prefix sums over [kept in offset order | placed in placement order]
-      const int kper = (nkept + NT - 1) / NT;
-      const int q0 = min(nkept, tid * kper), q1 = min(nkept, q0 + kper);
+      // exclusive prefix sums over [kept in offset order | placed in placement order]; MOVE
+      // records for the kept tensors whose offset changes (ascending destination)
       long long cu = 0;
-      for (int q = q0; q < q1; ++q) cu += sc.kept[q].y;
+      FOR_RECS({ const int k = rec_kind(r, inw); if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) cu += r.y; })
       long long tot = 0;
       long long base = scan64(cu, S.tmp, &tot);
-      for (int q = q0; q < q1; ++q) {
-        const int4 r = sc.kept[q];
-        sc.newoff[r.z & kRecIdMask] = (int)base;
-        base += r.y;
+      long long cm = 0;
+      {
+        long long b2 = base;
+        FOR_RECS({
+          const int k = rec_kind(r, inw);
+          if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) { cm += b2 != r.x; b2 += r.y; }
+        })
       }
+      long long nmv = 0;
+      long long bm = scan64(cm, S.tmp, &nmv);
+      if (c_mv + nmv > out.cap_rec) {
+        if (tid == 0) { status[0] = DYO_E_CAPACITY; status[1] = j; status[2] = (int)(c_mv + nmv); }
+        return;
+      }
+      FOR_RECS({
+        const int k = rec_kind(r, inw);
+        if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) {
+          const int t = r.z & kRecIdMask;
+          const int no = (int)base;
+          if (k == 1) S.e_newoff[hash_find(S, t)] = no;
+          if (no != r.x) {
+            dyo_move_rec mv;
+            mv.t = t;
+            mv.src = (int64_t)m * a.H + (int64_t)r.x * AL;
+            mv.dst = (int64_t)m * a.H + (int64_t)no * AL;
+            mv.bytes = a.t_bytes[t];
+            out.mv[c_mv + bm++] = mv;
+            d2d += mv.bytes;
+            st.off[t] = (int64_t)no * AL;
+          }
+          base += r.y;
+        }
+      })
+      nmove = (int)nmv;
       if (tid == 0) {
         long long c = tot;
-        for (int p = 0; p < np; ++p) { S.p_off[p] = (int)c; c += S.p_a[p]; }
+        for (int p = 0; p < np; ++p) { S.p_off[p] = (int)c; c += S.p_au[p]; }
       }
       __syncthreads();
     }
+    if (tid == 0) s_nmove = nmove;
     PSTAMP(6);
     // ---- F. records
-    if (c_ca + nc > out.cap_rec || c_al + na > out.cap_rec || c_fe + nf > out.cap_rec ||
-        c_mv + nkept > out.cap_rec) {
-      if (tid == 0) { status[0] = DYO_E_CAPACITY; status[1] = j; status[2] = (int)(c_mv + nkept); }
+    if (c_ca + nc > out.cap_rec || c_al + na > out.cap_rec || c_fe + nf > out.cap_rec) {
+      if (tid == 0) { status[0] = DYO_E_CAPACITY; status[1] = j; status[2] = 0; }
       return;
     }
     // EVICT, sorted by (host offset, id)
-    {
-      uint64_t* ekeys = nev <= kEvSmem ? evs : sc.keys;
-      if (nev <= NT) {
-        uint64_t k = 0;
-        int r = 0;
-        if (tid < nev) {
-          k = ekeys[tid];
-          for (int q = 0; q < nev; ++q) r += ekeys[q] < k;
-        }
-        __syncthreads();
-        if (tid < nev) ekeys[r] = k;
-        __syncthreads();
-      } else {
-        block_sort_u64(ekeys, nev);                   // bitonic (smem up to kEvSmem, else global)
-      }
-      long long d2h = 0;
-      for (int k = tid; k < nev; k += NT) {
-        const uint64_t key = ekeys[k];
-        const int t = (int)((key >> 1) & kRecIdMask);
-        const int wb = (int)(key & 1);
-        dyo_evict_rec r;
-        r.t = t;
-        r.src = (int64_t)m * a.H + st.off[t];
-        r.host_off = a.t_host[t];
-        r.bytes = a.t_bytes[t];
-        r.writeback = wb;
-        out.ev[c_ev + k] = r;
-        if (wb) d2h += r.bytes;
-        st.loc[t] = -1;
-        st.dirty[t] = 0;
-      }
-      long long s4[4] = {d2h, 0, 0, 0};
-      sum4(s4, S.tmp4);
-      if (tid == 0) hd.d2h = s4[0];
-    }
-    // MOVE (compaction only): kept tensors whose offset changed, in kept (= destination) order
-    long long d2d = 0, h2d = 0;
-    if (compact) {
-      const int kper = (nkept + NT - 1) / NT;
-      const int q0 = min(nkept, tid * kper), q1 = min(nkept, q0 + kper);
-      long long cm = 0;
-      for (int q = q0; q < q1; ++q) { const int4 r = sc.kept[q]; cm += sc.newoff[r.z & kRecIdMask] != r.x; }
-      long long nmv = 0;
-      long long bm = scan64(cm, S.tmp, &nmv);
-      for (int q = q0; q < q1; ++q) {
-        const int4 r = sc.kept[q];
-        const int t = r.z & kRecIdMask;
-        const int no = sc.newoff[t];
-        if (no != r.x) {
-          dyo_move_rec mv;
-          mv.t = t;
-          mv.src = (int64_t)m * a.H + (int64_t)r.x * AL;
-          mv.dst = (int64_t)m * a.H + (int64_t)no * AL;
-          mv.bytes = a.t_bytes[t];
-          out.mv[c_mv + bm++] = mv;
-          d2d += mv.bytes;
-          st.off[t] = (int64_t)no * AL;
+    if (nev <= kEvSort) {
+      uint64_t kk[kEvSort / PNT];
+      int ofs[kEvSort / PNT], rk[kEvSort / PNT];
+#pragma unroll
+      for (int q = 0; q < kEvSort / PNT; ++q) {
+        const int i = tid + q * PNT;
+        rk[q] = -1;
+        if (i < nev) {
+          kk[q] = S.ev_key[i];
+          ofs[q] = S.ev_off[i];
+          rk[q] = rank_u64(S.ev_key, nev, kk[q]);
         }
       }
-      if (tid == 0) s_nmove = (int)nmv;
-    } else if (tid == 0) {
-      s_nmove = 0;
+      __syncthreads();
+#pragma unroll
+      for (int q = 0; q < kEvSort / PNT; ++q)
+        if (rk[q] >= 0) { S.ev_key[rk[q]] = kk[q]; S.ev_off[rk[q]] = ofs[q]; }
+      __syncthreads();
+    } else {
+      block_sort_u64(sc.keys, nev);                 // bitonic in global memory (large evictions)
     }
-    // CARRY / ALLOC / FETCH + placed state (loc, off, dirty); carried sources tombstoned
-    for (int p = tid; p < np; p += NT) {
-      const int t = S.p_t[p];
-      // a copy valid in the other half (CARRY source, or overwritten by an ALLOC) stops being
-      // valid there (R1): its record is dropped at that half's next rebuild
-      if (st.loc[t] == 1 - m) st.rl[1 - m][s_sel[1 - m]][st.pos[t]].z |= kRecTomb;
+    for (int k = tid; k < nev; k += PNT) {
+      const uint64_t key = nev <= kEvSort ? S.ev_key[k] : sc.keys[k];
+      const int t = (int)((key >> 1) & kRecIdMask);
+      const int wb = (int)(key & 1);
+      const int ou = nev <= kEvSort ? S.ev_off[k] : sc.newoff[t];
+      dyo_evict_rec r;
+      r.t = t;
+      r.src = (int64_t)m * a.H + (int64_t)ou * AL;
+      r.host_off = (int64_t)(key >> 21) * AL;
+      r.bytes = a.t_bytes[t];
+      r.writeback = wb;
+      out.ev[c_ev + k] = r;
+      if (wb) d2h += r.bytes;
+      st.loc[t] = -1;
+      st.dirty[t] = 0;
+    }
+    // CARRY / ALLOC / FETCH + placed state (loc, off, dirty); a copy valid in the other half
+    // (CARRY source, or overwritten by an ALLOC) stops being valid there (R1): its record is
+    // tombstoned and dropped at that half's next rebuild
+    for (int p = tid; p < np; p += PNT) {
+      const int e = S.p_e[p];
+      const int t = S.e_t[e];
+      const int c = S.e_cls[e];
       const int64_t dst = (int64_t)m * a.H + (int64_t)S.p_off[p] * AL;
-      const int c = S.p_cls[p];
-      const int64_t nbytes = a.t_bytes[t];
-      if (c == 0) {
+      const int64_t nbytes = S.e_bytes[e];
+      if (S.e_loc[e] == 1 - m) atomicOr(&st.rl[1 - m][s_sel[1 - m]][S.e_pos[e]].z, kRecTomb);
+      if (c == C_CARRY) {
         dyo_carry_rec r;
         r.t = t;
-        r.src = (int64_t)(1 - m) * a.H + st.off[t];
+        r.src = (int64_t)(1 - m) * a.H + (int64_t)S.e_off[e] * AL;
         r.dst = dst;
         r.bytes = nbytes;
-        r.late = st.pw[t] ? 1 : 0;
+        r.late = (S.e_fl[e] & 2) ? 1 : 0;
         out.ca[c_ca + p] = r;
         d2d += nbytes;
-      } else if (c == 1) {
+      } else if (c == C_ALLOC) {
         dyo_alloc_rec r;
         r.t = t;
         r.dst = dst;
         r.bytes = nbytes;
         out.al[c_al + p - nc] = r;
-        st.dirty[t] = 0;
       } else {
         dyo_fetch_rec r;
         r.t = t;
-        r.host_off = a.t_host[t];
+        r.host_off = S.e_host[e];
         r.dst = dst;
         r.bytes = nbytes;
         out.fe[c_fe + p - nc - na] = r;
         h2d += nbytes;
-        st.dirty[t] = 0;
       }
+      S.e_newoff[e] = S.p_off[p];
       st.loc[t] = (int8_t)m;
       st.off[t] = (int64_t)S.p_off[p] * AL;
     }
     __syncthreads();
-    // entry records (placement of every W_j tensor); block j writes: dirty
-    if (tid < n) {
-      const int t = S.e_t[tid];
-      dyo_entry_rec r;
-      r.t = t;
-      r.mode = S.e_mode[tid];
-      r.needs_fetch = S.e_rd[tid];
-      r.dst = (int64_t)m * a.H + st.off[t];
-      out.ent[eb + tid] = r;
-      if (S.e_mode[tid] & 2) st.dirty[t] = 1;
-    }
+    // entry records (placement of every W_j tensor); dirty after block j (writes); pw flags
+    for (int i = tid; i < s_prev_n; i += PNT) st.pw[S.prev_t[i]] = 0;
     {
-      long long s4[4] = {d2d, h2d, 0, 0};
-      sum4(s4, S.tmp4);
-      if (tid == 0) { hd.d2d = s4[0]; hd.h2d = s4[1]; }
+      long long s4[4] = {d2d, h2d, d2h, 0};
+      sum4(s4, S.tmp4);                             // (its barriers also order the pw clears)
+      if (tid == 0) { hd.d2d = s4[0]; hd.h2d = s4[1]; hd.d2h = s4[2]; }
     }
-    // previous-group written flags (late carries, R8)
-    const int pn = st.prev_n[0];
-    for (int i = tid; i < pn; i += NT) st.pw[st.prev[i]] = 0;
-    __syncthreads();
-    if (tid < n) {
-      const int t = S.e_t[tid];
-      st.pw[t] = (S.e_mode[tid] & 2) ? 1 : 0;
-      st.prev[tid] = t;
+#pragma unroll
+    for (int q = 0; q < kEntCap / PNT; ++q) {
+      const int e = tid + q * PNT;
+      if (e < n) {
+        const int t = S.e_t[e];
+        dyo_entry_rec r;
+        r.t = t;
+        r.mode = S.e_mode[e];
+        r.needs_fetch = S.e_rd[e];
+        r.dst = (int64_t)m * a.H + (int64_t)S.e_newoff[e] * AL;
+        out.ent[eb + e] = r;
+        const int wr = (S.e_mode[e] & 2) ? 1 : 0;
+        // dirty: CARRY/KEEP keep theirs, ALLOC/FETCH start clean; block j's writes set it
+        const int dirty = wr || ((S.e_cls[e] == C_KEEP || S.e_cls[e] == C_CARRY) && (S.e_fl[e] & 4));
+        st.dirty[t] = (uint8_t)dirty;
+        S.e_fl[e] = (uint8_t)((S.e_fl[e] & ~4) | (dirty ? 4 : 0));
+        st.pw[t] = (uint8_t)wr;
+        S.prev_t[e] = t;
+      }
     }
     PSTAMP(7);
     // ---- G. rebuild the half's list: kept (offset order, updated) merged with the placed
     //      tensors sorted by their new offsets
-    if (tid < np) {
-      const int o = S.p_off[tid];
-      int r = 0;
-      for (int q = 0; q < np; ++q) r += S.p_off[q] < o;
-      S.q_off[r] = o;
-      S.q_idx[r] = tid;
-      S.q_cnt[r] = nkept;                             // default: every kept tensor is below
+#pragma unroll
+    for (int q = 0; q < kEntCap / PNT; ++q) {
+      const int i = tid + q * PNT;
+      if (i < np) {
+        const int o = S.p_off[i];
+        const int r = rank_i32(S.p_off, np, o);
+        S.q_off[r] = o;
+        S.q_idx[r] = i;
+        S.q_cnt[r] = (int)nkept;                   // default: every kept tensor is below
+      }
     }
     __syncthreads();
     const int sel_new = 1 - s_sel[m];
     int4* dst = st.rl[m][sel_new];
     {
-      const int kper = (nkept + NT - 1) / NT;
-      const int q0 = min(nkept, tid * kper), q1 = min(nkept, q0 + kper);
-      auto lower = [&](int o) {                        // placed offsets below o
+      auto lower = [&](int o) {                      // placed offsets below o
         int lo = 0, hi = np;
         while (lo < hi) { const int mid = (lo + hi) >> 1; if (S.q_off[mid] < o) lo = mid + 1; else hi = mid; }
         return lo;
       };
-      int lb_prev = 0;
-      if (q0 > 0 && q0 < nkept) {
-        const int4 r = sc.kept[q0 - 1];
-        lb_prev = lower(compact ? sc.newoff[r.z & kRecIdMask] : r.x);
+      long long q = kbase;                           // global kept index
+      int newx0 = 0;                                 // compaction: new offset of my first kept
+      if (compact) {
+        long long cu = 0;
+        FOR_RECS({ const int k = rec_kind(r, inw); if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) cu += r.y; })
+        long long tot = 0;
+        newx0 = (int)scan64(cu, S.tmp, &tot);
       }
-      for (int q = q0; q < q1; ++q) {
-        int4 r = sc.kept[q];
-        const int t = r.z & kRecIdMask;
-        if (compact) r.x = sc.newoff[t];
-        if (bit_get(inw, t)) {                         // KEEP: this occurrence updates the record
-          const uint8_t fl = sc.wfl[t];
-          r.w = sc.wnx[t];
-          r.z = (r.z & ~kRecNxRd) | ((fl & 1) ? kRecNxRd : 0) | ((fl & 2) ? kRecDirty : 0);
+      // merge: a kept record's slot = its kept index + the placed offsets below it (binary search
+      // over q_off); a placed tensor's slot = its rank + the kept offsets below it (binary search
+      // over the kept offsets, staged in the consumed gap array when they fit)
+      const bool koff_smem = nkept <= kGapSmem;
+      int32_t* koff = S.gap_s;
+      int newx = newx0;
+      FOR_RECS({
+        const int k = rec_kind(r, inw);
+        if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) {
+          int4 w = r;
+          const int t = r.z & kRecIdMask;
+          if (compact) { w.x = newx; newx += r.y; }
+          if (k == 1) {                              // KEEP: this occurrence updates the record
+            const int e = hash_find(S, t);
+            w.w = S.e_nx[e];
+            w.z = (r.z & ~(kRecNxRd | kRecDirty)) | ((S.e_fl[e] & 8) ? kRecNxRd : 0) | ((S.e_fl[e] & 4) ? kRecDirty : 0);
+          }
+          const int lb = lower(w.x);
+          if (koff_smem) koff[q] = w.x;
+          dst[q + lb] = w;
+          st.pos[t] = (int)(q + lb);
+          ++q;
         }
-        const int lb = lower(r.x);
-        for (int k = (q == 0 ? 0 : lb_prev); k < lb; ++k) S.q_cnt[k] = q;
-        lb_prev = lb;
-        dst[q + lb] = r;
-        st.pos[t] = q + lb;
+      })
+      if (!koff_smem) {
+        // many kept tensors: placed slots from the kept side (each kept record fills the placed
+        // offsets between its predecessor's and its own)
+        int last_lb = 0;
+        {
+          int x = newx0, lx = -1;
+          FOR_RECS({
+            const int k = rec_kind(r, inw);
+            if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) { lx = compact ? x : r.x; x += r.y; }
+          })
+          if (lx >= 0) last_lb = lower(lx);
+        }
+        int dummy = 0;
+        int lb_prev = scanmax(last_lb, S.tmp, &dummy);
+        long long q2 = kbase;
+        int x2 = newx0;
+        FOR_RECS({
+          const int k = rec_kind(r, inw);
+          if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) {
+            const int xo = compact ? x2 : r.x;
+            x2 += r.y;
+            const int lb = lower(xo);
+            for (int x = lb_prev; x < lb; ++x) S.q_cnt[x] = (int)q2;
+            lb_prev = lb;
+            ++q2;
+          }
+        })
+      } else {
+        __syncthreads();
+#pragma unroll
+        for (int qq = 0; qq < kEntCap / PNT; ++qq) {
+          const int i = tid + qq * PNT;
+          if (i < np) {
+            const int o = S.q_off[i];
+            int lo = 0, hi = (int)nkept;
+            while (lo < hi) { const int mid = (lo + hi) >> 1; if (koff[mid] < o) lo = mid + 1; else hi = mid; }
+            S.q_cnt[i] = lo;
+          }
+        }
       }
     }
     __syncthreads();
-    if (tid < np) {
-      const int p = S.q_idx[tid];
-      const int t = S.p_t[p];
-      const uint8_t fl = sc.wfl[t];
-      int4 r;
-      r.x = S.p_off[p];
-      r.y = S.p_a[p];
-      r.z = t | ((a.t_flags[t] & 1) ? kRecTransient : 0) | ((fl & 1) ? kRecNxRd : 0) | (st.dirty[t] ? kRecDirty : 0);
-      r.w = sc.wnx[t];
-      dst[tid + S.q_cnt[tid]] = r;
-      st.pos[t] = tid + S.q_cnt[tid];
+#pragma unroll
+    for (int qq = 0; qq < kEntCap / PNT; ++qq) {
+      const int i = tid + qq * PNT;
+      if (i < np) {
+        const int p = S.q_idx[i];
+        const int e = S.p_e[p];
+        const int t = S.e_t[e];
+        const uint8_t fl = S.e_fl[e];
+        int4 r;
+        r.x = S.p_off[p];
+        r.y = S.e_au[e];
+        r.z = t | ((fl & 1) ? kRecTransient : 0) | ((fl & 8) ? kRecNxRd : 0) | ((fl & 4) ? kRecDirty : 0);
+        r.w = S.e_nx[e];
+        dst[i + S.q_cnt[i]] = r;
+        st.pos[t] = i + S.q_cnt[i];
+      }
     }
-    if (tid < n) { const int t = S.e_t[tid]; atomicAnd(&inw[t >> 5], ~(1u << (t & 31))); }
+#pragma unroll
+    for (int q = 0; q < kEntCap / PNT; ++q) {
+      const int e = tid + q * PNT;
+      if (e < n) { const int t = S.e_t[e]; atomicAnd(&inw[t >> 5], ~(1u << (t & 31))); }
+    }
+    for (int h = tid; h < kHash; h += PNT) S.h_key[h] = -1;
     // ---- header
     if (tid == 0) {
-      s_n[m] = nkept + np;
+      s_n[m] = (int)nkept + np;
       s_sel[m] = sel_new;
-      st.prev_n[0] = n;
+      s_prev_n = n;
       hd.half = m;
       hd.n_ent = n;
       hd.n_evict = nev;
@@ -816,7 +1122,9 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
     __syncthreads();
     PSTAMP(8);
   }
+  for (int i = tid; i < s_prev_n; i += PNT) st.prev[i] = S.prev_t[i];
   if (tid == 0) {
+    st.prev_n[0] = s_prev_n;
     st.G[0] = G0 + Kt;
     for (int h = 0; h < 2; ++h) { st.rl_meta[h] = s_n[h]; st.rl_meta[2 + h] = s_sel[h]; }
     out.counts[0] = Kt;
@@ -864,7 +1172,7 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
                         int max_groups, cudaStream_t s) {
   static uint64_t attr_done = 0;                   // bit d: set on device d
   const uint64_t bit = 1ull << current_device();
-  const size_t base = (sizeof(PlanSmem) + 15) / 16 * 16 + (size_t)kEvSmem * 8;
+  const size_t base = (sizeof(PlanSmem) + 15) / 16 * 16;
   const int inw_smem = a.T <= kInwSmemWords * 32 ? 1 : 0;
   const size_t smem = base + (inw_smem ? (size_t)kInwSmemWords * 4 : 0);
   if (!(attr_done & bit)) {
@@ -881,7 +1189,7 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
   bucket_scan_kernel<<<1, NT, 0, s>>>(a, sc);
   bucket_fill_kernel<<<grid, 256, 0, s>>>(a, pd, sc);
   bucket_sort_kernel<<<grid * 2, 256, 0, s>>>(a, pd, sc);
-  plan_kernel<<<1, NT, smem, s>>>(a, pd, policy, in, work, sc, out, inw_smem);
+  plan_kernel<<<1, PNT, smem, s>>>(a, pd, policy, in, work, sc, out, inw_smem);
   return cudaGetLastError();
 }
 

@@ -28,4 +28,5 @@ for step in range(3):
         info = d.plan_info(J) if J < d.K else {}
         print(f"{cfg} step {step}: plan {tm['plan']['ms'] * 1e3:.1f} us; K {d.K}; transition {J} "
               f"(ent {info.get('n_entries')}, ev {info.get('n_evict')}, mv {info.get('n_move')}, ca {info.get('n_carry')}, "
-              f"al {info.get('n_alloc')}, fe {info.get('n_fetch')}) cycles:", dif, "total", int(st[8] - st[0]) if st[8] else None)
+              f"al {info.get('n_alloc')}, fe {info.get('n_fetch')}) cycles:", dif, "total", int(st[8] - st[0]) if st[8] else None,
+              f"nm {st[60]} ng {st[61]} kept {st[62]} regmode {st[63]}")

@@ -75,6 +75,27 @@ def n_choices(site):
     return len(site.branches) if isinstance(site, If) else site.hi - site.lo + 1
 
 
+def nested_ids(program):
+    """ids of the sites nested inside another site's arm or body (reading R16): such a site
+    executes once per execution of its enclosing arm / loop iteration, each time with its own
+    choice; only top-level sites carry branch-head logits."""
+    out = set()
+
+    def rec(items, inside):
+        for it in items:
+            if isinstance(it, If):
+                if inside:
+                    out.add(id(it))
+                for br in it.branches:
+                    rec(br, True)
+            elif isinstance(it, Loop):
+                if inside:
+                    out.add(id(it))
+                rec(it.body, True)
+    rec(program, False)
+    return out
+
+
 def bind(op, k, b=0):
     """The operator as executed in iteration k of its innermost enclosing loop by prediction b
     of its batch (reading R13): an access (t, m, stride_k, stride_b) names tensor
@@ -101,18 +122,23 @@ def bind(op, k, b=0):
     return Op(op.idioms, op.inputs, tuple(acc), op.name)
 
 
-def resolve(program, choices, b=0):
+def resolve(program, choices, b=0, nested=None):
     """Executed row sequence for given site choices (choices[i] = choice index of preorder
     site i; If -> branch index, Loop -> trip count lo + index).
 
     Each row is (op or None). An executed If contributes one control row followed by the
     chosen branch; a Loop with n iterations contributes n+1 control rows (n continue tests
     plus the exit test, reading R2): [Z, body, Z, body, ..., Z]. b = the prediction's index in
-    its batch (per-sample tensors, reading R13)."""
+    its batch (per-sample tensors, reading R13). nested: the choices of the nested sites'
+    executions in execution order (reading R16; their entries in `choices` are unused)."""
     site_list = sites(program)
     index = {id(s): i for i, s in enumerate(site_list)}
+    inner = nested_ids(program)
+    it_nested = iter(nested or ())
 
     def choice_of(s):
+        if id(s) in inner:
+            return next(it_nested)
         i = index[id(s)]
         if s.tie >= 0:
             i = s.tie

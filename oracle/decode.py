@@ -35,6 +35,7 @@ class Prediction:
     slots: list             # raw decoded block head, K_max x 10 ints
     near_ties: list = field(default_factory=list)
     matched: bool = True    # traversal: exact match found
+    nested: list = field(default_factory=list)   # nested-site executions' choices (R16)
 
 
 def decode_block_head(y, K_max, near):
@@ -57,9 +58,13 @@ def decode_block_head(y, K_max, near):
 def decode_branch_head(y, program, K_max, near):
     """Branch head -> choice index for every site in preorder (reading R4, R6)."""
     sl = A.sites(program)
+    inner = A.nested_ids(program)
     off = 10 * K_max
     choices = [0] * len(sl)
     for i, s in enumerate(sl):
+        if id(s) in inner:
+            choices[i] = -1            # R16: resolved per execution by the traversal
+            continue
         if s.tie >= 0:
             choices[i] = choices[s.tie]
             continue
@@ -158,6 +163,202 @@ def traversal(program, pred_blocks, b=0):
     return best[1], best[2], False
 
 
+# ---- nested sites (reading R16) ---------------------------------------------------------
+# A site nested in another site's arm or loop body executes once per execution of its
+# enclosure, each time with its own choice, and carries no branch-head logits. With the
+# top-level choices fixed, the path is a sequence of rows and choice points (one per nested
+# execution, in execution order). The paper's mapping "enumerates and traverses each possible
+# branch" whenever a control flow is met: the executions' choices are visited in
+# lexicographic order of the execution-ordered choice sequence (lower branch index / trip count
+# first); the first path whose cut at the predicted cumulative counts gives exactly the
+# predicted vectors wins; otherwise the path with the closest operator count, first in
+# the same order.
+
+def _atoms(program, choices, b):
+    """The path of fixed top-level `choices` as atoms: ('row', op_or_None) and
+    ('choice', [arm_atoms, ...]) for every nested execution; arm c of a nested If is its
+    branch c, arm c of a nested Loop is its execution with trip count lo + c."""
+    sl = A.sites(program)
+    index = {id(s): i for i, s in enumerate(sl)}
+    inner = A.nested_ids(program)
+
+    def loop_rows(it, n, k_out):
+        out = []
+        for i in range(n):
+            out.append(("row", None))
+            out.extend(rec(it.body, n - 1 - i if it.rev else i))
+        out.append(("row", None))
+        return out
+
+    def rec(items, k):
+        out = []
+        for it in items:
+            if isinstance(it, Op):
+                out.append(("row", A.bind(it, k, b)))
+            elif id(it) in inner:
+                if it.tie >= 0:
+                    raise ValueError("a nested site cannot replay another site (R6, R16)")
+                if isinstance(it, If):
+                    out.append(("row", None))
+                    out.append(("choice", [rec(br, k) for br in it.branches]))
+                else:
+                    out.append(("choice", [loop_rows(it, it.lo + c, k) for c in range(A.n_choices(it))]))
+            else:
+                i = index[id(it)]
+                c = choices[it.tie if it.tie >= 0 else i]
+                if isinstance(it, If):
+                    out.append(("row", None))
+                    out.extend(rec(it.branches[c], k))
+                else:
+                    out.extend(loop_rows(it, it.lo + c, k))
+        return out
+    return rec(program, None)
+
+
+def _feed(g, acc, row, pred):
+    """One row into the running block vector of group g (R4 cut); None when no extension of
+    the prefix can match (every element is >= 0, so running sums only grow)."""
+    if g >= len(pred):
+        return None
+    sig = A.row_sig(row)
+    acc = (acc[0] + 1,) + tuple(acc[1 + e] + sig[e] for e in range(9))
+    p = pred[g]
+    sat = tuple(A.sat(x) for x in acc)
+    if any(sat[e] > p[e] for e in range(10)):
+        return None
+    if acc[0] == p[0]:
+        if sat != tuple(p):
+            return None
+        return g + 1, (0,) * 10
+    return g, acc
+
+
+def nested_exact(atoms, pred):
+    """First (lexicographic) resolution of the choice points whose rows, cut at the predicted
+    cumulative counts, give exactly the predicted vectors: (nested choices, rows) or None.
+    Depth-first in execution order; a prefix is abandoned as soon as it cannot match (_feed);
+    a failed state (continuation, group, running vector) is remembered - the search from it is
+    deterministic - so the search is polynomial on repetitive programs (both are
+    result-preserving)."""
+    failed = set()
+    rows, nested = [], []
+    zero = (0,) * 10
+
+    def go(stack, g, acc):
+        while stack:
+            lst, i = stack[-1]
+            if i == len(lst):
+                stack = stack[:-1]
+                continue
+            atom = lst[i]
+            stack = stack[:-1] + ((lst, i + 1),)
+            if atom[0] == "row":
+                r = _feed(g, acc, atom[1], pred)
+                if r is None:
+                    return False
+                g, acc = r
+                rows.append(atom[1])
+            else:
+                key = (tuple((id(l), j) for l, j in stack), g, acc)
+                if key in failed:
+                    return False
+                mr, mn = len(rows), len(nested)
+                for c, arm in enumerate(atom[1]):
+                    nested.append(c)
+                    if go(stack + ((arm, 0),), g, acc):
+                        return True
+                    del rows[mr:]
+                    del nested[mn:]
+                failed.add(key)
+                return False
+        return g == len(pred) and acc == zero
+
+    if go(((atoms, 0),), 0, zero):
+        return list(nested), list(rows)
+    return None
+
+
+def _all_resolutions(atoms, cap=200_000):
+    """Every resolution of the choice points in lexicographic order: (nested, rows)."""
+    count = [0]
+
+    def rec(stack, rows, nest):
+        rows = list(rows)
+        while stack:
+            lst, i = stack[-1]
+            if i == len(lst):
+                stack = stack[:-1]
+                continue
+            atom = lst[i]
+            stack = stack[:-1] + ((lst, i + 1),)
+            if atom[0] == "choice":
+                for c, arm in enumerate(atom[1]):
+                    yield from rec(stack + ((arm, 0),), rows, nest + [c])
+                return
+            rows.append(atom[1])
+        count[0] += 1
+        if count[0] > cap:
+            raise RuntimeError("too many resolutions for the exhaustive fallback")
+        yield nest, rows
+    yield from rec(((atoms, 0),), [], [])
+
+
+def nested_traversal(program, choices, pred_blocks, b=0):
+    """Reading R16 with the top-level choices fixed (branch head): (nested, rows, matched)."""
+    atoms = _atoms(program, choices, b)
+    pred = [tuple(v) for v in pred_blocks]
+    hit = nested_exact(atoms, pred)
+    if hit is not None:
+        return hit[0], hit[1], True
+    total = sum(v[0] for v in pred)
+    best = None
+    for nest, rows in _all_resolutions(atoms):
+        d = abs(len(rows) - total)
+        if best is None or d < best[0]:
+            best = (d, nest, rows)
+    return best[1], best[2], False
+
+
+def top_choice_vectors(program):
+    """Top-level choice vectors in lexicographic order (preorder; nested sites -1; a tied site
+    replays its target)."""
+    sl = A.sites(program)
+    inner = A.nested_ids(program)
+    free = [i for i, s in enumerate(sl) if id(s) not in inner and s.tie < 0]
+
+    def rec(k, cur):
+        if k == len(free):
+            v = [-1 if id(s) in inner else 0 for s in sl]
+            for i, s in enumerate(sl):
+                if id(s) in inner:
+                    continue
+                v[i] = cur[free.index(s.tie)] if s.tie >= 0 else cur[free.index(i)]
+            yield v
+            return
+        for c in range(A.n_choices(sl[free[k]])):
+            yield from rec(k + 1, cur + [c])
+    yield from rec(0, [])
+
+
+def traversal_nested(program, pred_blocks, b=0):
+    """Reading R16 without a branch head: top-level vectors in lexicographic order, each with
+    its nested executions in lexicographic order; first exact match, else the closest count
+    (first in the same order). Returns (choices, nested, rows, matched)."""
+    pred = [tuple(v) for v in pred_blocks]
+    for ch in top_choice_vectors(program):
+        hit = nested_exact(_atoms(program, ch, b), pred)
+        if hit is not None:
+            return ch, hit[0], hit[1], True
+    total = sum(v[0] for v in pred)
+    best = None
+    for ch in top_choice_vectors(program):
+        for nest, rows in _all_resolutions(_atoms(program, ch, b)):
+            d = abs(len(rows) - total)
+            if best is None or d < best[0]:
+                best = (d, ch, nest, rows)
+    return best[1], best[2], best[3], False
+
+
 def tensor_sets(path, groups):
     """W_j (reading R8): tensors accessed by the group's operators, in order of first access
     (row order; within an operator ascending tensor id); mode = union of the group's accesses;
@@ -185,11 +386,18 @@ def decode(wl, y, branch_head=True, b=0):
     slots = decode_block_head(y, wl.K_max, near)
     counts_slots = [v for v in slots if v[0] != 0]
     matched = True
+    nested = []
+    has_nested = bool(A.nested_ids(wl.program))
     if branch_head:
         choices = decode_branch_head(y, wl.program, wl.K_max, near)
-        path = A.resolve(wl.program, choices, b)
+        if has_nested:
+            nested, path, matched = nested_traversal(wl.program, choices, counts_slots, b)
+        else:
+            path = A.resolve(wl.program, choices, b)
+    elif has_nested:
+        choices, nested, path, matched = traversal_nested(wl.program, counts_slots, b)
     else:
         choices, path, matched = traversal(wl.program, counts_slots, b)
     groups = cut(len(path), [v[0] for v in counts_slots])
     blocks = [A.block10(path[s:e]) for s, e in groups]
-    return Prediction(choices, path, groups, blocks, tensor_sets(path, groups), slots, near, matched)
+    return Prediction(choices, path, groups, blocks, tensor_sets(path, groups), slots, near, matched, nested)

@@ -204,9 +204,11 @@ def _host_layout(tensors_bytes, align):
 
 
 def n_branch_logits(program):
-    """Count of free (untied) branch-head logits: structure bookkeeping of the input."""
+    """Count of free (untied) branch-head logits: structure bookkeeping of the input. Only
+    top-level sites carry logits; a site nested in another site's arm or body has none
+    (reading R16)."""
     n = 0
-    for it in _walk(program):
+    for it in program:
         if isinstance(it, If) and it.tie < 0:
             n += len(it.branches)
         elif isinstance(it, Loop) and it.tie < 0:
@@ -231,8 +233,12 @@ def actual_choices(wl, sample, zipf_s=1.2):
     tied sites replay their target (reading R6). Deterministic; no method arithmetic."""
     rng = np.random.default_rng((int(wl.seed) * 1_000_003 + int(sample)) & 0x7FFFFFFF)
     sl = [it for it in _walk(wl.program) if isinstance(it, (If, Loop))]
+    top = {id(it) for it in wl.program}
     out = []
     for it in sl:
+        if id(it) not in top:
+            out.append(-1)                 # nested site: per-execution choices (R16), not drawn
+            continue
         if it.tie >= 0:
             out.append(out[it.tie])
             continue

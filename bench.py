@@ -39,7 +39,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="dyo", choices=["dyo", "reference"])
-    ap.add_argument("--config", default="moe", choices=["moe", "tiny", "af", "lstm"])
+    ap.add_argument("--config", default="moe", choices=["moe", "tiny", "af", "lstm", "tree"])
     ap.add_argument("--policy", type=int, default=1)
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--budget-gib", type=float, default=0.0)
@@ -57,6 +57,9 @@ CONFIG_DESC = {
     "af": "AlphaFold-Evoformer-shaped trace, 48 blocks x recycle 1..4, MSA 128x256, 2 GiB budget (BASELINE configs[2])",
     "lstm": "variable-length 2-layer LSTM (length U{16..512}, 4 task heads), batch of 64 predictions planned per "
             "step, 35,860 tensors of 2-4 KiB (+ 4 MiB weights), 48 MiB budget (BASELINE configs[3], var-length variant)",
+    "tree": "Tree-LSTM over random binary parse trees (leaves U{8..64}, 2n-1 node loop with a nested leaf/internal If "
+            "resolved per node by the traversal, reading R16), batch of 64 predictions planned per step, 33,031 tensors "
+            "of 2-4 KiB (+ 14 MiB weights/grads), 256 MiB budget (BASELINE configs[3], Tree-LSTM primary)",
 }
 
 

@@ -198,9 +198,20 @@ dyo_status dyo_arch_check(const dyo_arch* arch, int32_t align, dyo_arch_summary*
  * arch has no branch head (no GPU needed; used by the CPU test suite). slots: K_max x 10 decoded
  * block-head vectors (a slot with count 0 is empty); choices (n_sites int32 out): the choice of
  * every site, preorder; *matched = 1 for an exact match, 0 for the closest-count fallback.
- * DYO_E_UNSUPPORTED for nested control flow, DYO_E_CAPACITY if the search exceeds its budget. */
+ * DYO_E_UNSUPPORTED for nested control flow (R16 needs a branch head), DYO_E_CAPACITY if the
+ * search exceeds its budget. */
 dyo_status dyo_traverse_check(const dyo_arch* arch, const int32_t* slots, int32_t* choices, int32_t* matched,
                               char* err, int32_t errlen);
+
+/* Host-only run of the nested-site decode (R16) that dyo_pilot_predict uses for arches with
+ * nested sites (no GPU needed; used by the CPU test suite): slots = K_max x 10 decoded block-head
+ * vectors, top_choices = the choice of every site in preorder (nested sites ignored). Outputs the
+ * nested executions' choices (cap ints; *n_nested), the path's operator per row (path_ops may be
+ * NULL; -1 for control rows; *path_len rows) and *matched. DYO_E_STATE if the arch has no nested
+ * sites, DYO_E_CAPACITY if an output is too small. */
+dyo_status dyo_nested_check(const dyo_arch* arch, const int32_t* slots, const int32_t* top_choices, int32_t* nested,
+                            int32_t cap, int32_t* n_nested, int32_t* path_ops, int32_t path_cap, int32_t* path_len,
+                            int32_t* matched, char* err, int32_t errlen);
 
 /* Load pilot weights (copied to the device, rows padded to 16 bytes). F and O must match the
  * arch: F = pad16(3 + D_s + 10*S_max + 10*h); O >= 10*K_max + branch logits. */
@@ -234,6 +245,17 @@ dyo_status dyo_prediction_get(dyo_ctx* ctx, int32_t b, int32_t* K, int32_t* bloc
  * of the last dyo_pilot_predict matched a path exactly, 0 if the closest-operator-count
  * fallback of P:L147 was taken. DYO_E_STATE with a branch head. Host-side; no sync. */
 dyo_status dyo_prediction_matched(dyo_ctx* ctx, int32_t b, int32_t* matched);
+/* Nested sites (reading R16: a site inside a top-level loop body or If arm executes once per
+ * iteration / arm execution with its own choice; only Ifs with operator-only arms may nest, and
+ * only with a branch head - DYO_E_UNSUPPORTED at load otherwise): the choices of prediction b's
+ * nested executions in execution order, resolved on the host against the block head by the
+ * paper's traversal (exact match, else the closest operator count) - which is also
+ * why dyo_pilot_predict synchronises its stream once for such arches. out (host, cap ints) may
+ * be NULL to query *n; DYO_E_CAPACITY if cap < *n. *n = 0 for arches without nested sites. The
+ * prediction's `choices` (dyo_prediction_get) hold -1 for nested sites; dyo_prediction_matched
+ * reports whether the nested resolution matched exactly. */
+dyo_status dyo_prediction_nested(dyo_ctx* ctx, int32_t b, int32_t* out, int32_t cap, int32_t* n);
+
 /* Tensor-set entries of group g of prediction b (host out, capacity cap entries of 3 int32:
  * tensor, mode, needs_fetch); *n receives the count (DYO_E_CAPACITY if cap < n). */
 dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* out, int32_t cap,

@@ -303,6 +303,42 @@ def _all_resolutions(atoms, cap=200_000):
     yield from rec(((atoms, 0),), [], [])
 
 
+def closest_flat(atoms, total):
+    """P:L147's fallback for a path whose choice points are flat (arms hold rows only): the
+    first resolution, in lexicographic order, among those whose row count is closest to
+    `total`. The row count is the fixed rows plus the chosen arms' lengths, so the reachable
+    counts after each choice point are sets (suffix sums); choosing at every point the lowest
+    arm from which a closest count stays reachable gives the lexicographically first such
+    resolution. (tests/test_oracle_nested.py checks it against the exhaustive enumeration.)"""
+    fixed = sum(1 for a in atoms if a[0] == "row")
+    points = [[len(arm) for arm in a[1]] for a in atoms if a[0] == "choice"]
+    suffix = [set() for _ in range(len(points) + 1)]
+    suffix[-1] = {0}
+    for i in range(len(points) - 1, -1, -1):
+        suffix[i] = {v + l for v in suffix[i + 1] for l in points[i]}
+    dbest = min(abs(fixed + v - total) for v in suffix[0])
+    targets = {total - dbest, total + dbest}
+    nest, used = [], fixed
+    for i, lens in enumerate(points):
+        for c, l in enumerate(lens):
+            if any((t - used - l) in suffix[i + 1] for t in targets):
+                nest.append(c)
+                used += l
+                break
+    it = iter(nest)
+    rows = []
+    for a in atoms:
+        if a[0] == "row":
+            rows.append(a[1])
+        else:
+            rows.extend(r[1] for r in a[1][next(it)])
+    return nest, rows
+
+
+def _flat(atoms):
+    return all(a[0] == "row" or all(x[0] == "row" for arm in a[1] for x in arm) for a in atoms)
+
+
 def nested_traversal(program, choices, pred_blocks, b=0):
     """Reading R16 with the top-level choices fixed (branch head): (nested, rows, matched)."""
     atoms = _atoms(program, choices, b)
@@ -311,6 +347,9 @@ def nested_traversal(program, choices, pred_blocks, b=0):
     if hit is not None:
         return hit[0], hit[1], True
     total = sum(v[0] for v in pred)
+    if _flat(atoms):
+        nest, rows = closest_flat(atoms, total)
+        return nest, rows, False
     best = None
     for nest, rows in _all_resolutions(atoms):
         d = abs(len(rows) - total)

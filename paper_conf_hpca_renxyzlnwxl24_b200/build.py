@@ -10,7 +10,7 @@ BUILD = os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CU = ["pilot.cu", "pilot_tc.cu", "decode.cu", "plan.cu", "copy.cu"]
-CPP = ["api.cpp", "traverse.cpp"]
+CPP = ["api.cpp", "traverse.cpp", "nested.cpp"]
 
 
 def _run(cmd):

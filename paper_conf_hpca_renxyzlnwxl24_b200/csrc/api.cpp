@@ -47,6 +47,12 @@ struct dyo_ctx {
   // logits / choices staging and the device choices the decode kernel replays
   int branch_head = 1;
   TravArch trav;
+  // nested sites (R16): the host resolves every prediction's path after the pilot
+  int nested = 0;
+  NestArch nest;
+  std::vector<int32_t> site_logit;            // host copy: logit offset of each site (-1: none)
+  int32_t* h_path = nullptr;                  // pinned: B x L_max ops | B x L_max iterations | B lengths
+  std::vector<std::vector<int32_t>> last_nested;   // nested executions' choices of each prediction
   // exact-match mis-prediction memo (R15): host mirror of the device table (ad.memo_*)
   struct Memo {
     int cap = 0, kw = 0, ns = 0, mask = 0, live = 0, tomb = 0;
@@ -239,8 +245,9 @@ void free_plan_host(dyo_ctx* c) {
     P.seg_used = 0;
   }
   fh(c->h_status); fh(c->h_counts); fh(c->h_loc); fh(c->h_off);
-  fh(c->h_forced[0]); fh(c->h_forced[1]); fh(c->h_matched); fh(c->h_rep);
+  fh(c->h_forced[0]); fh(c->h_forced[1]); fh(c->h_matched); fh(c->h_rep); fh(c->h_path);
   c->h_rep = nullptr;
+  c->h_path = nullptr;
   c->h_forced[0] = c->h_forced[1] = c->h_matched = nullptr;
   c->h_status = c->h_counts = nullptr;
   c->h_loc = nullptr;
@@ -300,6 +307,8 @@ struct ArchHost {
   std::vector<int32_t> t_flags, sig, acc_ptr, acc_t, acc_m, acc_s, acc_sb, site_rev;
   std::vector<int32_t> site_kind, site_nch, site_lo, site_tie, site_logit, site_arm_ptr, arm_first, arm_n;
   std::vector<int32_t> piece_kind, piece_a, piece_b, piece_c, seg_table;
+  int nested = 0;            // 1: some sites are nested (R16): the host resolves the paths
+  NestArch nest;
 };
 
 dyo_status hfail(std::string& err, dyo_status s, const char* fmt, ...) {
@@ -398,6 +407,28 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std
   if (expect_op != n_ops) return hfail(err, DYO_E_INVAL, "arch: %d ops in nodes, %d declared", expect_op, n_ops);
   const int n_sites = (int)site_node.size();
   if (n_sites > kMaxSites) return hfail(err, DYO_E_CAPACITY, "arch: too many sites");
+  // nesting (R16): a site inside another site's span executes per iteration / arm execution
+  std::vector<int> depth(n_sites, 0);
+  for (int s2 = 0; s2 < n_sites; ++s2)
+    for (int s1 = 0; s1 < s2; ++s1)
+      if (site_node[s2] <= site_node[s1] + A->node_span[site_node[s1]]) ++depth[s2];
+  std::vector<int> tied_to(n_sites, 0);
+  for (int s2 = 0; s2 < n_sites; ++s2)
+    if (A->node_tie[site_node[s2]] >= 0 && A->node_tie[site_node[s2]] < n_sites) tied_to[A->node_tie[site_node[s2]]] = 1;
+  for (int s2 = 0; s2 < n_sites; ++s2) {
+    if (!depth[s2]) continue;
+    const int i = site_node[s2];
+    if (A->node_kind[i] != 1 || depth[s2] > 1)
+      return hfail(err, DYO_E_UNSUPPORTED, "arch: site %d: only Ifs directly inside a top-level site may nest (R16)", s2);
+    for (int q = i + 1; q <= i + A->node_span[i]; ++q)
+      if (A->node_kind[q] == 1 || A->node_kind[q] == 2)
+        return hfail(err, DYO_E_UNSUPPORTED, "arch: nested site %d: its arms must hold operators only (R16)", s2);
+    if (A->node_tie[i] >= 0 || tied_to[s2])
+      return hfail(err, DYO_E_INVAL, "arch: nested site %d cannot replay or be replayed (R6, R16)", s2);
+    if (!A->branch_head)
+      return hfail(err, DYO_E_UNSUPPORTED, "arch: nested sites need a branch head (the traversal over nested sites is not built)");
+    h.nested = 1;
+  }
   int logit = 10 * A->K_max;
   int64_t L_max = 0;
   // walk the top level
@@ -420,6 +451,7 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std
     site_kind.push_back(k);
     const int tie = A->node_tie[i];
     if (tie >= s) return hfail(err, DYO_E_INVAL, "arch: site %d ties to a later site", s);
+    if (tie >= 0 && depth[tie]) return hfail(err, DYO_E_INVAL, "arch: site %d ties to a nested site", s);
     site_tie.push_back(tie);
     if (k == 1) {
       site_nch.push_back(A->node_a[i]);
@@ -434,8 +466,8 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std
       if (site_tie[tie] >= 0 || site_nch[tie] != site_nch[s] || site_kind[tie] != k)
         return hfail(err, DYO_E_INVAL, "arch: site %d tie target must be a free site of the same shape", s);
       site_logit.push_back(-1);
-    } else if (!A->branch_head) {
-      site_logit.push_back(-1);          // traversal decode: choices come from the host (R4)
+    } else if (!A->branch_head || depth[s]) {
+      site_logit.push_back(-1);          // traversal decode / nested site: choices from the host (R4, R16)
     } else {
       site_logit.push_back(logit);
       logit += site_nch[s];
@@ -454,6 +486,24 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std
     }
   }
   h.n_branch_logits = logit - 10 * A->K_max;
+  // longest row count of a node range (nested Ifs: control row + their longest arm)
+  auto range_maxlen = [&](int first, int last) {
+    int64_t L = 0;
+    for (int q = first; q < last;) {
+      const int kq = A->node_kind[q];
+      if (kq == 0) { ++L; ++q; }
+      else if (kq == 1) {
+        int64_t mx = 0;
+        int r = q + 1;
+        for (int br = 0; br < A->node_a[q]; ++br) { mx = std::max<int64_t>(mx, A->node_span[r]); r += 1 + A->node_span[r]; }
+        L += 1 + mx;
+        q += 1 + A->node_span[q];
+      } else {
+        ++q;
+      }
+    }
+    return L;
+  };
   for (int i = 0; i < N;) {
     const int k = A->node_kind[i];
     if (k == 0) {
@@ -466,15 +516,19 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std
       const int s = node_site[i];
       int fo; bool hs;
       const int n = count_ops(i + 1, A->node_span[i], &fo, &hs);
-      if (hs) return hfail(err, DYO_E_UNSUPPORTED, "arch: nested control flow under site %d (device decode needs top-level sites)", s);
+      (void)hs;                          // nested sites were validated above (R16)
       if (k == 1) {
-        int mx = 0;
-        for (int br = 0; br < site_nch[s]; ++br) mx = std::max(mx, arm_n[site_arm_ptr[s] + br]);
+        int64_t mx = 0;
+        int r = i + 1;
+        for (int br = 0; br < site_nch[s]; ++br) {
+          mx = std::max<int64_t>(mx, range_maxlen(r + 1, r + 1 + A->node_span[r]));
+          r += 1 + A->node_span[r];
+        }
         piece_kind.push_back(1); piece_a.push_back(s); piece_b.push_back(0); piece_c.push_back(0);
         L_max += 1 + mx;
       } else {
         piece_kind.push_back(2); piece_a.push_back(s); piece_b.push_back(fo); piece_c.push_back(n);
-        L_max += (int64_t)(site_lo[s] + site_nch[s] - 1) * (1 + n) + 1;
+        L_max += (int64_t)(site_lo[s] + site_nch[s] - 1) * (1 + range_maxlen(i + 1, i + 1 + A->node_span[i])) + 1;
       }
       i += 1 + A->node_span[i];
     } else {
@@ -517,6 +571,22 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std
 
   h.n_sites = n_sites;
   h.L_max = L_max;
+  if (h.nested) {
+    NestArch& na = h.nest;
+    na.kind.assign(A->node_kind, A->node_kind + N);
+    na.a.assign(A->node_a, A->node_a + N);
+    na.b.assign(A->node_b, A->node_b + N);
+    na.span.assign(A->node_span, A->node_span + N);
+    na.flags.assign(N, 0);
+    if (A->node_flags) na.flags.assign(A->node_flags, A->node_flags + N);
+    na.site_of.assign(N, -1);
+    for (int s2 = 0; s2 < n_sites; ++s2) na.site_of[site_node[s2]] = s2;
+    na.sig = sig;
+    na.site_lo = site_lo;
+    na.site_tie = site_tie;
+    na.top.assign(n_sites, 0);
+    for (int s2 = 0; s2 < n_sites; ++s2) na.top[s2] = depth[s2] ? 0 : 1;
+  }
   return DYO_OK;
 }
 
@@ -681,6 +751,10 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   ctx->n_ops = n_ops; ctx->n_sites = n_sites; ctx->K_max = A->K_max; ctx->F = ad.F;
   ctx->branch_head = A->branch_head ? 1 : 0;
   ad.branch_head = ctx->branch_head;
+  ctx->nested = h.nested;
+  ctx->nest = h.nest;
+  ctx->site_logit = site_logit;
+  ctx->last_nested.clear();
   ctx->trav = TravArch{h.sig, site_kind, site_nch, site_lo, site_tie, site_arm_ptr, arm_first, arm_n,
                        piece_kind, piece_a, piece_b, piece_c};
   ctx->O_min = 10 * A->K_max + ctx->n_branch_logits;
@@ -692,17 +766,23 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   pd.B = B;
 #define DA(p, n) if ((st = dalloc(ctx, own, &p, (size_t)(n)))) return st
   DA(pd.K, B); DA(pd.L, B); DA(pd.choices, (size_t)B * std::max(n_sites, 1)); DA(pd.rchoices, (size_t)B * std::max(n_sites, 1)); DA(pd.slots, (size_t)B * K * 10);
-  DA(pd.path, (size_t)B * ad.L_max); DA(pd.grp, (size_t)B * K * 2); DA(pd.blocks, (size_t)B * K * 10);
+  DA(pd.path, (size_t)B * ad.L_max); DA(pd.path_it, (size_t)B * ad.L_max); DA(pd.grp, (size_t)B * K * 2);
+  DA(pd.blocks, (size_t)B * K * 10);
   DA(pd.ent_n, (size_t)B * K); DA(pd.ent, (size_t)B * K * kEntCap); DA(pd.status, 4);
   pd.head_stride = 3 + n_sites + ((int)piece_kind.size() + 1) + (K + 1) + K;
   DA(pd.head, (size_t)B * pd.head_stride);
   DA(ctx->desc_dev, (size_t)B * std::max(A->D_s, 1)); DA(ctx->hist_dev, (size_t)B * std::max(A->h, 1));
   DA(ctx->hist_tab[0], (size_t)B * K * 10); DA(ctx->hist_tab[1], (size_t)B * K * 10);
   DA(ctx->hist_K[0], B); DA(ctx->hist_K[1], B);
-  if (!ctx->branch_head) {
+  if (!ctx->branch_head || ctx->nested) {
     int32_t* f = nullptr;
     DA(f, (size_t)B * std::max(n_sites, 1));
     ad.forced = ctx->d_forced = f;
+  }
+  if (ctx->nested) {                    // the decode kernels read the host-resolved paths (R16)
+    ad.hp_op = pd.path;
+    ad.hp_it = pd.path_it;
+    ad.hp_len = pd.L;
   }
   ctx->hist_B[0] = ctx->hist_B[1] = 0;
   ctx->hist_cur = 0;
@@ -738,11 +818,12 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   if ((st = hmap((void**)&ctx->h_loc, T))) return st;
   if ((st = hmap((void**)&ctx->h_off, sizeof(int64_t) * T))) return st;
   if ((st = hmap((void**)&ctx->h_rep, sizeof(int32_t) * (4 + 10 * (size_t)K + 2 * (size_t)std::max(n_sites, 1))))) return st;
-  if (!ctx->branch_head) {
+  if (!ctx->branch_head || ctx->nested) {
     for (int i = 0; i < 2; ++i)
       if ((st = hmap((void**)&ctx->h_forced[i], sizeof(int32_t) * B * std::max(n_sites, 1)))) return st;
     if ((st = hmap((void**)&ctx->h_matched, sizeof(int32_t) * B))) return st;
   }
+  if (ctx->nested && (st = hmap((void**)&ctx->h_path, sizeof(int32_t) * ((size_t)2 * B * ad.L_max + B)))) return st;
   memset(ctx->h_loc, 0xff, T);
   int32_t* d_status = nullptr;
   int32_t* d_counts = nullptr;
@@ -810,6 +891,33 @@ dyo_status dyo_traverse_check(const dyo_arch* A, const int32_t* slots, int32_t* 
     int m = 0;
     st = traverse_decode(t, slots, A->K_max, choices, &m, e);
     *matched = m;
+  }
+  if (err && errlen > 0) { strncpy(err, e.c_str(), errlen - 1); err[errlen - 1] = 0; }
+  return st;
+}
+
+dyo_status dyo_nested_check(const dyo_arch* A, const int32_t* slots, const int32_t* top_choices, int32_t* nested,
+                            int32_t cap, int32_t* n_nested, int32_t* path_ops, int32_t path_cap, int32_t* path_len,
+                            int32_t* matched, char* err, int32_t errlen) {
+  if (!A || !slots || !top_choices || !n_nested || !path_len || !matched) return DYO_E_INVAL;
+  ArchHost h;
+  std::string e;
+  dyo_status st = parse_arch(A, 256, 1, h, e);
+  if (!st && !h.nested) { e = "arch has no nested sites"; st = DYO_E_STATE; }
+  if (!st) {
+    std::vector<int32_t> pop, pit, nest;
+    int m = 0;
+    st = nested_decode(h.nest, slots, A->K_max, top_choices, pop, pit, nest, &m, e);
+    if (!st) {
+      *matched = m;
+      *n_nested = (int32_t)nest.size();
+      *path_len = (int32_t)pop.size();
+      if ((int32_t)nest.size() > cap || (path_ops && (int32_t)pop.size() > path_cap)) st = DYO_E_CAPACITY;
+      else {
+        if (nested) std::copy(nest.begin(), nest.end(), nested);
+        if (path_ops) std::copy(pop.begin(), pop.end(), path_ops);
+      }
+    }
   }
   if (err && errlen > 0) { strncpy(err, e.c_str(), errlen - 1); err[errlen - 1] = 0; }
   return st;
@@ -1065,7 +1173,7 @@ dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
   ctx->tc_dev = nullptr;
   if ((s = build_tc_plan(ctx, w))) return s;
   if (ctx->h_logits) { cudaFreeHost(ctx->h_logits); ctx->h_logits = nullptr; }
-  if (!ctx->branch_head)
+  if (!ctx->branch_head || ctx->nested)
     CK(cudaHostAlloc((void**)&ctx->h_logits, sizeof(double) * ctx->cfg.max_batch * w->O, cudaHostAllocPortable));
   ctx->pilot_ok = true;
   return DYO_OK;
@@ -1163,14 +1271,18 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
                       &fused, st));
     }
   }
-  if (!ctx->branch_head) {
-    // traversal decode: logits to the host, one sync, block head -> slots
-    // (R4: rint half-even of y * 2^sigma, clamped), path search, choices back to the device
+  if (!ctx->branch_head || ctx->nested) {
+    // host decode: logits to the host, one sync, block head -> slots (R4: rint
+    // half-even of y * 2^sigma, clamped); traversal over the top-level sites (no branch head)
+    // or, with nested sites (R16), the branch-head argmax (lowest index on ties) and the nested
+    // executions resolved against the block head; choices (and paths) back to the device
     const int O = ctx->ad.O, K = ctx->K_max, ns = ctx->n_sites;
     CK(cudaMemcpyAsync(ctx->h_logits, ctx->logits64, sizeof(double) * B * O, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     int32_t* hf = ctx->h_forced[cur];
     std::vector<int32_t> slots((size_t)K * 10);
+    if (ctx->nested) ctx->last_nested.assign(B, {});
+    const int64_t Lm = ctx->ad.L_max;
     for (int b = 0; b < B; ++b) {
       const double* y = ctx->h_logits + (size_t)b * O;
       for (int i = 0; i < K * 10; ++i) {
@@ -1178,11 +1290,37 @@ dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* 
         slots[i] = (int32_t)std::nearbyint(t);
       }
       int matched = 0;
-      dyo_status r = traverse_decode(ctx->trav, slots.data(), K, hf + (size_t)b * std::max(ns, 1), &matched, ctx->err);
-      if (r) return r;
+      int32_t* chb = hf + (size_t)b * std::max(ns, 1);
+      if (!ctx->nested) {
+        dyo_status r = traverse_decode(ctx->trav, slots.data(), K, chb, &matched, ctx->err);
+        if (r) return r;
+      } else {
+        for (int s2 = 0; s2 < ns; ++s2) {
+          const int off = ctx->site_logit[s2];
+          if (off < 0) { chb[s2] = -1; continue; }
+          int best = 0;
+          for (int c = 1; c < ctx->trav.site_nch[s2]; ++c)
+            if (y[off + c] > y[off + best]) best = c;
+          chb[s2] = best;
+        }
+        for (int s2 = 0; s2 < ns; ++s2)
+          if (ctx->trav.site_tie[s2] >= 0) chb[s2] = chb[ctx->trav.site_tie[s2]];
+        std::vector<int32_t> pop, pit;
+        dyo_status r = nested_decode(ctx->nest, slots.data(), K, chb, pop, pit, ctx->last_nested[b], &matched, ctx->err);
+        if (r) return r;
+        if ((int64_t)pop.size() > Lm) return fail(ctx, DYO_E_CAPACITY, "nested path of %zu rows > L_max", pop.size());
+        std::copy(pop.begin(), pop.end(), ctx->h_path + (size_t)b * Lm);
+        std::copy(pit.begin(), pit.end(), ctx->h_path + (size_t)B * Lm + (size_t)b * Lm);
+        ctx->h_path[(size_t)2 * B * Lm + b] = (int32_t)pop.size();
+      }
       ctx->h_matched[b] = matched;
     }
     if (ns > 0) CK(cudaMemcpyAsync(ctx->d_forced, hf, sizeof(int32_t) * B * ns, cudaMemcpyHostToDevice, st));
+    if (ctx->nested) {
+      CK(cudaMemcpyAsync(ctx->pd.path, ctx->h_path, sizeof(int32_t) * B * Lm, cudaMemcpyHostToDevice, st));
+      CK(cudaMemcpyAsync(ctx->pd.path_it, ctx->h_path + (size_t)B * Lm, sizeof(int32_t) * B * Lm, cudaMemcpyHostToDevice, st));
+      CK(cudaMemcpyAsync(ctx->pd.L, ctx->h_path + (size_t)2 * B * Lm, sizeof(int32_t) * B, cudaMemcpyHostToDevice, st));
+    }
   }
   if (!fused) {
     TScope ts(ctx, 1, st);
@@ -1415,8 +1553,19 @@ dyo_status dyo_memo_stats(dyo_ctx* ctx, int64_t* mispredictions, int32_t* live, 
 
 dyo_status dyo_prediction_matched(dyo_ctx* ctx, int32_t b, int32_t* matched) {
   if (!ctx || !matched || b < 0 || b >= ctx->last_B) return DYO_E_INVAL;
-  if (ctx->branch_head || !ctx->h_matched) return fail(ctx, DYO_E_STATE, "no traversal decode in this arch");
+  if ((ctx->branch_head && !ctx->nested) || !ctx->h_matched) return fail(ctx, DYO_E_STATE, "no traversal decode in this arch");
   *matched = ctx->h_matched[b];
+  return DYO_OK;
+}
+
+dyo_status dyo_prediction_nested(dyo_ctx* ctx, int32_t b, int32_t* out, int32_t cap, int32_t* n) {
+  if (!ctx || !n || b < 0 || b >= ctx->last_B) return DYO_E_INVAL;
+  if (!ctx->nested) { *n = 0; return DYO_OK; }
+  if (b >= (int)ctx->last_nested.size()) return fail(ctx, DYO_E_STATE, "no prediction");
+  const auto& v = ctx->last_nested[b];
+  *n = (int32_t)v.size();
+  if ((int32_t)v.size() > cap) return fail(ctx, DYO_E_CAPACITY, "need %zu", v.size());
+  if (out) std::copy(v.begin(), v.end(), out);
   return DYO_OK;
 }
 

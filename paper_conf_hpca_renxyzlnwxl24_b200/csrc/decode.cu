@@ -92,7 +92,7 @@ decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int 
       if (threadIdx.x == 0) pd.ent_n[(int64_t)b * Km + g] = 0;
       continue;
     }
-    if (threadIdx.x == 0) { H.L = h[0]; H.nk = h[1]; H.K = K; }
+    if (threadIdx.x == 0) { H.L = h[0]; H.nk = h[1]; H.K = K; H.b = b; }
     __syncthreads();
     const int* hc = h + 3;
     for (int i = threadIdx.x; i < ns; i += blockDim.x) H.choice[i] = hc[i];

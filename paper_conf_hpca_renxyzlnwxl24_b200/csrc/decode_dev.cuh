@@ -34,6 +34,7 @@ struct DecHead {
   int cntc[256];                       // non-empty counts in slot order
   int choice[kMaxSites];
   int L, nk, K;
+  int b;                               // the prediction (host-resolved paths, R16)
 };
 
 // Head of a prediction with runtime-sized arrays (the stand-alone group kernel carves them from
@@ -45,6 +46,7 @@ struct DecHeadDyn {
   int* cntc;
   int* choice;
   int L, nk, K;
+  int b;
 };
 
 // Group-build scratch for at most R access records (R a power of two).
@@ -291,9 +293,11 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
   __syncwarp();
   memo_lookup_warp(a, y, H, lane, rch);
   DSTAMP(1);
-  // 3. piece lengths -> exclusive scan -> piece starts (R2)
+  // 3. piece lengths -> exclusive scan -> piece starts (R2); a host-resolved path (nested
+  //    sites, R16) brings its own length
   int carry = 0;
-  for (int p0 = 0; p0 < a.n_pieces; p0 += 32) {
+  if (a.hp_len) carry = a.hp_len[b];
+  for (int p0 = 0; p0 < a.n_pieces && !a.hp_len; p0 += 32) {
     const int p = p0 + lane;
     int len = 0;
     if (p < a.n_pieces) {
@@ -332,6 +336,7 @@ static __device__ void head_decode_warp(const ArchDev& a, const double* __restri
     H.L = L;
     H.nk = nk;
     H.K = K;
+    H.b = b;
   }
   __syncwarp();
 }
@@ -348,6 +353,11 @@ __device__ __forceinline__ int group_end(const HT& H, int g) {
 // per-iteration tensors (R13; 0 outside loops, counted down in a reversed loop).
 template <class HT>
 __device__ __forceinline__ int row_op(const ArchDev& a, const HT& H, int r, int* it = nullptr) {
+  if (a.hp_op) {                                               // host-resolved path (R16)
+    const int64_t i = (int64_t)H.b * a.L_max + r;
+    if (it) *it = a.hp_it[i];
+    return a.hp_op[i];
+  }
   int lo = 0, hi = a.n_pieces - 1;
   while (lo < hi) {
     const int mid = (lo + hi + 1) >> 1;
@@ -552,7 +562,7 @@ static __device__ void write_head(const ArchDev& a, const DecHead& H, const doub
                            int32_t* __restrict__ hist_K) {
   for (int i = threadIdx.x; i < a.K_max * 10; i += blockDim.x) pd.slots[(int64_t)b * a.K_max * 10 + i] = slot_int(y, i);
   for (int i = threadIdx.x; i < a.n_sites; i += blockDim.x) pd.choices[(int64_t)b * a.n_sites + i] = H.choice[i];
-  if (H.L <= a.L_max)
+  if (H.L <= a.L_max && !a.hp_op)
     for (int r = threadIdx.x; r < H.L; r += blockDim.x) pd.path[(int64_t)b * a.L_max + r] = row_op(a, H, r);
   if (threadIdx.x == 0) {
     pd.K[b] = H.K;

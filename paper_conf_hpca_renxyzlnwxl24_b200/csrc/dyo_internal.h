@@ -119,6 +119,11 @@ struct ArchDev {
   const int32_t* piece_c;
   const int32_t* seg_table;  // S_max x 10
   int branch_head;           // 0: choices come from the host traversal (forced, R4)
+  // nested sites (R16): the host resolves every prediction's path (rows + iteration indices);
+  // the decode kernels read it instead of expanding top-level pieces (null otherwise)
+  const int32_t* hp_op;      // max_batch x L_max: operator of each row (-1 control)
+  const int32_t* hp_it;      // max_batch x L_max: iteration index of the row's loop (R13)
+  const int32_t* hp_len;     // max_batch: path length
   const int32_t* forced;     // max_batch x n_sites choices written by the traversal, or null
   // exact-match mis-prediction memo (R15; memo.cpp): live entries > 0 enables the
   // lookup in the head decode. index: open-addressing slots (entry id, -1 empty, -2 deleted)
@@ -139,6 +144,7 @@ struct PredDev {
   int32_t* rchoices;  // B x n_sites: the pilot's own (raw) choices, the memo key's half
   int32_t* slots;     // B x K_max x 10 (decoded block head)
   int32_t* path;      // B x L_max (operator index, -1 control)
+  int32_t* path_it;   // B x L_max iteration index (nested arches: written by the host)
   int32_t* grp;       // B x K_max x 2 (start, end rows)
   int32_t* blocks;    // B x K_max x 10 executed block vectors
   int32_t* ent_n;     // B x K_max entry counts
@@ -222,6 +228,21 @@ struct TravArch {
 // when an exact match was found (else the closest-count fallback of P:L147).
 dyo_status traverse_decode(const TravArch& A, const int32_t* slots, int K_max, int32_t* choices, int* matched,
                            std::string& err);
+
+// ---- host nested-site decode (nested.cpp, R16) -----------------------------
+// Program tree of an arch with nested sites: every nested site is an If directly inside a
+// top-level Loop body or If arm whose own arms hold operators only.
+struct NestArch {
+  std::vector<int32_t> kind, a, b, span, flags, site_of;   // per node (site_of: site index or -1)
+  std::vector<int32_t> sig;                                // n_ops x 9 saturated signatures
+  std::vector<int32_t> site_lo, site_tie, top;             // per site; top = 1 for top-level sites
+};
+// top_choices: n_sites ints (nested sites ignored). Outputs the path (operator per row, -1 for
+// control rows; iteration index per row), the nested executions' choices in execution order and
+// *matched (1 exact, 0 closest-count fallback).
+dyo_status nested_decode(const NestArch& N, const int32_t* slots, int K_max, const int32_t* top_choices,
+                         std::vector<int32_t>& path_op, std::vector<int32_t>& path_it, std::vector<int32_t>& nested,
+                         int* matched, std::string& err);
 
 // ---- launchers (implemented in the .cu files) ------------------------------------------
 cudaError_t launch_encode(const ArchDev& a, const int64_t* desc, const int32_t* hist,

@@ -675,7 +675,7 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   sp.dec_tab_cap = dec_table_words(a, kDecTabCap);
   // fuse the decode when each CTA decodes at most a few groups of its samples (traversal: the
   // host decides first, so the decode runs after it in the stand-alone kernels)
-  sp.fuse_decode = (a.branch_head && sp.Bs * a.K_max <= 2 * C) ? 1 : 0;
+  sp.fuse_decode = (a.branch_head && !a.hp_op && sp.Bs * a.K_max <= 2 * C) ? 1 : 0;
   sp.push_logits = (sp.fuse_decode && C > 1 && sp.Bs == 1 && p.n_stages > 1) ? 1 : 0;
   sp.tab_off = -1;
   const int act_bytes = 2 * sp.Bs * p.max_width * (int)sizeof(double);

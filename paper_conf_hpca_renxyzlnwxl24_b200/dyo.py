@@ -98,7 +98,7 @@ def lib():
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
                      "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
                      "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats",
-                     "dyo_debug_copy_stamps", "dyo_query", "dyo_set_timing"):
+                     "dyo_debug_copy_stamps", "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -110,7 +110,7 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
            "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
            "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps",
-           "dyo_query", "dyo_set_timing")
+           "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check")
 
 
 def _a(x, dt):
@@ -210,6 +210,21 @@ def traverse_check(wl, slots):
     err = C.create_string_buffer(512)
     st = lib().dyo_traverse_check(C.byref(arch), _p(sl, i32), _p(ch, i32), C.byref(m), err, 512)
     return st, ch[:n_sites].tolist(), m.value, err.value.decode()
+
+
+def nested_check(wl, slots, top_choices, cap=1 << 16):
+    """Host-only nested-site decode by libdyo (no GPU): (status, nested, path_ops, matched, err)."""
+    arch, keep = _arch_struct(wl)
+    sl = _a(slots, np.int32).reshape(-1)
+    assert sl.size == wl.K_max * 10
+    tc = _a([max(c, 0) if c is not None else 0 for c in top_choices] or [0], np.int32)
+    nest = np.zeros(cap, np.int32)
+    path = np.zeros(cap, np.int32)
+    nn, pl, m = i32(), i32(), i32()
+    err = C.create_string_buffer(512)
+    st = lib().dyo_nested_check(C.byref(arch), _p(sl, i32), _p(tc, i32), _p(nest, i32), cap, C.byref(nn),
+                                _p(path, i32), cap, C.byref(pl), C.byref(m), err, 512)
+    return st, nest[:nn.value].tolist(), path[:pl.value].tolist(), m.value, err.value.decode()
 
 
 class Dyo:
@@ -329,6 +344,13 @@ class Dyo:
         m = i32()
         self._check(self.L.dyo_prediction_matched(self.ctx, b, C.byref(m)))
         return m.value
+
+    def nested(self, b, cap=4096):
+        """Choices of prediction b's nested-site executions in execution order (reading R16)."""
+        out = np.zeros(cap, np.int32)
+        n = i32()
+        self._check(self.L.dyo_prediction_nested(self.ctx, b, _p(out, i32), cap, C.byref(n)))
+        return out[: n.value].tolist()
 
     def group_entries(self, b, g, cap=1024, stream=0):
         out = np.zeros((cap, 3), np.int32)

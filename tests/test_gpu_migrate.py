@@ -348,3 +348,11 @@ def test_af_fullsize_bytes():
     wl = WL.make("af", n_samples=4)
     m = run_bytes(wl, 1, 1, gpu_fill=True)
     assert m["dma"] > 0
+
+
+def test_tree_scaled_nested_bytes():
+    """Tree-LSTM with nested per-node sites (R16): the host-resolved paths drive the plan; every
+    read of every block and every host home checked (small hidden size, 4 predictions)."""
+    wl = WL.make("tree", n_samples=16, batch=4, max_leaves=16, hidden=128, budget=8 << 20)
+    m = run_bytes(wl, 2, 1, B=4)
+    assert m["zc"] + m["dma"] > 0

@@ -43,7 +43,7 @@ def test_encode_bitexact(name):
 
 @pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 16), ("moe", 1), ("moe", 8), ("af", 1), ("af", 3),
                                     ("lstm", 8), ("lstm", 64), ("moe", 64), ("af", 64), ("moe", 20), ("moe", 100),
-                                    ("af", 17)])
+                                    ("af", 17), ("tree", 4), ("tree", 64)])
 def test_pilot_logits(name, B):
     wl = WL.make(name, n_samples=max(16, B))
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
@@ -84,6 +84,9 @@ def test_predict_from_encoded_features(name, B):
 
 def _check_prediction(d, wl, b, pred):
     K, blocks, choices, rows = d.prediction(b, wl.K_max, len(A.sites(wl.program)), _stream())
+    if A.nested_ids(wl.program):          # R16: nested executions resolved by the host traversal
+        assert d.nested(b) == pred.nested
+        assert d.matched(b) == int(pred.matched)
     assert K == len(pred.groups)
     assert [tuple(r) for r in rows.tolist()] == pred.groups
     assert [tuple(v) for v in blocks.tolist()] == [tuple(v) for v in pred.blocks]
@@ -93,7 +96,8 @@ def _check_prediction(d, wl, b, pred):
         assert [tuple(e) for e in ent.tolist()] == [(t, m, int(f)) for t, m, f in pred.W[g]], f"group {g}"
 
 
-@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 8), ("moe", 1), ("moe", 4), ("af", 2), ("lstm", 8)])
+@pytest.mark.parametrize("name,B", [("tiny", 1), ("tiny", 8), ("moe", 1), ("moe", 4), ("af", 2), ("lstm", 8),
+                                    ("tree", 1), ("tree", 8), ("tree", 64)])
 def test_decode(name, B):
     wl = WL.make(name, n_samples=max(16, B))
     d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
@@ -248,6 +252,39 @@ def test_plan_bitexact_lstm_batch64_bench_config():
     d = _run_plan_steps(wl, 1, 64, 1)
     assert d.query("plan_syncs") == 1
     assert d.query("pilot_kernel") == 0
+    d.close()
+
+
+@pytest.mark.parametrize("policy", [0, 1])
+def test_plan_bitexact_tree_scaled(policy):
+    """Tree-LSTM (configs[3] primary): nested leaf/internal site per node (R16), per-(sample,
+    node) tensors (R13), batch of 8 predictions planned as one sequence, two steps."""
+    wl = WL.make("tree", n_samples=32, batch=8, max_leaves=24, budget=64 << 20)
+    _run_plan_steps(wl, 2, 8, policy).close()
+
+
+def test_plan_bitexact_tree_batch64_bench_config():
+    """The bench's Tree-LSTM configuration: 64 predictions, 1,024 transitions, RETAIN."""
+    wl = WL.make("tree", n_samples=64)
+    d = _run_plan_steps(wl, 1, 64, 1)
+    assert d.query("plan_syncs") == 1
+    d.close()
+
+
+def test_decode_tree_random_pilot_fallback():
+    """An unplanted (random) Tree-LSTM pilot: the nested executions fall back to the closest
+    operator count, exactly as the oracle."""
+    wl = WL.make("tree", n_samples=16, batch=4)
+    rng = np.random.default_rng(5)
+    Wo = wl.pilot.weights["out.W"]
+    Wo[:10 * wl.K_max] = rng.uniform(-1, 1, size=Wo[:10 * wl.K_max].shape).astype(np.float32)
+    wl.pilot.weights["out.b"][:10 * wl.K_max] = np.float32(2.0)
+    d = make_ctx(wl, max_batch=4, flags=F_NO_HOST_POOL)
+    d.predict(wl.samples[:4].copy(), hist_for(wl, 4), 4, stream=_stream())
+    r = oracle_step(wl, range(4), PL.initial_state(len(wl.tensors)), (), plan=False)
+    for b in range(4):
+        assert not r["preds"][b].near_ties
+        _check_prediction(d, wl, b, r["preds"][b])
     d.close()
 
 

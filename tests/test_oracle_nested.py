@@ -127,3 +127,21 @@ def test_branch_head_skips_nested_sites():
     y[10 + 2] = 1.0
     near = []
     assert D.decode_branch_head(y, prog, 1, near) == [2, -1]
+
+
+@settings(max_examples=80, deadline=None)
+@given(nested_programs(), st.data())
+def test_closest_flat_equals_exhaustive_fallback(prog, data):
+    """The suffix-set fallback (P:L147 for flat choice points) = the exhaustive enumeration's
+    first closest resolution."""
+    ch = data.draw(st.sampled_from(list(D.top_choice_vectors(prog))))
+    atoms = D._atoms(prog, ch, 0)
+    if not D._flat(atoms):
+        return
+    total = data.draw(st.integers(0, 40))
+    best = None
+    for nest, rows in D._all_resolutions(atoms):
+        d = abs(len(rows) - total)
+        if best is None or d < best[0]:
+            best = (d, nest, rows)
+    assert D.closest_flat(atoms, total) == (best[1], best[2])

@@ -672,7 +672,203 @@ def _plant_lstm_heads(pilot, K_max, min_len, max_len, tasks, rows_per_step, rows
         off += 1
 
 
-CONFIGS = {"tiny": make_tiny, "moe": make_moe, "af": make_af, "lstm": make_lstm}
+def _random_tree_postorder(rng, n):
+    """Post-order node types (0 leaf, 1 internal) of a random binary tree with n leaves
+    (uniform random split of the leaf span at every internal node)."""
+    out = []
+
+    def rec(m):
+        if m == 1:
+            out.append(0)
+            return
+        left = int(rng.integers(1, m))
+        rec(left)
+        rec(m - left)
+        out.append(1)
+    rec(n)
+    return out
+
+
+def make_tree(seed=0, n_samples=128, batch=64, min_leaves=8, max_leaves=64, hidden=512,
+              budget=256 * MiB, pilot_kind="P512", K_max=16, fwd_groups=8):
+    """Tree-LSTM over binary parse trees: configs[3]'s primary variant (survey §8(d) M3).
+
+    Per sample: embed; Loop F over the tree's nodes in post-order (trip 2n-1 in [15, 127] for
+    n leaves in U{8..64}) whose body is ONE If selecting the node type - a site nested in the
+    loop, so every node takes its own choice (reading R16): leaf (one cell op reading the
+    word's input x[b,k]) or internal (compose + norm ops reading the states of nodes k-1 and
+    k-2: the right child of a post-order node is k-1; the left child is approximated by k-2,
+    since child indices of an arbitrary parse tree are not a linear stride, R13); loss; Loop B
+    (tied to F, reversed) of a uniform node-backward op accumulating the weight gradients;
+    optimizer. Per-(sample, node) tensors use strided accesses (R13): h/c (2 KiB), saved
+    gates g (4 KiB, transient), input x (2 KiB); two leading pad slots keep k-2 in range.
+    The pilot is planted (a stand-in for a trained pilot): pass-through units
+    carry the descriptors N = 2n-1, the per-group leaf / internal counts of 8 forward groups
+    (even node split) and the node counts of 8 backward groups through every layer, and the
+    block head is the exact linear function of them - so the decode meets an exact match, and
+    the traversal orders each group's leaves before its internal nodes (the lexicographically
+    first resolution; order inside a block is not predicted). The trip-count logits
+    (2tN - t^2)/2048 put the argmax at t = N."""
+    rng = np.random.default_rng(seed)
+    tensors = []
+
+    def add(nb, transient, name):
+        tensors.append([nb, transient, name])
+        return len(tensors) - 1
+
+    hb, gb = hidden * 4, 4 * hidden * 2
+    W_leaf = add(4 * hidden * hidden * 2, False, "W_leaf")
+    W_comp = add(5 * 2 * hidden * hidden * 2, False, "W_comp")
+    gW_leaf = add(4 * hidden * hidden * 2, False, "gW_leaf")
+    gW_comp = add(5 * 2 * hidden * hidden * 2, False, "gW_comp")
+    pool = add(hb, True, "pool")
+    dpool = add(hb, True, "dpool")
+    loss = add(256, True, "loss")
+    max_nodes = 2 * max_leaves - 1
+    S = max_nodes + 2                                   # per-sample slots: 2 pads + nodes
+    h0 = len(tensors)
+    for b in range(batch):
+        for k in range(S):
+            add(hb, True, f"h[{b},{k - 2}]")
+    c0 = len(tensors)
+    for b in range(batch):
+        for k in range(S):
+            add(hb, True, f"c[{b},{k - 2}]")
+    g0 = len(tensors)
+    for b in range(batch):
+        for k in range(S):
+            add(gb, True, f"g[{b},{k - 2}]")
+    x0 = len(tensors)
+    for b in range(batch):
+        for k in range(S):
+            add(hb, False, f"x[{b},{k - 2}]")
+
+    def acc(*a):
+        return tuple(sorted(a, key=lambda e: e[0]))
+
+    Hd = hidden
+    leaf_sig = (0, 1, 0, 2, 4, 0)
+    comp_sig = (1, 0, 0, 3, 6, 0)
+    norm_sig = (0, 0, 1, 1, 2, 1)
+    bwd_sig = (1, 0, 0, 4, 8, 0)
+
+    def node(base, d):                                  # (tensor, mode, stride_k, stride_b) of slot k + d
+        return (base + 2 + d, None, 1, S)
+
+    def A_(base, d, m):
+        t, _, sk, sbb = node(base, d)
+        return (t, m, sk, sbb)
+
+    leaf_arm = [Op(leaf_sig, ((1, Hd), (Hd, 4 * Hd)),
+                   acc((W_leaf, R, 0, 0), (pool, RW, 0, 0), A_(h0, 0, W), A_(c0, 0, W), A_(g0, 0, W), A_(x0, 0, R)),
+                   "leaf")]
+    int_arm = [Op(comp_sig, ((1, 2 * Hd), (2 * Hd, 5 * Hd)),
+                  acc((W_comp, R, 0, 0), A_(h0, -2, R), A_(h0, -1, R), A_(h0, 0, W), A_(c0, -2, R), A_(c0, -1, R),
+                      A_(c0, 0, W), A_(g0, 0, W)), "compose"),
+               Op(norm_sig, ((1, Hd),), acc((pool, RW, 0, 0), A_(h0, 0, RW), A_(g0, 0, RW)), "norm")]
+    bwd_body = [Op(bwd_sig, ((1, Hd), (Hd, 5 * Hd)),
+                   acc((W_leaf, R, 0, 0), (W_comp, R, 0, 0), (gW_leaf, RW, 0, 0), (gW_comp, RW, 0, 0),
+                       (dpool, R, 0, 0), A_(h0, 0, R), A_(c0, 0, R), A_(g0, 0, R), A_(x0, 0, R)), "node_bwd")]
+    embed = Op((0, 1, 0, 0, 1, 0), ((max_nodes, Hd),), (), "embed")
+    loss_op = Op((0, 0, 0, 1, 2, 0), ((1, Hd),), acc((pool, R, 0, 0), (loss, W, 0, 0), (dpool, W, 0, 0)), "loss")
+    opt = Op((0, 0, 0, 0, 3, 0), ((4 * Hd, 2 * Hd),) * 2,
+             acc((W_leaf, RW, 0, 0), (W_comp, RW, 0, 0), (gW_leaf, RW, 0, 0), (gW_comp, RW, 0, 0)), "optimizer")
+    lo, hi = 2 * min_leaves - 1, max_nodes
+    program = [embed,
+               Loop([If([leaf_arm, int_arm])], lo, hi),
+               loss_op,
+               Loop(bwd_body, lo, hi, tie=0, rev=True),
+               opt]
+    sizes = [t[0] for t in tensors]
+    offs, _ = _host_layout(sizes, 256)
+    tens = [Tensor(t[0], offs[i], t[1], t[2]) for i, t in enumerate(tensors)]
+    # samples: trees, descriptors [N, leaves per forward group, internals per forward group,
+    # nodes per backward group]
+    bg = K_max - fwd_groups
+    D_s = 1 + 2 * fwd_groups + bg
+    trees, rows = [], []
+    for _ in range(n_samples):
+        n = int(rng.integers(min_leaves, max_leaves + 1))
+        ty = _random_tree_postorder(rng, n)
+        N = len(ty)
+        fw = [(g * N // fwd_groups, (g + 1) * N // fwd_groups) for g in range(fwd_groups)]
+        leaves = [sum(1 for k in range(a, b) if ty[k] == 0) for a, b in fw]
+        ints = [(b - a) - l for (a, b), l in zip(fw, leaves)]
+        bw = [((g + 1) * N // bg) - (g * N // bg) for g in range(bg)]
+        trees.append(ty)
+        rows.append([N] + leaves + ints + bw)
+    samples = np.asarray(rows, np.int64)
+    S_max, h = 16, 2
+    program_sites = n_branch_logits(program)
+    pilot = make_pilot(rng, pilot_kind, S_max, D_s, h, K_max, program_sites,
+                       xs_mean=[float(v) for v in samples.mean(axis=0)])
+    _plant_tree_heads(pilot, K_max, fwd_groups, lo, hi, D_s,
+                      {"embed": embed, "leaf": leaf_arm, "int": int_arm, "loss": loss_op, "bwd": bwd_body, "opt": opt})
+    return Workload("tree", LSTM, program, tens, S_max, D_s, h, K_max,
+                    budget=budget, align=256, policy=1, pilot=pilot, samples=samples,
+                    hist_ids=np.array([-2, -1], np.int32), seed=seed,
+                    notes={"batch": batch, "trees": trees, "fwd_groups": fwd_groups, "oracle_batch": 2})
+
+
+def _sig9(op):
+    """Operator signature bookkeeping for the planted head (Fig. 3 form: idioms ++ dimension
+    sums of the inputs) - input construction of the stand-in pilot, recomputed by neither side."""
+    dims = [sum(s[k] for s in op.inputs if len(s) > k) for k in range(3)]
+    return list(op.idioms) + dims
+
+
+def _plant_tree_heads(pilot, K_max, fwd_groups, lo, hi, D_s, ops):
+    """Pass-through units 0..D_s-1 carry the descriptors (feature units desc x 2^-10) through
+    every layer; the block head of slot g is the exact linear function of them (coefficients
+    x 2^(10 - sigma), R4 scaling) and the trip logits (2tN - t^2)/2048 (see make_tree)."""
+    w = pilot.weights
+    f0 = w["feat0.W"]
+    for i in range(D_s):
+        f0[i, :] = 0.0
+        f0[i, i] = 1.0
+        w["feat0.b"][i] = 0.0
+    for k in range(3):
+        for l in range(len(pilot.mlp)):
+            Wl = w[f"mlp{k}.{l}.W"]
+            for i in range(D_s):
+                Wl[i, :] = 0.0
+                Wl[i, i] = 1.0
+                w[f"mlp{k}.{l}.b"][i] = 0.0
+    Wo, bo = w["out.W"], w["out.b"]
+    Wo[: 10 * K_max, :] = 0.0
+    bo[: 10 * K_max] = 0.0
+    sg = {k: [_sig9(o) for o in v] if isinstance(v, list) else _sig9(v) for k, v in ops.items()}
+    leaf_v = [3] + sg["leaf"][0]                     # Z (loop test) + Z (If) + the leaf op
+    int_v = [4] + [a + b for a, b in zip(sg["int"][0], sg["int"][1])]
+    bwd_v = [2] + sg["bwd"][0]                       # Z + the backward op
+    bg = K_max - fwd_groups
+
+    def put(slot, unit, vec):
+        for e in range(10):
+            sigma = 4 if e < 7 else 10
+            Wo[10 * slot + e, unit] += np.float32(vec[e] * 2.0 ** (10 - sigma))
+
+    def bias(slot, vec):
+        for e in range(10):
+            sigma = 4 if e < 7 else 10
+            bo[10 * slot + e] += np.float32(vec[e] / 2.0 ** sigma)
+    for g in range(fwd_groups):
+        put(g, 1 + g, leaf_v)
+        put(g, 1 + fwd_groups + g, int_v)
+    bias(0, [1] + sg["embed"])
+    bias(fwd_groups - 1, [2] + sg["loss"])           # the loop's exit test + the loss op
+    for g in range(bg):
+        put(fwd_groups + g, 1 + 2 * fwd_groups + g, bwd_v)
+    bias(K_max - 1, [2] + sg["opt"])                 # the backward loop's exit test + optimizer
+    off = 10 * K_max
+    for t in range(lo, hi + 1):                      # Loop F trip-count logits
+        Wo[off, :] = 0.0
+        Wo[off, 0] = np.float32(t)
+        bo[off] = np.float32(-t * t / 2048.0)
+        off += 1
+
+
+CONFIGS = {"tiny": make_tiny, "moe": make_moe, "af": make_af, "lstm": make_lstm, "tree": make_tree}
 
 
 def make(name, seed=0, **kw):

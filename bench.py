@@ -264,6 +264,12 @@ def pilot_latency(torch, wl, dev, desc_dev, hist64, nS, s0):
             s0.synchronize()
             ss.append((time.perf_counter() - t0) * 1e6)
         out["single_shot_us"] = round(float(np.median(ss[5:])), 2)
+        if g1.query("host_decode"):
+            # the decode of this arch runs on the host (nested sites, R16): one stream sync per
+            # predict, so there is no graph to replay
+            out["note"] = "host-side decode (nested sites, R16): single-shot only, no graph replay"
+            g1.close()
+            return out
         cs = torch.cuda.Stream()
         for _ in range(3):
             g1.predict(desc_dev[:1], h1, 1, stream=cs.cuda_stream)

@@ -2155,6 +2155,7 @@ dyo_status dyo_query(dyo_ctx* ctx, int32_t what, int64_t* value) {
     case DYO_Q_PILOT_KERNEL: *value = ctx->last_tc; return DYO_OK;
     case DYO_Q_DECODE_FUSED: *value = ctx->last_fused; return DYO_OK;
     case DYO_Q_PLAN_SYNCS: *value = ctx->last_plan_syncs; return DYO_OK;
+    case DYO_Q_HOST_DECODE: *value = (!ctx->branch_head || ctx->nested) ? 1 : 0; return DYO_OK;
   }
   return DYO_E_INVAL;
 }

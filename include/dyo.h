@@ -294,6 +294,39 @@ dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** 
 dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half_free,
                        void* ev_prev_done, void* ev_ready);
 
+/* ---- On-demand fetch of mis-predicted tensors ("checks whether the tensor
+ * is in GPU memory ... migrates the tensors on demand", P:L197 tensor fault handler; DESIGN.md
+ * reading R17) --------------------------------------------------------------------------------
+ * When the pilot mis-predicts, block j (the rows [C_j, C_j+1) of the ACTUAL path, cut at the
+ * predicted counts: the operator counter of P:L178) touches tensors the plan did not make
+ * ready. Before block j runs, the runtime passes the actual accesses that may be missing.
+ * dyo_fault_config: allocates the device fault area (outside B; two halves used by alternate
+ *   blocks); 0 frees it. Synchronises the device.
+ * dyo_fault_fetch: j = the transition last enqueued by dyo_migrate (block j is next to run;
+ *   DYO_E_STATE otherwise - with faults the runtime enqueues transitions one block ahead).
+ *   For each id (modes: 1 read, 2 write, 3 read-write), dev_ptrs[i] (host array) receives:
+ *     - the tensor's planned slot if it is in the planned W_j and that entry is valid for the
+ *       access (read-first in the plan or a write-first access, and a write only where the plan
+ *       writes): the residency check;
+ *     - else a fault-area copy: read-first accesses copy the tensor's latest bytes - from its
+ *       valid device copy after transition j (for a tensor the plan ALLOCs in this transition,
+ *       its copy before it), else from its host home - on `stream`, after transition j's
+ *       migrations; ev_done (may be NULL) is recorded after the copies: block j waits on it.
+ *   Written faulted tensors are written back after block j ends, by the next dyo_migrate
+ *   (after its ev_prev_done): to the host home and to the tensor's valid device copy, before
+ *   that transition's EVICT and carries. The plan's residency is never changed, so plans
+ *   computed ahead stay valid. DYO_E_CAPACITY if a block's faults exceed half the area.
+ * dyo_fault_stats: faults served from the fault area, their bytes copied in, and accesses
+ *   found resident (any pointer may be NULL). */
+dyo_status dyo_fault_config(dyo_ctx* ctx, int64_t area_bytes);
+dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const int32_t* modes, int32_t n,
+                           void** dev_ptrs, void* stream, void* ev_done);
+dyo_status dyo_fault_stats(dyo_ctx* ctx, int64_t* faults, int64_t* bytes, int64_t* resident);
+/* Enqueues the pending write-backs of the last block's written faulted tensors on `stream`
+ * after ev_block_end (may be NULL) - what the next dyo_migrate would do; for the last block of
+ * a run. No-op without pending write-backs. */
+dyo_status dyo_fault_flush(dyo_ctx* ctx, void* stream, void* ev_block_end);
+
 /* Device address of tensor t after the last planned transition that placed it (NULL if it is
  * on the host). Valid until the next dyo_migrate that moves it. */
 dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr);

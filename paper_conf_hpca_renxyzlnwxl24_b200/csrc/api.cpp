@@ -116,6 +116,21 @@ struct dyo_ctx {
   int8_t* h_loc = nullptr;         // pinned mirrors of the committed residency
   int64_t* h_off = nullptr;
 
+  // on-demand fetch of mis-predicted tensors (reading R17)
+  char* fault_area = nullptr;
+  int64_t fault_cap = 0, fault_used = 0;
+  int fault_j = -1;                          // block whose faults occupy the area
+  struct FaultWb { int32_t t; char* src; };
+  std::vector<FaultWb> fault_wb;             // written faulted tensors of the last block
+  cudaEvent_t ev_fault_wb = nullptr;
+  int64_t n_faults = 0, fault_bytes = 0, n_fault_resident = 0;
+  // host replay of the residency after every migrated transition (FIFO over plans)
+  std::vector<int8_t> mig_loc;
+  std::vector<int64_t> mig_off;
+  std::vector<std::pair<int32_t, std::pair<int8_t, int64_t>>> mig_prev_alloc;   // ALLOC'd in the last transition
+  PlanSlot* last_mig_slot = nullptr;
+  int last_mig_j = -1;
+  int64_t last_mig_seq = -1;
   // migration
   cudaStream_t d2h = nullptr;      // ctx-owned stream for the EVICT (D2H) phase
   cudaStream_t side = nullptr;     // ctx-owned stream for early CARRY (overlaps FETCH)
@@ -645,6 +660,7 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_pred, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_memo, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_fault_wb, cudaEventDisableTiming);
   if (e != cudaSuccess) {
     dyo_destroy(ctx);
     return e == cudaErrorMemoryAllocation ? DYO_E_NOMEM : DYO_E_CUDA;
@@ -691,6 +707,8 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->aux) cudaStreamDestroy(ctx->aux);
   if (ctx->ev_pred) cudaEventDestroy(ctx->ev_pred);
   if (ctx->ev_memo) cudaEventDestroy(ctx->ev_memo);
+  if (ctx->ev_fault_wb) cudaEventDestroy(ctx->ev_fault_wb);
+  if (ctx->fault_area) cudaFree(ctx->fault_area);
   if (ctx->h_rep) cudaFreeHost(ctx->h_rep);
   if (ctx->h_memo_stage) cudaFreeHost(ctx->h_memo_stage);
   for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
@@ -869,6 +887,14 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
     P.ev_pending = false;
   }
   ctx->plan_seq = ctx->mig_seq = 0;
+  ctx->mig_loc.assign(T, -1);            // every tensor starts on the host
+  ctx->mig_off.assign(T, 0);
+  ctx->mig_prev_alloc.clear();
+  ctx->last_mig_slot = nullptr;
+  ctx->last_mig_j = -1;
+  ctx->fault_wb.clear();
+  ctx->fault_j = -1;
+  ctx->n_faults = ctx->fault_bytes = ctx->n_fault_resident = 0;
 #undef DA
   // ---- host pool (pinned, mapped: DMA and zero-copy kernels) ----
   ctx->host_bytes = pool;
@@ -1613,6 +1639,23 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
   PlanState& in = ctx->state[ctx->committed];
   PlanState& wk = ctx->state[1 - ctx->committed];
   {
+    // DYO_FAULT=drop_prefetch:p[:seed] - fault injection: read-first entries of the prediction
+    // dropped before planning (the runtime's accesses then fault them in, R17)
+    static int parsed = 0;
+    static double drop_p = 0.0;
+    static unsigned long long drop_seed = 0;
+    if (!parsed) {
+      parsed = 1;
+      if (const char* e = getenv("DYO_FAULT"))
+        if (strncmp(e, "drop_prefetch:", 14) == 0) {
+          char* q = nullptr;
+          drop_p = strtod(e + 14, &q);
+          if (q && *q == ':') drop_seed = strtoull(q + 1, nullptr, 10);
+        }
+    }
+    if (drop_p > 0.0) CK(launch_fault_drop(ctx->ad, ctx->pd, b0, n, drop_p, drop_seed, st));
+  }
+  {
     TScope ts(ctx, 2, st);
     CK(launch_plan(ctx->ad, ctx->pd, b0, n, ctx->cfg.policy, in, wk, ctx->sc, P.dout, ctx->max_groups, st));
   }
@@ -1827,6 +1870,21 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   } else {
     CK(cudaEventRecord(ctx->ev_entry, s));
     CK(cudaStreamWaitEvent(sd, ctx->ev_entry, 0));
+  }
+  // 0. write-backs of the faulted tensors block j-1 wrote (R17): after block j-1 ends, the
+  //    fault area's bytes go to the tensor's host home and to its valid device copy; this
+  //    transition's EVICT (D2H stream) and carries (after ev_moves) are ordered after them
+  if (!ctx->fault_wb.empty()) {
+    if (ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
+    for (const auto& w : ctx->fault_wb) {
+      const int64_t nb = ctx->t_bytes[w.t];
+      CK(cudaMemcpyAsync(host + ctx->t_host[w.t], w.src, nb, cudaMemcpyDeviceToHost, s));
+      if (ctx->mig_loc[w.t] >= 0)
+        CK(cudaMemcpyAsync(arena + ctx->mig_loc[w.t] * ctx->H + ctx->mig_off[w.t], w.src, nb, cudaMemcpyDeviceToDevice, s));
+    }
+    ctx->fault_wb.clear();
+    CK(cudaEventRecord(ctx->ev_fault_wb, s));
+    CK(cudaStreamWaitEvent(sd, ctx->ev_fault_wb, 0));
   }
   const int64_t stage_half = ctx->staging_bytes / 2 / 256 * 256;
   char* stage_pack = ctx->staging;                 // D2H stream
@@ -2045,8 +2103,134 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   TRACE("  transition %d issued", j);
   if (ev_ready) CK(cudaEventRecord((cudaEvent_t)ev_ready, s));
   CK(cudaEventRecord(P.ev_last, s));
+  // host replay of the residency after transition j (the fault path's residency check, R17)
+  {
+    const int m = h.half;
+    const int64_t mb = (int64_t)m * ctx->H;
+    ctx->mig_prev_alloc.clear();
+    for (int i = 0; i < h.n_evict; ++i) ctx->mig_loc[P.out.ev[h.o_evict + i].t] = -1;
+    for (int i = 0; i < h.n_move; ++i) ctx->mig_off[P.out.mv[h.o_move + i].t] = P.out.mv[h.o_move + i].dst - mb;
+    for (int i = 0; i < h.n_carry; ++i) {
+      const auto& r = P.out.ca[h.o_carry + i];
+      ctx->mig_loc[r.t] = (int8_t)m; ctx->mig_off[r.t] = r.dst - mb;
+    }
+    for (int i = 0; i < h.n_alloc; ++i) {
+      const auto& r = P.out.al[h.o_alloc + i];
+      ctx->mig_prev_alloc.push_back({(int32_t)r.t, {ctx->mig_loc[r.t], ctx->mig_off[r.t]}});
+      ctx->mig_loc[r.t] = (int8_t)m; ctx->mig_off[r.t] = r.dst - mb;
+    }
+    for (int i = 0; i < h.n_fetch; ++i) {
+      const auto& r = P.out.fe[h.o_fetch + i];
+      ctx->mig_loc[r.t] = (int8_t)m; ctx->mig_off[r.t] = r.dst - mb;
+    }
+    ctx->last_mig_slot = &P;
+    ctx->last_mig_j = j;
+    ctx->last_mig_seq = ctx->mig_seq;
+  }
   P.ev_pending = true;
   P.next_j = j + 1;
+  return DYO_OK;
+}
+
+// ---- on-demand fetch of mis-predicted tensors (R17) -------------
+dyo_status dyo_fault_config(dyo_ctx* ctx, int64_t area_bytes) {
+  if (!ctx || area_bytes < 0) return DYO_E_INVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  if (ctx->fault_area) { cudaFree(ctx->fault_area); ctx->fault_area = nullptr; }
+  ctx->fault_cap = ctx->fault_used = 0;
+  ctx->fault_wb.clear();
+  ctx->fault_j = -1;
+  if (area_bytes == 0) return DYO_OK;
+  CK(cudaMalloc(&ctx->fault_area, area_bytes));
+  ctx->fault_cap = area_bytes;
+  return DYO_OK;
+}
+
+dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const int32_t* modes, int32_t n,
+                           void** dev_ptrs, void* stream, void* ev_done) {
+  if (!ctx || (n > 0 && (!ids || !modes || !dev_ptrs)) || n < 0) return DYO_E_INVAL;
+  if (!ctx->fault_area) return fail(ctx, DYO_E_STATE, "dyo_fault_config first");
+  dyo_ctx::PlanSlot* P = ctx->last_mig_slot;
+  if (!P || j != ctx->last_mig_j || !P->valid || ctx->last_mig_seq != ctx->mig_seq)
+    return fail(ctx, DYO_E_STATE, "block %d is not the last migrated transition", j);
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t s = (cudaStream_t)stream;
+  const PlanHdr& h = P->out.hdr[j];
+  // the planned W_j with its placement (entry records of transition j, host copy)
+  std::vector<dyo_entry_rec> ent(h.n_ent);
+  if (h.n_ent) CK(cudaMemcpy(ent.data(), P->dout.ent + h.o_ent, sizeof(dyo_entry_rec) * h.n_ent, cudaMemcpyDeviceToHost));
+  if (ctx->fault_j != j) { ctx->fault_used = 0; ctx->fault_j = j; }
+  // copies after transition j's migrations (stream order with the ctx's last migrate)
+  CK(cudaStreamWaitEvent(s, P->ev_last, 0));
+  const int64_t AL = ctx->cfg.align;
+  for (int i = 0; i < n; ++i) {
+    const int t = ids[i], md = modes[i];
+    if (t < 0 || t >= ctx->T || md < 1 || md > 3) return fail(ctx, DYO_E_INVAL, "fault %d: tensor %d mode %d", i, t, md);
+    const dyo_entry_rec* e = nullptr;
+    for (const auto& r : ent)
+      if (r.t == t) { e = &r; break; }
+    // residency check: planned and valid for this access -> its slot. Valid: the
+    // plan fetched it (or the access writes first), and a write is one the plan knows about
+    // (a write the plan does not expect would leave a device copy it treats as clean)
+    if (e && (e->needs_fetch || !(md & 1)) && (!(md & 2) || (e->mode & 2))) {
+      dev_ptrs[i] = ctx->arena + e->dst;
+      ++ctx->n_fault_resident;
+      continue;
+    }
+    // miss: a fault-area copy from the tensor's latest bytes - its valid device copy after
+    // transition j (or, for a tensor the plan ALLOCs in this transition, its copy before it),
+    // else its host home
+    // the area's halves alternate between blocks: block j's half is still read by block j and
+    // by the write-backs migrate(j+1) enqueues; block j+2 reuses it after its EVICT waited for
+    // block j's end
+    const int64_t nb = ctx->t_bytes[t], ab = align_up(nb, AL);
+    const int64_t half = ctx->fault_cap / 2 / AL * AL;
+    if (ctx->fault_used + ab > half)
+      return fail(ctx, DYO_E_CAPACITY, "fault area: need %lld bytes per block", (long long)(ctx->fault_used + ab));
+    char* dst = ctx->fault_area + (j & 1) * half + ctx->fault_used;
+    ctx->fault_used += ab;
+    int8_t loc = ctx->mig_loc[t];
+    int64_t off = ctx->mig_off[t];
+    if (e) {
+      loc = -1;
+      for (const auto& pa : ctx->mig_prev_alloc)
+        if (pa.first == t) { loc = pa.second.first; off = pa.second.second; }
+    }
+    if (md & 1) {
+      if (loc >= 0) CK(cudaMemcpyAsync(dst, ctx->arena + loc * ctx->H + off, nb, cudaMemcpyDeviceToDevice, s));
+      else CK(cudaMemcpyAsync(dst, ctx->host_pool + ctx->t_host[t], nb, cudaMemcpyHostToDevice, s));
+      ctx->fault_bytes += nb;
+    }
+    if (md & 2) ctx->fault_wb.push_back({t, dst});
+    dev_ptrs[i] = dst;
+    ++ctx->n_faults;
+  }
+  if (ev_done) CK(cudaEventRecord((cudaEvent_t)ev_done, s));
+  return DYO_OK;
+}
+
+dyo_status dyo_fault_flush(dyo_ctx* ctx, void* stream, void* ev_block_end) {
+  if (!ctx) return DYO_E_INVAL;
+  if (ctx->fault_wb.empty()) return DYO_OK;
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t s = (cudaStream_t)stream;
+  if (ev_block_end) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_block_end, 0));
+  for (const auto& w : ctx->fault_wb) {
+    const int64_t nb = ctx->t_bytes[w.t];
+    CK(cudaMemcpyAsync(ctx->host_pool + ctx->t_host[w.t], w.src, nb, cudaMemcpyDeviceToHost, s));
+    if (ctx->mig_loc[w.t] >= 0)
+      CK(cudaMemcpyAsync(ctx->arena + ctx->mig_loc[w.t] * ctx->H + ctx->mig_off[w.t], w.src, nb, cudaMemcpyDeviceToDevice, s));
+  }
+  ctx->fault_wb.clear();
+  return DYO_OK;
+}
+
+dyo_status dyo_fault_stats(dyo_ctx* ctx, int64_t* faults, int64_t* bytes, int64_t* resident) {
+  if (!ctx) return DYO_E_INVAL;
+  if (faults) *faults = ctx->n_faults;
+  if (bytes) *bytes = ctx->fault_bytes;
+  if (resident) *resident = ctx->n_fault_resident;
   return DYO_OK;
 }
 

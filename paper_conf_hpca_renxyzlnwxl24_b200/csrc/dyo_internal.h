@@ -267,6 +267,8 @@ cudaError_t plan_debug_stamps(int j, unsigned long long* out);
 // device arrays (d) into the pinned mapped mirrors (h: device-side aliases) by the counts in
 // d.counts; nothing when d.status[0] != 0. Entry records are not copied.
 cudaError_t launch_plan_export(const PlanOut& d, const PlanOut& h, cudaStream_t s);
+cudaError_t launch_fault_drop(const ArchDev& a, const PredDev& pd, int b0, int nb, double p, uint64_t seed,
+                              cudaStream_t s);
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,
                           int32_t* hist_tab_out, int32_t* hist_K_out, cudaStream_t s);
 cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int policy,

@@ -1143,6 +1143,53 @@ cudaError_t plan_debug_stamps(int j, unsigned long long* out) {
   return e;
 }
 
+// ---- fault injection (DYO_FAULT=drop_prefetch:p[:seed], R17 tests and measurement) ------
+// Drops every read-first entry of the predictions' tensor sets whose splitmix64 hash of
+// (seed, b, k, t) is below lim (workloads.drop_prefetch is the test side's twin), keeping the
+// others in order: the plan then misses those tensors and the runtime faults them in.
+__device__ __forceinline__ uint64_t drop_hash(uint64_t seed, uint64_t b, uint64_t k, uint64_t t) {
+  uint64_t z = seed * 0x9E3779B97F4A7C15ull + (b << 40) + (k << 20) + t;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+__global__ void fault_drop_kernel(ArchDev a, PredDev pd, int b0, int nb, uint64_t lim, int all, uint64_t seed) {
+  __shared__ int warp_tmp[32];
+  for (int item = blockIdx.x; item < nb * a.K_max; item += gridDim.x) {
+    const int b = b0 + item / a.K_max, k = item % a.K_max;
+    if (k >= pd.K[b]) continue;
+    int2* ent = pd.ent + ((int64_t)b * a.K_max + k) * kEntCap;
+    const int n = pd.ent_n[(int64_t)b * a.K_max + k];
+    int base = 0;
+    for (int i0 = 0; i0 < n; i0 += blockDim.x) {
+      const int i = i0 + threadIdx.x;
+      int2 e = make_int2(0, 0);
+      int keep = 0;
+      if (i < n) {
+        e = ent[i];
+        const bool rd = (e.y >> 2) & 1;
+        keep = !(rd && (all || drop_hash(seed, (uint64_t)b, (uint64_t)k, (uint64_t)e.x) < lim));
+      }
+      int tot = 0;
+      const int p = block_scan(keep, warp_tmp, &tot);   // barriers: every read precedes the writes
+      if (keep) ent[base + p] = e;
+      base += tot;
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) pd.ent_n[(int64_t)b * a.K_max + k] = base;
+    __syncthreads();
+  }
+}
+
+cudaError_t launch_fault_drop(const ArchDev& a, const PredDev& pd, int b0, int nb, double p, uint64_t seed,
+                              cudaStream_t s) {
+  const int all = p >= 1.0 ? 1 : 0;
+  const uint64_t lim = all ? 0 : (uint64_t)(p * 18446744073709551616.0);
+  fault_drop_kernel<<<148, 256, 0, s>>>(a, pd, b0, nb, lim, all, seed);
+  return cudaGetLastError();
+}
+
 // 8-byte words of the record arrays, grid-stride over all six lists
 __global__ void plan_export_kernel(PlanOut d, PlanOut h) {
   if (d.status[0] != 0) return;

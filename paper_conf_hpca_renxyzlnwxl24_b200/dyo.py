@@ -98,7 +98,8 @@ def lib():
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
                      "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
                      "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats",
-                     "dyo_debug_copy_stamps", "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check"):
+                     "dyo_debug_copy_stamps", "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check",
+                     "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -110,7 +111,8 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
            "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
            "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps",
-           "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check")
+           "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check",
+           "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush")
 
 
 def _a(x, dt):
@@ -383,6 +385,28 @@ class Dyo:
     def migrate(self, j, stream=0, ev_half_free=None, ev_prev_done=None, ev_ready=None):
         """ev_*: cudaEvent_t handles (torch.cuda.Event.cuda_event) or None."""
         self._check(self.L.dyo_migrate(self.ctx, j, P(stream), P(ev_half_free), P(ev_prev_done), P(ev_ready)))
+
+    # ---- on-demand fetch of mis-predicted tensors (P:L184, L197; R17) ----
+    def fault_config(self, area_bytes):
+        self._check(self.L.dyo_fault_config(self.ctx, i64(area_bytes)))
+
+    def fault_fetch(self, j, ids, modes, stream=0, ev_done=None):
+        """Device addresses for block j's (possibly) missing accesses (list of ints)."""
+        ids_a = _a(ids, np.int32)
+        md = _a(modes, np.int32)
+        n = len(ids_a)
+        ptrs = (P * max(n, 1))()
+        self._check(self.L.dyo_fault_fetch(self.ctx, int(j), _p(ids_a, i32), _p(md, i32), n, ptrs, P(stream),
+                                           P(ev_done)))
+        return [ptrs[i] for i in range(n)]
+
+    def fault_flush(self, stream=0, ev_block_end=None):
+        self._check(self.L.dyo_fault_flush(self.ctx, P(stream), P(ev_block_end)))
+
+    def fault_stats(self):
+        f, b, r = i64(), i64(), i64()
+        self._check(self.L.dyo_fault_stats(self.ctx, C.byref(f), C.byref(b), C.byref(r)))
+        return {"faults": f.value, "bytes": b.value, "resident": r.value}
 
     def residency(self, t):
         p = P()

@@ -17,9 +17,10 @@ def make_ctx(wl, max_batch=1, flags=0, policy=None, **kw):
     return d
 
 
-def oracle_step(wl, sample_ids, state, table, policy=None, plan=True):
+def oracle_step(wl, sample_ids, state, table, policy=None, plan=True, drop=None):
     """Oracle for a batch of samples planned together (sample order); plan=False stops after
-    the decode."""
+    the decode. drop = (p, seed): the planned tensor sets lose their read-first entries chosen by
+    workloads.drop_prefetch (the DYO_FAULT injection); r["Ws"] holds the planned sets."""
     preds, feats, logits = [], [], []
     for b, s in enumerate(sample_ids):
         x = E.encode(wl, wl.samples[s], wl.hist_ids, table)
@@ -27,16 +28,19 @@ def oracle_step(wl, sample_ids, state, table, policy=None, plan=True):
         feats.append(x)
         logits.append(y)
         preds.append(D.decode(wl, y, branch_head=wl.notes.get("branch_head", True), b=b))
-    Ws = [Wj for p in preds for Wj in p.W]
+    if drop is not None:
+        Ws = [Wj for b, p in enumerate(preds) for Wj in WL.drop_prefetch(p.W, drop[0], drop[1], b)]
+    else:
+        Ws = [Wj for p in preds for Wj in p.W]
     new_table = [b for p in preds for b in p.blocks]
     if not plan:
-        return dict(feats=feats, logits=logits, preds=preds, trs=[], state=state, table=new_table, err=None)
+        return dict(feats=feats, logits=logits, preds=preds, trs=[], state=state, table=new_table, err=None, Ws=Ws)
     try:
         trs, st = PL.plan(state, wl, Ws, policy)
         err = None
     except PL.BudgetError as e:
         trs, st, err = [], state, e
-    return dict(feats=feats, logits=logits, preds=preds, trs=trs, state=st, table=new_table, err=err)
+    return dict(feats=feats, logits=logits, preds=preds, trs=trs, state=st, table=new_table, err=err, Ws=Ws)
 
 
 def hist_for(wl, B):

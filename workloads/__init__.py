@@ -876,6 +876,27 @@ def make(name, seed=0, **kw):
 
 
 # ----------------------------------------------------------------------------
+# fault injection (DYO_FAULT=drop_prefetch:p): a counter-based drop decision, implemented here
+# for the test side and independently in libdyo (api.cpp drop_hash)
+# ----------------------------------------------------------------------------
+
+def drop_hash(seed, b, k, t):
+    """splitmix64 of (seed, prediction b, group slot k, tensor t) -> uint64."""
+    M = (1 << 64) - 1
+    z = (int(seed) * 0x9E3779B97F4A7C15 + (int(b) << 40) + (int(k) << 20) + int(t)) & M
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M
+    return z ^ (z >> 31)
+
+
+def drop_prefetch(W, p, seed, b):
+    """The predicted tensor sets of prediction b with every read-first entry dropped when
+    drop_hash(seed, b, k, t) / 2^64 < p (the injected 'mis-prediction' of DYO_FAULT)."""
+    lim = int(p * (1 << 64)) if p < 1 else (1 << 64)
+    return [[e for e in Wk if not (e[2] and drop_hash(seed, b, k, e[0]) < lim)] for k, Wk in enumerate(W)]
+
+
+# ----------------------------------------------------------------------------
 # counter-based content generator (migration byte checks; both sides call it)
 # ----------------------------------------------------------------------------
 

@@ -172,7 +172,10 @@ def transition(state, wl, Ws, j, policy, choose=None, occ=None):
     live, dead = [], []
     for t in cands:
         d, e = next_use(Ws, t, j, occ)
-        is_dead = (e is None and wl.tensors[t].transient) or (e is not None and not e[2])
+        # R9: only a transient tensor can be dead (no later access, or its next access writes it
+        # first); a persistent tensor is never dropped on a predicted overwrite (R17: under a
+        # mis-prediction the overwrite may not happen)
+        is_dead = wl.tensors[t].transient and (e is None or not e[2])
         if is_dead:
             dead.append(t)
         else:

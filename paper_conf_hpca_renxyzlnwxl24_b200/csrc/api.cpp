@@ -123,7 +123,7 @@ struct dyo_ctx {
   struct FaultWb { int32_t t; char* src; };
   std::vector<FaultWb> fault_wb;             // written faulted tensors of the last block
   cudaEvent_t ev_fault_wb = nullptr;
-  int64_t n_faults = 0, fault_bytes = 0, n_fault_resident = 0;
+  int64_t n_faults = 0, fault_bytes = 0, n_fault_resident = 0, n_fault_repair = 0;
   // host replay of the residency after every migrated transition (FIFO over plans)
   std::vector<int8_t> mig_loc;
   std::vector<int64_t> mig_off;
@@ -894,7 +894,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   ctx->last_mig_j = -1;
   ctx->fault_wb.clear();
   ctx->fault_j = -1;
-  ctx->n_faults = ctx->fault_bytes = ctx->n_fault_resident = 0;
+  ctx->n_faults = ctx->fault_bytes = ctx->n_fault_resident = ctx->n_fault_repair = 0;
 #undef DA
   // ---- host pool (pinned, mapped: DMA and zero-copy kernels) ----
   ctx->host_bytes = pool;
@@ -2205,6 +2205,25 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
     if (md & 2) ctx->fault_wb.push_back({t, dst});
     dev_ptrs[i] = dst;
     ++ctx->n_faults;
+  }
+  // repair: a tensor the plan expects block j to write first (its slot was not fetched, and the
+  // plan will treat it as dirty) that the actual block does not write through that slot would
+  // later be written back with the slot's stale bytes: its latest bytes are copied into the
+  // slot now (from its previous device copy, else its host home)
+  for (const auto& r : ent) {
+    if (r.needs_fetch) continue;
+    bool written = false;
+    for (int i = 0; i < n && !written; ++i)
+      written = ids[i] == r.t && (modes[i] & 2) && dev_ptrs[i] == ctx->arena + r.dst;
+    if (written) continue;
+    int8_t loc = -1;
+    int64_t off = 0;
+    for (const auto& pa : ctx->mig_prev_alloc)
+      if (pa.first == r.t) { loc = pa.second.first; off = pa.second.second; }
+    const int64_t nb = ctx->t_bytes[r.t];
+    if (loc >= 0) CK(cudaMemcpyAsync(ctx->arena + r.dst, ctx->arena + loc * ctx->H + off, nb, cudaMemcpyDeviceToDevice, s));
+    else CK(cudaMemcpyAsync(ctx->arena + r.dst, ctx->host_pool + ctx->t_host[r.t], nb, cudaMemcpyHostToDevice, s));
+    ++ctx->n_fault_repair;
   }
   if (ev_done) CK(cudaEventRecord((cudaEvent_t)ev_done, s));
   return DYO_OK;

@@ -376,7 +376,8 @@ __device__ __forceinline__ int rec_kind(int4 r, const uint32_t* inw) {
   if (r.z & kRecTomb) return 0;
   const int t = r.z & kRecIdMask;
   if (bit_get(inw, t)) return 1;
-  const bool dead = (r.w < 0 && (r.z & kRecTransient)) || (r.w >= 0 && !(r.z & kRecNxRd));
+  // R9: only a transient tensor can be dead (no later access, or written first next)
+  const bool dead = (r.z & kRecTransient) && (r.w < 0 || !(r.z & kRecNxRd));
   return dead ? 2 : 3;
 }
 

@@ -313,9 +313,9 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
  *       its copy before it), else from its host home - on `stream`, after transition j's
  *       migrations; ev_done (may be NULL) is recorded after the copies: block j waits on it.
  *   `ids` must list every access of the actual block (not only the suspected misses): a tensor
- *   the plan expects block j to write first (slot not fetched, treated as dirty afterwards)
- *   that the actual block does not write through its slot gets its latest bytes copied into
- *   that slot (the repair), so no later write-back publishes stale bytes.
+ *   the plan ALLOCs at transition j (slot not filled, treated as dirty afterwards) that the
+ *   actual block does not write through its slot gets its latest bytes copied into that slot
+ *   (the repair), so no later write-back publishes stale bytes.
  *   Written faulted tensors are written back after block j ends, by the next dyo_migrate
  *   (after its ev_prev_done): to the host home and to the tensor's valid device copy, before
  *   that transition's EVICT and carries. The plan's residency is never changed, so plans

@@ -2192,11 +2192,8 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
     ctx->fault_used += ab;
     int8_t loc = ctx->mig_loc[t];
     int64_t off = ctx->mig_off[t];
-    if (e) {
-      loc = -1;
-      for (const auto& pa : ctx->mig_prev_alloc)
-        if (pa.first == t) { loc = pa.second.first; off = pa.second.second; }
-    }
+    for (const auto& pa : ctx->mig_prev_alloc)       // ALLOC'd at j: its slot holds no bytes yet
+      if (pa.first == t) { loc = pa.second.first; off = pa.second.second; }
     if (md & 1) {
       if (loc >= 0) CK(cudaMemcpyAsync(dst, ctx->arena + loc * ctx->H + off, nb, cudaMemcpyDeviceToDevice, s));
       else CK(cudaMemcpyAsync(dst, ctx->host_pool + ctx->t_host[t], nb, cudaMemcpyHostToDevice, s));
@@ -2206,23 +2203,24 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
     dev_ptrs[i] = dst;
     ++ctx->n_faults;
   }
-  // repair: a tensor the plan expects block j to write first (its slot was not fetched, and the
-  // plan will treat it as dirty) that the actual block does not write through that slot would
-  // later be written back with the slot's stale bytes: its latest bytes are copied into the
-  // slot now (from its previous device copy, else its host home)
-  for (const auto& r : ent) {
-    if (r.needs_fetch) continue;
+  // repair: a tensor the plan ALLOCs at transition j (its slot holds no bytes; the plan expects
+  // block j to write it and treats it as dirty afterwards) that the actual block does not write
+  // through that slot would later be written back with the slot's stale bytes: its latest bytes
+  // are copied into the slot now (from its previous device copy, else its host home)
+  for (const auto& pa : ctx->mig_prev_alloc) {
+    const int t = pa.first;
+    const dyo_entry_rec* e = nullptr;
+    for (const auto& r : ent)
+      if (r.t == t) { e = &r; break; }
+    if (!e) continue;
     bool written = false;
     for (int i = 0; i < n && !written; ++i)
-      written = ids[i] == r.t && (modes[i] & 2) && dev_ptrs[i] == ctx->arena + r.dst;
+      written = ids[i] == t && (modes[i] & 2) && dev_ptrs[i] == ctx->arena + e->dst;
     if (written) continue;
-    int8_t loc = -1;
-    int64_t off = 0;
-    for (const auto& pa : ctx->mig_prev_alloc)
-      if (pa.first == r.t) { loc = pa.second.first; off = pa.second.second; }
-    const int64_t nb = ctx->t_bytes[r.t];
-    if (loc >= 0) CK(cudaMemcpyAsync(ctx->arena + r.dst, ctx->arena + loc * ctx->H + off, nb, cudaMemcpyDeviceToDevice, s));
-    else CK(cudaMemcpyAsync(ctx->arena + r.dst, ctx->host_pool + ctx->t_host[r.t], nb, cudaMemcpyHostToDevice, s));
+    const int8_t loc = pa.second.first;
+    const int64_t off = pa.second.second, nb = ctx->t_bytes[t];
+    if (loc >= 0) CK(cudaMemcpyAsync(ctx->arena + e->dst, ctx->arena + loc * ctx->H + off, nb, cudaMemcpyDeviceToDevice, s));
+    else CK(cudaMemcpyAsync(ctx->arena + e->dst, ctx->host_pool + ctx->t_host[t], nb, cudaMemcpyHostToDevice, s));
     ++ctx->n_fault_repair;
   }
   if (ev_done) CK(cudaEventRecord((cudaEvent_t)ev_done, s));

@@ -56,6 +56,7 @@ def run_faults(wl, steps, policy=1, drop=None, mispredict=False, area=256 << 20)
     table = ()
     ver = [0] * len(wl.tensors)
     n_fault = n_slot = 0
+    hist = {}                                     # diagnostics: tensor -> [(step, block, kind, mode, planned)]
     for s in range(steps):
         smp = s % len(wl.samples)
         r = oracle_step(wl, [smp], st, table, policy, drop=drop)
@@ -77,6 +78,12 @@ def run_faults(wl, steps, policy=1, drop=None, mispredict=False, area=256 << 20)
             cls = F.classify(r["Ws"][j], Aj)
             ptrs = d.fault_fetch(j, [t for t, _, _ in cls], [m for _, m, _ in cls], stream.cuda_stream)
             planned = {int(e[0]): int(e[3]) for e in d.plan_records(j, "entries").tolist()}
+            pl = {t: (mm, rd) for t, mm, rd in r["Ws"][j]}
+            for (t, m, kind), p in zip(cls, ptrs):
+                hist.setdefault(t, []).append((s, j, kind, m, pl.get(t)))
+            for t, mm, rd in r["Ws"][j]:
+                if t not in {x for x, _, _ in cls}:
+                    hist.setdefault(t, []).append((s, j, "planned-only", mm, rd))
             for (t, m, kind), p in zip(cls, ptrs):
                 if kind == "slot":
                     assert p == base + planned[t], f"step {s} block {j}: tensor {t} not served from its slot"
@@ -103,8 +110,11 @@ def run_faults(wl, steps, policy=1, drop=None, mispredict=False, area=256 << 20)
         if ten.transient:
             continue
         if st.loc[t] != PL.HOST:
-            assert torch.equal(_view(base + st.loc[t] * H + st.off[t], ten.nbytes), _words(t, ver[t], ten.nbytes)), \
-                f"resident copy of {t}"
+            got = _view(base + st.loc[t] * H + st.off[t], ten.nbytes)
+            if not torch.equal(got, _words(t, ver[t], ten.nbytes)):
+                have = [v for v in range(ver[t] + 1) if torch.equal(got, _words(t, v, ten.nbytes))]
+                raise AssertionError(f"resident copy of {t} ({ten.name}): has version {have}, latest {ver[t]}; "
+                                     f"history {hist.get(t)}")
         else:
             assert np.array_equal(pool[ten.host_off: ten.host_off + ten.nbytes], M.content_bytes(t, ver[t], ten.nbytes)), \
                 f"host home of {t}"

@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--budget-gib", type=float, default=0.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-faults", action="store_true", help="skip the on-demand fetch measurement")
     ap.add_argument("--dist-backend", default=None, help="nccl (default with CUDA) or gloo")
     ap.add_argument("--compute", default="auto", choices=["auto", "none", "emulate"],
                     help="emulate the DyNN's per-group compute with spin kernels (auto: on for af)")
@@ -346,6 +347,47 @@ def mispredict_stream(torch, wl, dev, s0, n_distinct=16, repeats=4):
     return out
 
 
+def fault_stream(torch, d, wl, desc_dev, hist_dev, nS, B, s0, s1, steps=4, p_drop=0.05, seed=11):
+    """On-demand fetch (R17) measured with the library's fault injection: each step's read-first
+    entries are dropped from the plan with probability p_drop (dyo_fault_inject), the runtime
+    migrates one block ahead and asks dyo_fault_fetch for every access of the actual (undropped)
+    block. Reports faults and fault bytes per step and the step time with and without drops (the
+    same block-by-block protocol, wall clock, no compute emulation). Outside the timed region."""
+    import numpy as np
+    d.fault_config(512 << 20)
+    out = {"p_drop": p_drop, "steps": steps}
+    for p in (0.0, p_drop):
+        d.fault_inject(p, seed)
+        st0 = d.fault_stats()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for k in range(steps):
+            i0 = (k * B) % nS
+            d.predict(desc_dev[i0: i0 + B], hist_dev, B, stream=s0.cuda_stream)
+            acts = []
+            for b in range(B):
+                K, _, _, _ = d.prediction(b, wl.K_max, 0, s0.cuda_stream)
+                acts += [d.group_entries(b, g, stream=s0.cuda_stream) for g in range(K)]
+            Kp = d.plan(stream=s0.cuda_stream)
+            for j in range(Kp):
+                d.migrate(j, s1.cuda_stream)
+                e = acts[j]
+                modes = [int(m) for m in e[:, 1]] if len(e) else []
+                d.fault_fetch(j, [int(t) for t in e[:, 0]] if len(e) else [], modes, s1.cuda_stream)
+            d.fault_flush(s1.cuda_stream)
+        torch.cuda.synchronize()
+        ms = (time.perf_counter() - t0) * 1e3 / steps
+        st1 = d.fault_stats()
+        key = "with_drops" if p > 0 else "without_drops"
+        out[key] = {"ms_per_step_wall": round(ms, 3),
+                    "faults_per_step": round((st1["faults"] - st0["faults"]) / steps, 2),
+                    "fault_bytes_per_step": int((st1["bytes"] - st0["bytes"]) / steps),
+                    "slot_accesses_per_step": round((st1["resident"] - st0["resident"]) / steps, 1)}
+    d.fault_inject(0.0, 0)
+    d.fault_config(0)
+    return out
+
+
 def calibrate_spin(torch):
     """GPU cycles per microsecond of torch.cuda._sleep (the compute emulation's spin kernel)."""
     s = torch.cuda.Stream()
@@ -550,6 +592,13 @@ def run_dyo(args):
     e2e_s = time.perf_counter() - t0
     e2e_bytes = None
 
+    faults = None
+    if rank == 0 and not args.no_faults:
+        _log("faults")
+        try:
+            faults = fault_stream(torch, d, wl, desc_dev, hist_dev, nS, B, s0, s1)
+        except Exception as e:                  # reported, never fatal to the headline line
+            faults = {"error": str(e)[:200]}
     peaks, peak_src = measured_peaks()
     _log("pilot loop")
     # pilot latency at batch 1 (the cluster GEMV kernel, decode fused) and throughput at batch 64
@@ -699,6 +748,7 @@ def run_dyo(args):
         "predictions_per_s": round(1e6 / pred_us, 1),
         "pilot_latency_b1": lat,
         "mispredictions": mis,
+        "faults": faults,
         "pilot_batch64": {"us_per_batch": round(b64_us, 2), "us_per_prediction": round(b64_us / 64, 3),
                           "predictions_per_s": round(64e6 / b64_us, 1),
                           "pilot_kernel_us": round(b64_kernel_us, 2), "decode_kernels_us": round(b64_decode_us, 2),

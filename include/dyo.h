@@ -330,6 +330,12 @@ dyo_status dyo_fault_stats(dyo_ctx* ctx, int64_t* faults, int64_t* bytes, int64_
  * after ev_block_end (may be NULL) - what the next dyo_migrate would do; for the last block of
  * a run. No-op without pending write-backs. */
 dyo_status dyo_fault_flush(dyo_ctx* ctx, void* stream, void* ev_block_end);
+/* Fault injection (tests / measurement): from the next dyo_plan on, every read-first entry of the
+ * planned predictions whose splitmix64 hash of (seed, prediction, group slot, tensor) is below
+ * p x 2^64 is dropped before planning (workloads.drop_prefetch is the test side's twin), so the
+ * runtime faults it in. p < 0 restores the DYO_FAULT=drop_prefetch:p[:seed] environment
+ * setting (default off); p = 0 disables. DYO_E_INVAL for p > 1. */
+dyo_status dyo_fault_inject(dyo_ctx* ctx, double p, uint64_t seed);
 
 /* Device address of tensor t after the last planned transition that placed it (NULL if it is
  * on the host). Valid until the next dyo_migrate that moves it. */

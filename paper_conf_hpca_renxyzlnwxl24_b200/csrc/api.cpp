@@ -124,6 +124,8 @@ struct dyo_ctx {
   std::vector<FaultWb> fault_wb;             // written faulted tensors of the last block
   cudaEvent_t ev_fault_wb = nullptr;
   int64_t n_faults = 0, fault_bytes = 0, n_fault_resident = 0, n_fault_repair = 0;
+  double drop_p = -1.0;                      // dyo_fault_inject (< 0: DYO_FAULT environment)
+  unsigned long long drop_seed = 0;
   // host replay of the residency after every migrated transition (FIFO over plans)
   std::vector<int8_t> mig_loc;
   std::vector<int64_t> mig_off;
@@ -1642,17 +1644,19 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
     // DYO_FAULT=drop_prefetch:p[:seed] - fault injection: read-first entries of the prediction
     // dropped before planning (the runtime's accesses then fault them in, R17)
     static int parsed = 0;
-    static double drop_p = 0.0;
-    static unsigned long long drop_seed = 0;
+    static double env_p = 0.0;
+    static unsigned long long env_seed = 0;
     if (!parsed) {
       parsed = 1;
       if (const char* e = getenv("DYO_FAULT"))
         if (strncmp(e, "drop_prefetch:", 14) == 0) {
           char* q = nullptr;
-          drop_p = strtod(e + 14, &q);
-          if (q && *q == ':') drop_seed = strtoull(q + 1, nullptr, 10);
+          env_p = strtod(e + 14, &q);
+          if (q && *q == ':') env_seed = strtoull(q + 1, nullptr, 10);
         }
     }
+    const double drop_p = ctx->drop_p >= 0.0 ? ctx->drop_p : env_p;
+    const unsigned long long drop_seed = ctx->drop_p >= 0.0 ? ctx->drop_seed : env_seed;
     if (drop_p > 0.0) CK(launch_fault_drop(ctx->ad, ctx->pd, b0, n, drop_p, drop_seed, st));
   }
   {
@@ -2224,6 +2228,13 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
     ++ctx->n_fault_repair;
   }
   if (ev_done) CK(cudaEventRecord((cudaEvent_t)ev_done, s));
+  return DYO_OK;
+}
+
+dyo_status dyo_fault_inject(dyo_ctx* ctx, double p, uint64_t seed) {
+  if (!ctx || !(p <= 1.0)) return DYO_E_INVAL;
+  ctx->drop_p = p;
+  ctx->drop_seed = seed;
   return DYO_OK;
 }
 

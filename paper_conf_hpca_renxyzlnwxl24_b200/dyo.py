@@ -99,7 +99,7 @@ def lib():
                      "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
                      "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats",
                      "dyo_debug_copy_stamps", "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check",
-                     "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush"):
+                     "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush", "dyo_fault_inject"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -112,7 +112,7 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
            "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps",
            "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check",
-           "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush")
+           "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush", "dyo_fault_inject")
 
 
 def _a(x, dt):
@@ -399,6 +399,9 @@ class Dyo:
         self._check(self.L.dyo_fault_fetch(self.ctx, int(j), _p(ids_a, i32), _p(md, i32), n, ptrs, P(stream),
                                            P(ev_done)))
         return [ptrs[i] for i in range(n)]
+
+    def fault_inject(self, p, seed=0):
+        self._check(self.L.dyo_fault_inject(self.ctx, C.c_double(p), C.c_uint64(seed)))
 
     def fault_flush(self, stream=0, ev_block_end=None):
         self._check(self.L.dyo_fault_flush(self.ctx, P(stream), P(ev_block_end)))

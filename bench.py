@@ -366,7 +366,7 @@ def fault_stream(torch, d, wl, desc_dev, hist_dev, nS, B, s0, s1, steps=4, p_dro
             d.predict(desc_dev[i0: i0 + B], hist_dev, B, stream=s0.cuda_stream)
             acts = []
             for b in range(B):
-                K, _, _, _ = d.prediction(b, wl.K_max, 0, s0.cuda_stream)
+                K, _, _, _ = d.prediction(b, wl.K_max, 4096, s0.cuda_stream)   # >= n_sites (kMaxSites)
                 acts += [d.group_entries(b, g, stream=s0.cuda_stream) for g in range(K)]
             Kp = d.plan(stream=s0.cuda_stream)
             for j in range(Kp):

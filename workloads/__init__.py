@@ -875,6 +875,21 @@ def make(name, seed=0, **kw):
     return CONFIGS[name](seed=seed, **kw)
 
 
+def op_time_ns(op):
+    """Synthetic compute time of an operator (ns): 1 + (sum over its inputs of the element
+    count) / 64 - the trace's execution time for the partition labels (P:L168 'execution time of
+    each operator'); an input of both sides, no method arithmetic. Control rows take 0."""
+    if op is None:
+        return 0
+    n = 0
+    for shp in op.inputs:
+        e = 1
+        for d in shp:
+            e *= int(d)
+        n += e
+    return 1 + n // 64
+
+
 # ----------------------------------------------------------------------------
 # fault injection (DYO_FAULT=drop_prefetch:p): a counter-based drop decision, implemented here
 # for the test side and independently in libdyo (api.cpp drop_hash)

@@ -337,6 +337,55 @@ dyo_status dyo_fault_flush(dyo_ctx* ctx, void* stream, void* ev_block_end);
  * setting (default off); p = 0 disables. DYO_E_INVAL for p > 1. */
 dyo_status dyo_fault_inject(dyo_ctx* ctx, double p, uint64_t seed);
 
+/* ---- Partition labels (§IV-D: Sentinel-style labels that "maximize the
+ * overlap between tensor migration and training computation without violating the GPU memory
+ * capacity"; §V L203-L205 the partition simulator; §VI-G L275 the heuristics; R18) ----
+ * One sample's execution trace: L rows of the loaded arch (path_ops: operator per row, -1 for a
+ * control row; path_it: the row's iteration index, R13; b: the per-sample binding), compute time
+ * per operator op_time_ns (n_ops int64, host). Block j = rows [c_j, c_j+1) needs the aligned bytes
+ * of its tensor set (<= H), migrates the bytes of the tensors it reads first, and hides that
+ * migration (ceil(bytes * 1000 / bw) ns, bw in bytes per microsecond) behind block j-1's compute;
+ * exposed = sum over j >= 1 of max(0, migration_j - compute_j-1).
+ * method 0: the overlap partition - minimum exposed time over K-block partitions within the
+ *   capacity, the lexicographically smallest cut vector among the minimisers (GPU dynamic
+ *   programming over (block, previous block start, block end));
+ * method 1 / 2 / 3: even operators / even compute time / even accessed bytes (cut j after the
+ *   longest prefix holding at most j/K of the total, kept non-empty).
+ * cuts (host, K+1 ints) receives 0 = c_0 < ... < c_K = L, *exposed the ns, *feasible (may be
+ * NULL) whether every block fits H (method 0: 0 and *exposed = -1 when none does). L <= 4096;
+ * synchronises `stream`. DYO_E_CAPACITY if a block start meets more than 4096 distinct tensors. */
+dyo_status dyo_partition(dyo_ctx* ctx, const int32_t* path_ops, const int32_t* path_it, int32_t L, int32_t b,
+                         const int64_t* op_time_ns, int32_t K, int32_t method, int64_t H, int64_t bw, int32_t* cuts,
+                         int64_t* exposed, int32_t* feasible, void* stream);
+
+/* ---- Pilot training (§IV-D, §V: LeakyReLU, SGD, learning rate 0.01;
+ * DESIGN.md reading R19) ------------------------------------------------------------------
+ * A trainer holds an fp64 copy of a pilot (the weights of w, widened exactly) and trains the
+ * feature layers, the MLP of nn_type (the only one that runs) and the output layer.
+ * dyo_trainer_step: one SGD step on a minibatch - feat (device, B x F fp32: dyo_encode_features
+ *   output) and target (device, B x O fp32: label block vectors in R4 block-head units and
+ *   one-hot branch choices) - on L = (1/2B) sum ||y - t||^2, on `stream`; *loss (may be NULL)
+ *   receives the loss before the step (synchronises the stream). B <= max_batch.
+ * dyo_trainer_export: every weight array of the pilot in dyo_pilot_desc order (feature layers
+ *   W then b; MLP k = 0..2, layer l: W then b; out W then b) into blob (host fp64, cap doubles;
+ *   NULL to query *n); the untrained MLPs keep their weights. Synchronises the device.
+ * Deterministic: every sum runs in a fixed order. */
+typedef struct dyo_trainer dyo_trainer;
+dyo_status dyo_trainer_create(const dyo_pilot_desc* w, int32_t nn_type, int32_t max_batch, int32_t device,
+                              dyo_trainer** out);
+dyo_status dyo_trainer_step(dyo_trainer* tr, const float* feat, const float* target, int32_t B, double lr,
+                            double* loss, void* stream);
+dyo_status dyo_trainer_export(dyo_trainer* tr, double* blob, int64_t cap, int64_t* n);
+dyo_status dyo_trainer_destroy(dyo_trainer* tr);
+
+/* The resolved path (R2 rows: operator per row, -1 for a control row; iteration index per row,
+ * R13) of the loaded arch for the given site choices (n_sites ints, preorder; nested sites
+ * ignored) and nested executions' choices (R16, execution order) - the execution trace of a
+ * sample whose control flow is known (partition labels, R18). Host-only; DYO_E_CAPACITY with the
+ * needed length in *L if cap is too small. */
+dyo_status dyo_trace_path(dyo_ctx* ctx, const int32_t* choices, const int32_t* nested, int32_t n_nested, int32_t* ops,
+                          int32_t* its, int32_t cap, int32_t* L);
+
 /* Device address of tensor t after the last planned transition that placed it (NULL if it is
  * on the host). Valid until the next dyo_migrate that moves it. */
 dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr);

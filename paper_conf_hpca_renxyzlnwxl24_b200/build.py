@@ -9,7 +9,7 @@ OUT = os.path.join(HERE, "libdyo.so")
 BUILD = os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-CU = ["pilot.cu", "pilot_tc.cu", "decode.cu", "plan.cu", "copy.cu"]
+CU = ["pilot.cu", "pilot_tc.cu", "decode.cu", "plan.cu", "copy.cu", "partition.cu", "train.cu"]
 CPP = ["api.cpp", "traverse.cpp", "nested.cpp"]
 
 

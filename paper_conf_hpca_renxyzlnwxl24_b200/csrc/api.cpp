@@ -133,6 +133,9 @@ struct dyo_ctx {
   PlanSlot* last_mig_slot = nullptr;
   int last_mig_j = -1;
   int64_t last_mig_seq = -1;
+  // partition labels (R18): device scratch grown on demand
+  void* part_buf = nullptr;
+  size_t part_bytes = 0;
   // migration
   cudaStream_t d2h = nullptr;      // ctx-owned stream for the EVICT (D2H) phase
   cudaStream_t side = nullptr;     // ctx-owned stream for early CARRY (overlaps FETCH)
@@ -588,7 +591,7 @@ dyo_status parse_arch(const dyo_arch* A, int64_t AL, int max_b, ArchHost& h, std
 
   h.n_sites = n_sites;
   h.L_max = L_max;
-  if (h.nested) {
+  {                                      // the program tree (nested decode, dyo_trace_path)
     NestArch& na = h.nest;
     na.kind.assign(A->node_kind, A->node_kind + N);
     na.a.assign(A->node_a, A->node_a + N);
@@ -711,6 +714,7 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->ev_memo) cudaEventDestroy(ctx->ev_memo);
   if (ctx->ev_fault_wb) cudaEventDestroy(ctx->ev_fault_wb);
   if (ctx->fault_area) cudaFree(ctx->fault_area);
+  if (ctx->part_buf) cudaFree(ctx->part_buf);
   if (ctx->h_rep) cudaFreeHost(ctx->h_rep);
   if (ctx->h_memo_stage) cudaFreeHost(ctx->h_memo_stage);
   for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
@@ -1586,6 +1590,24 @@ dyo_status dyo_prediction_matched(dyo_ctx* ctx, int32_t b, int32_t* matched) {
   return DYO_OK;
 }
 
+dyo_status dyo_trace_path(dyo_ctx* ctx, const int32_t* choices, const int32_t* nested, int32_t n_nested, int32_t* ops,
+                          int32_t* its, int32_t cap, int32_t* L) {
+  if (!ctx || !choices || !L || (n_nested > 0 && !nested)) return DYO_E_INVAL;
+  if (!ctx->arch_ok) return fail(ctx, DYO_E_STATE, "load the arch first");
+  for (int s2 = 0; s2 < ctx->n_sites; ++s2)
+    if (ctx->nest.top[s2] && (choices[s2] < 0 || choices[s2] >= ctx->trav.site_nch[s2]))
+      return fail(ctx, DYO_E_INVAL, "choice %d of site %d", choices[s2], s2);
+  std::vector<int32_t> pop, pit;
+  std::string e;
+  dyo_status st = trace_path(ctx->nest, choices, nested, n_nested, pop, pit, e);
+  if (st) return fail(ctx, st, "%s", e.c_str());
+  *L = (int32_t)pop.size();
+  if ((int32_t)pop.size() > cap) return fail(ctx, DYO_E_CAPACITY, "need %zu rows", pop.size());
+  if (ops) std::copy(pop.begin(), pop.end(), ops);
+  if (its) std::copy(pit.begin(), pit.end(), its);
+  return DYO_OK;
+}
+
 dyo_status dyo_prediction_nested(dyo_ctx* ctx, int32_t b, int32_t* out, int32_t cap, int32_t* n) {
   if (!ctx || !n || b < 0 || b >= ctx->last_B) return DYO_E_INVAL;
   if (!ctx->nested) { *n = 0; return DYO_OK; }
@@ -2133,6 +2155,61 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   }
   P.ev_pending = true;
   P.next_j = j + 1;
+  return DYO_OK;
+}
+
+// ---- partition labels (R18) ----------------------
+dyo_status dyo_partition(dyo_ctx* ctx, const int32_t* path_ops, const int32_t* path_it, int32_t L, int32_t b,
+                         const int64_t* op_time_ns, int32_t K, int32_t method, int64_t H, int64_t bw, int32_t* cuts,
+                         int64_t* exposed, int32_t* feasible, void* stream) {
+  if (!ctx || !path_ops || !path_it || !op_time_ns || !cuts || !exposed) return DYO_E_INVAL;
+  if (!ctx->arch_ok) return fail(ctx, DYO_E_STATE, "load the arch first");
+  if (L < 1 || K < 1 || K > L || L > 4096 || method < 0 || method > 3 || bw < 1 || H < 0 || b < 0 ||
+      b >= ctx->cfg.max_batch)
+    return fail(ctx, DYO_E_INVAL, "partition: L=%d K=%d method=%d", L, K, method);
+  for (int r = 0; r < L; ++r)
+    if (path_ops[r] < -1 || path_ops[r] >= ctx->n_ops) return fail(ctx, DYO_E_INVAL, "row %d: operator %d", r, path_ops[r]);
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t lay = (size_t)L * (L + 1);
+  const size_t need_b = 3 * lay * 8 + (method == 0 ? (size_t)K * lay * 8 : 0) + (size_t)L * 8 + (size_t)ctx->n_ops * 8 +
+                        (size_t)(K + 1) * 4 + 64 + 16;
+  if (need_b > ctx->part_bytes) {
+    if (ctx->part_buf) { CK(cudaStreamSynchronize(s)); cudaFree(ctx->part_buf); ctx->part_buf = nullptr; ctx->part_bytes = 0; }
+    CK(cudaMalloc(&ctx->part_buf, need_b));
+    ctx->part_bytes = need_b;
+  }
+  char* q = static_cast<char*>(ctx->part_buf);
+  long long* need = reinterpret_cast<long long*>(q); q += lay * 8;
+  long long* fetch = reinterpret_cast<long long*>(q); q += lay * 8;
+  long long* comp = reinterpret_cast<long long*>(q); q += lay * 8;
+  long long* f = reinterpret_cast<long long*>(q); if (method == 0) q += (size_t)K * lay * 8;
+  long long* ons = reinterpret_cast<long long*>(q); q += (size_t)ctx->n_ops * 8;
+  int32_t* ops = reinterpret_cast<int32_t*>(q); q += (size_t)L * 4;
+  int32_t* its = reinterpret_cast<int32_t*>(q); q += (size_t)L * 4;
+  long long* res = reinterpret_cast<long long*>(q); q += 16;
+  int* ovf = reinterpret_cast<int*>(q); q += 16;
+  int32_t* dcuts = reinterpret_cast<int32_t*>(q);
+  CK(cudaMemcpyAsync(ops, path_ops, (size_t)L * 4, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(its, path_it, (size_t)L * 4, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(ons, op_time_ns, (size_t)ctx->n_ops * 8, cudaMemcpyHostToDevice, s));
+  CK(cudaMemsetAsync(ovf, 0, 4, s));
+  CK(cudaMemsetAsync(res, 0, 16, s));
+  CK(launch_partition(ctx->ad, ops, its, L, b, ons, K, method, H, bw, need, fetch, comp, f, dcuts, res, ovf, s));
+  long long hres[2] = {0, 0};
+  int hovf = 0;
+  CK(cudaMemcpyAsync(hres, res, 16, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&hovf, ovf, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(cuts, dcuts, (size_t)(K + 1) * 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (hovf) return fail(ctx, DYO_E_CAPACITY, "partition: more distinct tensors per block start than the hash holds");
+  if (method == 0) {
+    *exposed = hres[0];
+    if (feasible) *feasible = hres[0] >= 0 ? 1 : 0;
+  } else {
+    *exposed = hres[0];
+    if (feasible) *feasible = (int32_t)hres[1];
+  }
   return DYO_OK;
 }
 

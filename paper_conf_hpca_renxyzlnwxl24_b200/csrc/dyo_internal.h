@@ -244,6 +244,10 @@ dyo_status nested_decode(const NestArch& N, const int32_t* slots, int K_max, con
                          std::vector<int32_t>& path_op, std::vector<int32_t>& path_it, std::vector<int32_t>& nested,
                          int* matched, std::string& err);
 
+// The path of given top-level choices and nested executions' choices (execution order).
+dyo_status trace_path(const NestArch& N, const int32_t* choices, const int32_t* nested, int n_nested,
+                      std::vector<int32_t>& path_op, std::vector<int32_t>& path_it, std::string& err);
+
 // ---- launchers (implemented in the .cu files) ------------------------------------------
 cudaError_t launch_encode(const ArchDev& a, const int64_t* desc, const int32_t* hist,
                           const int32_t* hist_tab, const int32_t* hist_K, int hist_B, int B, float* feat,
@@ -267,6 +271,10 @@ cudaError_t plan_debug_stamps(int j, unsigned long long* out);
 // device arrays (d) into the pinned mapped mirrors (h: device-side aliases) by the counts in
 // d.counts; nothing when d.status[0] != 0. Entry records are not copied.
 cudaError_t launch_plan_export(const PlanOut& d, const PlanOut& h, cudaStream_t s);
+cudaError_t launch_partition(const ArchDev& a, const int32_t* ops, const int32_t* its, int L, int b,
+                             const long long* op_ns, int K, int method, long long H, long long bw, long long* need,
+                             long long* fetch, long long* comp, long long* f, int32_t* cuts, long long* result,
+                             int* overflow, cudaStream_t s);
 cudaError_t launch_fault_drop(const ArchDev& a, const PredDev& pd, int b0, int nb, double p, uint64_t seed,
                               cudaStream_t s);
 cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, int B,

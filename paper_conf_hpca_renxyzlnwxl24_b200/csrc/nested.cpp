@@ -271,4 +271,29 @@ dyo_status nested_decode(const NestArch& N, const int32_t* slots, int K_max, con
   return DYO_OK;
 }
 
+dyo_status trace_path(const NestArch& N, const int32_t* choices, const int32_t* nested, int n_nested,
+                      std::vector<int32_t>& path_op, std::vector<int32_t>& path_it, std::string& err) {
+  const Flat F = flatten(N, choices);
+  path_op.clear();
+  path_it.clear();
+  int ci = 0;
+  for (const Atom& a : F.at) {
+    if (a.type == 0) {
+      path_op.push_back(a.op);
+      path_it.push_back(a.it);
+      continue;
+    }
+    if (ci >= n_nested) { err = "trace: fewer nested choices than nested executions"; return DYO_E_INVAL; }
+    const int c = nested[ci++];
+    if (c < 0 || c >= a.narm) { err = "trace: nested choice out of range"; return DYO_E_INVAL; }
+    const Arm& arm = F.arms[a.arm0 + c];
+    for (int q = 0; q < arm.n_ops; ++q) {
+      path_op.push_back(arm.first_op + q);
+      path_it.push_back(a.it);
+    }
+  }
+  if (ci != n_nested) { err = "trace: more nested choices than nested executions"; return DYO_E_INVAL; }
+  return DYO_OK;
+}
+
 }  // namespace dyo

@@ -99,7 +99,9 @@ def lib():
                      "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
                      "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats",
                      "dyo_debug_copy_stamps", "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check",
-                     "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush", "dyo_fault_inject"):
+                     "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush", "dyo_fault_inject", "dyo_partition",
+                     "dyo_trace_path", "dyo_trainer_create", "dyo_trainer_step", "dyo_trainer_export",
+                     "dyo_trainer_destroy"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
@@ -112,7 +114,8 @@ EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_d
            "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
            "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps",
            "dyo_query", "dyo_set_timing", "dyo_prediction_nested", "dyo_nested_check",
-           "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush", "dyo_fault_inject")
+           "dyo_fault_config", "dyo_fault_fetch", "dyo_fault_stats", "dyo_fault_flush", "dyo_fault_inject", "dyo_partition",
+           "dyo_trace_path", "dyo_trainer_create", "dyo_trainer_step", "dyo_trainer_export", "dyo_trainer_destroy")
 
 
 def _a(x, dt):
@@ -227,6 +230,95 @@ def nested_check(wl, slots, top_choices, cap=1 << 16):
     st = lib().dyo_nested_check(C.byref(arch), _p(sl, i32), _p(tc, i32), _p(nest, i32), cap, C.byref(nn),
                                 _p(path, i32), cap, C.byref(pl), C.byref(m), err, 512)
     return st, nest[:nn.value].tolist(), path[:pl.value].tolist(), m.value, err.value.decode()
+
+
+def _pilot_desc(spec, keep, slope=0.01):
+    """dyo_pilot_desc of a PilotSpec (arrays kept alive in `keep`)."""
+    w = spec.weights
+
+    def arr(x, dt=np.float32):
+        x = _a(x, dt)
+        keep.append(x)
+        return x
+
+    def ptrs(names):
+        lst = [_p(arr(w[n]), f32) for n in names]
+        pa = (PF32 * max(1, len(lst)))(*lst)
+        keep.append(pa)
+        return pa
+    nf = len(spec.feature)
+    fo = arr([f[0] for f in spec.feature] or [0], np.int32)
+    fl = arr([f[1] for f in spec.feature] or [0], np.int32)
+    fu = arr([f[2] for f in spec.feature] or [0], np.int32)
+    mi = arr([m[0] for m in spec.mlp], np.int32)
+    mo = arr([m[1] for m in spec.mlp], np.int32)
+    fW = ptrs([f"feat{i}.W" for i in range(nf)])
+    fb = ptrs([f"feat{i}.b" for i in range(nf)])
+    mW = ptrs([f"mlp{k}.{l}.W" for k in range(3) for l in range(len(spec.mlp))])
+    mb = ptrs([f"mlp{k}.{l}.b" for k in range(3) for l in range(len(spec.mlp))])
+    oW, ob = arr(w["out.W"]), arr(w["out.b"])
+    return PilotDesc(spec.F, spec.O, nf, _p(fo, i32), _p(fl, i32), _p(fu, i32), fW, fb, len(spec.mlp),
+                     _p(mi, i32), _p(mo, i32), mW, mb, spec.out_in, _p(oW, f32), _p(ob, f32), slope)
+
+
+def weight_names(spec):
+    """Weight arrays in dyo_pilot_desc / dyo_trainer_export order."""
+    names = []
+    for i in range(len(spec.feature)):
+        names += [f"feat{i}.W", f"feat{i}.b"]
+    for k in range(3):
+        for l in range(len(spec.mlp)):
+            names += [f"mlp{k}.{l}.W", f"mlp{k}.{l}.b"]
+    return names + ["out.W", "out.b"]
+
+
+class Trainer:
+    """dyo_trainer: SGD on a pilot's fp64 copy (reading R19)."""
+
+    def __init__(self, spec, nn_type, max_batch, device=0):
+        self.L = lib()
+        self.spec = spec
+        keep = []
+        d = _pilot_desc(spec, keep)
+        self.tr = P()
+        st = self.L.dyo_trainer_create(C.byref(d), int(nn_type), int(max_batch), int(device), C.byref(self.tr))
+        if st:
+            raise DyoError(st, "dyo_trainer_create")
+
+    def step(self, feat, target, B, lr=0.01, stream=0, want_loss=True):
+        loss = C.c_double(0.0)
+        st = self.L.dyo_trainer_step(self.tr, P(Dyo._ptr(feat)), P(Dyo._ptr(target)), int(B), C.c_double(lr),
+                                     C.byref(loss) if want_loss else None, P(stream))
+        if st:
+            raise DyoError(st, "dyo_trainer_step")
+        return loss.value
+
+    def weights(self):
+        """{name: float64 array} of every weight array (trained and untouched)."""
+        n = i64()
+        self.L.dyo_trainer_export(self.tr, None, 0, C.byref(n))
+        blob = np.zeros(n.value, np.float64)
+        st = self.L.dyo_trainer_export(self.tr, blob.ctypes.data_as(C.POINTER(C.c_double)), n.value, C.byref(n))
+        if st:
+            raise DyoError(st, "dyo_trainer_export")
+        out, o = {}, 0
+        for name in weight_names(self.spec):
+            shp = np.shape(self.spec.weights[name])
+            k = int(np.prod(shp))
+            out[name] = blob[o:o + k].reshape(shp)
+            o += k
+        return out
+
+    def close(self):
+        if self.tr:
+            self.L.dyo_trainer_destroy(self.tr)
+            self.tr = P()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class Dyo:
@@ -385,6 +477,32 @@ class Dyo:
     def migrate(self, j, stream=0, ev_half_free=None, ev_prev_done=None, ev_ready=None):
         """ev_*: cudaEvent_t handles (torch.cuda.Event.cuda_event) or None."""
         self._check(self.L.dyo_migrate(self.ctx, j, P(stream), P(ev_half_free), P(ev_prev_done), P(ev_ready)))
+
+    def trace_path(self, choices, nested=(), cap=1 << 20):
+        """(ops, its) of the resolved path for the given site choices / nested choices."""
+        ch = _a(list(choices) or [0], np.int32)
+        ne = _a(list(nested) or [0], np.int32)
+        ops = np.zeros(cap, np.int32)
+        its = np.zeros(cap, np.int32)
+        L = i32()
+        self._check(self.L.dyo_trace_path(self.ctx, _p(ch, i32), _p(ne, i32), len(nested), _p(ops, i32), _p(its, i32),
+                                          cap, C.byref(L)))
+        return ops[:L.value].copy(), its[:L.value].copy()
+
+    # ---- partition labels (P:L164-L170, L275; R18) ----
+    METHODS = {"overlap": 0, "even_ops": 1, "even_time": 2, "even_size": 3}
+
+    def partition(self, path_ops, path_it, b, op_time_ns, K, method, H, bw, stream=0):
+        """(cuts, exposed_ns, feasible) of one trace (R18); method in METHODS."""
+        ops = _a(path_ops, np.int32)
+        its = _a(path_it, np.int32)
+        ons = _a(op_time_ns, np.int64)
+        cuts = np.zeros(K + 1, np.int32)
+        ex, fe = i64(), i32()
+        self._check(self.L.dyo_partition(self.ctx, _p(ops, i32), _p(its, i32), len(ops), int(b), _p(ons, i64), int(K),
+                                         self.METHODS[method] if isinstance(method, str) else int(method), i64(H),
+                                         i64(bw), _p(cuts, i32), C.byref(ex), C.byref(fe), P(stream)))
+        return cuts.tolist(), ex.value, bool(fe.value)
 
     # ---- on-demand fetch of mis-predicted tensors (P:L184, L197; R17) ----
     def fault_config(self, area_bytes):

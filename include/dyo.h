@@ -364,7 +364,7 @@ dyo_status dyo_partition(dyo_ctx* ctx, const int32_t* path_ops, const int32_t* p
  * feature layers, the MLP of nn_type (the only one that runs) and the output layer.
  * dyo_trainer_step: one SGD step on a minibatch - feat (device, B x F fp32: dyo_encode_features
  *   output) and target (device, B x O fp32: label block vectors in R4 block-head units and
- *   one-hot branch choices) - on L = (1/2B) sum ||y - t||^2, on `stream`; *loss (may be NULL)
+ *   one-hot branch choices) - on L = (1/(B O)) sum (y - t)^2, on `stream`; *loss (may be NULL)
  *   receives the loss before the step (synchronises the stream). B <= max_batch.
  * dyo_trainer_export: every weight array of the pilot in dyo_pilot_desc order (feature layers
  *   W then b; MLP k = 0..2, layer l: W then b; out W then b) into blob (host fp64, cap doubles;

@@ -5,9 +5,10 @@ DESIGN.md reading R19).
 Oracle - test infrastructure only (see oracle/__init__.py).
 
 Loss (reading R19; the paper names no loss): for a minibatch of B samples with pilot outputs y_b
-and targets t_b (the label block vectors in the block-head units of R4 - count / 16, idiom sums
-/ 16, dimension sums / 1024 - and, in the branch head, the one-hot of each free site's actual
-choice), L = (1 / 2B) sum_b ||y_b - t_b||^2. One SGD step: every parameter p <- p - lr dL/dp,
+(O logits each) and targets t_b (the label block vectors in the block-head units of R4 - count /
+16, idiom sums / 16, dimension sums / 1024 - and, in the branch head, the one-hot of each free
+site's actual choice), the mean squared error L = (1 / (B O)) sum_b ||y_b - t_b||^2 (PyTorch's
+MSELoss default reduction). One SGD step: every parameter p <- p - lr dL/dp,
 where the parameters are the feature layers, the MLP selected by the NN type (the only one that
 runs) and the output layer. fp64 throughout (the pilot's fp32 weights are widened
 exactly; a trained pilot is rounded back to fp32 to be loaded).
@@ -59,9 +60,10 @@ def loss_and_grads(spec, w, X, Tgt, nn_type):
     B = X.shape[0]
     y, cache = forward(spec, w, X, nn_type)
     diff = y - Tgt
-    L = float((diff * diff).sum() / (2.0 * B))
+    N = diff.size
+    L = float((diff * diff).sum() / N)
     g = {}
-    d = diff / B                                   # dL/dy
+    d = 2.0 * diff / N                             # dL/dy
     # output layer (linear)
     name, z, _ = cache[-1]
     g["out.W"] = d.T @ z

@@ -3,4 +3,4 @@
 The product path is libdyo.so (include/dyo.h) — hand-written sm_100a CUDA kernels plus a C++
 DMA engine; `dyo` is its thin ctypes binding. No CPU fallback exists.
 """
-from .dyo import Dyo, DyoError, lib, LIB_PATH, EXPORTS  # noqa: F401
+from .dyo import Dyo, DyoError, Trainer, lib, LIB_PATH, EXPORTS  # noqa: F401

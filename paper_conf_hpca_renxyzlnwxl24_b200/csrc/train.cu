@@ -1,5 +1,5 @@
 // Pilot training on the GPU (§IV-D, §V: LeakyReLU, SGD, learning rate 0.01;
-// DESIGN.md reading R19): minibatch SGD on L = (1/2B) sum_b ||y_b - t_b||^2 over the feature
+// DESIGN.md reading R19): minibatch SGD on the mean squared error over the feature
 // layers, the MLP selected by the NN type and the output layer, in fp64 (the pilot's fp32
 // weights widen exactly; export rounds back to fp32 for dyo_load_pilot).
 //
@@ -68,7 +68,8 @@ __global__ void fwd_kernel(const double* __restrict__ W, const double* __restric
   }
 }
 
-// dL/dy = (y - t) / B and the loss (one block, fixed-order reduction)
+// L = (1 / (B O)) sum (y - t)^2 (MSELoss, mean), dL/dy = 2 (y - t) / (B O) (one block,
+// fixed-order reduction)
 __global__ void loss_kernel(const double* __restrict__ y, const double* __restrict__ t, double* __restrict__ dy, int B,
                             int O, double* __restrict__ loss) {
   __shared__ double part[1024];
@@ -76,7 +77,7 @@ __global__ void loss_kernel(const double* __restrict__ y, const double* __restri
   const int64_t n = (int64_t)B * O;
   for (int64_t i = threadIdx.x; i < n; i += blockDim.x) {
     const double d = y[i] - t[i];
-    dy[i] = d / B;
+    dy[i] = 2.0 * d / (double)n;
     s = fma(d, d, s);
   }
   part[threadIdx.x] = s;
@@ -85,7 +86,7 @@ __global__ void loss_kernel(const double* __restrict__ y, const double* __restri
     if ((int)threadIdx.x < w) part[threadIdx.x] += part[threadIdx.x + w];
     __syncthreads();
   }
-  if (threadIdx.x == 0) *loss = part[0] / (2.0 * B);
+  if (threadIdx.x == 0) *loss = part[0] / (double)n;
 }
 
 // gradient w.r.t. the pre-activation: times LeakyReLU'(v) (sign of the post-activation)

@@ -63,7 +63,8 @@ def test_lr_zero_and_unselected_mlps_unchanged():
 
 
 def test_output_bias_step_closed_form():
-    """dL/db_out = mean over the batch of (y - t): one step moves the output bias by lr * that."""
+    """dL/db_out = (2 / (B O)) sum over the batch of (y - t): one step moves the output bias by lr
+    times that."""
     spec = _small_spec(4)
     w = TR.widen(spec)
     rng = np.random.default_rng(5)
@@ -71,8 +72,8 @@ def test_output_bias_step_closed_form():
     y, _ = TR.forward(spec, w, X, 0)
     b0 = w["out.b"].copy()
     L = TR.sgd_step(spec, w, X, T, 0, lr=0.01)
-    assert np.allclose(w["out.b"], b0 - 0.01 * (y - T).mean(axis=0), rtol=0, atol=1e-15)
-    assert abs(L - ((y - T) ** 2).sum() / 6) <= 1e-12 * L
+    assert np.allclose(w["out.b"], b0 - 0.01 * 2 * (y - T).sum(axis=0) / (3 * 7), rtol=0, atol=1e-15)
+    assert abs(L - ((y - T) ** 2).sum() / 21) <= 1e-12 * L
 
 
 def test_sgd_decreases_loss_on_a_fixed_batch():

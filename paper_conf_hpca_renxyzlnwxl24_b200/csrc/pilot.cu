@@ -636,6 +636,9 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   }
   StagePlan sp{};
   sp.Bs = B < kBs ? 1 : kBs;
+  // a wide pilot whose 8-sample activation buffers do not fit shared memory runs one sample per
+  // cluster (the batch-1 kernel, one cluster per prediction)
+  if (sp.Bs > 1 && 2 * kBs * p.max_width * (int)sizeof(double) + kDmmaRedBytes + 4096 > kDynCap) sp.Bs = 1;
   if (sp.Bs > 1) {
     // batch path: every cluster of the launch must be co-resident (one wave; measured on MoE
     // B = 64: 8 clusters of 16 CTAs -> 7 active -> two waves, 117 us; of 8 CTAs -> 74 us), so

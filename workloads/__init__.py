@@ -769,7 +769,7 @@ def make_tree(seed=0, n_samples=128, batch=64, min_leaves=8, max_leaves=64, hidd
     bwd_body = [Op(bwd_sig, ((1, Hd), (Hd, 5 * Hd)),
                    acc((W_leaf, R, 0, 0), (W_comp, R, 0, 0), (gW_leaf, RW, 0, 0), (gW_comp, RW, 0, 0),
                        (dpool, R, 0, 0), A_(h0, 0, R), A_(c0, 0, R), A_(g0, 0, R), A_(x0, 0, R)), "node_bwd")]
-    embed = Op((0, 1, 0, 0, 1, 0), ((max_nodes, Hd),), (), "embed")
+    embed = Op((0, 1, 0, 0, 1, 0), ((max_nodes, Hd),), acc((pool, W, 0, 0)), "embed")     # resets the pooled state
     loss_op = Op((0, 0, 0, 1, 2, 0), ((1, Hd),), acc((pool, R, 0, 0), (loss, W, 0, 0), (dpool, W, 0, 0)), "loss")
     opt = Op((0, 0, 0, 0, 3, 0), ((4 * Hd, 2 * Hd),) * 2,
              acc((W_leaf, RW, 0, 0), (W_comp, RW, 0, 0), (gW_leaf, RW, 0, 0), (gW_comp, RW, 0, 0)), "optimizer")

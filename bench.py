@@ -793,10 +793,64 @@ def run_dyo(args):
             comp["gpu_speedup"] = {"pilot_decode": round((comp["pilot_us_per_prediction"] + comp["decode_us_per_prediction"])
                                                          / max(pred_us, 1e-9), 1),
                                    "plan": round(comp["plan_us_per_step"] / max(plan_us, 1e-9), 1)}
-    print(json.dumps(out), flush=True)
     d.close()
+    if world == 1 and not args.no_cpu_baseline:
+        _log("compiled cpu planner")
+        try:
+            out["cpu_baseline"]["compiled_planner"] = compiled_planner_leg(torch, wl, local, dev_inputs, B, s0, args.steps,
+                                                                           plan_us)
+        except Exception as e:                  # reported, never fatal to the headline line
+            out["cpu_baseline"]["compiled_planner"] = {"error": str(e)[:200]}
+    print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def compiled_planner_leg(torch, wl, dev, inputs, B, s0, n_steps, gpu_plan_us):
+    """K2's honest baseline: the compiled single-core CPU planner (baseline/cpu_planner.cpp, g++
+    -O3, bit-exact with oracle/plan.py - tests/test_cpu_planner.py) planning the same W sets the GPU
+    planner plans. A fresh manager predicts each step on the GPU; its tensor sets are read back
+    (untimed), the CPU planner plans them (timed, one host core) and the GPU planner plans them
+    too; both start from an empty arena, so every transition's byte counts must agree."""
+    import numpy as np
+    sys.path.insert(0, os.path.join(ROOT, "baseline"))
+    import cpu_planner
+    from paper_conf_hpca_renxyzlnwxl24_b200 import Dyo
+    dc = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, device=dev, flags=0)
+    dc.load(wl)
+    cp = cpu_planner.CpuPlanner(wl)
+    n_sites = 4096
+    t_cpu, n_tr, mism, steps = 0.0, 0, 0, 0
+    for k in range(n_steps):
+        desc, hist = inputs(k)
+        dc.predict(desc, hist, B, stream=s0.cuda_stream)
+        Ws = []
+        for b in range(B):
+            K, _, _, _ = dc.prediction(b, wl.K_max, n_sites, stream=s0.cuda_stream)
+            for g in range(K):
+                Ws.append([tuple(int(x) for x in e) for e in dc.group_entries(b, g, cap=1 << 16, stream=s0.cuda_stream)])
+        t0 = time.perf_counter()
+        st, trs = cp.plan(Ws)
+        t_cpu += time.perf_counter() - t0
+        K = dc.plan(stream=s0.cuda_stream)
+        if st != 0 or K != len(trs):
+            mism += 1
+            break
+        for j in range(K):
+            info = dc.plan_info(j)
+            if (info["h2d"], info["d2h"], info["d2d"]) != (trs[j]["h2d"], trs[j]["d2h"], trs[j]["d2d"]):
+                mism += 1
+        n_tr += K
+        steps += 1
+    torch.cuda.synchronize()
+    dc.close()
+    cp.close()
+    cpu_us = t_cpu / max(1, steps) * 1e6
+    return {"plan_us_per_step": round(cpu_us, 1), "transitions_per_step": round(n_tr / max(1, steps), 2),
+            "steps": steps, "cores": 1, "transition_mismatches_vs_gpu": mism,
+            "gpu_plan_us": round(gpu_plan_us, 2), "gpu_speedup": round(cpu_us / max(gpu_plan_us, 1e-9), 2),
+            "sample": "the bench's first %d step inputs, W sets of the GPU decode, planned from an empty arena" % steps,
+            "kind": "compiled single-core planner (baseline/cpu_planner.cpp, g++ -O3 -march=x86-64-v3)"}
 
 
 def step_bound_ms(trs, h2d_gbs, d2h_gbs):

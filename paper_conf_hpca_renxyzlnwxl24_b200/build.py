@@ -26,6 +26,7 @@ def build(force=False, verbose=False):
     srcs = [os.path.join(CSRC, f) for f in CU + CPP] + [os.path.join(CSRC, "dyo_internal.h"), os.path.join(CSRC, "decode_dev.cuh"), os.path.join(CSRC, "pilot_common.cuh"),
                                                        os.path.join(HERE, "..", "include", "dyo.h")]
     if not force and os.path.exists(OUT) and all(os.path.getmtime(OUT) >= os.path.getmtime(s) for s in srcs):
+        build_cpu_baseline()
         return OUT
     objs = []
     for f in CU:
@@ -41,7 +42,19 @@ def build(force=False, verbose=False):
               "-c", os.path.join(CSRC, f), "-o", o])
         objs.append(o)
     _run([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", OUT, *objs])
+    build_cpu_baseline()
     return OUT
+
+
+def build_cpu_baseline():
+    """The compiled single-core CPU planner (baseline/cpu_planner.cpp): a bench/test baseline,
+    not part of libdyo."""
+    src = os.path.join(HERE, "..", "baseline", "cpu_planner.cpp")
+    out = os.path.join(HERE, "..", "baseline", "libcpuplan.so")
+    if os.path.exists(out) and os.path.getmtime(out) >= os.path.getmtime(src):
+        return out
+    _run(["g++", "-O3", "-march=x86-64-v3", "-std=c++17", "-shared", "-fPIC", "-o", out, src])
+    return out
 
 
 if __name__ == "__main__":

@@ -667,6 +667,7 @@ def run_dyo(args):
         return
 
     value = bytes_all / (ms_max * 1e-3) / 1e9
+    host_numa = d.query("host_numa")
     # dominant kernel of the timed region among libdyo's kernels
     kern = {k: tm[k] for k in ("pilot", "decode", "plan", "copy_d2d", "copy_zc")}
     dom = max(kern, key=lambda k: kern[k]["ms"])
@@ -777,6 +778,9 @@ def run_dyo(args):
         "mechanisms": ctr,
         "gpu_launches": int(launches),
         "clocks": clk.summary(),
+        "host_pool": {"numa_node": host_numa, "gpu_topology": gpu_topology(local),
+                      "note": "pinned tensor homes bound to the GPU's NUMA node (mbind before cudaHostRegister; "
+                              "-1 = the platform reports no node)"},
         "e2e": {"value": round(bytes_all / e2e_max / 1e9, 3), "unit": "GB/s",
                 "h2d_bytes_per_step": int(wl.D_s * 8 + wl.h * 4), "d2h_bytes_per_step": int(16 * 4 + 9 * len(wl.tensors)),
                 "note": "dyo_* calls with pinned host sample descriptors; plan lists + residency read back each step"},
@@ -851,6 +855,23 @@ def compiled_planner_leg(torch, wl, dev, inputs, B, s0, n_steps, gpu_plan_us):
             "gpu_plan_us": round(gpu_plan_us, 2), "gpu_speedup": round(cpu_us / max(gpu_plan_us, 1e-9), 2),
             "sample": "the bench's first %d step inputs, W sets of the GPU decode, planned from an empty arena" % steps,
             "kind": "compiled single-core planner (baseline/cpu_planner.cpp, g++ -O3 -march=x86-64-v3)"}
+
+
+def gpu_topology(local):
+    """This GPU's row of `nvidia-smi topo -m` (GPU <-> GPU / NIC links, CPU and NUMA affinity) and
+    its PCIe link, for the multi-manager report (survey §8(e)); None if nvidia-smi is missing."""
+    import subprocess
+    try:
+        topo = subprocess.run(["nvidia-smi", "topo", "-m"], capture_output=True, text=True, timeout=20).stdout
+        lines = [ln for ln in topo.splitlines() if ln.strip()]
+        head = lines[0].split() if lines else []
+        row = next((ln for ln in lines[1:] if ln.split() and ln.split()[0] == f"GPU{local}"), None)
+        link = subprocess.run(["nvidia-smi", "-i", str(local), "--query-gpu=pci.bus_id,pcie.link.gen.current,"
+                               "pcie.link.width.current", "--format=csv,noheader"],
+                              capture_output=True, text=True, timeout=20).stdout.strip()
+        return {"header": " ".join(head), "row": " ".join(row.split()) if row else None, "pcie": link}
+    except (OSError, subprocess.SubprocessError):
+        return None
 
 
 def step_bound_ms(trs, h2d_gbs, d2h_gbs):

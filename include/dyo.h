@@ -398,6 +398,10 @@ dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr);
  *   DYO_Q_PLAN_SYNCS: host synchronisations taken by the last successful dyo_plan (1, §8(b)).
  *   DYO_Q_HOST_DECODE: 1 if the loaded arch's decode runs on the host (no branch head, or nested
  *     sites: dyo_pilot_predict synchronises its stream once, so it cannot be graph-captured).
+ *   DYO_Q_HOST_NUMA: NUMA node the pinned host pool is bound to (survey §8(e): each GPU's
+ *     manager uses its own host link): the node sysfs reports for the device's PCI address (or
+ *     $DYO_HOST_NUMA), pages bound with mbind before cudaHostRegister; -1 if the platform reports
+ *     no node or binding failed, in which case the pool is a plain cudaHostAlloc.
  * DYO_E_INVAL for a NULL ctx / value or an unknown `what`. */
 /* Measurement switch at run time: sets or clears DYO_F_TIMING (the only flag that may change
  * after dyo_create; DYO_E_INVAL for any other bit). With it clear no timing events are recorded,
@@ -408,6 +412,7 @@ dyo_status dyo_set_timing(dyo_ctx* ctx, int32_t on);
 #define DYO_Q_DECODE_FUSED 1
 #define DYO_Q_PLAN_SYNCS 2
 #define DYO_Q_HOST_DECODE 3
+#define DYO_Q_HOST_NUMA 4
 dyo_status dyo_query(dyo_ctx* ctx, int32_t what, int64_t* value);
 
 /* Per-ctx counters of the last dyo_plan / dyo_migrate calls (bytes by mechanism, launches). */

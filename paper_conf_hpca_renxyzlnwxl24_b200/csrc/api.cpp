@@ -12,6 +12,11 @@
 #include <string>
 #include <vector>
 
+#include <cctype>
+#include <sys/mman.h>
+#include <sys/syscall.h>
+#include <unistd.h>
+
 #include "dyo_internal.h"
 
 using namespace dyo;
@@ -40,6 +45,8 @@ struct dyo_ctx {
   int64_t staging_bytes = 0;
   char* host_pool = nullptr;
   int64_t host_bytes = 0;
+  int host_numa = -1;              // NUMA node the pool was bound to (-1: unbound, cudaHostAlloc)
+  bool host_registered = false;    // pool = mmap + mbind + cudaHostRegister (free with munmap)
   // prediction
   PredDev pd{};
   double* logits64 = nullptr;      // fp64 logits (decode decisions, R4)
@@ -689,6 +696,62 @@ void memo_free(dyo_ctx* ctx) {
   ctx->ad.memo_hits = nullptr;
 }
 
+// ---- NUMA-local pinned host pool (survey §8(e): each GPU's manager migrates over its own
+// host link, so its tensor homes belong on the GPU's NUMA node). The node comes from sysfs for the
+// device's PCI address; the pages are bound there (mbind, preferred) before cudaHostRegister faults
+// them in. Without a node (or if any step fails) the pool falls back to cudaHostAlloc.
+static int device_numa_node(int device) {
+  if (const char* e = getenv("DYO_HOST_NUMA")) return atoi(e);   // -1 disables binding
+  char bus[32] = {0};
+  if (cudaDeviceGetPCIBusId(bus, sizeof bus, device) != cudaSuccess) return -1;
+  for (char* c = bus; *c; ++c) *c = (char)tolower(*c);
+  char path[96];
+  snprintf(path, sizeof path, "/sys/bus/pci/devices/%s/numa_node", bus);
+  FILE* f = fopen(path, "r");
+  if (!f) return -1;
+  int node = -1;
+  if (fscanf(f, "%d", &node) != 1) node = -1;
+  fclose(f);
+  return node;
+}
+
+static void host_pool_free(dyo_ctx* ctx) {
+  if (!ctx->host_pool) return;
+  if (ctx->host_registered) {
+    cudaHostUnregister(ctx->host_pool);
+    munmap(ctx->host_pool, (size_t)std::max<int64_t>(ctx->host_bytes, 64));
+  } else {
+    cudaFreeHost(ctx->host_pool);
+  }
+  ctx->host_pool = nullptr;
+  ctx->host_registered = false;
+}
+
+static dyo_status host_pool_alloc(dyo_ctx* ctx, int64_t bytes) {
+  const size_t n = (size_t)std::max<int64_t>(bytes, 64);
+  ctx->host_numa = -1;
+  ctx->host_registered = false;
+  const int node = device_numa_node(ctx->device);
+  if (node >= 0 && node < 64) {
+    void* p = mmap(nullptr, n, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+    if (p != MAP_FAILED) {
+      unsigned long mask = 1UL << node;
+      const int MPOL_PREFERRED_ = 1;
+      bool ok = syscall(SYS_mbind, p, n, MPOL_PREFERRED_, &mask, 64UL, 0U) == 0;
+      if (ok && cudaHostRegister(p, n, cudaHostRegisterMapped | cudaHostRegisterPortable) == cudaSuccess) {
+        ctx->host_pool = (char*)p;
+        ctx->host_registered = true;
+        ctx->host_numa = node;
+        return DYO_OK;
+      }
+      cudaGetLastError();
+      munmap(p, n);
+    }
+  }
+  CK(cudaHostAlloc((void**)&ctx->host_pool, n, cudaHostAllocMapped | cudaHostAllocPortable));
+  return DYO_OK;
+}
+
 dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (!ctx) return DYO_E_INVAL;
   cudaSetDevice(ctx->device);
@@ -697,7 +760,7 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   free_owned(ctx, ctx->pilot_dev);
   memo_free(ctx);
   free_plan_host(ctx);
-  if (ctx->host_pool) cudaFreeHost(ctx->host_pool);
+  host_pool_free(ctx);
   if (ctx->h_logits) cudaFreeHost(ctx->h_logits);
   if (ctx->arena) cudaFree(ctx->arena);
   if (ctx->staging) cudaFree(ctx->staging);
@@ -732,7 +795,7 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
   memo_free(ctx);
   ctx->memo.mispredictions = 0;
   free_plan_host(ctx);
-  if (ctx->host_pool) { cudaFreeHost(ctx->host_pool); ctx->host_pool = nullptr; }
+  host_pool_free(ctx);
   ctx->arch_ok = false;
   const int64_t AL = ctx->cfg.align;
   ArchHost h;
@@ -904,8 +967,10 @@ dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
 #undef DA
   // ---- host pool (pinned, mapped: DMA and zero-copy kernels) ----
   ctx->host_bytes = pool;
-  if (!(ctx->cfg.flags & DYO_F_NO_HOST_POOL))
-    CK(cudaHostAlloc((void**)&ctx->host_pool, std::max<int64_t>(pool, 64), cudaHostAllocMapped | cudaHostAllocPortable));
+  if (!(ctx->cfg.flags & DYO_F_NO_HOST_POOL)) {
+    dyo_status hst = host_pool_alloc(ctx, pool);
+    if (hst) return hst;
+  }
   ctx->arch_ok = true;
   ctx->pilot_ok = false;
   return DYO_OK;
@@ -2445,6 +2510,7 @@ dyo_status dyo_query(dyo_ctx* ctx, int32_t what, int64_t* value) {
     case DYO_Q_DECODE_FUSED: *value = ctx->last_fused; return DYO_OK;
     case DYO_Q_PLAN_SYNCS: *value = ctx->last_plan_syncs; return DYO_OK;
     case DYO_Q_HOST_DECODE: *value = (!ctx->branch_head || ctx->nested) ? 1 : 0; return DYO_OK;
+    case DYO_Q_HOST_NUMA: *value = ctx->host_numa; return DYO_OK;
   }
   return DYO_E_INVAL;
 }

@@ -593,7 +593,7 @@ class Dyo:
     def set_timing(self, on):
         self._check(self.L.dyo_set_timing(self.ctx, 1 if on else 0))
 
-    QUERIES = {"pilot_kernel": 0, "decode_fused": 1, "plan_syncs": 2, "host_decode": 3}
+    QUERIES = {"pilot_kernel": 0, "decode_fused": 1, "plan_syncs": 2, "host_decode": 3, "host_numa": 4}
 
     def query(self, what):
         """dyo_query: 'pilot_kernel' (0 K1 cluster GEMV, 1 K1-TC), 'decode_fused', 'plan_syncs'."""

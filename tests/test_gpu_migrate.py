@@ -356,3 +356,30 @@ def test_tree_scaled_nested_bytes():
     wl = WL.make("tree", n_samples=16, batch=4, max_leaves=16, hidden=128, budget=8 << 20)
     m = run_bytes(wl, 2, 1, B=4)
     assert m["zc"] + m["dma"] > 0
+
+
+def _sysfs_numa_node(dev):
+    bus = torch.cuda.get_device_properties(dev)
+    pci = "%04x:%02x:%02x.0" % (bus.pci_domain_id, bus.pci_bus_id, bus.pci_device_id)
+    try:
+        with open(f"/sys/bus/pci/devices/{pci}/numa_node") as f:
+            return int(f.read().strip())
+    except OSError:
+        return -1
+
+
+def test_host_pool_numa_local_and_exact(monkeypatch):
+    """Survey §8(e) / P:L259: the pinned tensor homes sit on the GPU's NUMA node (mbind before
+    cudaHostRegister) when the platform reports one; bytes through that pool stay exact; the
+    DYO_HOST_NUMA=-1 override falls back to cudaHostAlloc."""
+    wl = WL.make("tiny", n_samples=16)
+    node = _sysfs_numa_node(0)
+    d = make_ctx(wl)
+    assert d.query("host_numa") == node
+    d.close()
+    m = run_bytes(wl, 2, 1)
+    assert m["dma"] > 0
+    monkeypatch.setenv("DYO_HOST_NUMA", "-1")
+    d = make_ctx(wl)
+    assert d.query("host_numa") == -1
+    d.close()

@@ -820,7 +820,8 @@ def compiled_planner_leg(torch, wl, dev, inputs, B, s0, n_steps, gpu_plan_us):
     sys.path.insert(0, os.path.join(ROOT, "baseline"))
     import cpu_planner
     from paper_conf_hpca_renxyzlnwxl24_b200 import Dyo
-    dc = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, device=dev, flags=0)
+    # plan-only manager (DYO_F_NO_HOST_POOL = 4): its plans are never migrated, each supersedes the last
+    dc = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, device=dev, flags=4)
     dc.load(wl)
     cp = cpu_planner.CpuPlanner(wl)
     n_sites = 4096

@@ -38,10 +38,12 @@ def run_checked(state, wl, Ws, policy, vs=None):
         tr = transition(st, wl, Ws, j, policy)
         # I3: nothing block j-1 uses is evicted or compacted at transition j
         assert not prev_set & {r[0] for r in tr.evict}, "I3 evict"
-        assert not prev_set & {r[0] for r in tr.move}, "I3 move"
+        assert tr.late_all or not prev_set & {r[0] for r in tr.move}, "I3 move"   # R20: late_all waits
         check_layout(st, wl)
-        for t, _, _ in Ws[j]:                       # I2: W_j resident in half m
-            assert st.loc[t] == tr.half, f"I2: tensor {t} not in half {tr.half}"
+        shared = {t for t, _ in tr.share}
+        for t, _, _ in Ws[j]:                       # I2: W_j resident in half m (or SHARE'd, R20)
+            assert st.loc[t] == tr.half or (t in shared and st.loc[t] == 1 - tr.half), \
+                f"I2: tensor {t} not in half {tr.half}"
         vs.apply(tr)
         bad = vs.run_block(Ws[j], tr.half, st, H)   # I4/I5 via versions read by block j
         assert not bad, f"stale read of tensors {bad} at block {j}"

@@ -60,14 +60,14 @@ class ByteSim:
         bad = []
         for t, mode, rd in Wj:
             nb = self.wl.tensors[t].nbytes
-            base = half * self.H + state.off[t]
+            base = state.loc[t] * self.H + state.off[t]      # half m, or 1-m when SHARE'd (R20)
             if rd and self._checked(t) and not np.array_equal(self.dev[base: base + nb],
                                                               content_bytes(t, self.ver[t], nb)):
                 bad.append(t)
         for t, mode, rd in Wj:
             if mode & W:
                 nb = self.wl.tensors[t].nbytes
-                base = half * self.H + state.off[t]
+                base = state.loc[t] * self.H + state.off[t]      # half m, or 1-m when SHARE'd (R20)
                 self.fresh.add(t)
                 self.ver[t] += 1
                 self.dev[base: base + nb] = content_bytes(t, self.ver[t], nb)
@@ -105,7 +105,7 @@ class VersionSim:
     def run_block(self, Wj, half, state, H):
         bad = []
         for t, mode, rd in Wj:
-            base = half * H + state.off[t]
+            base = state.loc[t] * H + state.off[t]          # half m, or 1-m when SHARE'd (R20)
             checked = not self.wl.tensors[t].transient or t in self.fresh
             if rd and checked and self.dev_ver.get(base) != (t, self.ver[t]):
                 bad.append(t)
@@ -113,5 +113,5 @@ class VersionSim:
             if mode & W:
                 self.fresh.add(t)
                 self.ver[t] += 1
-                self.dev_ver[half * H + state.off[t]] = (t, self.ver[t])
+                self.dev_ver[state.loc[t] * H + state.off[t]] = (t, self.ver[t])
         return bad

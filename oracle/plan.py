@@ -20,6 +20,13 @@ Transition j, in order:
      compacted: exclusive prefix sums over [kept by old offset | CARRY | ALLOC | FETCH]
   5. operation order (P:L180 evict first, then prefetch): EVICT writebacks, MOVE (compaction,
      ascending destination), CARRY, FETCH; then block j marks its written tensors dirty.
+
+Policy bit SHARE (reading R20): a tensor of W_j valid in half 1-m that the next group
+W_{j+1} also holds stays where it is (SHARE, no copy, no space in half m): block j reads it in
+the other half, and transition j+1 finds it in its own half (KEEP). While block j runs, transition
+j+1 must not move it, so a compaction of a half holding tensors of the running block waits for
+that block's end (the transition is `late_all`: its MOVE / CARRY / FETCH run after block j-1).
+Without SHARE every W_j tensor is in half m when block j starts (R1: ping-pong by D2D).
 """
 from __future__ import annotations
 
@@ -31,6 +38,7 @@ from workloads import R, W
 HOST = -1
 INF = 1 << 62
 PAPER, RETAIN = 0, 1
+SHARE = 2          # policy bit (R20); policy & 1 selects RETAIN
 
 
 class BudgetError(Exception):
@@ -61,6 +69,8 @@ class Transition:
     carry: list      # (t, src_abs, dst_abs, nbytes, late)
     alloc: list      # (t, dst_abs, nbytes)
     fetch: list      # (t, host_off, dst_abs, nbytes)
+    share: list = field(default_factory=list)   # (t, abs) of the W_j tensors left in half 1-m (R20)
+    late_all: bool = False                      # R20: MOVE / CARRY / FETCH wait for block j-1's end
     h2d: int = 0
     d2h: int = 0
     d2d: int = 0
@@ -150,22 +160,29 @@ def transition(state, wl, Ws, j, policy, choose=None, occ=None):
     a, nb, host_off = tensor_table(wl)
     m = (state.G + j) % 2
     Wj = Ws[j]
-    need = sum(a[t] for t, _, _ in Wj)
-    if need > H:
-        raise BudgetError(f"transition {j}: W_j needs {need} B > H = {H} B")
     in_w = {t for t, _, _ in Wj}
     prev_written = {t for t, mode, _ in state.prev if mode & W}
+    share_on = bool(policy & SHARE)
+    nxt = {t for t, _, _ in Ws[j + 1]} if share_on and j + 1 < len(Ws) else set()
+    # R20: tensors of the running block j-1 in half m (left there by SHARE at transition j-1)
+    pinned = {t for t, _, _ in state.prev if state.loc[t] == m}
 
-    keep, carry, alloc, fetch = [], [], [], []
+    keep, carry, alloc, fetch, share = [], [], [], [], []
     for t, mode, rd in Wj:
         if state.loc[t] == m:
             keep.append(t)
+        elif state.loc[t] == 1 - m and t in nxt:
+            share.append(t)
         elif state.loc[t] == 1 - m and rd:
             carry.append(t)
         elif rd:
             fetch.append(t)
         else:
             alloc.append(t)
+    shared = set(share)
+    need = sum(a[t] for t, _, _ in Wj if t not in shared)
+    if need > H:
+        raise BudgetError(f"transition {j}: W_j needs {need} B > H = {H} B")
 
     # eviction candidates: other valid tensors of half m
     cands = [t for t in range(T) if state.loc[t] == m and t not in in_w]
@@ -198,7 +215,9 @@ def transition(state, wl, Ws, j, policy, choose=None, occ=None):
     kept_all = sorted(keep + retained, key=lambda t: state.off[t])
     placed = sorted(carry) + sorted(alloc) + sorted(fetch, key=lambda t: (host_off[t], t))
     new_off = first_fit(kept_all, placed, state.off, a, H)
+    late_all = False
     if new_off is None:                   # fragmentation: compact (R11 fallback)
+        late_all = bool(pinned)           # R20: it moves tensors block j-1 is using: after its end
         new_off, cur = {}, 0
         for t in kept_all + placed:
             new_off[t] = cur
@@ -214,7 +233,8 @@ def transition(state, wl, Ws, j, policy, choose=None, occ=None):
     fetch_l = [(t, host_off[t], m * H + new_off[t], nb[t])
                for t in sorted(fetch, key=lambda t: (host_off[t], t))]
 
-    tr = Transition(j, m, need, evict, move, carry_l, alloc_l, fetch_l)
+    tr = Transition(j, m, need, evict, move, carry_l, alloc_l, fetch_l,
+                    [(t, (1 - m) * H + state.off[t]) for t in share], late_all)
     tr.h2d = sum(r[3] for r in fetch_l)
     tr.d2h = sum(r[3] for r in evict if r[4])
     tr.d2d = sum(r[3] for r in move) + sum(r[3] for r in carry_l)

@@ -78,6 +78,8 @@ struct StagePlan {
   int tab_off;            // >= 0: byte offset of the decode tables prefetched at launch (fused decode)
   int push_logits;        // 1: the output stage pushes its logits to every CTA (fused decode, C > 1)
   int red_off;            // batch path (BS > 1): byte offset of the DMMA tile table + K-split partials
+  int wbuf;               // doubles per sample of each activation buffer: the widest stage, and the
+                          // O logits when the output stage pushes them into a buffer (push_logits)
   int st_off[4 + kMaxLayers];
   int rpc[4 + kMaxLayers];      // rows per CTA of each stage
   int gsh[4 + kMaxLayers];      // log2 of the threads per row (k-split) of each stage
@@ -250,7 +252,7 @@ __device__ __forceinline__ void dmma_stage(const PilotDev& p, const StageDev& st
 
 // grid = n_clusters * C (cluster dims C set at launch). Dynamic smem:
 //   [mbarriers: n_stages (weights) + 2 (activation buffers)][staged weight slices]
-//   [activations 2 x BS x max_width doubles]
+//   [activations 2 x BS x wbuf doubles (wbuf = max_width, or O when the logits are pushed)]
 // With fuse_decode the weight region is reused for the decode (DecHead / DecGroup) afterwards.
 template <int BS>
 __global__ void __launch_bounds__(kPilotThreads)
@@ -295,7 +297,7 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();                       // descriptors + barrier inits visible in the CTA
-  const int W = p.max_width;
+  const int W = spc.wbuf;
   double* buf[2] = {act, act + BS * W};
   // ---- 0. TMA: lane si of warp 0 issues stage si's weight slice (all stages in flight at once)
   if (tid < p.n_stages && sp.st_off[tid] >= 0) {
@@ -681,7 +683,11 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   sp.fuse_decode = (a.branch_head && !a.hp_op && sp.Bs * a.K_max <= 2 * C) ? 1 : 0;
   sp.push_logits = (sp.fuse_decode && C > 1 && sp.Bs == 1 && p.n_stages > 1) ? 1 : 0;
   sp.tab_off = -1;
-  const int act_bytes = 2 * sp.Bs * p.max_width * (int)sizeof(double);
+  // the output stage's buffer holds O logits per sample when they are pushed (O may exceed every
+  // hidden width: MoE P512 O = 544 > 512; a narrow pilot, H256, would overflow the region)
+  const int o4 = (p.O + 3) / 4 * 4;
+  sp.wbuf = (sp.push_logits && o4 > p.max_width) ? o4 : p.max_width;
+  const int act_bytes = 2 * sp.Bs * sp.wbuf * (int)sizeof(double);
   const int base = ((2 * (4 + kMaxLayers) + 2) * 8 + 127) / 128 * 128;
   const int budget = kDynCap - act_bytes - (sp.Bs > 1 ? kDmmaRedBytes + 256 : 0);
   int off = base;

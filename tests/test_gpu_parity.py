@@ -62,6 +62,25 @@ def test_pilot_logits(name, B):
     d.close()
 
 
+@pytest.mark.parametrize("width", [32, 64, 128, 256, 1024, 2048])
+@pytest.mark.parametrize("B", [1, 64])
+def test_pilot_logits_width_sweep(width, B):
+    """The width-sweep pilots ("H<w>": P512's topology at hidden width w) meet the same
+    north_star gate at batch 1 and 64 (each width picks its own cluster size / samples per cluster)."""
+    wl = WL.make_moe(n_samples=max(16, B), pilot_kind=f"H{width}")
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    logits = torch.zeros((B, wl.pilot.O), device="cuda")
+    d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, stream=_stream())
+    torch.cuda.synchronize()
+    ids = range(0, B, 7) if B > 8 else range(B)
+    r = oracle_step(wl, ids, PL.initial_state(len(wl.tensors)), (), plan=False)
+    y = logits.cpu().numpy()
+    for i, b in enumerate(ids):
+        g1, g2, _ = logit_gates(y[b], r["feats"][i], wl.pilot, wl.nn_type)
+        assert g2.all() and g1.all(), f"width {width} sample {b}"
+    d.close()
+
+
 @pytest.mark.parametrize("name,B", [("tiny", 1), ("moe", 2), ("af", 1), ("lstm", 4)])
 def test_predict_from_encoded_features(name, B):
     """The unfused entry: dyo_encode_features -> device features -> dyo_pilot_predict(feat=...)

@@ -102,7 +102,7 @@ def test_pool_mode_belady_is_optimal(seed):
 
 
 @pytest.mark.parametrize("name,steps", [("tiny", 6), ("moe", 3), ("af", 1)])
-@pytest.mark.parametrize("policy", [0, 1])
+@pytest.mark.parametrize("policy", [0, 1, 2, 3])
 def test_invariants_on_configs(name, steps, policy):
     wl = WL.make(name)
     st_ = PL.initial_state(len(wl.tensors))
@@ -137,8 +137,71 @@ def test_invariants_random(seed):
     tens, Ws, budget = _random_trace(rng, T=9, K=7, budget=int(rng.choice([2048, 3072, 8192])))
     wl = _wl(tens, budget)
     st_ = PL.initial_state(len(tens))
-    for policy in (0, 1):
+    for policy in (0, 1, 2, 3):
         try:
             INV.run_checked(st_, wl, Ws, policy)
         except PL.BudgetError:
             pass
+
+
+@pytest.mark.parametrize("K", [2, 3, 6, 7])
+@pytest.mark.parametrize("policy", [0, 1])
+def test_share_running_state_closed_form(K, policy):
+    """R20 closed form: a running state t0 read and written by every block (the AlphaFold MSA/pair
+    state) ping-pongs by K-1 late carries without SHARE; with SHARE it never moves except a final
+    carry when it sits in the wrong half at the plan's last transition (K even), and every block
+    still reads the latest version (run_checked: I1-I5 on versions)."""
+    tens = [[512, 0, False]] + [[256, 512 + 256 * k, True] for k in range(K)]
+    wl = _wl(tens, 4096, policy)
+    Ws = [[(0, RW, True), (1 + k, W, False)] for k in range(K)]
+    trs, _, _ = INV.run_checked(PL.initial_state(K + 1), wl, Ws, policy)
+    carries = [(tr.j, r[0], r[4]) for tr in trs for r in tr.carry]
+    assert carries == [(j, 0, True) for j in range(1, K)]
+    trs, _, _ = INV.run_checked(PL.initial_state(K + 1), wl, Ws, policy | PL.SHARE)
+    carries = [(tr.j, r[0], r[4]) for tr in trs for r in tr.carry]
+    assert carries == ([(K - 1, 0, True)] if K % 2 == 0 else [])
+    assert [tr.j for tr in trs if tr.share] == [j for j in range(1, K - 1) if j % 2 == 1]
+    assert sum(tr.d2d for tr in trs) == (512 if K % 2 == 0 else 0)
+
+
+def test_share_needs_the_next_group_and_frees_half_m():
+    """R20 eligibility: only a tensor the next group also holds stays in the other half (a tensor
+    used by j-1 and j only is carried as in R1), and a SHARE'd tensor takes no room in half m."""
+    wl = _wl([[512, 0, False], [512, 512, False], [512, 1024, True]], 2048, 1)   # H = 1024
+    Ws = [[(0, R, True), (1, R, True)], [(0, R, True), (1, R, True)], [(0, R, True), (2, W, False)]]
+    trs, _, _ = INV.run_checked(PL.initial_state(3), wl, Ws, 1 | PL.SHARE)
+    assert trs[1].share == [(0, 0)] and [r[0] for r in trs[1].carry] == [1]
+    assert trs[1].need == 512
+    # without SHARE block 1 needs both in half 1 (1024 = H): fits, both carried
+    trs, _, _ = INV.run_checked(PL.initial_state(3), wl, Ws, 1)
+    assert [r[0] for r in trs[1].carry] == [0, 1] and trs[1].need == 1024
+
+
+def _share_late_checked(seed):
+    """R20: a transition compacts a half holding tensors of the running block j-1 only as a late
+    transition (after block j-1 ends); otherwise no MOVE touches W_{j-1} (I3, run_checked)."""
+    rng = np.random.default_rng(seed)
+    tens, Ws, budget = _random_trace(rng, T=9, K=8, budget=int(rng.choice([1536, 2048, 3072])))
+    wl = _wl(tens, budget)
+    try:
+        trs, _, _ = INV.run_checked(PL.initial_state(len(tens)), wl, Ws, 1 | PL.SHARE)
+    except PL.BudgetError:
+        return []
+    for j, tr in enumerate(trs):
+        pinned = {t for t, _ in (trs[j - 1].share if j else [])}
+        if tr.late_all:
+            assert pinned
+        if pinned & {r[0] for r in tr.move}:
+            assert tr.late_all
+    return trs
+
+
+@pytest.mark.parametrize("seed", [204, 505, 710, 1227])     # seeds whose plans compact under SHARE'd tensors
+def test_share_late_all_cases(seed):
+    assert any(tr.late_all for tr in _share_late_checked(seed))
+
+
+@settings(max_examples=60, deadline=None)
+@given(st.integers(0, 10 ** 6))
+def test_share_late_all_random(seed):
+    _share_late_checked(seed)

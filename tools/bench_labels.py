@@ -176,7 +176,8 @@ epochs = 20 if quick else 200
 for ep in range(epochs):
     for b0 in range(0, n_train, 64):
         L = tr.step(feats[b0:b0 + 64], T[b0:b0 + 64], 64, lr=0.01, stream=s0.cuda_stream, want_loss=(b0 == 0))
-    losses.append(L)
+        if b0 == 0:
+            losses.append(L)           # the epoch's first minibatch loss (the others are not read back)
 w = tr.weights()
 tr.close()
 import copy

@@ -7,7 +7,7 @@ from paper_conf_hpca_renxyzlnwxl24_b200 import Dyo
 cfg = sys.argv[1] if len(sys.argv) > 1 else "moe"
 B = int(sys.argv[2]) if len(sys.argv) > 2 else 64
 wl = WL.make(cfg, n_samples=max(64, B))
-d = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, flags=4 | 8)
+d = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, flags=4 | 8 | 32)   # 32: DYO_F_PILOT_TC
 d.load(wl)
 s = torch.cuda.current_stream()
 desc = torch.from_numpy(wl.samples[:B].copy()).cuda()

@@ -82,17 +82,20 @@ int32_t cpu_plan(void* sp, int32_t T, const int64_t* bytes, const int64_t* host_
     const int m = (int)((st.G + j) & 1);
     const int e0 = ent_ptr[j], e1 = ent_ptr[j + 1];
     int64_t need = 0;
-    for (int e = e0; e < e1; ++e) need += a[ent_t[e]];
-    if (need > H) return -3;
     keep.clear(); carry.clear(); alloc.clear(); fetch.clear();
     for (int e = e0; e < e1; ++e) {
       const int t = ent_t[e];
       inw[t] = 1;
+      // R20 (policy bit 2): valid in the other half and held by the next group -> stays there
+      const bool share = (policy & 2) && st.loc[t] == 1 - m && nxt[e] == j + 1;
+      if (!share) need += a[t];
       if (st.loc[t] == m) keep.push_back(t);
+      else if (share) continue;
       else if (st.loc[t] == 1 - m && ent_rd[e]) carry.push_back(t);
       else if (ent_rd[e]) fetch.push_back(t);
       else alloc.push_back(t);
     }
+    if (need > H) return -3;
     // candidates of half m
     live.clear();
     evicted.clear();
@@ -106,7 +109,7 @@ int32_t cpu_plan(void* sp, int32_t T, const int64_t* bytes, const int64_t* host_
       if (!dead) live.emplace_back(nx[t] < 0 ? (int64_t)1 << 62 : (int64_t)(nx[t] - j), a[t], t);
     }
     std::vector<int32_t> ret;
-    if (policy == 1) {
+    if (policy & 1) {
       std::sort(live.begin(), live.end());
       int64_t used = 0;
       for (auto& x : live) {

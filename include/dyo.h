@@ -50,7 +50,9 @@ typedef struct dyo_ctx dyo_ctx;
 typedef struct {
   int64_t budget;         /* B: device arena bytes, split in two equal halves (R7) */
   int32_t align;          /* ALIGN in bytes (power of two >= 16; 256 in all configs) */
-  int32_t policy;         /* 0 = PAPER (evict every unused tensor), 1 = RETAIN (R10) */
+  int32_t policy;         /* bit 0: 0 = PAPER (evict every unused tensor), 1 = RETAIN (R10);
+                             bit 1: SHARE (R20): a W_j tensor valid in the other half that
+                             W_{j+1} also holds stays in place (no D2D carry) */
   int32_t max_batch;      /* max predictions per dyo_pilot_predict call (1..1024) */
   int32_t max_groups;     /* max groups per dyo_plan (sum over its predictions), <= 65535 */
   int32_t max_entries;    /* capacity of tensor-set entries per dyo_plan (0 = 512 per group) */
@@ -158,6 +160,9 @@ typedef struct {
   int32_t n_evict, n_move, n_carry, n_alloc, n_fetch;
   int64_t need;                 /* aligned bytes of W_j */
   int64_t h2d, d2h, d2d;        /* algorithmic bytes (FETCH; written-back EVICT; MOVE + CARRY) */
+  int32_t n_share;              /* R20: W_j tensors left in half 1-m (their entry records' dst) */
+  int32_t late_all;             /* R20: 1 if MOVE / CARRY / FETCH wait for block j-1 (compaction of a
+                                   half holding tensors block j-1 SHARE'd); dyo_migrate honours it */
 } dyo_transition_info;
 
 /* Plan records as stored by libdyo (little-endian int64 fields, absolute device offsets into

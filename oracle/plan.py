@@ -200,7 +200,7 @@ def transition(state, wl, Ws, j, policy, choose=None, occ=None):
     room = H - need
     if choose is not None:
         retained = list(choose(live, room))
-    elif policy == RETAIN:
+    elif policy & RETAIN:                  # bit 0 (bit 1 is SHARE, R20)
         retained = prefix_cut(live, room)
     else:
         retained = []

@@ -646,7 +646,7 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   ctx->device = device;
   dyo_config& c = ctx->cfg;
   if (c.align <= 0 || (c.align & (c.align - 1)) || c.align < 16 || c.budget < 2 * c.align ||
-      c.max_batch < 1 || c.max_batch > 1024 || c.policy < 0 || c.policy > 1) {
+      c.max_batch < 1 || c.max_batch > 1024 || c.policy < 0 || c.policy > 3) {
     delete ctx;
     return DYO_E_INVAL;
   }
@@ -1791,6 +1791,8 @@ dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info) {
   info->half = h.half; info->n_entries = h.n_ent; info->n_evict = h.n_evict; info->n_move = h.n_move;
   info->n_carry = h.n_carry; info->n_alloc = h.n_alloc; info->n_fetch = h.n_fetch;
   info->need = h.need; info->h2d = h.h2d; info->d2h = h.d2h; info->d2d = h.d2d;
+  info->n_share = h.flags >> 1;
+  info->late_all = h.flags & 1;
   return DYO_OK;
 }
 
@@ -2052,6 +2054,9 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   TRACE("  evict phase issued");
   CK(cudaEventRecord(ctx->ev_evict, sd));
   CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
+  // R20: this transition compacts a half that holds tensors the running block j-1 SHARE'd, so
+  //      its MOVE / CARRY / FETCH wait for block j-1 to end (the EVICTs above never touch them)
+  if ((h.flags & 1) && ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
 
   // 2. MOVE (compaction, R11/R12), ascending destination. Processed in order, moves are safe
   //    (new <= old and every destination ends below the later sources), but run in parallel a

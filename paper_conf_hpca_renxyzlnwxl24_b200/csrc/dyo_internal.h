@@ -22,7 +22,7 @@ constexpr int kMaxSites = 4096;
 constexpr int kEntCap = 1024;             // tensor-set entries per group (records before dedupe)
 constexpr int kPlanThreads = 1024;
 
-enum OpClass : int8_t { C_KEEP = 0, C_CARRY = 1, C_ALLOC = 2, C_FETCH = 3 };
+enum OpClass : int8_t { C_KEEP = 0, C_CARRY = 1, C_ALLOC = 2, C_FETCH = 3, C_SHARE = 4 };   // C_SHARE: R20
 
 // ---- pilot --------------------------------------------------------------------------
 constexpr int kMaxLayers = 16;
@@ -174,7 +174,7 @@ struct PlanState {
   int32_t* pos;       // T: index of a valid tensor's record in its half's current list
 };
 struct PlanHdr {      // per transition (device + pinned mirror)
-  int32_t half, n_ent, n_evict, n_move, n_carry, n_alloc, n_fetch, pad;
+  int32_t half, n_ent, n_evict, n_move, n_carry, n_alloc, n_fetch, flags;   // flags: bit 0 late_all, >> 1 n_share (R20)
   int64_t need, h2d, d2h, d2d;
   int64_t o_ent, o_evict, o_move, o_carry, o_alloc, o_fetch;  // record offsets
 };

@@ -423,9 +423,11 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
   }
   for (int w = tid; w < nwords; w += PNT) inw[w] = 0u;
   for (int h = tid; h < kHash; h += PNT) S.h_key[h] = -1;
-  __shared__ int s_n[2], s_sel[2], s_prev_n;
+  __shared__ int s_n[2], s_sel[2], s_prev_n, s_prev_share;
+  const bool share_on = (policy & 2) != 0;        // R20
   if (tid == 0) {
     s_prev_n = in.prev_n[0];
+    s_prev_share = 0;      // a plan's last transition never SHAREs (no next group): nothing pinned at j = 0
     for (int h = 0; h < 2; ++h) { s_n[h] = in.rl_meta[h]; s_sel[h] = in.rl_meta[2 + h]; }
   }
   __syncthreads();
@@ -474,7 +476,11 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
         const int64_t host = a.t_host[t], bytes = a.t_bytes[t];
         const int nx = sc.nxt[eb + e];
         const int nxrd = sc.nxt_rd[eb + e];
-        const int c = l == m ? C_KEEP : (l == 1 - m && rd ? C_CARRY : (rd ? C_FETCH : C_ALLOC));
+        // R20 (policy bit 2): a tensor valid in the other half that the next group also holds
+        // stays there (SHARE); nx == j + 1 <=> t is in W_{j+1} of this plan
+        const int c = l == m ? C_KEEP
+                    : (l == 1 - m && share_on && nx == j + 1) ? C_SHARE
+                    : (l == 1 - m && rd ? C_CARRY : (rd ? C_FETCH : C_ALLOC));
         S.e_t[e] = t;
         S.e_off[e] = (int)(off / AL);
         S.e_pos[e] = pos;
@@ -492,15 +498,16 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
         uint32_t h = hash_t(t);
         while (atomicCAS(&S.h_key[h], -1, t) != -1) h = (h + 1) & (kHash - 1);
         S.h_val[h] = e;
-        v4[0] += au;
-        v4[1] += c == C_CARRY;
+        v4[0] += c == C_SHARE ? 0 : au;               // a SHARE'd tensor takes no room in half m
+        v4[1] += (c == C_CARRY) + ((long long)(c == C_SHARE) << 32);
         v4[2] += c == C_ALLOC;
         v4[3] += c == C_FETCH;
       }
     }
     sum4(v4, S.tmp4);
     const long long need_u = v4[0];
-    const int nc = (int)v4[1], na = (int)v4[2], nf = (int)v4[3];
+    const int nc = (int)(v4[1] & 0xffffffffll), na = (int)v4[2], nf = (int)v4[3];
+    const int nsh = (int)(v4[1] >> 32);
     if (need_u > Hu) {
       if (tid == 0) { status[0] = DYO_E_BUDGET; status[1] = j; status[2] = 0; }
       return;
@@ -527,7 +534,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
       live_u = w4[0];
     }
     // eviction rule: 0 evict every live candidate (PAPER), 1 keep all (RETAIN, fits), 2 cut
-    const int rule = policy == 0 ? 0 : (live_u <= room ? 1 : 2);
+    const int rule = (policy & 1) == 0 ? 0 : (live_u <= room ? 1 : 2);
     PSTAMP(2);
     // ---- C. RETAIN prefix cut by radix select: the smallest key K* whose prefix sum of
     //      aligned sizes (keys ascending) exceeds the room; keys >= K* are evicted
@@ -671,7 +678,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
 #pragma unroll
     for (int q = 0; q < kEntCap / PNT; ++q) {
       const int e = tid + q * PNT;
-      if (e < n && S.e_cls[e] != C_KEEP) {
+      if (e < n && S.e_cls[e] != C_KEEP && S.e_cls[e] != C_SHARE) {
         const int c = S.e_cls[e], t = S.e_t[e];
         const uint64_t rank = c == C_CARRY ? 0 : (c == C_ALLOC ? 1 : 2);
         const uint64_t mid = c == C_FETCH ? (uint64_t)(S.e_host[e] / AL) : 0;
@@ -965,11 +972,11 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
         r.t = t;
         r.mode = S.e_mode[e];
         r.needs_fetch = S.e_rd[e];
-        r.dst = (int64_t)m * a.H + (int64_t)S.e_newoff[e] * AL;
+        r.dst = (int64_t)(S.e_cls[e] == C_SHARE ? 1 - m : m) * a.H + (int64_t)S.e_newoff[e] * AL;
         out.ent[eb + e] = r;
         const int wr = (S.e_mode[e] & 2) ? 1 : 0;
         // dirty: CARRY/KEEP keep theirs, ALLOC/FETCH start clean; block j's writes set it
-        const int dirty = wr || ((S.e_cls[e] == C_KEEP || S.e_cls[e] == C_CARRY) && (S.e_fl[e] & 4));
+        const int dirty = wr || ((S.e_cls[e] == C_KEEP || S.e_cls[e] == C_CARRY || S.e_cls[e] == C_SHARE) && (S.e_fl[e] & 4));
         st.dirty[t] = (uint8_t)dirty;
         S.e_fl[e] = (uint8_t)((S.e_fl[e] & ~4) | (dirty ? 4 : 0));
         st.pw[t] = (uint8_t)wr;
@@ -1108,6 +1115,9 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
       hd.n_carry = nc;
       hd.n_alloc = na;
       hd.n_fetch = nf;
+      // R20: a compaction of a half holding tensors the running block j-1 SHARE'd waits for its end
+      hd.flags = (compact && s_prev_share > 0 ? 1 : 0) | (nsh << 1);
+      s_prev_share = nsh;
       hd.need = need_u * AL;
       hd.o_evict = c_ev;
       hd.o_move = c_mv;

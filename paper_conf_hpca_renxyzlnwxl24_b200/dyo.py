@@ -57,7 +57,8 @@ class ArchSummary(C.Structure):
 
 class TransitionInfo(C.Structure):
     _fields_ = [("half", i32), ("n_entries", i32), ("n_evict", i32), ("n_move", i32), ("n_carry", i32),
-                ("n_alloc", i32), ("n_fetch", i32), ("need", i64), ("h2d", i64), ("d2h", i64), ("d2d", i64)]
+                ("n_alloc", i32), ("n_fetch", i32), ("need", i64), ("h2d", i64), ("d2h", i64), ("d2d", i64),
+                ("n_share", i32), ("late_all", i32)]
 
 
 class Counters(C.Structure):

@@ -21,7 +21,8 @@ def planner():
 
 
 @pytest.mark.parametrize("name,steps,B,policy,kw", [
-    ("tiny", 6, 1, 1, {}), ("tiny", 6, 1, 0, {}), ("moe", 3, 1, 1, {}),
+    ("tiny", 6, 1, 1, {}), ("tiny", 6, 1, 0, {}), ("moe", 3, 1, 1, {}), ("tiny", 6, 1, 3, {}), ("af", 1, 1, 3, {}),
+    ("lstm", 2, 8, 3, {"batch": 8, "max_len": 96, "n_samples": 32}),
     ("lstm", 2, 8, 1, {"batch": 8, "max_len": 96, "n_samples": 32}),
     ("tree", 2, 8, 1, {"batch": 8, "max_leaves": 24, "budget": 64 << 20, "n_samples": 32})])
 def test_cpu_planner_bitexact(planner, name, steps, B, policy, kw):

@@ -162,7 +162,7 @@ def test_lstm_scaled_small_tensors_zero_copy():
     assert m["zc"] > 0
 
 
-def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0, lookahead=False):
+def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0, lookahead=False, spin=0):
     """The full event protocol, enqueued asynchronously: emulated compute block j runs on its own
     stream after ready[j]; transition j's EVICT waits end[j-2], its late carries end[j-1].
     Read mismatches are accumulated on the device; the host syncs once per step."""
@@ -208,6 +208,8 @@ def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0, lookahead=False)
             d.migrate(j, s_copy.cuda_stream, hf.cuda_event, pd.cuda_event, ready[j].cuda_event)
             s_comp.wait_event(ready[j])
             with torch.cuda.stream(s_comp):
+                if spin:                       # a long block: transition j+1 overlaps it
+                    torch.cuda._sleep(spin)
                 for (t, mode, rd, dst) in ents[j]:
                     nb = wl.tensors[t].nbytes
                     if rd and (not wl.tensors[t].transient or t in fresh):
@@ -383,3 +385,36 @@ def test_host_pool_numa_local_and_exact(monkeypatch):
     d = make_ctx(wl)
     assert d.query("host_numa") == -1
     d.close()
+
+
+def _tiny_share_late():
+    wl = WL.make("tiny", seed=0, n_samples=32)
+    wl.budget = 384 << 20            # RETAIN + SHARE here: ~45 SHARE'd tensors and 9 late_all compactions in 10 steps
+    from oracle import run as OR
+    trs = [t for r in OR.run(wl, 6, policy=3) for t in r.transitions]
+    assert any(t.late_all for t in trs) and any(t.share for t in trs)
+    return wl
+
+
+def test_share_bytes_tiny():
+    """R20 SHARE: blocks read SHARE'd tensors in the other half; compactions under the running
+    block's tensors wait for its end (late_all); every read sees its latest version."""
+    run_bytes(_tiny_share_late(), 6, 3)
+
+
+def test_share_pipelined_long_blocks():
+    """The asynchronous protocol with long emulated blocks (spin before the reads): a late_all
+    transition that did not wait for block j-1 would move its tensors under it."""
+    run_pipelined(_tiny_share_late(), 6, 3, spin=2_000_000)
+
+
+def test_share_af_scaled():
+    wl = WL.make_af(seed=1, n_samples=8, act_mib=1, weight_mib=1, blocks=8, budget=64 << 20)
+    for t in wl.tensors:
+        t.nbytes = min(t.nbytes, 1 << 20)
+    off = 0
+    for t in wl.tensors:
+        t.host_off = off
+        off += (t.nbytes + 255) // 256 * 256
+    run_bytes(wl, 3, 3)
+    run_pipelined(wl, 2, 3, spin=200_000)

@@ -148,12 +148,17 @@ def _run_plan_steps(wl, steps, B=1, policy=None, flags=F_NO_HOST_POOL):
                 assert (info["half"], info["h2d"], info["d2h"], info["d2d"], info["need"]) == \
                     (tr.half, tr.h2d, tr.d2h, tr.d2d, tr.need), f"step {s} transition {j}"
                 assert gpu_lists(d, j) == tr_lists(tr), f"step {s} transition {j}"
+                # R20: SHARE'd tensors (their entry records point into half 1-m) and late_all
+                assert (info["n_share"], info["late_all"]) == (len(tr.share), int(tr.late_all)), f"step {s} tr {j}"
+                if tr.share:
+                    ent = {int(e[0]): int(e[3]) for e in d.plan_records(j, 5)}
+                    assert all(ent[t] == dst for t, dst in tr.share), f"step {s} transition {j}"
             st = r["state"]
         table = r["table"]
     return d
 
 
-@pytest.mark.parametrize("policy", [0, 1])
+@pytest.mark.parametrize("policy", [0, 1, 2, 3])
 @pytest.mark.parametrize("name,steps,B", [("tiny", 8, 1), ("tiny", 3, 8), ("moe", 6, 1), ("af", 3, 1)])
 def test_plan_bitexact(name, steps, B, policy):
     wl = WL.make(name, n_samples=32)
@@ -165,8 +170,8 @@ def test_plan_tight_budgets_and_errors(budget_mib):
     """Tight budgets: evictions with writeback, compaction, and DYO_E_BUDGET (transactional)."""
     wl = WL.make("tiny", n_samples=32)
     wl.budget = budget_mib << 20
-    _run_plan_steps(wl, 10, 1, 0).close()
-    _run_plan_steps(wl, 10, 1, 1).close()
+    for policy in (0, 1, 3):
+        _run_plan_steps(wl, 10, 1, policy).close()
 
 
 def test_unplanted_pilot_random_partitions():
@@ -251,7 +256,7 @@ def test_plan_bitexact_traversal():
     _run_plan_steps(wl, 4, 2, 1).close()
 
 
-@pytest.mark.parametrize("policy", [0, 1])
+@pytest.mark.parametrize("policy", [0, 1, 3])
 def test_plan_bitexact_lstm_scaled(policy):
     """Var-length LSTM (configs[3] variant): per-timestep / per-sample tensors (R13), reversed
     backward loop, batch of 8 predictions planned as one sequence, two consecutive steps."""
@@ -264,17 +269,19 @@ def test_plan_bitexact_lstm_fullsize():
     _run_plan_steps(wl, 1, 8, 1).close()
 
 
-def test_plan_bitexact_lstm_batch64_bench_config():
+@pytest.mark.parametrize("policy", [1, 3])
+def test_plan_bitexact_lstm_batch64_bench_config(policy):
     """The bench's LSTM configuration: 64 predictions (K1-TC + batch decode), 1,024 transitions
-    planned as one sequence, RETAIN; every record of every transition bit-exact, one host sync."""
+    planned as one sequence, RETAIN (+ SHARE, R20); every record of every transition bit-exact,
+    one host sync."""
     wl = WL.make("lstm", n_samples=64)
-    d = _run_plan_steps(wl, 1, 64, 1)
+    d = _run_plan_steps(wl, 1, 64, policy)
     assert d.query("plan_syncs") == 1
     assert d.query("pilot_kernel") == 0
     d.close()
 
 
-@pytest.mark.parametrize("policy", [0, 1])
+@pytest.mark.parametrize("policy", [0, 1, 3])
 def test_plan_bitexact_tree_scaled(policy):
     """Tree-LSTM (configs[3] primary): nested leaf/internal site per node (R16), per-(sample,
     node) tensors (R13), batch of 8 predictions planned as one sequence, two steps."""

@@ -10,7 +10,8 @@ budgets = [float(x) for x in (sys.argv[1] if len(sys.argv) > 1 else "1,2,4,8,16,
 rows = []
 for b in budgets:
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--config", "af", "--budget-gib", str(b),
-                        "--steps", os.environ.get("SWEEP_STEPS", "4"), "--warmup", "2", "--no-cpu-baseline"], capture_output=True, text=True)
+                        "--steps", os.environ.get("SWEEP_STEPS", "4"), "--warmup", "2", "--no-cpu-baseline", "--no-faults",
+                        "--policy", os.environ.get("SWEEP_POLICY", "1")], capture_output=True, text=True)
     try:
         d = json.loads(r.stdout.strip().splitlines()[-1])
     except Exception:
@@ -25,4 +26,4 @@ for b in budgets:
     rows.append(row)
     print(json.dumps(row), flush=True)
 ok = [r for r in rows if r["exposed_frac"] is not None and r["exposed_frac"] <= 0.05]
-print(json.dumps({"B_star_0_gib": min(r["budget_gib"] for r in ok) if ok else None, "rows": rows}))
+print(json.dumps({"policy": int(os.environ.get("SWEEP_POLICY", "1")), "B_star_0_gib": min(r["budget_gib"] for r in ok) if ok else None, "rows": rows}))

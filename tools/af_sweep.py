@@ -20,10 +20,15 @@ for b in budgets:
     ce = d.get("compute_emulation") or {}
     row = {"budget_gib": b, "ms_per_step": d["ms_per_step"], "compute_ms": ce.get("compute_ms_per_step"),
            "exposed_ms": ce.get("exposed_ms_per_step"), "exposed_frac": ce.get("exposed_frac_of_compute"),
+           "compute_only_ms": ce.get("compute_only_ms_per_step"), "exposed_vs_compute_only_ms": ce.get("exposed_vs_compute_only_ms"),
+           "exposed_vs_compute_only_frac": ce.get("exposed_vs_compute_only_frac"),
            "migration_gbs": d["value"], "h2d_GB_step": round(d["h2d_bytes_per_step"] / 1e9, 3),
            "d2h_GB_step": round(d["d2h_bytes_per_step"] / 1e9, 3), "plan_us": d["plan_us"],
            "h2d_dma_gbs": d["pcie"]["h2d_dma_gbs"], "d2h_dma_gbs": d["pcie"]["d2h_dma_gbs"]}
     rows.append(row)
     print(json.dumps(row), flush=True)
 ok = [r for r in rows if r["exposed_frac"] is not None and r["exposed_frac"] <= 0.05]
-print(json.dumps({"policy": int(os.environ.get("SWEEP_POLICY", "1")), "B_star_0_gib": min(r["budget_gib"] for r in ok) if ok else None, "rows": rows}))
+ok2 = [r for r in rows if r.get("exposed_vs_compute_only_frac") is not None and r["exposed_vs_compute_only_frac"] <= 0.05]
+print(json.dumps({"policy": int(os.environ.get("SWEEP_POLICY", "1")),
+                  "B_star_0_gib": min(r["budget_gib"] for r in ok) if ok else None,
+                  "B_star_0_gib_vs_compute_only": min(r["budget_gib"] for r in ok2) if ok2 else None, "rows": rows}))

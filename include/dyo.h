@@ -70,6 +70,9 @@ typedef struct {
 #define DYO_F_PILOT_TC 32     /* batches >= 16 on K1-TC (tcgen05 kind::tf32, 3xTF32, fp32 accumulation; reading
                                * R14's componentwise tolerance) instead of the default K1 batch path (fp64
                                * DMMA tensor-core tiles, fp64 accumulation: the north_star gate) */
+#define DYO_F_STRICT_ORDER 64 /* R12's strict phase order in dyo_migrate: every FETCH waits for the whole EVICT
+                               * phase (default: reading R21, a FETCH DMA waits only for block j-2 and the
+                               * write-backs whose device range it overwrites) */
 
 /* Static architecture: the DyNN program in preorder, its operators and the
  * tensor table. All arrays are HOST memory; dyo_load_arch copies what it needs. */
@@ -294,8 +297,13 @@ dyo_status dyo_plan_records(dyo_ctx* ctx, int32_t j, int32_t list, const void** 
  *   run or one K5 zero-copy gather), late CARRY after ev_prev_done (end of block j-1; may be
  *   NULL), and finally ev_ready (may be NULL), which block j must wait on.
  * Because EVICT_j only waits for block j-2, it overlaps transition j-1's fetches (P:L176's
- * double buffer; PCIe is full duplex). Host-non-blocking; all transitions of a plan may be
- * enqueued at once. */
+ * double buffer; PCIe is full duplex). Reading R21 (default; DYO_F_STRICT_ORDER restores R12's
+ * phase order): in a transition without compaction MOVEs and with at most 64 write-backs, each
+ * FETCH DMA waits only for ev_half_free and for the write-backs whose device range it overwrites,
+ * so the H2D link starts while later write-backs still run D2H; CARRYs, zero-copy fetches and
+ * ev_ready still follow the whole EVICT phase. The plan (layout, records, bytes) is unchanged.
+ * A late_all transition (R20) runs MOVE / CARRY / FETCH after ev_prev_done.
+ * Host-non-blocking; all transitions of a plan may be enqueued at once. */
 dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half_free,
                        void* ev_prev_done, void* ev_ready);
 

@@ -147,6 +147,7 @@ struct dyo_ctx {
   cudaStream_t d2h = nullptr;      // ctx-owned stream for the EVICT (D2H) phase
   cudaStream_t side = nullptr;     // ctx-owned stream for early CARRY (overlaps FETCH)
   cudaEvent_t ev_entry = nullptr, ev_evict = nullptr, ev_moves = nullptr, ev_carry = nullptr;
+  std::vector<cudaEvent_t> ev_wb;   // R21: one per write-back copy group of a transition (D2H stream order)
   dyo_counters ctr{};
   int sm_count = 148;
   // DYO_F_TIMING: event pairs per launch kind
@@ -782,6 +783,7 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->h_memo_stage) cudaFreeHost(ctx->h_memo_stage);
   for (auto& t : ctx->tm) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+  for (auto e : ctx->ev_wb) cudaEventDestroy(e);
   if (ctx->ev_ref) cudaEventDestroy(ctx->ev_ref);
   delete ctx;
   return DYO_OK;
@@ -1983,6 +1985,30 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   char* stage_pack = ctx->staging;                 // D2H stream
   char* stage_move = ctx->staging + stage_half;    // copy stream
 
+  // R21: FETCH DMAs wait only for the write-backs whose device range they overwrite (and for
+  //      block j-2, the last user of half m), not for the whole EVICT phase. Applies when the
+  //      transition has no compaction MOVEs and a bounded number of write-backs; otherwise the
+  //      phase order is strict (R12). wb_iv: (src range, index of its copy group's event).
+  int n_wb = 0;
+  for (int i = 0; i < h.n_evict; ++i) n_wb += P.out.ev[h.o_evict + i].writeback ? 1 : 0;
+  const bool relaxed = h.n_move == 0 && ev_half_free && n_wb > 0 && n_wb <= 64 &&
+                       !(ctx->cfg.flags & DYO_F_STRICT_ORDER) && !(h.flags & 1);
+  struct WbIv { int64_t lo, hi; int ev; };
+  std::vector<WbIv> wb_iv;
+  int n_wb_ev = 0;
+  auto wb_mark = [&](const dyo_evict_rec* ev0, int a0, int a1, bool only_wb) -> dyo_status {
+    if (!relaxed) return DYO_OK;
+    if (n_wb_ev == (int)ctx->ev_wb.size()) {
+      cudaEvent_t e;
+      CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+      ctx->ev_wb.push_back(e);
+    }
+    CK(cudaEventRecord(ctx->ev_wb[n_wb_ev], sd));
+    for (int q = a0; q < a1; ++q)
+      if (!only_wb || ev0[q].writeback) wb_iv.push_back({ev0[q].src, ev0[q].src + ev0[q].bytes, n_wb_ev});
+    ++n_wb_ev;
+    return DYO_OK;
+  };
   // 1. EVICT writebacks (D2H): host runs (ascending host offset) -> DMA (direct, or K3 packed
   //    through staging when the device sources are scattered), or one zero-copy scatter launch
   //    (K5) for the runs below dma_min
@@ -2011,6 +2037,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
           CK(cudaMemcpyAsync(host + r.host_off, arena + r.dev_off, r.bytes, cudaMemcpyDeviceToHost, sd)); }
         ctx->ctr.d2h_dma += r.bytes;
         ctx->ctr.n_dma++;
+        if (dyo_status s1 = wb_mark(ev, r.first, r.first + r.count, true)) return s1;
       } else if (r.bytes >= dma_min && !(ctx->cfg.flags & DYO_F_NO_PACK)) {
         int q = r.first;
         while (q < r.first + r.count) {
@@ -2022,6 +2049,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
               CK(cudaMemcpyAsync(host + ev[q].host_off, arena + ev[q].src, ev[q].bytes, cudaMemcpyDeviceToHost, sd)); }
             ctx->ctr.d2h_dma += ev[q].bytes;
             ctx->ctr.n_dma++;
+            if (dyo_status s1 = wb_mark(ev, q, q + 1, true)) return s1;
             ++q;
             continue;
           }
@@ -2033,6 +2061,9 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
             CK(cudaMemcpyAsync(host + base, stage_pack, len, cudaMemcpyDeviceToHost, sd)); }
           ctx->ctr.d2h_packed += len;
           ctx->ctr.n_dma++;
+          // the pack kernel read the sources: their ranges are free once it has run, but the
+          // staging buffer is reused by the next pack only after this DMA - mark after the DMA
+          if (dyo_status s1 = wb_mark(ev, q, q2, true)) return s1;
           q = q2;
         }
       } else {
@@ -2049,11 +2080,40 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
       }
       dyo_status s1 = launch_segs(ctx, g0, sd, zc_grid, 4);
       if (s1) return s1;
+      if (relaxed) {
+        if (n_wb_ev == (int)ctx->ev_wb.size()) {
+          cudaEvent_t e;
+          CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+          ctx->ev_wb.push_back(e);
+        }
+        CK(cudaEventRecord(ctx->ev_wb[n_wb_ev], sd));
+        for (int q : small) wb_iv.push_back({ev[q].src, ev[q].src + ev[q].bytes, n_wb_ev});
+        ++n_wb_ev;
+      }
     }
   }
   TRACE("  evict phase issued");
   CK(cudaEventRecord(ctx->ev_evict, sd));
-  CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
+  if (relaxed) {
+    CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_half_free, 0));   // block j-2 done: half m is ours
+    std::sort(wb_iv.begin(), wb_iv.end(), [](const WbIv& x, const WbIv& y) { return x.lo < y.lo; });
+  } else {
+    CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
+  }
+  int wb_waited = -1;   // s has waited the copy groups [0, wb_waited] (they complete in order on sd)
+  auto wait_wb = [&](int64_t lo, int64_t hi) -> dyo_status {
+    if (!relaxed) return DYO_OK;
+    int need = -1;
+    auto it = std::upper_bound(wb_iv.begin(), wb_iv.end(), lo, [](int64_t v, const WbIv& x) { return v < x.lo; });
+    if (it != wb_iv.begin()) --it;   // the interval starting at or before lo may reach into [lo, hi)
+    for (; it != wb_iv.end() && it->lo < hi; ++it)
+      if (it->hi > lo) need = std::max(need, it->ev);
+    if (need > wb_waited) {
+      CK(cudaStreamWaitEvent(s, ctx->ev_wb[need], 0));
+      wb_waited = need;
+    }
+    return DYO_OK;
+  };
   // R20: this transition compacts a half that holds tensors the running block j-1 SHARE'd, so
   //      its MOVE / CARRY / FETCH wait for block j-1 to end (the EVICTs above never touch them)
   if ((h.flags & 1) && ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
@@ -2142,6 +2202,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
     if (early > 0) {
       CK(cudaEventRecord(ctx->ev_moves, s));
       CK(cudaStreamWaitEvent(ctx->side, ctx->ev_moves, 0));
+      if (relaxed) CK(cudaStreamWaitEvent(ctx->side, ctx->ev_evict, 0));   // carry destinations: every write-back done
       dyo_status s1 = d2d_records(ctx, ca, P.dout.ca + h.o_carry, 0, h.n_carry, 1, 2, 3, 4, 0, arena, arena, 0,
                                   ctx->side, d2d_grid);
       if (s1) return s1;
@@ -2164,6 +2225,7 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
       }
       const int64_t bytes = fe[k - 1].host_off + fe[k - 1].bytes - fe[i].host_off;
       if (bytes >= dma_min) {
+        if (dyo_status s1 = wait_wb(fe[i].dst, fe[i].dst + bytes)) return s1;
         TRACE("  h2d dma host_off=%lld dst=%lld bytes=%lld", (long long)fe[i].host_off, (long long)fe[i].dst, (long long)bytes);
         { TScope ts(ctx, 5, s, bytes);
           CK(cudaMemcpyAsync(arena + fe[i].dst, host + fe[i].host_off, bytes, cudaMemcpyHostToDevice, s)); }
@@ -2178,10 +2240,14 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
       }
       i = k;
     }
+    if (relaxed && P.seg_used > g0) CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));   // small fetches: after all
     dyo_status s1 = launch_segs(ctx, g0, s, zc_grid, 4);
     if (s1) return s1;
   }
   if (carry_side) CK(cudaStreamWaitEvent(s, ctx->ev_carry, 0));
+  // R21: late carries and block j (ALLOC'd tensors it writes, CARRY destinations) need every
+  //      write-back of this transition done
+  if (relaxed) CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
   // 4. late CARRY: block j-1 writes them, so they wait for its end
   {
     const dyo_carry_rec* ca = P.out.ca + h.o_carry;

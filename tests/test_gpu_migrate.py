@@ -418,3 +418,15 @@ def test_share_af_scaled():
         off += (t.nbytes + 255) // 256 * 256
     run_bytes(wl, 3, 3)
     run_pipelined(wl, 2, 3, spin=200_000)
+
+
+@pytest.mark.parametrize("strict", [0, 64])
+def test_moe_scaled_fetch_after_overlapping_writebacks(strict):
+    """R21: with the default per-range order a FETCH DMA waits only for the write-backs it
+    overwrites (gradients written back in backward, experts fetched into their slots);
+    DYO_F_STRICT_ORDER (64) keeps R12's whole-phase order. Bytes exact both ways, also under the
+    asynchronous event protocol."""
+    wl = WL.make_moe(seed=5, n_samples=8, expert_mib=1, act_mib=1, budget=96 << 20)
+    m = run_bytes(wl, 4, 1, flags=strict, dma_min=1 << 20)
+    assert m["dma"] > 0
+    run_pipelined(wl, 3, 1, dma_min=1 << 20)

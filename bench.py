@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--budget-gib", type=float, default=0.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-faults", action="store_true", help="skip the on-demand fetch measurement")
+    ap.add_argument("--strict-order", action="store_true",
+                    help="DYO_F_STRICT_ORDER: R12's whole-phase EVICT -> FETCH order instead of R21's per-range order")
     ap.add_argument("--dist-backend", default=None, help="nccl (default with CUDA) or gloo")
     ap.add_argument("--compute", default="auto", choices=["auto", "none", "emulate"],
                     help="emulate the DyNN's per-group compute with spin kernels (auto: on for af)")
@@ -451,7 +453,8 @@ def run_dyo(args):
     wl = make_workload(args, rank)
     _log("workload built")
     B = wl.notes.get("batch", 1)          # predictions planned per step (lstm: a minibatch of 64)
-    d = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, device=local, flags=0)   # headline: uninstrumented
+    d = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, device=local,
+            flags=64 if args.strict_order else 0)   # headline: uninstrumented
     d.load(wl)
     _log("ctx loaded")
     s0 = torch.cuda.current_stream()
@@ -763,7 +766,8 @@ def run_dyo(args):
                             "time not counted"),
         "vs_baseline": None, "dtype": "f32 weights / f64 accumulate (pilot); int64 (plan); u8 (migrate)",
         "data": "synthetic",
-        "config": {"workload": args.config, "desc": CONFIG_DESC[args.config], "policy": "RETAIN" if args.policy else "PAPER",
+        "config": {"workload": args.config, "desc": CONFIG_DESC[args.config], "policy": ("RETAIN" if args.policy & 1 else "PAPER") + ("+SHARE (R20)" if args.policy & 2 else ""),
+                   "migrate_order": "R12 strict" if args.strict_order else "R21 per-range",
                    "budget_bytes": wl.budget, "tensors": len(wl.tensors),
                    "l2": "inputs larger than L2 (every step moves >= 1 GiB through HBM and PCIe)",
                    "parallelism": f"{world} independent managers (replicas, no collective on the path)"},

@@ -8,8 +8,9 @@ from paper_conf_hpca_renxyzlnwxl24_b200 import Dyo
 cfg = sys.argv[1] if len(sys.argv) > 1 else "moe"
 B = int(sys.argv[2]) if len(sys.argv) > 2 else 1
 Js = [int(x) for x in sys.argv[3:]] or [3]
+POL = int(os.environ.get("PLAN_POLICY", "-1"))
 wl = WL.make(cfg, n_samples=max(64, B))
-d = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, flags=4 | 8)
+d = Dyo(wl.budget, wl.align, wl.policy if POL < 0 else POL, max_batch=B, flags=4 | 8)
 d.load(wl)
 s = torch.cuda.current_stream().cuda_stream
 desc = torch.from_numpy(wl.samples.copy()).cuda()

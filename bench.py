@@ -495,8 +495,9 @@ def run_dyo(args):
             if K <= 64:     # record-level detail for the R21 step bound (small plans: MoE, AF steps)
                 ev = d.plan_records(j, "evict")
                 fe = d.plan_records(j, "fetch")
+                late = bool(info["n_carry"]) and bool(d.plan_records(j, "carry")[:, 4].any())
                 trs.append((info["h2d"], info["d2h"], [(int(r[1]), int(r[3])) for r in ev if r[4]],
-                            [(int(r[2]), int(r[3])) for r in fe], info["n_move"], info["late_all"]))
+                            [(int(r[2]), int(r[3])) for r in fe], info["n_move"], info["late_all"], late))
             else:
                 trs.append((info["h2d"], info["d2h"]))
         per_tr.append(trs)
@@ -521,6 +522,8 @@ def run_dyo(args):
                 bend[j].record(s_comp)
         if emulate:
             s1.wait_stream(s_comp)
+        elif K:
+            s1.wait_event(ready[K - 1])      # R21: the last ready[] may be joined off the copy stream
 
     def run_steps(n, first, inputs):
         """n steps with plan lookahead: step i's transitions are enqueued, then step i+1 is
@@ -941,8 +944,10 @@ def step_bound_ms(trs, h2d_gbs, d2h_gbs, strict=False):
         for dst, nb in tr[3]:
             dep = max([e for lo, hi, e in iv if dst < hi and dst + nb > lo] or [0.0])
             f = max(f, dep) + nb / (h2d_gbs * 1e6)
-        f_end = max(f, e_end)
-        ready.append(f_end)
+        # ready[j] joins FETCH_j and EVICT_j; the copy stream itself waits EVICT_j only when the
+        # transition has late carries
+        f_end = max(f, e_end) if tr[6] else f
+        ready.append(max(f, e_end))
     return ready[-1] if ready else 0.0
 
 

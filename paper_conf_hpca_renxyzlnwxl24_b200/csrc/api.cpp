@@ -148,6 +148,8 @@ struct dyo_ctx {
   cudaStream_t side = nullptr;     // ctx-owned stream for early CARRY (overlaps FETCH)
   cudaEvent_t ev_entry = nullptr, ev_evict = nullptr, ev_moves = nullptr, ev_carry = nullptr;
   std::vector<cudaEvent_t> ev_wb;   // R21: one per write-back copy group of a transition (D2H stream order)
+  cudaStream_t join = nullptr;      // R21: ready[j] = FETCH_j + EVICT_j joined off the copy stream
+  cudaEvent_t ev_tail = nullptr;
   dyo_counters ctr{};
   int sm_count = 148;
   // DYO_F_TIMING: event pairs per launch kind
@@ -674,6 +676,8 @@ dyo_status dyo_create(const dyo_config* cfg, int32_t device, dyo_ctx** outp) {
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_pred, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_memo, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_fault_wb, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->join, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->ev_tail, cudaEventDisableTiming);
   if (e != cudaSuccess) {
     dyo_destroy(ctx);
     return e == cudaErrorMemoryAllocation ? DYO_E_NOMEM : DYO_E_CUDA;
@@ -769,6 +773,8 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
     if (P.ev_last) cudaEventDestroy(P.ev_last);
   if (ctx->ev_entry) cudaEventDestroy(ctx->ev_entry);
   if (ctx->ev_evict) cudaEventDestroy(ctx->ev_evict);
+  if (ctx->join) cudaStreamDestroy(ctx->join);
+  if (ctx->ev_tail) cudaEventDestroy(ctx->ev_tail);
   if (ctx->d2h) cudaStreamDestroy(ctx->d2h);
   if (ctx->side) cudaStreamDestroy(ctx->side);
   if (ctx->ev_moves) cudaEventDestroy(ctx->ev_moves);
@@ -2246,13 +2252,17 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   }
   if (carry_side) CK(cudaStreamWaitEvent(s, ctx->ev_carry, 0));
   // R21: late carries and block j (ALLOC'd tensors it writes, CARRY destinations) need every
-  //      write-back of this transition done
-  if (relaxed) CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
+  //      write-back of this transition done. Without late carries the copy stream does not wait:
+  //      ready[j] joins FETCH_j and EVICT_j on the join stream, so FETCH_{j+1} (the other half)
+  //      may start while EVICT_j's write-backs still run
+  bool any_late = false;
+  for (int i = 0; i < h.n_carry; ++i) any_late |= P.out.ca[h.o_carry + i].late != 0;
+  const bool join = relaxed && !any_late;
+  if (relaxed && any_late) CK(cudaStreamWaitEvent(s, ctx->ev_evict, 0));
   // 4. late CARRY: block j-1 writes them, so they wait for its end
   {
     const dyo_carry_rec* ca = P.out.ca + h.o_carry;
-    bool any = false;
-    for (int i = 0; i < h.n_carry; ++i) any |= ca[i].late != 0;
+    const bool any = any_late;
     if (any) {
       if (ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
       for (int i = 0; i < h.n_carry; ++i)
@@ -2263,8 +2273,16 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
     }
   }
   TRACE("  transition %d issued", j);
-  if (ev_ready) CK(cudaEventRecord((cudaEvent_t)ev_ready, s));
-  CK(cudaEventRecord(P.ev_last, s));
+  if (join) {
+    CK(cudaEventRecord(ctx->ev_tail, s));
+    CK(cudaStreamWaitEvent(ctx->join, ctx->ev_tail, 0));
+    CK(cudaStreamWaitEvent(ctx->join, ctx->ev_evict, 0));
+    if (ev_ready) CK(cudaEventRecord((cudaEvent_t)ev_ready, ctx->join));
+    CK(cudaEventRecord(P.ev_last, ctx->join));
+  } else {
+    if (ev_ready) CK(cudaEventRecord((cudaEvent_t)ev_ready, s));
+    CK(cudaEventRecord(P.ev_last, s));
+  }
   // host replay of the residency after transition j (the fault path's residency check, R17)
   {
     const int m = h.half;

@@ -162,11 +162,11 @@ def test_lstm_scaled_small_tensors_zero_copy():
     assert m["zc"] > 0
 
 
-def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0, lookahead=False, spin=0):
+def run_pipelined(wl, steps, policy=None, dma_min=0, staging=0, lookahead=False, spin=0, flags=0):
     """The full event protocol, enqueued asynchronously: emulated compute block j runs on its own
     stream after ready[j]; transition j's EVICT waits end[j-2], its late carries end[j-1].
     Read mismatches are accumulated on the device; the host syncs once per step."""
-    d = make_ctx(wl, policy=policy, dma_min_bytes=dma_min, staging_bytes=staging)
+    d = make_ctx(wl, policy=policy, dma_min_bytes=dma_min, staging_bytes=staging, flags=flags)
     pool = d.host_pool_array()
     for t, ten in enumerate(wl.tensors):
         pool[ten.host_off: ten.host_off + ten.nbytes] = M.content_bytes(t, 0, ten.nbytes)
@@ -429,4 +429,5 @@ def test_moe_scaled_fetch_after_overlapping_writebacks(strict):
     wl = WL.make_moe(seed=5, n_samples=8, expert_mib=1, act_mib=1, budget=96 << 20)
     m = run_bytes(wl, 4, 1, flags=strict, dma_min=1 << 20)
     assert m["dma"] > 0
-    run_pipelined(wl, 3, 1, dma_min=1 << 20)
+    run_pipelined(wl, 3, 1, dma_min=1 << 20, flags=strict)
+    run_pipelined(wl, 3, 1, dma_min=1 << 20, flags=strict, spin=500_000)

@@ -188,7 +188,10 @@ dyo_status dyo_destroy(dyo_ctx* ctx);
 
 /* Load the static architecture (copies it; builds the AFM segment table (R3), operator
  * signatures, site table and tensor table on the device; allocates the pinned, mapped host
- * pool sized to max(host_off + bytes)). Resets residency: all tensors on the host. */
+ * pool sized to max(host_off + bytes), bound to the GPU's NUMA node - DYO_Q_HOST_NUMA). Resets
+ * residency: all tensors on the host. DYO_E_NOMEM if the pool exceeds ~94% of the node's
+ * MemAvailable (one manager per GPU pins from the same host RAM), DYO_E_INVAL for a malformed
+ * program, DYO_E_UNSUPPORTED for a Loop nested in a dynamic site. */
 dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* arch);
 
 /* Host-only check of an arch (no GPU needed; used by the CPU test suite): runs the same parse

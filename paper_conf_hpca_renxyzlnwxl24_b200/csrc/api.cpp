@@ -732,8 +732,26 @@ static void host_pool_free(dyo_ctx* ctx) {
   ctx->host_registered = false;
 }
 
+// MemAvailable of /proc/meminfo in bytes (-1 if unreadable): several managers on one node pin
+// their pools from the same RAM (one per GPU), so a pool that cannot fit is refused up front
+// (DYO_E_NOMEM) instead of letting pinning drive the host into the OOM killer.
+static int64_t host_mem_available() {
+  FILE* f = fopen("/proc/meminfo", "r");
+  if (!f) return -1;
+  char line[256];
+  int64_t kb = -1;
+  while (fgets(line, sizeof line, f))
+    if (sscanf(line, "MemAvailable: %lld kB", (long long*)&kb) == 1) break;
+  fclose(f);
+  return kb < 0 ? -1 : kb * 1024;
+}
+
 static dyo_status host_pool_alloc(dyo_ctx* ctx, int64_t bytes) {
   const size_t n = (size_t)std::max<int64_t>(bytes, 64);
+  const int64_t avail = host_mem_available();
+  if (avail > 0 && (int64_t)n > avail - (avail >> 4))
+    return fail(ctx, DYO_E_NOMEM, "host pool of %lld MiB exceeds the node's available memory (%lld MiB)",
+                (long long)(n >> 20), (long long)(avail >> 20));
   ctx->host_numa = -1;
   ctx->host_registered = false;
   const int node = device_numa_node(ctx->device);

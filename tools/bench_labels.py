@@ -72,6 +72,39 @@ for budget_gib in (3.0, 0.5, 0.25):
 d.close()
 out["partition"] = res
 
+# the same comparison on the AlphaFold-shaped trace over a budget sweep (E13 on the E7 sweep,
+# P:L249-L253, L275): recycle-1 samples (path <= 4096 rows), K = 32 blocks
+wl = WL.make("af", n_samples=64)
+d = Dyo(wl.budget, wl.align, wl.policy, max_batch=1, flags=4)
+d.load(wl)
+op_ns = [WL.op_time_ns(o) for o in op_list(wl)]
+paths = []
+for s in range(64):
+    ch = [max(c, 0) for c in WL.actual_choices(wl, s)]
+    ops, its = d.trace_path(ch)
+    if len(ops) <= 4096:
+        paths.append((ops, its))
+    if len(paths) >= (4 if quick else 8):
+        break
+res = {}
+Kaf = 32
+for budget_gib in (1.0, 2.0, 4.0, 8.0):
+    H = int(budget_gib * (1 << 30)) // 2
+    agg = {m: [] for m in ("overlap", "even_ops", "even_time", "even_size")}
+    feas = {m: 0 for m in agg}
+    for ops, its in paths:
+        for m in agg:
+            cuts, ex, ok = d.partition(ops, its, 0, op_ns, Kaf, m, H, 50_000)
+            if ok:
+                agg[m].append(ex)
+                feas[m] += 1
+    res[f"B={budget_gib}GiB"] = {
+        "trace_rows": [len(p[0]) for p in paths], "K": Kaf, "samples": len(paths), "bw_GBps": 50,
+        "mean_exposed_us": {m: (round(float(np.mean(v)) / 1e3, 2) if v else None) for m, v in agg.items()},
+        "feasible": feas}
+d.close()
+out["partition_af_sweep"] = res
+
 # ---- training (R19) ------------------------------------------------------------------------
 wl = WL.make("moe", n_samples=64)
 B = 64

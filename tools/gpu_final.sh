@@ -2,7 +2,7 @@
 # Round measurement: GPU tests, smoke, bench lines (all configs), reference arm, launch list,
 # ncu captures of the top kernels. Outputs under gpurun_out/r02/.
 cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
-O=gpurun_out/r02; mkdir -p $O
+O=gpurun_out/${OUT:-r02}; mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1 || { tail -20 $O/build.log; exit 1; }
 nvidia-smi > $O/nvidia_smi.txt 2>&1; nvidia-smi topo -m > $O/topo.txt 2>&1
 if [ "${SKIP_TESTS:-0}" != 1 ]; then
@@ -12,6 +12,9 @@ timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>
 for cfg in ${CFGS:-moe lstm tree af}; do
   timeout 1200 python bench.py --config $cfg --steps 10 --warmup 3 > $O/bench_$cfg.log 2>&1; echo "bench $cfg rc=$?"
 done
+# B*0 demonstration: the AlphaFold-shaped trace at 16 GiB with SHARE (R20), exposed vs the compute-only harness
+timeout 1200 python bench.py --config af --policy 3 --budget-gib 16 --steps 6 --warmup 3 --no-cpu-baseline > $O/bench_af16_share.log 2>&1; echo "bench af16 share rc=$?"
+timeout 900 python bench.py --config moe --steps 10 --warmup 3 --no-cpu-baseline --no-faults --strict-order > $O/bench_moe_strict.log 2>&1; echo "bench moe strict rc=$?"
 timeout 900 python bench.py --impl reference --steps 3 --warmup 1 > $O/bench_reference.log 2>&1; echo "ref rc=$?"
 if [ "${SKIP_NCU:-0}" != 1 ]; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_moe.csv \

@@ -288,7 +288,6 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
   uint64_t* wbar = reinterpret_cast<uint64_t*>(smem_raw);           // one per stage
   uint64_t* abar = wbar + (4 + kMaxLayers);                         // two activation buffers
   double* act = reinterpret_cast<double*>(smem_raw + spc.act_off);
-  if (blockIdx.x == 0 && tid == 0) { pd.status[0] = 0; pd.status[1] = 0; }
   if (tid == 0) {
     for (int i = 0; i < 4 + kMaxLayers; ++i) mbar_init(&wbar[i], 1);
     mbar_init(&abar[0], 1);
@@ -329,6 +328,13 @@ pilot_kernel(const __grid_constant__ ArchDev a, const PilotDev* __restrict__ pde
   }
   // the decode tables ride the same launch-time TMA stream (used only by the epilogue)
   if (sp.tab_off >= 0 && tid == 32) prefetch_dec_tables(a, reinterpret_cast<int*>(smem_raw + sp.tab_off), &abar[2]);
+  // Programmatic dependent launch: everything above reads only what dyo_load_arch / dyo_load_pilot
+  // wrote (descriptors, weights, decode tables), so it may overlap the previous kernel of the
+  // stream; from here on (features, the history table, prediction outputs) the previous kernel's
+  // writes must be visible. The next prediction may then start its own prologue.
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (blockIdx.x == 0 && tid == 0) { pd.status[0] = 0; pd.status[1] = 0; }
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   stamp(1, stamp_on);
   // ---- 1. the sub-batch's feature vectors into buf[0] (overlaps the weight stream)
   for (int bb = 0; bb < nb; ++bb) {
@@ -735,13 +741,20 @@ cudaError_t launch_pilot(const ArchDev& a, const PilotDev& p, const PilotDev* p_
   cfg.blockDim = dim3(kPilotThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = C;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  // programmatic stream serialization: the launch may begin while the stream's previous kernel
+  // finishes (the kernel waits with griddepcontrol.wait before touching dependent data);
+  // DYO_PILOT_PDL=0 turns it off (measurement)
+  static int pdl = -1;
+  if (pdl < 0) { const char* e = getenv("DYO_PILOT_PDL"); pdl = (e && e[0] == '0') ? 0 : 1; }
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = pdl ? 2 : 1;
   if (fused) *fused = sp.fuse_decode;
   if (sp.Bs == 1)
     return cudaLaunchKernelEx(&cfg, pilot_kernel<1>, a, p_dev, sp, feat_or_null, desc, hist, hist_tab, hist_K, hist_B,

@@ -62,6 +62,32 @@ def test_pilot_logits(name, B):
     d.close()
 
 
+@pytest.mark.parametrize("name,B", [("moe", 1), ("tiny", 1), ("moe", 8)])
+def test_pilot_back_to_back_chained_history(name, B):
+    """Consecutive predictions on one stream with no host sync between them (the pilot launches
+    with programmatic dependent launch: its prologue overlaps the previous kernel): every
+    prediction's logits match the oracle fed the previous prediction's block table (R3 history),
+    and the last decode is exact."""
+    wl = WL.make(name, n_samples=8 * B)
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    outs = [torch.zeros((B, wl.pilot.O), device="cuda") for _ in range(8)]
+    for k in range(8):
+        d.predict(wl.samples[k * B:(k + 1) * B].copy(), hist_for(wl, B), B, outs[k], stream=_stream())
+    torch.cuda.synchronize()
+    table = ()
+    r = None
+    for k in range(8):
+        r = oracle_step(wl, range(k * B, (k + 1) * B), PL.initial_state(len(wl.tensors)), table, plan=False)
+        y = outs[k].cpu().numpy()
+        for b in range(B):
+            g1, g2, _ = logit_gates(y[b], r["feats"][b], wl.pilot, wl.nn_type)
+            assert g1.all() and g2.all(), f"prediction {k} sample {b}"
+        table = r["table"]
+    for b in range(B):
+        _check_prediction(d, wl, b, r["preds"][b])
+    d.close()
+
+
 @pytest.mark.parametrize("width", [32, 64, 128, 256, 1024, 2048])
 @pytest.mark.parametrize("B", [1, 64])
 def test_pilot_logits_width_sweep(width, B):

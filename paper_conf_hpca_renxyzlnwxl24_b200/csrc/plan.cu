@@ -543,6 +543,36 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
       FOR_RECS(cnt += rec_kind(r, inw) == 3;)
       long long nlive = 0;
       long long kb = scan64(cnt, S.tmp, &nlive);
+      if (nlive <= kEvSort) {
+        // few live candidates: rank selection in shared memory (keys are unique, so the ranks
+        // are a permutation): sizes in key order, one block scan, the first rank whose prefix
+        // exceeds the room -> its key is the threshold (the same K* as the radix select below)
+        uint64_t* keys = S.ev_key;                      // free until phase D
+        uint64_t* sorted = S.pkey;                      // free until phase E
+        int32_t* szs = S.gap_s;                         // free until phase D
+        FOR_RECS(if (rec_kind(r, inw) == 3) keys[kb++] = live_key(r, j);)
+        __syncthreads();
+        const int nl = (int)nlive;
+        for (int i = tid; i < nl; i += PNT) {
+          const uint64_t k = keys[i];
+          const int rk = rank_u64(keys, nl, k);
+          sorted[rk] = k;
+          szs[rk] = (int32_t)((k >> 20) & ((1u << 28) - 1));
+        }
+        __syncthreads();
+        const int per_k = (nl + PNT - 1) / PNT;
+        const int r0 = min(nl, tid * per_k), r1 = min(nl, r0 + per_k);
+        long long ls = 0;
+        for (int q = r0; q < r1; ++q) ls += szs[q];
+        long long tot = 0;
+        long long c = scan64(ls, S.tmp, &tot);
+        if (c <= room)                                  // exactly one thread's chunk crosses the room
+          for (int q = r0; q < r1; ++q) {
+            c += szs[q];
+            if (c > room) { s_thresh = sorted[q]; break; }
+          }
+        __syncthreads();
+      } else {
       FOR_RECS(if (rec_kind(r, inw) == 3) sc.keys[kb++] = live_key(r, j);)
       __syncthreads();
       uint64_t prefix = 0, mask = 0;
@@ -603,6 +633,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
         if ((key & mask) == prefix) s_thresh = key;
       }
       __syncthreads();
+      }
     }
     const uint64_t thresh = rule == 2 ? s_thresh : 0;
     PSTAMP(3);

@@ -10,6 +10,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include <cctype>
@@ -131,6 +132,11 @@ struct dyo_ctx {
   std::vector<FaultWb> fault_wb;             // written faulted tensors of the last block
   cudaEvent_t ev_fault_wb = nullptr;
   int64_t n_faults = 0, fault_bytes = 0, n_fault_resident = 0, n_fault_repair = 0;
+  // copy descriptors of the fault copies: two halves alternating between blocks like the fault
+  // area; the host rewrites a half only after the launch that read it (ev_fseg) has run
+  CopySeg* fault_segs = nullptr;
+  int64_t fseg_cap = 0, fseg_used = 0;
+  cudaEvent_t ev_fseg[2] = {nullptr, nullptr};
   double drop_p = -1.0;                      // dyo_fault_inject (< 0: DYO_FAULT environment)
   unsigned long long drop_seed = 0;
   // host replay of the residency after every migrated transition (FIFO over plans)
@@ -802,6 +808,8 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
   if (ctx->ev_memo) cudaEventDestroy(ctx->ev_memo);
   if (ctx->ev_fault_wb) cudaEventDestroy(ctx->ev_fault_wb);
   if (ctx->fault_area) cudaFree(ctx->fault_area);
+  if (ctx->fault_segs) cudaFreeHost(ctx->fault_segs);
+  for (auto e : ctx->ev_fseg) if (e) cudaEventDestroy(e);
   if (ctx->part_buf) cudaFree(ctx->part_buf);
   if (ctx->h_rep) cudaFreeHost(ctx->h_rep);
   if (ctx->h_memo_stage) cudaFreeHost(ctx->h_memo_stage);
@@ -1995,12 +2003,15 @@ dyo_status dyo_migrate(dyo_ctx* ctx, int32_t j, void* copy_stream, void* ev_half
   //    transition's EVICT (D2H stream) and carries (after ev_moves) are ordered after them
   if (!ctx->fault_wb.empty()) {
     if (ev_prev_done) CK(cudaStreamWaitEvent(s, (cudaEvent_t)ev_prev_done, 0));
+    const int64_t seg0 = P.seg_used;                 // one segment-copy launch for all of them
     for (const auto& w : ctx->fault_wb) {
       const int64_t nb = ctx->t_bytes[w.t];
-      CK(cudaMemcpyAsync(host + ctx->t_host[w.t], w.src, nb, cudaMemcpyDeviceToHost, s));
-      if (ctx->mig_loc[w.t] >= 0)
-        CK(cudaMemcpyAsync(arena + ctx->mig_loc[w.t] * ctx->H + ctx->mig_off[w.t], w.src, nb, cudaMemcpyDeviceToDevice, s));
+      if (!push_seg(ctx, w.src, host + ctx->t_host[w.t], nb)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors (fault write-backs)");
+      if (ctx->mig_loc[w.t] >= 0 &&
+          !push_seg(ctx, w.src, arena + ctx->mig_loc[w.t] * ctx->H + ctx->mig_off[w.t], nb))
+        return fail(ctx, DYO_E_CAPACITY, "copy descriptors (fault write-backs)");
     }
+    if (dyo_status s1 = launch_segs(ctx, seg0, s, 16, 4)) return s1;
     ctx->fault_wb.clear();
     CK(cudaEventRecord(ctx->ev_fault_wb, s));
     CK(cudaStreamWaitEvent(sd, ctx->ev_fault_wb, 0));
@@ -2397,6 +2408,11 @@ dyo_status dyo_fault_config(dyo_ctx* ctx, int64_t area_bytes) {
   if (area_bytes == 0) return DYO_OK;
   CK(cudaMalloc(&ctx->fault_area, area_bytes));
   ctx->fault_cap = area_bytes;
+  if (!ctx->fault_segs) {
+    ctx->fseg_cap = 1 << 16;                     // per half
+    CK(cudaHostAlloc((void**)&ctx->fault_segs, sizeof(CopySeg) * 2 * ctx->fseg_cap, cudaHostAllocMapped | cudaHostAllocPortable));
+    for (auto& e : ctx->ev_fseg) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
   return DYO_OK;
 }
 
@@ -2410,19 +2426,44 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
   CK(cudaSetDevice(ctx->device));
   cudaStream_t s = (cudaStream_t)stream;
   const PlanHdr& h = P->out.hdr[j];
-  // the planned W_j with its placement (entry records of transition j, host copy)
-  std::vector<dyo_entry_rec> ent(h.n_ent);
-  if (h.n_ent) CK(cudaMemcpy(ent.data(), P->dout.ent + h.o_ent, sizeof(dyo_entry_rec) * h.n_ent, cudaMemcpyDeviceToHost));
-  if (ctx->fault_j != j) { ctx->fault_used = 0; ctx->fault_j = j; }
-  // copies after transition j's migrations (stream order with the ctx's last migrate)
+  // the planned W_j with its placement: the plan's entry records, copied to the host once per
+  // plan (the first fault fetch or dyo_plan_records), then a tensor -> entry index for block j
+  if (!P->ent_host) {
+    if (P->n_ent) CK(cudaMemcpy(P->out.ent, P->dout.ent, sizeof(dyo_entry_rec) * P->n_ent, cudaMemcpyDeviceToHost));
+    P->ent_host = true;
+  }
+  const dyo_entry_rec* ent = P->out.ent + h.o_ent;
+  std::unordered_map<int32_t, int32_t> ent_of;
+  ent_of.reserve((size_t)h.n_ent * 2);
+  for (int q = 0; q < h.n_ent; ++q) ent_of.emplace((int32_t)ent[q].t, q);
+  auto find_ent = [&](int t) -> const dyo_entry_rec* {
+    auto it = ent_of.find(t);
+    return it == ent_of.end() ? nullptr : ent + it->second;
+  };
+  if (ctx->fault_j != j) {
+    ctx->fault_used = 0;
+    ctx->fault_j = j;
+    CK(cudaEventSynchronize(ctx->ev_fseg[j & 1]));    // block j-2's fault copies have run
+    ctx->fseg_used = 0;
+  }
+  // copies after transition j's migrations (stream order with the ctx's last migrate); the
+  // fault copies of the call go to the SM copy kernel as one launch (device and mapped pinned
+  // host sources alike) instead of one cudaMemcpyAsync per tensor
   CK(cudaStreamWaitEvent(s, P->ev_last, 0));
+  CopySeg* fsegs = ctx->fault_segs + (int64_t)(j & 1) * ctx->fseg_cap;
+  const int64_t seg0 = ctx->fseg_used;
+  auto push_fault = [&](const char* src, char* dst, int64_t bytes) -> bool {
+    for (int64_t o = 0; o < bytes; o += kChunk) {
+      if (ctx->fseg_used >= ctx->fseg_cap) return false;
+      fsegs[ctx->fseg_used++] = CopySeg{src + o, dst + o, std::min(kChunk, bytes - o)};
+    }
+    return true;
+  };
   const int64_t AL = ctx->cfg.align;
   for (int i = 0; i < n; ++i) {
     const int t = ids[i], md = modes[i];
     if (t < 0 || t >= ctx->T || md < 1 || md > 3) return fail(ctx, DYO_E_INVAL, "fault %d: tensor %d mode %d", i, t, md);
-    const dyo_entry_rec* e = nullptr;
-    for (const auto& r : ent)
-      if (r.t == t) { e = &r; break; }
+    const dyo_entry_rec* e = find_ent(t);
     // residency check: planned and valid for this access -> its slot. Valid: the
     // plan fetched it (or the access writes first), and a write is one the plan knows about
     // (a write the plan does not expect would leave a device copy it treats as clean)
@@ -2448,8 +2489,8 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
     for (const auto& pa : ctx->mig_prev_alloc)       // ALLOC'd at j: its slot holds no bytes yet
       if (pa.first == t) { loc = pa.second.first; off = pa.second.second; }
     if (md & 1) {
-      if (loc >= 0) CK(cudaMemcpyAsync(dst, ctx->arena + loc * ctx->H + off, nb, cudaMemcpyDeviceToDevice, s));
-      else CK(cudaMemcpyAsync(dst, ctx->host_pool + ctx->t_host[t], nb, cudaMemcpyHostToDevice, s));
+      const char* src = loc >= 0 ? ctx->arena + loc * ctx->H + off : ctx->host_pool + ctx->t_host[t];
+      if (!push_fault(src, dst, nb)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors (faults)");
       ctx->fault_bytes += nb;
     }
     if (md & 2) ctx->fault_wb.push_back({t, dst});
@@ -2462,9 +2503,7 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
   // are copied into the slot now (from its previous device copy, else its host home)
   for (const auto& pa : ctx->mig_prev_alloc) {
     const int t = pa.first;
-    const dyo_entry_rec* e = nullptr;
-    for (const auto& r : ent)
-      if (r.t == t) { e = &r; break; }
+    const dyo_entry_rec* e = find_ent(t);
     if (!e) continue;
     bool written = false;
     for (int i = 0; i < n && !written; ++i)
@@ -2472,10 +2511,18 @@ dyo_status dyo_fault_fetch(dyo_ctx* ctx, int32_t j, const int32_t* ids, const in
     if (written) continue;
     const int8_t loc = pa.second.first;
     const int64_t off = pa.second.second, nb = ctx->t_bytes[t];
-    if (loc >= 0) CK(cudaMemcpyAsync(ctx->arena + e->dst, ctx->arena + loc * ctx->H + off, nb, cudaMemcpyDeviceToDevice, s));
-    else CK(cudaMemcpyAsync(ctx->arena + e->dst, ctx->host_pool + ctx->t_host[t], nb, cudaMemcpyHostToDevice, s));
+    const char* src = loc >= 0 ? ctx->arena + loc * ctx->H + off : ctx->host_pool + ctx->t_host[t];
+    if (!push_fault(src, ctx->arena + e->dst, nb)) return fail(ctx, DYO_E_CAPACITY, "copy descriptors (faults)");
     ++ctx->n_fault_repair;
   }
+  if (ctx->fseg_used > seg0) {
+    CopySeg* dptr = nullptr;
+    CK(cudaHostGetDevicePointer((void**)&dptr, fsegs + seg0, 0));
+    TScope ts(ctx, 4, s, 0);
+    CK(launch_copy_segments(dptr, (int)(ctx->fseg_used - seg0), kChunk, 16, s));
+    ctx->ctr.n_kernels++;
+  }
+  CK(cudaEventRecord(ctx->ev_fseg[j & 1], s));
   if (ev_done) CK(cudaEventRecord((cudaEvent_t)ev_done, s));
   return DYO_OK;
 }

@@ -543,7 +543,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
       FOR_RECS(cnt += rec_kind(r, inw) == 3;)
       long long nlive = 0;
       long long kb = scan64(cnt, S.tmp, &nlive);
-      if (nlive <= kEvSort) {
+      if (nlive <= 256) {
         // few live candidates: rank selection in shared memory (keys are unique, so the ranks
         // are a permutation): sizes in key order, one block scan, the first rank whose prefix
         // exceeds the room -> its key is the threshold (the same K* as the radix select below)

@@ -641,6 +641,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
     //      Pass 1 counts kept / evicted / gaps after my first kept record (local), pass 2 writes.
     long long kbase = 0, nkept = 0;                 // this thread's first kept index; total kept
     int nev = 0;
+    int pe0_keep = 0;                               // end of the kept record before my first (phase G)
     int last_x = -1;                                // old offset of this thread's last kept record
     {
       long long ck = 0, ce = 0, cg = 0;
@@ -661,6 +662,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
       })
       int pe_all = 0;
       const int pe0 = scanmax(last_end, S.tmp, &pe_all);   // end of the kept record before my first
+      pe0_keep = pe0;
       if (first_x >= 0 && first_x > pe0) ++cg;
       long long tot = 0;
       const long long b = scan64((ck << 42) | (ce << 21) | cg, S.tmp, &tot);
@@ -1045,11 +1047,14 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
         long long tot = 0;
         newx0 = (int)scan64(cu, S.tmp, &tot);
       }
-      // merge: a kept record's slot = its kept index + the placed offsets below it (binary search
-      // over q_off); a placed tensor's slot = its rank + the kept offsets below it (binary search
-      // over the kept offsets, staged in the consumed gap array when they fit)
-      const bool koff_smem = nkept <= kGapSmem;
-      int32_t* koff = S.gap_s;
+      // merge (one pass, no per-record search): a kept record's slot = its kept index + the placed
+      // offsets below it; a placed tensor's slot = its rank + the kept records below it. No placed
+      // offset lies inside a kept range, so a thread's pointer into the ascending placed offsets
+      // starts below its first kept record (one binary search from the end of the previous kept
+      // record, pe0) and advances linearly: the placed tensors it passes get this record's kept
+      // index. Placed tensors above the last kept record keep the default nkept; after a
+      // compaction every placed tensor lies above every kept one.
+      int ptr = compact ? 0 : lower(pe0_keep);
       int newx = newx0;
       FOR_RECS({
         const int k = rec_kind(r, inw);
@@ -1062,53 +1067,14 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
             w.w = S.e_nx[e];
             w.z = (r.z & ~(kRecNxRd | kRecDirty)) | ((S.e_fl[e] & 8) ? kRecNxRd : 0) | ((S.e_fl[e] & 4) ? kRecDirty : 0);
           }
-          const int lb = lower(w.x);
-          if (koff_smem) koff[q] = w.x;
+          if (!compact)
+            while (ptr < np && S.q_off[ptr] < w.x) { S.q_cnt[ptr] = (int)q; ++ptr; }
+          const int lb = compact ? 0 : ptr;
           dst[q + lb] = w;
           st.pos[t] = (int)(q + lb);
           ++q;
         }
       })
-      if (!koff_smem) {
-        // many kept tensors: placed slots from the kept side (each kept record fills the placed
-        // offsets between its predecessor's and its own)
-        int last_lb = 0;
-        {
-          int x = newx0, lx = -1;
-          FOR_RECS({
-            const int k = rec_kind(r, inw);
-            if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) { lx = compact ? x : r.x; x += r.y; }
-          })
-          if (lx >= 0) last_lb = lower(lx);
-        }
-        int dummy = 0;
-        int lb_prev = scanmax(last_lb, S.tmp, &dummy);
-        long long q2 = kbase;
-        int x2 = newx0;
-        FOR_RECS({
-          const int k = rec_kind(r, inw);
-          if (k != 0 && !rec_evicted(r, k, rule, thresh, j)) {
-            const int xo = compact ? x2 : r.x;
-            x2 += r.y;
-            const int lb = lower(xo);
-            for (int x = lb_prev; x < lb; ++x) S.q_cnt[x] = (int)q2;
-            lb_prev = lb;
-            ++q2;
-          }
-        })
-      } else {
-        __syncthreads();
-#pragma unroll
-        for (int qq = 0; qq < kEntCap / PNT; ++qq) {
-          const int i = tid + qq * PNT;
-          if (i < np) {
-            const int o = S.q_off[i];
-            int lo = 0, hi = (int)nkept;
-            while (lo < hi) { const int mid = (lo + hi) >> 1; if (koff[mid] < o) lo = mid + 1; else hi = mid; }
-            S.q_cnt[i] = lo;
-          }
-        }
-      }
     }
     __syncthreads();
 #pragma unroll

@@ -753,6 +753,8 @@ def run_dyo(args):
     shares = {k: round(v["ms"] / ms_instr, 4) for k, v in tm.items()}
     bound_ms = step_bound_ms(timed_trs, probe["h2d"], probe["d2h"]) / args.steps
     bound_strict_ms = step_bound_ms(timed_trs, probe["h2d"], probe["d2h"], strict=True) / args.steps
+    bidir = bidir_probe(torch)
+    bound_fluid_ms = step_bound_fluid_ms(timed_trs, probe["h2d"], probe["d2h"], bidir) / args.steps
     dma_h2d = tm["dma_h2d"]
     dma_d2h = tm["dma_d2h"]
     h2d_link = dma_h2d["bytes"] / (dma_h2d["ms"] * 1e-3) / 1e9 if dma_h2d["ms"] else None
@@ -768,12 +770,15 @@ def run_dyo(args):
         "instrumented_ms_per_step": round(ms_instr / args.steps, 3),
         "step_bound_ms": round(bound_ms, 3),
         "step_bound_strict_ms": round(bound_strict_ms, 3),
+        "step_bound_link_ms": round(bound_fluid_ms, 3),
+        "frac_of_link_bound": round(bound_fluid_ms / (ms_max / args.steps), 4) if ms_max else None,
         "frac_of_step_bound": round(bound_ms / (ms_max / args.steps), 4) if ms_max else None,
         "step_bound_note": ("critical path of the timed steps' per-transition H2D / D2H bytes at the probe's "
                             "per-direction rates: EVICT_j (D2H stream, in order) after block j-2; FETCH_j "
                             "after the write-backs overlapping its destination (R21; strict: after the whole "
                             "EVICT_j, R12); block j = ready[j] (no compute emulation) - D2D, plan and pilot "
-                            "time not counted"),
+                            "time not counted; step_bound_link_ms: the same DAG with both directions sharing the "
+                            "measured bidirectional aggregate while they overlap (fluid model)"),
         "vs_baseline": None, "dtype": "f32 weights / f64 accumulate (pilot); int64 (plan); u8 (migrate)",
         "data": "synthetic",
         "config": {"workload": args.config, "desc": CONFIG_DESC[args.config], "policy": ("RETAIN" if args.policy & 1 else "PAPER") + ("+SHARE (R20)" if args.policy & 2 else ""),
@@ -816,6 +821,7 @@ def run_dyo(args):
                  "d2h_dma_gbs": round(d2h_link, 2) if d2h_link else None,
                  "peak_theoretical_gbs": PCIE_GEN5_X16,
                  "probe_h2d_gbs": round(probe["h2d"], 2), "probe_d2h_gbs": round(probe["d2h"], 2),
+                 "probe_bidir_gbs": round(bidir, 2),
                  "frac_h2d_of_theoretical": round(h2d_link / PCIE_GEN5_X16, 4) if h2d_link else None,
                  "frac_d2h_of_theoretical": round(d2h_link / PCIE_GEN5_X16, 4) if d2h_link else None,
                  "step_gbs_per_gpu": round(value / world, 3)},
@@ -956,6 +962,89 @@ def step_bound_ms(trs, h2d_gbs, d2h_gbs, strict=False):
         f_end = max(f, e_end) if tr[6] else f
         ready.append(max(f, e_end))
     return ready[-1] if ready else 0.0
+
+
+def step_bound_fluid_ms(trs, h2d_gbs, d2h_gbs, bidir_gbs):
+    """The record-level DAG of step_bound_ms (R21 where it applies), simulated as a fluid model
+    of the PCIe link: each direction alone runs at its probe rate, both at once share the
+    measured bidirectional aggregate (in proportion to their solo rates). Transitions without
+    record detail (large plans) are one write-back and one fetch task each. ms."""
+    rh, rd = h2d_gbs * 1e6, d2h_gbs * 1e6                     # bytes per ms
+    both = bidir_gbs * 1e6
+    bh, bd = both * rh / (rh + rd), both * rd / (rh + rd)
+    bh, bd = min(bh, rh), min(bd, rd)
+    # tasks: (queue, bytes, deps); queue 0 = D2H (in order), 1 = H2D (in order)
+    tasks, ready_deps = [], []
+    for j, tr in enumerate(trs):
+        relaxed = len(tr) > 2 and tr[4] == 0 and not tr[5] and 0 < len(tr[2]) <= 64
+        half = ready_deps[j - 2] if j >= 2 else []
+        wb_ids, iv = [], []
+        if len(tr) > 2:
+            for src, nb in tr[2]:
+                tasks.append((0, nb, list(half)))
+                wb_ids.append(len(tasks) - 1)
+                iv.append((src, src + nb, len(tasks) - 1))
+        elif tr[1]:
+            tasks.append((0, tr[1], list(half)))
+            wb_ids.append(len(tasks) - 1)
+        fe_ids = []
+        fetches = tr[3] if len(tr) > 2 else ([(0, tr[0])] if tr[0] else [])
+        for dst, nb in fetches:
+            if relaxed:
+                dep = [k for lo, hi, k in iv if dst < hi and dst + nb > lo]
+                deps = list(half) + dep[-1:]
+            else:
+                deps = list(half) + wb_ids
+            tasks.append((1, nb, deps))
+            fe_ids.append(len(tasks) - 1)
+        ready_deps.append((fe_ids + wb_ids) or half)
+    n = len(tasks)
+    rem = [float(t[1]) for t in tasks]
+    done = [None] * n
+    qs = [[k for k in range(n) if tasks[k][0] == q] for q in (0, 1)]
+    head = [0, 0]
+    t = 0.0
+    while head[0] < len(qs[0]) or head[1] < len(qs[1]):
+        run = []
+        for q in (0, 1):
+            if head[q] < len(qs[q]):
+                k = qs[q][head[q]]
+                if all(done[d] is not None for d in tasks[k][2]):
+                    run.append((q, k))
+        if not run:
+            return float("nan")          # cannot happen: dependencies point backwards
+        two = len(run) == 2
+        rate = {0: bd if two else rd, 1: bh if two else rh}
+        dt = min(rem[k] / rate[q] for q, k in run)
+        t += dt
+        for q, k in run:
+            rem[k] -= dt * rate[q]
+            if rem[k] <= 1e-6:
+                done[k] = t
+                head[q] += 1
+    return t
+
+
+def bidir_probe(torch, nbytes=256 << 20, reps=3):
+    """Aggregate GB/s of one H2D and one D2H copy running at once (two streams)."""
+    h1 = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    h2 = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d1 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    d2 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(s1)
+    s2.wait_event(a)
+    for _ in range(reps):
+        with torch.cuda.stream(s1):
+            d1.copy_(h1, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h2.copy_(d2, non_blocking=True)
+    s1.wait_stream(s2)
+    b.record(s1)
+    b.synchronize()
+    return 2 * nbytes * reps / (a.elapsed_time(b) * 1e-3) / 1e9
 
 
 def _log(msg):

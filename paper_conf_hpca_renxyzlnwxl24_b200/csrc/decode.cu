@@ -28,6 +28,7 @@ __device__ __forceinline__ int* head_of(const PredDev& pd, int b) { return pd.he
 
 __global__ void __launch_bounds__(kDecThreads)
 decode_head_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int32_t* __restrict__ hist_K) {
+  pdl_enter();
   extern __shared__ __align__(16) unsigned char dsm[];
   HeadSmem& S = *reinterpret_cast<HeadSmem*>(dsm);
   double* ys = reinterpret_cast<double*>(dsm + kHeadSmemBytes);
@@ -61,6 +62,7 @@ decode_head_kernel(ArchDev a, const double* __restrict__ logits, PredDev pd, int
 template <int R>
 __global__ void __launch_bounds__(kDecThreads)
 decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int tab_cap, int pending_pass) {
+  pdl_enter();
   extern __shared__ __align__(16) unsigned char dsm[];
   DecGroupT<R>& G = *reinterpret_cast<DecGroupT<R>*>(dsm);
   int* hw = reinterpret_cast<int*>(dsm + (sizeof(DecGroupT<R>) + 15) / 16 * 16);
@@ -145,21 +147,18 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
     if (e != cudaSuccess) return e;
     hsm_set = hsm;
   }
-  decode_head_kernel<<<B, kDecThreads, hsm, s>>>(a, logits, pd, hist_K_out);
-  cudaError_t e = cudaGetLastError();
+  cudaError_t e = launch_pdl(decode_head_kernel, dim3(B), dim3(kDecThreads), hsm, s, a, logits, pd, hist_K_out);
   if (e != cudaSuccess) return e;
   // PredDev.B = the allocation's batch: the kernels walk B x K_max items of this call only
   PredDev pb = pd;
   pb.B = B;
-  decode_groups_kernel<kRecSmall><<<B * a.K_max, kDecThreads, smA, s>>>(a, pb, hist_tab_out, tab_cap, 0);
-  e = cudaGetLastError();
+  e = launch_pdl(decode_groups_kernel<kRecSmall>, dim3(B * a.K_max), dim3(kDecThreads), smA, s, a, pb, hist_tab_out, tab_cap, 0);
   if (e != cudaSuccess) return e;
   static int sms_d[64] = {};
   int& sms = sms_d[dv];
   if (!sms) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dv);
   const int gB = B * a.K_max < 2 * sms ? B * a.K_max : 2 * sms;
-  decode_groups_kernel<kRecCap><<<gB, kDecThreads, smB, s>>>(a, pb, hist_tab_out, tab_cap, 1);
-  return cudaGetLastError();
+  return launch_pdl(decode_groups_kernel<kRecCap>, dim3(gB), dim3(kDecThreads), smB, s, a, pb, hist_tab_out, tab_cap, 1);
 }
 
 }  // namespace dyo

@@ -5,6 +5,34 @@
 
 namespace dyo {
 
+// Programmatic dependent launch (PDL) for kernel chains on one stream: a kernel launched with
+// launch_pdl may be scheduled while its predecessor finishes; pdl_enter() at its top waits for
+// the predecessor grid's completion and memory flush (griddepcontrol.wait) before anything
+// reads its outputs, then lets this kernel's own successor be scheduled (every CTA has started,
+// so a waiting successor never holds slots the primary still needs). DYO_PDL=0 disables it.
+__device__ __forceinline__ void pdl_enter() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+int pdl_enabled();   // api / launch side: 1 unless DYO_PDL=0
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
 // Exclusive scan of one int per thread over the block; *total gets the sum (all threads).
 // warp_tmp: >= 32 ints of shared memory. Contains three __syncthreads().
 __device__ __forceinline__ int block_scan(int v, int* warp_tmp, int* total) {

@@ -36,6 +36,12 @@
 
 namespace dyo {
 
+int pdl_enabled() {
+  static int v = -1;
+  if (v < 0) { const char* e = getenv("DYO_PDL"); v = (e && e[0] == '0') ? 0 : 1; }
+  return v;
+}
+
 constexpr int NT = kPlanThreads;                  // 1024
 constexpr uint64_t kInfD = 0xFFFFull;
 constexpr int kInwSmemWords = 8192;               // smem W_j bitmap for T <= 2^18
@@ -100,6 +106,7 @@ __device__ __forceinline__ bool bit_get(const uint32_t* b, int t) { return (b[t 
 // ---- 0. group list + entry bases -------------------------------------------------------
 __global__ void __launch_bounds__(NT, 1)
 plan_prep_kernel(ArchDev a, PredDev pd, int b0, int nb, PlanScratch sc, PlanOut out, int max_groups) {
+  pdl_enter();
   __shared__ long long tmp[32];
   __shared__ int s_fail;
   const int tid = threadIdx.x;
@@ -141,6 +148,7 @@ plan_prep_kernel(ArchDev a, PredDev pd, int b0, int nb, PlanScratch sc, PlanOut 
 
 // ---- bucket kernels: next occurrence of every entry's tensor ---------------------------
 __global__ void bucket_init_kernel(ArchDev a, PlanScratch sc) {
+  pdl_enter();
   for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < a.T; t += gridDim.x * blockDim.x) {
     sc.bcnt[t] = 0;
     sc.bfill[t] = 0;
@@ -159,6 +167,7 @@ __device__ __forceinline__ const int2* group_entries(const ArchDev& a, const Pre
 
 // one block per group (grid-stride)
 __global__ void bucket_count_kernel(ArchDev a, PredDev pd, PlanScratch sc) {
+  pdl_enter();
   const int Kt = sc.Kt[0];
   for (int g = blockIdx.x; g < Kt; g += gridDim.x) {
     int n;
@@ -169,6 +178,7 @@ __global__ void bucket_count_kernel(ArchDev a, PredDev pd, PlanScratch sc) {
 
 // exclusive scan of the bucket counts (one CTA, a contiguous chunk of tensors per thread)
 __global__ void __launch_bounds__(NT, 1) bucket_scan_kernel(ArchDev a, PlanScratch sc) {
+  pdl_enter();
   __shared__ long long tmp[32];
   if (sc.Kt[0] < 0) return;
   const int T = a.T, per = (T + NT - 1) / NT;
@@ -186,6 +196,7 @@ __global__ void __launch_bounds__(NT, 1) bucket_scan_kernel(ArchDev a, PlanScrat
 }
 
 __global__ void bucket_fill_kernel(ArchDev a, PredDev pd, PlanScratch sc) {
+  pdl_enter();
   const int Kt = sc.Kt[0];
   for (int g = blockIdx.x; g < Kt; g += gridDim.x) {
     int n;
@@ -201,6 +212,7 @@ __global__ void bucket_fill_kernel(ArchDev a, PredDev pd, PlanScratch sc) {
 // group), then every entry learns the next group holding the tensor and whether that
 // occurrence reads it first; the tensor learns its first occurrence in the plan
 __global__ void bucket_sort_kernel(ArchDev a, PredDev pd, PlanScratch sc) {
+  pdl_enter();
   if (sc.Kt[0] < 0) return;
   const int lane = threadIdx.x & 31;
   const int warps = (gridDim.x * blockDim.x) >> 5;
@@ -401,6 +413,7 @@ __device__ __forceinline__ bool rec_evicted(int4 r, int k, int rule, uint64_t th
 __global__ void __launch_bounds__(PNT, 1)
 plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanScratch sc, PlanOut out,
             int inw_smem) {
+  pdl_enter();
   extern __shared__ __align__(16) unsigned char smem_raw[];
   PlanSmem& S = *reinterpret_cast<PlanSmem*>(smem_raw);
   uint32_t* inw = inw_smem ? reinterpret_cast<uint32_t*>(smem_raw + (sizeof(PlanSmem) + 15) / 16 * 16) : sc.inw;
@@ -1200,6 +1213,7 @@ cudaError_t launch_fault_drop(const ArchDev& a, const PredDev& pd, int b0, int n
 
 // 8-byte words of the record arrays, grid-stride over all six lists
 __global__ void plan_export_kernel(PlanOut d, PlanOut h) {
+  pdl_enter();
   if (d.status[0] != 0) return;
   const int K = d.counts[0];
   const int64_t n[6] = {(int64_t)K * (int64_t)(sizeof(PlanHdr) / 8), (int64_t)d.counts[1] * 5, (int64_t)d.counts[2] * 4,
@@ -1218,7 +1232,8 @@ __global__ void plan_export_kernel(PlanOut d, PlanOut h) {
 cudaError_t launch_plan_export(const PlanOut& d, const PlanOut& h, cudaStream_t s) {
   static_assert(sizeof(PlanHdr) % 8 == 0 && sizeof(dyo_evict_rec) == 40 && sizeof(dyo_move_rec) == 32 &&
                 sizeof(dyo_carry_rec) == 40 && sizeof(dyo_alloc_rec) == 24 && sizeof(dyo_fetch_rec) == 32, "record layout");
-  plan_export_kernel<<<64, 256, 0, s>>>(d, h);
+  cudaError_t le = launch_pdl(plan_export_kernel, dim3(64), dim3(256), 0, s, d, h);
+  if (le != cudaSuccess) return le;
   return cudaGetLastError();
 }
 
@@ -1237,14 +1252,15 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
     attr_done |= bit;
   }
   if (nb > NT) return cudaErrorInvalidValue;
-  plan_prep_kernel<<<1, NT, 0, s>>>(a, pd, b0, nb, sc, out, max_groups);
+  cudaError_t le = launch_pdl(plan_prep_kernel, dim3(1), dim3(NT), 0, s, a, pd, b0, nb, sc, out, max_groups);
+  if (le != cudaSuccess) return le;
   const int grid = 296;
-  bucket_init_kernel<<<grid, 256, 0, s>>>(a, sc);
-  bucket_count_kernel<<<grid, 256, 0, s>>>(a, pd, sc);
-  bucket_scan_kernel<<<1, NT, 0, s>>>(a, sc);
-  bucket_fill_kernel<<<grid, 256, 0, s>>>(a, pd, sc);
-  bucket_sort_kernel<<<grid * 2, 256, 0, s>>>(a, pd, sc);
-  plan_kernel<<<1, PNT, smem, s>>>(a, pd, policy, in, work, sc, out, inw_smem);
+  if ((le = launch_pdl(bucket_init_kernel, dim3(grid), dim3(256), 0, s, a, sc)) != cudaSuccess) return le;
+  if ((le = launch_pdl(bucket_count_kernel, dim3(grid), dim3(256), 0, s, a, pd, sc)) != cudaSuccess) return le;
+  if ((le = launch_pdl(bucket_scan_kernel, dim3(1), dim3(NT), 0, s, a, sc)) != cudaSuccess) return le;
+  if ((le = launch_pdl(bucket_fill_kernel, dim3(grid), dim3(256), 0, s, a, pd, sc)) != cudaSuccess) return le;
+  if ((le = launch_pdl(bucket_sort_kernel, dim3(grid * 2), dim3(256), 0, s, a, pd, sc)) != cudaSuccess) return le;
+  if ((le = launch_pdl(plan_kernel, dim3(1), dim3(PNT), smem, s, a, pd, policy, in, work, sc, out, inw_smem)) != cudaSuccess) return le;
   return cudaGetLastError();
 }
 

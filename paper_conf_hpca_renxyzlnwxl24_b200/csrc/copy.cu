@@ -122,6 +122,23 @@ struct RecCursor {
   }
 };
 
+// Grid barrier of a cooperative multi-wave launch: every CTA's copies of the wave have read
+// their sources (the elected thread waited for its bulk stores, the threads' byte tails are
+// done) before any CTA starts the next wave, whose destinations may overlap them (a compaction
+// wave ends where a later move's destination meets an earlier move's source).
+__device__ __forceinline__ void copy_grid_barrier(unsigned int* ctr, unsigned int target) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(ctr, 1u);
+    unsigned int v;
+    do {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+    } while ((int)(v - target) < 0);
+  }
+  __syncthreads();
+}
+
 template <int kTmaStages, int kTmaChunk>
 __global__ void __launch_bounds__(kRecThreads)
 copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
@@ -131,9 +148,18 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
   __shared__ int s_i0;
   __shared__ int64_t s_off0;
   constexpr int L = kTmaStages - 1;          // loads kept in flight ahead of the store cursor
-  const RecCopyArgs* a = &args;
   unsigned long long t_enter = 0, t_scan = 0;
-  if (a->stamps != nullptr && threadIdx.x == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_enter));
+  if (args.stamps != nullptr && threadIdx.x == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_enter));
+  const int nwaves = args.n_waves > 1 ? args.n_waves : 1;
+  for (int wv = 0; wv < nwaves; ++wv) {
+  RecCopyArgs aw = args;
+  if (nwaves > 1) {
+    const int r0 = wv ? args.wave_end[wv - 1] : 0;
+    aw.rec = args.rec + (int64_t)r0 * args.stride;
+    aw.n = args.wave_end[wv] - r0;
+    aw.total = args.wave_total[wv];
+  }
+  const RecCopyArgs* a = &aw;
   // the stream: the records' bodies, or the single range's body (0 when unaligned)
   const bool single = a->rec == nullptr;
   const int64_t T = !single ? a->total
@@ -209,6 +235,8 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
       }
     }
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    // the next wave initialises the barriers again
+    for (int q = 0; q < kTmaStages; ++q) asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(su32(&bar[q])) : "memory");
   }
   // < 16-byte tails and unaligned records: byte copies, record k by CTA k % grid
   if (single) {
@@ -225,6 +253,9 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
       for (int64_t x = (al ? nb & ~(int64_t)15 : 0) + threadIdx.x; x < nb; x += blockDim.x) dp[x] = sp[x];
     }
   }
+  if (wv + 1 < nwaves) copy_grid_barrier(args.gbar, args.gbar_base + (unsigned)(wv + 1) * gridDim.x);
+  }   // waves
+  const RecCopyArgs* a = &args;
   // exit stamp after every copy of the CTA, the byte tails included
   if (a->stamps != nullptr) {
     __syncthreads();
@@ -244,7 +275,7 @@ copy_records_tma_kernel(const __grid_constant__ RecCopyArgs args) {
 }
 
 template <int S, int C>
-static cudaError_t launch_ring(const RecCopyArgs& a, int grid, cudaStream_t s) {
+static cudaError_t launch_ring(const RecCopyArgs& a, int grid, cudaStream_t s, int* grid_used) {
   static uint64_t attr_done = 0;                  // bit d: attributes set on device d
   const uint64_t bit = 1ull << current_device();
   const int smem = S * C;
@@ -260,11 +291,27 @@ static cudaError_t launch_ring(const RecCopyArgs& a, int grid, cudaStream_t s) {
       }
     attr_done |= bit;
   }
+  if (a.n_waves > 1) {
+    // multi-wave: the whole grid, co-resident (cooperative launch) for the grid barriers
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kRecThreads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeCooperative;
+    at[0].val.cooperative = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    if (grid_used) *grid_used = grid;
+    return cudaLaunchKernelEx(&cfg, copy_records_tma_kernel<S, C>, a);
+  }
   // at least one chunk per CTA; enough CTAs for the tail loop over the records
   int64_t g = (a.total + C - 1) / C;
   if (a.rec != nullptr && g < a.n) g = a.n;
   if (g > grid) g = grid;
   if (g < 1) g = 1;
+  if (grid_used) *grid_used = (int)g;
   copy_records_tma_kernel<S, C><<<(int)g, kRecThreads, smem, s>>>(a);
   return cudaGetLastError();
 }
@@ -327,7 +374,7 @@ int64_t copy_stamps_read(unsigned long long* host, int64_t cap) {
   return (int64_t)n;
 }
 
-cudaError_t launch_copy_records(const RecCopyArgs& a0, int grid, cudaStream_t s) {
+cudaError_t launch_copy_records(const RecCopyArgs& a0, int grid, cudaStream_t s, int* grid_used) {
   if (a0.total <= 0 && (a0.rec == nullptr || a0.n <= 0)) return cudaSuccess;
   RecCopyArgs a = a0;
   static int stamps_on = -1;
@@ -345,11 +392,11 @@ cudaError_t launch_copy_records(const RecCopyArgs& a0, int grid, cudaStream_t s)
   grid *= tma_ctas_per_sm();
   cudaError_t e;
   switch (tma_ring()) {
-    case 1: e = launch_ring<8, 16 << 10>(a, grid, s); break;
-    case 2: e = launch_ring<4, 32 << 10>(a, grid, s); break;
-    case 3: e = launch_ring<6, 32 << 10>(a, grid, s); break;
-    case 4: e = launch_ring<3, 64 << 10>(a, grid, s); break;
-    default: e = launch_ring<kTmaStages, kTmaChunk>(a, grid, s); break;
+    case 1: e = launch_ring<8, 16 << 10>(a, grid, s, grid_used); break;
+    case 2: e = launch_ring<4, 32 << 10>(a, grid, s, grid_used); break;
+    case 3: e = launch_ring<6, 32 << 10>(a, grid, s, grid_used); break;
+    case 4: e = launch_ring<3, 64 << 10>(a, grid, s, grid_used); break;
+    default: e = launch_ring<kTmaStages, kTmaChunk>(a, grid, s, grid_used); break;
   }
   if (e == cudaSuccess && stamps_on == 2) {
     copy_mark_kernel<<<1, 1, 0, s>>>(g_stamps, a.launch, 1);

@@ -291,6 +291,7 @@ cudaError_t launch_copy_segments(const CopySeg* segs_dev_or_mapped, int n, int64
 // rec == nullptr: one range of `total` bytes from src_base to dst_base. total = sum over the
 // selected records of their 16-byte-aligned bodies (bytes & ~15, or 0 when src or dst is not
 // 16-byte aligned): the host computes it with rec_body() below.
+constexpr int kMaxWaves = 24;    // compaction waves per record-copy launch (grid barrier between)
 struct RecCopyArgs {
   const int64_t* rec;
   int32_t stride, n, f_src, f_dst, f_bytes, f_late;
@@ -301,11 +302,19 @@ struct RecCopyArgs {
   int64_t total;
   unsigned long long* stamps;  // measurement aid (DYO_COPY_STAMPS): 4 x u64 per CTA, or null
   int64_t launch;              // launch index for the stamps
+  // n_waves > 1: the records are processed as consecutive waves [wave_end[w-1], wave_end[w])
+  // (relative to rec) of wave_total[w] body bytes each, every CTA arriving at a grid barrier
+  // (counter gbar, target gbar_base + (w+1) * grid) between waves; cooperative launch
+  int32_t n_waves;
+  int32_t wave_end[kMaxWaves];
+  int64_t wave_total[kMaxWaves];
+  unsigned int* gbar;
+  unsigned int gbar_base;
 };
 int64_t copy_stamps_read(unsigned long long* host, int64_t cap);
 inline int64_t rec_body(const char* src, const char* dst, int64_t bytes) {
   return ((((uintptr_t)src) | ((uintptr_t)dst)) & 15) == 0 ? (bytes & ~(int64_t)15) : 0;
 }
-cudaError_t launch_copy_records(const RecCopyArgs& a, int grid, cudaStream_t s);
+cudaError_t launch_copy_records(const RecCopyArgs& a, int grid, cudaStream_t s, int* grid_used = nullptr);
 
 }  // namespace dyo

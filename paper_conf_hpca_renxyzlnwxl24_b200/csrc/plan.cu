@@ -265,7 +265,8 @@ __global__ void bucket_sort_kernel(ArchDev a, PredDev pd, PlanScratch sc) {
 // transition; larger halves re-read their chunk in RPT-record windows (same code, same order).
 // Every W_j entry's per-tensor state is gathered into shared memory in one round trip (phase A)
 // and everything after it that concerns W_j (placement, records, rebuild) reads shared memory.
-constexpr int PNT = 512;
+constexpr int kPlanBig = 512;                     // planner threads (large halves)
+constexpr int kPlanSmall = 128;                   // small problems: fewer warps per barrier
 constexpr int RPT = 16;                           // records per thread kept in registers
 constexpr int kHash = 2048;                       // W_j: tensor -> entry (open addressing)
 constexpr int kGapSmem = 4096;                    // gaps in shared memory up to this
@@ -410,6 +411,7 @@ __device__ __forceinline__ bool rec_evicted(int4 r, int k, int rule, uint64_t th
     }                                                                                           \
   }
 
+template <int PNT>
 __global__ void __launch_bounds__(PNT, 1)
 plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanScratch sc, PlanOut out,
             int inw_smem) {
@@ -593,7 +595,7 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
       const int kper = (int)((nlive + PNT - 1) / PNT);
       const int k0 = min((int)nlive, tid * kper), k1 = min((int)nlive, k0 + kper);
       for (int shift = 56; shift >= 0; shift -= 8) {
-        if (tid < 256) { S.hist[tid] = 0; S.hcnt[tid] = 0; }
+        for (int hb = tid; hb < 256; hb += PNT) { S.hist[hb] = 0; S.hcnt[hb] = 0; }
         __syncthreads();
         for (int k = k0; k < k1; ++k) {
           const uint64_t key = sc.keys[k];
@@ -1246,11 +1248,20 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
   const int inw_smem = a.T <= kInwSmemWords * 32 ? 1 : 0;
   const size_t smem = base + (inw_smem ? (size_t)kInwSmemWords * 4 : 0);
   if (!(attr_done & bit)) {
-    cudaError_t e = cudaFuncSetAttribute(plan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(plan_kernel<kPlanBig>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)(base + (size_t)kInwSmemWords * 4));
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(plan_kernel<kPlanSmall>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(base + (size_t)kInwSmemWords * 4));
     if (e != cudaSuccess) return e;
     attr_done |= bit;
   }
+  // small problems (every resident record of a half fits 16 registers of 128 threads) run with
+  // 4 warps: the per-transition cost is barrier latency, which grows with the warps waited on.
+  // DYO_PLAN_THREADS=128|512 forces one (measurement; both are tested bit-exact)
+  static int forced = -1;
+  if (forced < 0) { const char* e = getenv("DYO_PLAN_THREADS"); forced = e ? atoi(e) : 0; }
+  const bool small = forced == 128 || (forced != 512 && a.T <= kPlanSmall * 16);
   if (nb > NT) return cudaErrorInvalidValue;
   cudaError_t le = launch_pdl(plan_prep_kernel, dim3(1), dim3(NT), 0, s, a, pd, b0, nb, sc, out, max_groups);
   if (le != cudaSuccess) return le;
@@ -1260,7 +1271,11 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
   if ((le = launch_pdl(bucket_scan_kernel, dim3(1), dim3(NT), 0, s, a, sc)) != cudaSuccess) return le;
   if ((le = launch_pdl(bucket_fill_kernel, dim3(grid), dim3(256), 0, s, a, pd, sc)) != cudaSuccess) return le;
   if ((le = launch_pdl(bucket_sort_kernel, dim3(grid * 2), dim3(256), 0, s, a, pd, sc)) != cudaSuccess) return le;
-  if ((le = launch_pdl(plan_kernel, dim3(1), dim3(PNT), smem, s, a, pd, policy, in, work, sc, out, inw_smem)) != cudaSuccess) return le;
+  if (small)
+    le = launch_pdl(plan_kernel<kPlanSmall>, dim3(1), dim3(kPlanSmall), smem, s, a, pd, policy, in, work, sc, out, inw_smem);
+  else
+    le = launch_pdl(plan_kernel<kPlanBig>, dim3(1), dim3(kPlanBig), smem, s, a, pd, policy, in, work, sc, out, inw_smem);
+  if (le != cudaSuccess) return le;
   return cudaGetLastError();
 }
 

@@ -1256,12 +1256,12 @@ cudaError_t launch_plan(const ArchDev& a, const PredDev& pd, int b0, int nb, int
     if (e != cudaSuccess) return e;
     attr_done |= bit;
   }
-  // small problems (every resident record of a half fits 16 registers of 128 threads) run with
-  // 4 warps: the per-transition cost is barrier latency, which grows with the warps waited on.
-  // DYO_PLAN_THREADS=128|512 forces one (measurement; both are tested bit-exact)
+  // DYO_PLAN_THREADS=128: the 4-warp planner (measured slower than 512 threads even on the small
+  // MoE / AF halves - 0.56 vs 0.47 ms, 3.2 vs 2.7 ms per plan - the per-transition latency is
+  // the threads' serial work between barriers, not the barriers; kept as a tested variant)
   static int forced = -1;
   if (forced < 0) { const char* e = getenv("DYO_PLAN_THREADS"); forced = e ? atoi(e) : 0; }
-  const bool small = forced == 128 || (forced != 512 && a.T <= kPlanSmall * 16);
+  const bool small = forced == 128 && a.T <= kPlanSmall * 16 * 64;
   if (nb > NT) return cudaErrorInvalidValue;
   cudaError_t le = launch_pdl(plan_prep_kernel, dim3(1), dim3(NT), 0, s, a, pd, b0, nb, sc, out, max_groups);
   if (le != cudaSuccess) return le;

@@ -965,39 +965,36 @@ def step_bound_ms(trs, h2d_gbs, d2h_gbs, strict=False):
 
 
 def step_bound_fluid_ms(trs, h2d_gbs, d2h_gbs, bidir_gbs):
-    """The record-level DAG of step_bound_ms (R21 where it applies), simulated as a fluid model
-    of the PCIe link: each direction alone runs at its probe rate, both at once share the
-    measured bidirectional aggregate (in proportion to their solo rates). Transitions without
-    record detail (large plans) are one write-back and one fetch task each. ms."""
+    """The record-level DAG of step_bound_ms (the same dependencies: each direction's queue in
+    order, EVICT_j after ready[j-2], FETCH_j after the whole EVICT_j (R12) or after the write-backs
+    it overwrites (R21), ready[j] after both queues' work of transition j) simulated as a fluid
+    model of the PCIe link: each direction alone runs at its probe rate, both at once share the
+    measured bidirectional aggregate (in proportion to their solo rates). ms."""
     rh, rd = h2d_gbs * 1e6, d2h_gbs * 1e6                     # bytes per ms
     both = bidir_gbs * 1e6
-    bh, bd = both * rh / (rh + rd), both * rd / (rh + rd)
-    bh, bd = min(bh, rh), min(bd, rd)
-    # tasks: (queue, bytes, deps); queue 0 = D2H (in order), 1 = H2D (in order)
-    tasks, ready_deps = [], []
+    bh, bd = min(both * rh / (rh + rd), rh), min(both * rd / (rh + rd), rd)
+    tasks, ready_deps = [], []                                 # task: (queue 0 D2H / 1 H2D, bytes, deps)
+    last = [None, None]                                        # latest task of each queue so far
     for j, tr in enumerate(trs):
         relaxed = len(tr) > 2 and tr[4] == 0 and not tr[5] and 0 < len(tr[2]) <= 64
         half = ready_deps[j - 2] if j >= 2 else []
-        wb_ids, iv = [], []
-        if len(tr) > 2:
-            for src, nb in tr[2]:
-                tasks.append((0, nb, list(half)))
-                wb_ids.append(len(tasks) - 1)
-                iv.append((src, src + nb, len(tasks) - 1))
-        elif tr[1]:
-            tasks.append((0, tr[1], list(half)))
-            wb_ids.append(len(tasks) - 1)
-        fe_ids = []
+        iv = []
+        wbs = tr[2] if len(tr) > 2 else ([(0, tr[1])] if tr[1] else [])
+        for src, nb in wbs:
+            tasks.append((0, nb, list(half)))
+            last[0] = len(tasks) - 1
+            iv.append((src, src + nb, last[0]))
+        evict_end = [last[0]] if last[0] is not None else []
         fetches = tr[3] if len(tr) > 2 else ([(0, tr[0])] if tr[0] else [])
         for dst, nb in fetches:
             if relaxed:
                 dep = [k for lo, hi, k in iv if dst < hi and dst + nb > lo]
                 deps = list(half) + dep[-1:]
             else:
-                deps = list(half) + wb_ids
+                deps = list(half) + evict_end
             tasks.append((1, nb, deps))
-            fe_ids.append(len(tasks) - 1)
-        ready_deps.append((fe_ids + wb_ids) or half)
+            last[1] = len(tasks) - 1
+        ready_deps.append(list(half) + [k for k in last if k is not None])
     n = len(tasks)
     rem = [float(t[1]) for t in tasks]
     done = [None] * n
@@ -1022,7 +1019,7 @@ def step_bound_fluid_ms(trs, h2d_gbs, d2h_gbs, bidir_gbs):
             if rem[k] <= 1e-6:
                 done[k] = t
                 head[q] += 1
-    return t
+    return max([t for t in done if t is not None] or [0.0])
 
 
 def bidir_probe(torch, nbytes=256 << 20, reps=3):

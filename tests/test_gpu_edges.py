@@ -62,3 +62,32 @@ def test_ragged_tensor_core_batches(name, B):
     r1 = oracle_step(wl, [B], PL.initial_state(len(wl.tensors)), r["table"], plan=False)
     _check_prediction(d, wl, 0, r1["preds"][0])
     d.close()
+
+
+def test_max_batch_1024_predict_and_plan():
+    """Maximum sizes: the largest prediction batch the ABI accepts (max_batch 1024) on the tiny
+    workload - 1,024 predictions in one dyo_pilot_predict (batch kernel, clusters co-resident by
+    the launch's cluster-size choice), decoded on the GPU, then one plan of their 8,192 groups:
+    logits (north_star gate) and decodes on a sample of the predictions, every transition of the
+    plan bit-exact with the oracle."""
+    from gpu_harness import logit_gates
+    B = 1024
+    wl = WL.make("tiny", n_samples=B)
+    d = make_ctx(wl, max_batch=B, flags=F_NO_HOST_POOL)
+    logits = torch.zeros((B, wl.pilot.O), device="cuda")
+    d.predict(wl.samples[:B].copy(), hist_for(wl, B), B, logits, stream=_stream())
+    r = oracle_step(wl, range(B), PL.initial_state(len(wl.tensors)), ())
+    assert r["err"] is None
+    y = logits.cpu().numpy()
+    for b in list(range(0, B, 97)) + [B - 1]:
+        g1, g2, _ = logit_gates(y[b], r["feats"][b], wl.pilot, wl.nn_type)
+        assert g1.all() and g2.all(), f"prediction {b}"
+        _check_prediction(d, wl, b, r["preds"][b])
+    K = d.plan(stream=_stream())
+    assert K == len(r["trs"]) == sum(len(p.W) for p in r["preds"])
+    for j, tr in enumerate(r["trs"]):
+        info = d.plan_info(j)
+        assert (info["half"], info["h2d"], info["d2h"], info["d2d"], info["need"]) == \
+            (tr.half, tr.h2d, tr.d2h, tr.d2d, tr.need), f"transition {j}"
+        assert gpu_lists(d, j) == tr_lists(tr), f"transition {j}"
+    d.close()

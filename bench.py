@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--budget-gib", type=float, default=0.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-faults", action="store_true", help="skip the on-demand fetch measurement")
+    ap.add_argument("--sm-copy", action="store_true",
+                    help="DYO_F_SM_COPY: device moves by the SM vector-copy kernel (host-built work items) instead of TMA")
     ap.add_argument("--strict-order", action="store_true",
                     help="DYO_F_STRICT_ORDER: R12's whole-phase EVICT -> FETCH order instead of R21's per-range order")
     ap.add_argument("--dist-backend", default=None, help="nccl (default with CUDA) or gloo")
@@ -454,7 +456,7 @@ def run_dyo(args):
     _log("workload built")
     B = wl.notes.get("batch", 1)          # predictions planned per step (lstm: a minibatch of 64)
     d = Dyo(wl.budget, wl.align, wl.policy, max_batch=B, device=local,
-            flags=64 if args.strict_order else 0)   # headline: uninstrumented
+            flags=(64 if args.strict_order else 0) | (16 if args.sm_copy else 0))   # headline: uninstrumented
     d.load(wl)
     _log("ctx loaded")
     s0 = torch.cuda.current_stream()

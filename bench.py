@@ -483,11 +483,18 @@ def run_dyo(args):
 
     per_tr = []                               # (h2d, d2h) of every transition planned (step bound)
 
-    def plan_next(desc, hist):
-        """Predict + plan one step (the plan is double-buffered: this may run while the previous
-        step's transitions are still migrating)."""
+    def plan_start(desc, hist):
+        """Predict + launch the plan of one step (dyo_plan_async: the host goes on enqueuing the
+        previous step's transitions while the planner runs)."""
         d.predict(desc, hist, B, stream=s0.cuda_stream)
-        K = d.plan(stream=s0.cuda_stream)
+        d.plan_async(stream=s0.cuda_stream)
+
+    def plan_next(desc=None, hist=None):
+        """Complete a plan (dyo_plan_wait: the one host sync) and read its byte counts; with
+        inputs, predict + plan first."""
+        if desc is not None:
+            plan_start(desc, hist)
+        K = d.plan_wait()
         h2d = d2h = 0
         trs = []
         for j in range(K):
@@ -528,18 +535,21 @@ def run_dyo(args):
             s1.wait_event(ready[K - 1])      # R21: the last ready[] may be joined off the copy stream
 
     def run_steps(n, first, inputs):
-        """n steps with plan lookahead: step i's transitions are enqueued, then step i+1 is
-        predicted and planned while they run."""
+        """n steps with plan lookahead: step i+1 is predicted and its planner launched, step i's
+        transitions are enqueued while the planner runs (dyo_plan_async), then the plan is
+        completed (dyo_plan_wait) while step i migrates."""
         tot = [0, 0, 0]
         pending = plan_next(*inputs(first))
         for i in range(n):
             K, h2d, d2h = pending
+            if i + 1 < n:
+                plan_start(*inputs(first + i + 1))
             enqueue(K)
             tot[0] += K
             tot[1] += h2d
             tot[2] += d2h
             if i + 1 < n:
-                pending = plan_next(*inputs(first + i + 1))
+                pending = plan_next()
         return tot
 
     def barrier():

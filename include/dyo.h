@@ -283,6 +283,15 @@ dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* out, i
  * migrations of the plan two generations back to finish. In a plan-only ctx
  * (DYO_F_NO_HOST_POOL) each plan supersedes the previous ones. */
 dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* stream);
+/* dyo_plan in two halves, so the host can enqueue the previous plan's transitions while this
+ * plan's kernels run: dyo_plan_async launches the planner (same arguments and checks as dyo_plan,
+ * no synchronisation); dyo_plan_wait takes the one synchronisation and commits the plan (K_out,
+ * DYO_E_BUDGET / DYO_E_CAPACITY as dyo_plan, state unchanged on error). Between the two only
+ * dyo_migrate (of older plans), dyo_fault_* and the read-only queries of the previous plan are
+ * allowed; dyo_pilot_predict, dyo_residency and dyo_load_* return DYO_E_STATE, as does a second
+ * dyo_plan_async or a dyo_plan_wait without a pending plan. */
+dyo_status dyo_plan_async(dyo_ctx* ctx, int32_t b0, int32_t n, void* stream);
+dyo_status dyo_plan_wait(dyo_ctx* ctx, int32_t* K_out);
 
 /* Host copies of the most recent plan (valid until the dyo_plan after next). */
 dyo_status dyo_plan_info(dyo_ctx* ctx, int32_t j, dyo_transition_info* info);

@@ -155,6 +155,8 @@ struct dyo_ctx {
   cudaEvent_t ev_entry = nullptr, ev_evict = nullptr, ev_moves = nullptr, ev_carry = nullptr;
   std::vector<cudaEvent_t> ev_wb;   // R21: one per write-back copy group of a transition (D2H stream order)
   cudaStream_t join = nullptr;      // R21: ready[j] = FETCH_j + EVICT_j joined off the copy stream
+  bool plan_pending = false;        // dyo_plan_async issued, dyo_plan_wait not yet called
+  cudaStream_t plan_stream = nullptr;
   unsigned int* gbar = nullptr;     // grid-barrier counter of the multi-wave compaction launches
   unsigned int gbar_issued = 0;     // arrivals the launches enqueued so far (stream order on copy_stream)
   cudaEvent_t ev_tail = nullptr;
@@ -827,6 +829,7 @@ dyo_status dyo_destroy(dyo_ctx* ctx) {
 }
 
 dyo_status dyo_load_arch(dyo_ctx* ctx, const dyo_arch* A) {
+  if (ctx && ctx->plan_pending) return fail(ctx, DYO_E_STATE, "dyo_load_arch: a plan is pending (dyo_plan_wait first)");
   if (!ctx || !A) return DYO_E_INVAL;
   CK(cudaSetDevice(ctx->device));
   CK(cudaDeviceSynchronize());
@@ -1221,6 +1224,7 @@ static dyo_status build_tc_plan(dyo_ctx* ctx, const dyo_pilot_desc* w) {
 }
 
 dyo_status dyo_load_pilot(dyo_ctx* ctx, const dyo_pilot_desc* w) {
+  if (ctx && ctx->plan_pending) return fail(ctx, DYO_E_STATE, "dyo_load_pilot: a plan is pending (dyo_plan_wait first)");
   if (!ctx || !w) return DYO_E_INVAL;
   if (!ctx->arch_ok) return fail(ctx, DYO_E_STATE, "load the arch first");
   CK(cudaSetDevice(ctx->device));
@@ -1371,6 +1375,7 @@ dyo_status dyo_encode_features(dyo_ctx* ctx, const dyo_sample* s, int32_t B, flo
 
 dyo_status dyo_pilot_predict(dyo_ctx* ctx, const float* feat, const dyo_sample* s, int32_t B,
                              float* logits, void* stream) {
+  if (ctx && ctx->plan_pending) return fail(ctx, DYO_E_STATE, "dyo_pilot_predict: a plan is pending (dyo_plan_wait first)");
   if (!ctx) return DYO_E_INVAL;
   if (!ctx->arch_ok || !ctx->pilot_ok) return fail(ctx, DYO_E_STATE, "load arch and pilot first");
   if (B < 1 || B > ctx->cfg.max_batch) return fail(ctx, DYO_E_INVAL, "B=%d out of [1, max_batch]", B);
@@ -1741,8 +1746,11 @@ dyo_status dyo_group_entries(dyo_ctx* ctx, int32_t b, int32_t g, int32_t* outp, 
   return DYO_OK;
 }
 
-dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* stream) {
+static dyo_status plan_complete(dyo_ctx* ctx, int32_t* K_out);
+
+dyo_status dyo_plan_async(dyo_ctx* ctx, int32_t b0, int32_t n, void* stream) {
   if (!ctx) return DYO_E_INVAL;
+  if (ctx->plan_pending) return fail(ctx, DYO_E_STATE, "a plan is pending: dyo_plan_wait first");
   if (!ctx->arch_ok || ctx->last_B <= 0) return fail(ctx, DYO_E_STATE, "no prediction to plan");
   if (n < 0) { b0 = 0; n = ctx->last_B; }
   if (b0 < 0 || n < 1 || b0 + n > ctx->last_B) return fail(ctx, DYO_E_INVAL, "prediction range");
@@ -1795,6 +1803,29 @@ dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* s
   CK(launch_plan_export(P.dout, P.hout, st));
   CK(cudaMemcpyAsync(ctx->h_loc, wk.loc, ctx->T, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(ctx->h_off, wk.off, sizeof(int64_t) * ctx->T, cudaMemcpyDeviceToHost, st));
+  ctx->plan_pending = true;
+  ctx->plan_stream = st;
+  return DYO_OK;
+}
+
+dyo_status dyo_plan_wait(dyo_ctx* ctx, int32_t* K_out) {
+  if (!ctx) return DYO_E_INVAL;
+  if (!ctx->plan_pending) return fail(ctx, DYO_E_STATE, "no pending plan");
+  return plan_complete(ctx, K_out);
+}
+
+dyo_status dyo_plan(dyo_ctx* ctx, int32_t b0, int32_t n, int32_t* K_out, void* stream) {
+  dyo_status s0 = dyo_plan_async(ctx, b0, n, stream);
+  if (s0) return s0;
+  return plan_complete(ctx, K_out);
+}
+
+static dyo_status plan_complete(dyo_ctx* ctx, int32_t* K_out) {
+  ctx->plan_pending = false;
+  CK(cudaSetDevice(ctx->device));
+  cudaStream_t st = ctx->plan_stream;
+  dyo_ctx::PlanSlot& P = ctx->slot[ctx->plan_seq & 1];
+  PlanState& in = ctx->state[ctx->committed];
   CK(cudaStreamSynchronize(st));     // the one synchronisation of the hot path (DMA sizes to host)
   ctx->last_plan_syncs = 1;
   const int32_t status = ctx->h_status[0];
@@ -2620,6 +2651,7 @@ dyo_status dyo_fault_stats(dyo_ctx* ctx, int64_t* faults, int64_t* bytes, int64_
 }
 
 dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr) {
+  if (ctx && ctx->plan_pending) return fail(ctx, DYO_E_STATE, "dyo_residency: a plan is pending (dyo_plan_wait first)");
   if (!ctx || !dev_ptr || t < 0 || t >= ctx->T) return DYO_E_INVAL;
   const int8_t l = ctx->h_loc[t];
   *dev_ptr = l < 0 ? nullptr : ctx->arena + (int64_t)l * ctx->H + ctx->h_off[t];

@@ -95,7 +95,7 @@ def lib():
         L.dyo_last_error.argtypes = [P]
         for name in ("dyo_create", "dyo_destroy", "dyo_load_arch", "dyo_load_pilot", "dyo_host_pool",
                      "dyo_arena", "dyo_encode_features", "dyo_pilot_predict", "dyo_prediction_get",
-                     "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records", "dyo_migrate",
+                     "dyo_group_entries", "dyo_plan", "dyo_plan_async", "dyo_plan_wait", "dyo_plan_info", "dyo_plan_records", "dyo_migrate",
                      "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
                      "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
                      "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats",
@@ -110,7 +110,8 @@ def lib():
 
 EXPORTS = ("dyo_strerror", "dyo_last_error", "dyo_version", "dyo_create", "dyo_destroy", "dyo_load_arch",
            "dyo_load_pilot", "dyo_host_pool", "dyo_arena", "dyo_encode_features", "dyo_pilot_predict",
-           "dyo_prediction_get", "dyo_prediction_matched", "dyo_group_entries", "dyo_plan", "dyo_plan_info", "dyo_plan_records",
+           "dyo_prediction_get", "dyo_prediction_matched", "dyo_group_entries", "dyo_plan", "dyo_plan_async", "dyo_plan_wait",
+           "dyo_plan_info", "dyo_plan_records",
            "dyo_migrate", "dyo_residency", "dyo_get_counters", "dyo_get_timings", "dyo_arch_check",
            "dyo_debug_pilot_stamps", "dyo_debug_plan_stamps", "dyo_debug_copy", "dyo_traverse_check",
            "dyo_debug_floor", "dyo_memo_config", "dyo_report", "dyo_memo_stats", "dyo_debug_copy_stamps",
@@ -456,6 +457,15 @@ class Dyo:
     def plan(self, b0=0, n=-1, stream=0):
         K = i32()
         self._check(self.L.dyo_plan(self.ctx, b0, n, C.byref(K), P(stream)))
+        self.K = K.value
+        return self.K
+
+    def plan_async(self, b0=0, n=-1, stream=0):
+        self._check(self.L.dyo_plan_async(self.ctx, b0, n, P(stream)))
+
+    def plan_wait(self):
+        K = i32()
+        self._check(self.L.dyo_plan_wait(self.ctx, C.byref(K)))
         self.K = K.value
         return self.K
 

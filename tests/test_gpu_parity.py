@@ -422,3 +422,41 @@ def test_pilot_logits_tensor_cores(name, B):
     print(f"{name} B={B}: {n_tie} predictions with a documented argmax near-tie")
     assert n_tie == 0, "decisions differ from the oracle's on a seeded config"
     d.close()
+
+
+def test_plan_async_wait_overlaps_migration_and_guards():
+    """dyo_plan_async / dyo_plan_wait: the same plan as dyo_plan (records bit-exact with the
+    oracle), the previous plan's transitions may be enqueued in between, and the calls that would
+    race with the running planner are refused (DYO_E_STATE = -5)."""
+    wl = WL.make("moe", n_samples=16)
+    wl.tensors = wl.tensors
+    d = make_ctx(wl, max_batch=1)
+    st = PL.initial_state(len(wl.tensors))
+    table = ()
+    cs = _stream()
+    prev_K = 0
+    for s in range(3):
+        r = oracle_step(wl, [s], st, table)
+        d.predict(wl.samples[[s]].copy(), hist_for(wl, 1), 1, stream=cs)
+        d.plan_async(stream=cs)
+        with pytest.raises(Exception) as ei:
+            d.predict(wl.samples[[s]].copy(), hist_for(wl, 1), 1, stream=cs)
+        assert getattr(ei.value, "status", None) == -5
+        with pytest.raises(Exception) as ei:
+            d.plan_async(stream=cs)
+        assert getattr(ei.value, "status", None) == -5
+        for j in range(prev_K):                     # the previous plan migrates meanwhile
+            d.migrate(j, cs)
+        K = d.plan_wait()
+        assert K == len(r["trs"])
+        for j, tr in enumerate(r["trs"]):
+            assert gpu_lists(d, j) == tr_lists(tr), f"step {s} transition {j}"
+        with pytest.raises(Exception) as ei:
+            d.plan_wait()
+        assert getattr(ei.value, "status", None) == -5
+        prev_K = K
+        st, table = r["state"], r["table"]
+    for j in range(prev_K):
+        d.migrate(j, cs)
+    torch.cuda.synchronize()
+    d.close()

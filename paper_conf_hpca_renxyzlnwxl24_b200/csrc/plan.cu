@@ -914,9 +914,18 @@ plan_kernel(ArchDev a, PredDev pd, int policy, PlanState in, PlanState st, PlanS
         }
       })
       nmove = (int)nmv;
-      if (tid == 0) {
-        long long c = tot;
-        for (int p = 0; p < np; ++p) { S.p_off[p] = (int)c; c += S.p_au[p]; }
+      {
+        // placed tensors after the kept run: exclusive prefix sums of their aligned sizes
+        // (contiguous placements per thread, one block scan)
+        constexpr int PP = kEntCap / PNT;
+        const int p0 = tid * PP;
+        long long ls = 0;
+#pragma unroll
+        for (int q = 0; q < PP; ++q) if (p0 + q < np) ls += S.p_au[p0 + q];
+        long long ptot = 0;
+        long long c = tot + scan64(ls, S.tmp, &ptot);
+#pragma unroll
+        for (int q = 0; q < PP; ++q) if (p0 + q < np) { S.p_off[p0 + q] = (int)c; c += S.p_au[p0 + q]; }
       }
       __syncthreads();
     }

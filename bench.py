@@ -763,12 +763,17 @@ def run_dyo(args):
     except OSError:
         pass
     shares = {k: round(v["ms"] / ms_instr, 4) for k, v in tm.items()}
-    bound_ms = step_bound_ms(timed_trs, probe["h2d"], probe["d2h"]) / args.steps
-    bound_strict_ms = step_bound_ms(timed_trs, probe["h2d"], probe["d2h"], strict=True) / args.steps
-    bidir = bidir_probe(torch)
-    bound_fluid_ms = step_bound_fluid_ms(timed_trs, probe["h2d"], probe["d2h"], bidir) / args.steps
     dma_h2d = tm["dma_h2d"]
     dma_d2h = tm["dma_d2h"]
+    # a bound needs rates no lower than the link delivered in the step: the probe (one sample,
+    # noisy on a busy box) or the DMA rate seen in the step, whichever is higher
+    rate_h = max(probe["h2d"], dma_h2d["bytes"] / (dma_h2d["ms"] * 1e6) if dma_h2d["ms"] else 0.0)
+    rate_d = max(probe["d2h"], dma_d2h["bytes"] / (dma_d2h["ms"] * 1e6) if dma_d2h["ms"] else 0.0)
+    bound_strict_ms = step_bound_ms(timed_trs, rate_h, rate_d, strict=True) / args.steps
+    # the bound of the order the run used (--strict-order: R12 everywhere)
+    bound_ms = bound_strict_ms if args.strict_order else step_bound_ms(timed_trs, rate_h, rate_d) / args.steps
+    bidir = max(bidir_probe(torch), bidir_probe(torch))
+    bound_fluid_ms = step_bound_fluid_ms(timed_trs, rate_h, rate_d, bidir, strict=args.strict_order) / args.steps
     h2d_link = dma_h2d["bytes"] / (dma_h2d["ms"] * 1e-3) / 1e9 if dma_h2d["ms"] else None
     d2h_link = dma_d2h["bytes"] / (dma_d2h["ms"] * 1e-3) / 1e9 if dma_d2h["ms"] else None
     plan_us = tm["plan"]["ms"] * 1e3 / max(1, tm["plan"]["launches"])
@@ -976,7 +981,7 @@ def step_bound_ms(trs, h2d_gbs, d2h_gbs, strict=False):
     return ready[-1] if ready else 0.0
 
 
-def step_bound_fluid_ms(trs, h2d_gbs, d2h_gbs, bidir_gbs):
+def step_bound_fluid_ms(trs, h2d_gbs, d2h_gbs, bidir_gbs, strict=False):
     """The record-level DAG of step_bound_ms (the same dependencies: each direction's queue in
     order, EVICT_j after ready[j-2], FETCH_j after the whole EVICT_j (R12) or after the write-backs
     it overwrites (R21), ready[j] after both queues' work of transition j) simulated as a fluid
@@ -988,7 +993,7 @@ def step_bound_fluid_ms(trs, h2d_gbs, d2h_gbs, bidir_gbs):
     tasks, ready_deps = [], []                                 # task: (queue 0 D2H / 1 H2D, bytes, deps)
     last = [None, None]                                        # latest task of each queue so far
     for j, tr in enumerate(trs):
-        relaxed = len(tr) > 2 and tr[4] == 0 and not tr[5] and 0 < len(tr[2]) <= 64
+        relaxed = not strict and len(tr) > 2 and tr[4] == 0 and not tr[5] and 0 < len(tr[2]) <= 64
         half = ready_deps[j - 2] if j >= 2 else []
         iv = []
         wbs = tr[2] if len(tr) > 2 else ([(0, tr[1])] if tr[1] else [])

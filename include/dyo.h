@@ -416,8 +416,9 @@ dyo_status dyo_trace_path(dyo_ctx* ctx, const int32_t* choices, const int32_t* n
 dyo_status dyo_residency(dyo_ctx* ctx, int32_t t, void** dev_ptr);
 
 /* Introspection of the last calls (tests and measurement; host-only, no synchronisation).
- *   DYO_Q_PILOT_KERNEL: kernel the last dyo_pilot_predict ran: 0 = K1 cluster GEMV (batch < 16,
- *     or DYO_PILOT_TC=0), 1 = K1-TC (tcgen05 tensor cores, batch >= 16).
+ *   DYO_Q_PILOT_KERNEL: kernel the last dyo_pilot_predict ran: 0 = K1 (cluster GEMV at batch < 8,
+ *     fp64 DMMA tensor-core tiles at batch >= 8; fp64 accumulation), 1 = K1-TC (tcgen05 3xTF32,
+ *     opt-in DYO_F_PILOT_TC, batch >= 16).
  *   DYO_Q_DECODE_FUSED: 1 if the last dyo_pilot_predict decoded in K1's epilogue, 0 if it
  *     launched the stand-alone decode kernels.
  *   DYO_Q_PLAN_SYNCS: host synchronisations taken by the last successful dyo_plan (1, §8(b)).

@@ -79,7 +79,7 @@ decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int 
   bool staged = false;
   ArchDev A = a;
   const int n_items = pd.B * Km;
-  for (int item = blockIdx.x; item < n_items; item += (pending_pass ? gridDim.x : n_items)) {
+  for (int item = blockIdx.x; item < n_items; item += gridDim.x) {
     const int b = item / Km, g = item % Km;
     if (pending_pass) {
       if (threadIdx.x == 0) s_todo = pd.ent_n[(int64_t)b * Km + g] == -1;
@@ -152,7 +152,14 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
   // PredDev.B = the allocation's batch: the kernels walk B x K_max items of this call only
   PredDev pb = pd;
   pb.B = B;
-  e = launch_pdl(decode_groups_kernel<kRecSmall>, dim3(B * a.K_max), dim3(kDecThreads), smA, s, a, pb, hist_tab_out, tab_cap, 0);
+  // first pass: one item per CTA while the batch fits a few CTAs per SM (MoE / LSTM: 64 x 16
+  // slots, one wave); larger batches (AF: 64 x 256 slots) loop over items grid-stride, so each CTA
+  // stages the decode tables once instead of once per slot
+  static int sms1_d[64] = {};
+  int& sms1 = sms1_d[dv];
+  if (!sms1) cudaDeviceGetAttribute(&sms1, cudaDevAttrMultiProcessorCount, dv);
+  const int gA = B * a.K_max < 8 * sms1 ? B * a.K_max : 8 * sms1;
+  e = launch_pdl(decode_groups_kernel<kRecSmall>, dim3(gA), dim3(kDecThreads), smA, s, a, pb, hist_tab_out, tab_cap, 0);
   if (e != cudaSuccess) return e;
   static int sms_d[64] = {};
   int& sms = sms_d[dv];

@@ -4,6 +4,7 @@
 // (prediction, group slot)). No materialised path.
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <cstdlib>
 
 #include "decode_dev.cuh"
 
@@ -115,6 +116,158 @@ decode_groups_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int 
   }
 }
 
+// First pass, one WARP per (prediction, group slot): the groups of <= 64 access records (the
+// common case: MoE / AF / LSTM blocks) need no block barrier at all - rows, counts and signature
+// sums by lane, a warp scan for the record positions, the record sort / dedup of build_group's
+// warp path - so a CTA builds kDecThreads/32 groups at once instead of one. A group with more
+// records is left pending (ent_n = -1) for the full-capacity block pass, exactly as before.
+constexpr int kWarpRec = 64;
+struct WarpGroupSmem {
+  int32_t rec_t[kWarpRec];
+  int32_t rec_m[kWarpRec];
+  uint64_t key[kWarpRec];
+};
+struct WarpHead {                    // same member names as DecHead (build helpers are templated)
+  int* start;
+  int* cum;
+  int* cntc;
+  int* choice;
+  int L, nk, K;
+  int b;
+};
+
+__global__ void __launch_bounds__(kDecThreads)
+decode_groups_warp_kernel(ArchDev a, PredDev pd, int32_t* __restrict__ hist_tab, int tab_cap, int hw_words) {
+  pdl_enter();
+  extern __shared__ __align__(16) unsigned char dsm[];
+  const int nwarps = blockDim.x >> 5, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  WarpGroupSmem* WG = reinterpret_cast<WarpGroupSmem*>(dsm);
+  int* hw_all = reinterpret_cast<int*>(dsm + sizeof(WarpGroupSmem) * nwarps);
+  int* tabs = hw_all + (size_t)hw_words * nwarps;
+  const ArchDev A = stage_decode_tables(a, tabs, tab_cap);   // once per CTA (ends with a barrier)
+  WarpGroupSmem& G = WG[warp];
+  int* hw = hw_all + (size_t)hw_words * warp;
+  const int ns = a.n_sites, np = a.n_pieces, Km = a.K_max;
+  WarpHead H;
+  H.start = hw;
+  H.cum = hw + np + 1;
+  H.cntc = H.cum + Km + 1;
+  H.choice = H.cntc + Km;
+  const int n_items = pd.B * Km;
+  for (int item = blockIdx.x * nwarps + warp; item < n_items; item += gridDim.x * nwarps) {
+    const int b = item / Km, g = item % Km;
+    const int* h = head_of(pd, b);
+    const int K = h[2];
+    int32_t* ent_n = pd.ent_n + (int64_t)b * Km + g;
+    if (g >= K) {
+      if (lane == 0) *ent_n = 0;
+      continue;
+    }
+    H.L = h[0]; H.nk = h[1]; H.K = K; H.b = b;
+    const int* hc = h + 3;
+    for (int i = lane; i < ns; i += 32) H.choice[i] = hc[i];
+    const int* hs = hc + ns;
+    for (int i = lane; i <= np; i += 32) H.start[i] = hs[i];
+    const int* hcum = hs + np + 1;
+    const int* hcnt = hcum + Km + 1;
+    for (int i = lane; i < H.nk; i += 32) { H.cum[i] = hcum[i]; H.cntc[i] = hcnt[i]; }
+    __syncwarp();
+    const int s = group_start(H, g), e = group_end(H, g);
+    const int nrows = e - s;
+    if (lane == 0) {
+      pd.grp[((int64_t)b * Km + g) * 2] = s;
+      pd.grp[((int64_t)b * Km + g) * 2 + 1] = e;
+    }
+    // rows in contiguous chunks per lane: access counts and signature sums
+    const int chunk = (nrows + 31) / 32;
+    const int rs = s + lane * chunk, re = min(e, rs + chunk);
+    long long sg[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
+    int cnt = 0;
+    for (int r = rs; r < re; ++r) {
+      const int op = row_op(A, H, r);
+      if (op >= 0) {
+        cnt += A.acc_ptr[op + 1] - A.acc_ptr[op];
+#pragma unroll
+        for (int k = 0; k < 9; ++k) sg[k] += A.op_sig[(int64_t)op * 9 + k];
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < 9; ++k)
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) sg[k] += __shfl_xor_sync(0xffffffffu, sg[k], o);
+    const int inc = warp_incl_scan(cnt, lane);
+    const int n = __shfl_sync(0xffffffffu, inc, 31);
+    if (n > kWarpRec) {                          // the full-capacity block pass builds it
+      if (lane == 0) *ent_n = -1;
+      __syncwarp();
+      continue;
+    }
+    int pos = inc - cnt;
+    for (int r = rs; r < re; ++r) {
+      int it = 0;
+      const int op = row_op(A, H, r, &it);
+      if (op < 0) continue;
+      for (int q = A.acc_ptr[op]; q < A.acc_ptr[op + 1]; ++q, ++pos) {
+        G.rec_t[pos] = A.acc_t[q] + A.acc_s[q] * it + A.acc_sb[q] * b;   // R13 (validated at load)
+        G.rec_m[pos] = A.acc_m[q];
+      }
+    }
+    // block vector (R1) of the group: lanes 0..9
+    if (lane < 10) {
+      int v;
+      if (lane == 0) {
+        v = min(nrows, kSat);
+      } else {
+        long long x = 0;
+#pragma unroll
+        for (int k = 0; k < 9; ++k) if (k == lane - 1) x = sg[k];
+        v = (int)min(x, (long long)kSat);
+      }
+      pd.blocks[((int64_t)b * Km + g) * 10 + lane] = v;
+      hist_tab[((int64_t)b * Km + g) * 10 + lane] = v;
+    }
+    __syncwarp();
+    // records -> tensors in first-access order with their mode union (build_group's warp path)
+    uint64_t x = lane < n ? ((uint64_t)(uint32_t)G.rec_t[lane] << 32) | ((uint64_t)lane << 2) | (uint64_t)G.rec_m[lane] : ~0ull;
+    uint64_t z = lane + 32 < n ? ((uint64_t)(uint32_t)G.rec_t[lane + 32] << 32) | ((uint64_t)(lane + 32) << 2) |
+                                     (uint64_t)G.rec_m[lane + 32]
+                               : ~0ull;
+    warp_sort64(x, z, lane);
+    G.key[lane] = x;
+    G.key[lane + 32] = z;
+    __syncwarp();
+    uint64_t o[2];
+#pragma unroll
+    for (int hh = 0; hh < 2; ++hh) {
+      const int i = lane + 32 * hh;
+      o[hh] = ~0ull;
+      if (i < n) {
+        const uint32_t t = (uint32_t)(G.key[i] >> 32);
+        if (i == 0 || (uint32_t)(G.key[i - 1] >> 32) != t) {
+          const uint32_t p0 = (uint32_t)(G.key[i] & 0xffffffffu) >> 2;
+          const uint32_t m0 = (uint32_t)G.key[i] & 3u;
+          uint32_t mu = m0;
+          for (int k = i + 1; k < n && (uint32_t)(G.key[k] >> 32) == t; ++k) mu |= (uint32_t)G.key[k] & 3u;
+          o[hh] = ((uint64_t)p0 << 32) | ((uint64_t)t << 3) | (mu << 1) | (m0 & 1u);
+        }
+      }
+    }
+    warp_sort64(o[0], o[1], lane);
+    const int u = __popc(__ballot_sync(0xffffffffu, o[0] != ~0ull)) + __popc(__ballot_sync(0xffffffffu, o[1] != ~0ull));
+    int2* ent = pd.ent + ((int64_t)b * Km + g) * kEntCap;
+#pragma unroll
+    for (int hh = 0; hh < 2; ++hh) {
+      const int i = lane + 32 * hh;
+      if (i < u) {
+        const uint32_t lo = (uint32_t)(o[hh] & 0xffffffffu);
+        ent[i] = make_int2((int)(lo >> 3), (int)(((lo >> 1) & 3u) | ((lo & 1u) << 2)));
+      }
+    }
+    if (lane == 0) *ent_n = u;
+    __syncwarp();
+  }
+}
+
 template <int R>
 size_t groups_smem(const ArchDev& a, int tab_cap) {
   const int hw = (a.n_pieces + 1 + 2 * a.K_max + 1 + a.n_sites + 3) / 4 * 4;
@@ -158,8 +311,26 @@ cudaError_t launch_decode(const ArchDev& a, const double* logits, PredDev& pd, i
   static int sms1_d[64] = {};
   int& sms1 = sms1_d[dv];
   if (!sms1) cudaDeviceGetAttribute(&sms1, cudaDevAttrMultiProcessorCount, dv);
-  const int gA = B * a.K_max < 8 * sms1 ? B * a.K_max : 8 * sms1;
-  e = launch_pdl(decode_groups_kernel<kRecSmall>, dim3(gA), dim3(kDecThreads), smA, s, a, pb, hist_tab_out, tab_cap, 0);
+  static int warp_on = -1;
+  if (warp_on < 0) { const char* ev = getenv("DYO_DECODE_WARP"); warp_on = (ev && ev[0] == '0') ? 0 : 1; }
+  if (warp_on) {
+    // one warp per group slot (<= 64 records; larger groups pending for the block pass)
+    const int hw_words = (a.n_pieces + 1 + 2 * a.K_max + 1 + a.n_sites + 3) / 4 * 4;
+    const int nw = kDecThreads / 32;
+    const size_t smW = sizeof(WarpGroupSmem) * nw + (size_t)hw_words * 4 * nw + (size_t)tab_cap * 4;
+    static size_t setW_d[64] = {};
+    if (smW > setW_d[dv]) {
+      cudaError_t ee = cudaFuncSetAttribute(decode_groups_warp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smW);
+      if (ee != cudaSuccess) return ee;
+      setW_d[dv] = smW;
+    }
+    const int items = B * a.K_max, blocks = (items + nw - 1) / nw;
+    const int gW = blocks < 8 * sms1 ? blocks : 8 * sms1;
+    e = launch_pdl(decode_groups_warp_kernel, dim3(gW), dim3(kDecThreads), smW, s, a, pb, hist_tab_out, tab_cap, hw_words);
+  } else {
+    const int gA = B * a.K_max < 8 * sms1 ? B * a.K_max : 8 * sms1;
+    e = launch_pdl(decode_groups_kernel<kRecSmall>, dim3(gA), dim3(kDecThreads), smA, s, a, pb, hist_tab_out, tab_cap, 0);
+  }
   if (e != cudaSuccess) return e;
   static int sms_d[64] = {};
   int& sms = sms_d[dv];

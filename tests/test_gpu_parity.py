@@ -429,7 +429,6 @@ def test_plan_async_wait_overlaps_migration_and_guards():
     oracle), the previous plan's transitions may be enqueued in between, and the calls that would
     race with the running planner are refused (DYO_E_STATE = -5)."""
     wl = WL.make("moe", n_samples=16)
-    wl.tensors = wl.tensors
     d = make_ctx(wl, max_batch=1)
     st = PL.initial_state(len(wl.tensors))
     table = ()
